@@ -1,0 +1,422 @@
+#!/usr/bin/env python
+"""Benchmark of the PDL-mapped blocked matmul (BASELINE.json metric:
+"matmul GFLOP/s at 1/2/4/8 B200 and % of tensor-core peak").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--dtype f64|f32]
+                    [--config C4] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...      (one process per GPU)
+
+A step is one pass of the whole hot path over one batch
+of synthetic input: at N = 1 one FP64 DGEMM task (paper's precision,
+PAPER.md L1402-1406) of config C4 (16384^3, tile 1024) through
+task_matmul + pdl_run; at N > 1 the operand-panel exchange over NCCL
+(all-gather in grid rows / columns) followed by each Worker's rectangle.
+Strong scaling: the same 16384^3 problem is split over the N Workers.
+
+Timed region (value): operands resident in HBM (N = 1: whole matrices; N > 1:
+each Worker's unique chunks), W warm-up steps, then K steps bracketed by a
+barrier + torch.cuda.synchronize(), CUDA events on the launching stream, max
+over ranks.  Inputs (6 GiB FP64) are far larger than the 126 MB L2.
+e2e: the same metric with host (pinned) operands through the public API,
+host<->device copies inside the timed region.
+
+Rank 0 prints ONE JSON line.  --impl reference times the CPU oracle
+(oracle/, a plain triple loop accumulating in double) on a bounded row sample
+of the same workload -- the reference arm of this tier.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "matmul GFLOP/s at 1/2/4/8 B200 and % of tensor-core peak"
+PROFILES = os.path.join(ROOT, "profiles")
+# FP64 DMMA peak measured on this box class with tools/microbench (mma.sync
+# m8n8k4 from registers, 148 x 2 CTAs): profiles/r01_microbench.json.
+FP64_DMMA_PEAK_TFLOPS = 37.0
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--dtype", choices=("f64", "f32"), default="f64")
+    p.add_argument("--config", default="C4")
+    p.add_argument("--impl", choices=("ours", "reference"), default="ours")
+    p.add_argument("--e2e-steps", type=int, default=3)
+    p.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle sample budget")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cublas", action="store_true")
+    return p.parse_args()
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except OSError:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+def tensor_peak(dtype):
+    """Precision-matched tensor-core peak (TFLOP/s) and where it comes from."""
+    pk, src = peaks()
+    if dtype == "f64":
+        return FP64_DMMA_PEAK_TFLOPS, "FP64 DMMA measured (tools/microbench, profiles/r01_microbench.json)"
+    # TF32 = bf16 measured burst x nominal tf32/bf16 ratio (1.1 / 2.25)
+    return pk["bf16_tflops"] * 1.1 / 2.25, f"TF32 = {src} bf16 burst {pk['bf16_tflops']} x 1.1/2.25"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.path = None
+
+    def __enter__(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+            time.sleep(0.3)
+        except OSError:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.2)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.path or not os.path.exists(self.path):
+            return None
+        rows = []
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append((float(parts[1]), float(parts[2]), parts[5:9]))
+            except ValueError:
+                continue
+        os.unlink(self.path)
+        if not rows:
+            return None
+        maxmhz = max(r[1] for r in rows)
+        loaded = [r for r in rows if r[0] > 0.5 * maxmhz] or rows
+        names = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[2][i].lower() == "active"})
+        return {"sm_mhz": float(np.median([r[0] for r in loaded])), "sm_max_mhz": maxmhz,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def ncu_traffic(dtype, cfg):
+    """DRAM bytes per launch of the dominant kernel from a committed ncu capture."""
+    path = os.path.join(PROFILES, "ncu_traffic.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get(f"{dtype}/{cfg}")
+    except (OSError, ValueError):
+        return None
+
+
+def host_inputs(cfg, np_dtype):
+    return W.config_inputs(cfg, np_dtype)
+
+
+def cpu_baseline(A, B, seconds):
+    """Time the oracle (as it stands) on a bounded row sample of the workload."""
+    import oracle
+    M, K = A.shape
+    N = B.shape[1]
+    rng = np.random.Generator(np.random.PCG64(99))
+    t0 = time.perf_counter()
+    oracle.matmul(A, B, rows=rng.integers(0, M, size=2), with_mag=False)
+    t1 = time.perf_counter()
+    per_row = max((t1 - t0) / 2, 1e-6)
+    nrows = int(max(2, min(M, seconds / per_row)))
+    rows = rng.integers(0, M, size=nrows)
+    t0 = time.perf_counter()
+    oracle.matmul(A, B, rows=rows, with_mag=False)
+    dt = time.perf_counter() - t0
+    gflops = 2.0 * nrows * N * K / dt / 1e9
+    return {"value": round(gflops, 3), "unit": "GFLOP/s", "cores": oracle.max_threads(), "kind": "oracle",
+            "sample": f"{nrows} random rows x all {N} columns of the {M}x{N}x{K} product "
+                      f"({2.0 * nrows * N * K:.3g} FLOP, {dt:.1f} s, double accumulation)"}
+
+
+def run_reference(args):
+    """Reference arm: the CPU oracle on the box's host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    c = W.CONFIGS[args.config]
+    np_dtype = np.float64 if args.dtype == "f64" else np.float32
+    A, B = host_inputs(args.config, np_dtype)
+    import oracle
+    rng = np.random.Generator(np.random.PCG64(5))
+    per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    t0 = time.perf_counter()
+    oracle.matmul(A, B, rows=rng.integers(0, c.M, size=2), with_mag=False)
+    per_row = max((time.perf_counter() - t0) / 2, 1e-6)
+    nrows = int(max(1, min(c.M, per_step / per_row)))
+    flops = 2.0 * nrows * c.N * c.K
+    for _ in range(args.warmup):
+        oracle.matmul(A, B, rows=rng.integers(0, c.M, size=nrows), with_mag=False)
+    times = []
+    for _ in range(args.steps):
+        rows = rng.integers(0, c.M, size=nrows)
+        t0 = time.perf_counter()
+        oracle.matmul(A, B, rows=rows, with_mag=False)
+        times.append(time.perf_counter() - t0)
+    ms = 1e3 * sum(times) / len(times)
+    value = flops / (ms / 1e3) / 1e9
+    line = {"metric": METRIC, "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
+            "data": "synthetic", "impl": "reference",
+            "config": {"workload": f"{args.config} {c.M}x{c.N}x{c.K} ({args.dtype}), oracle row sample",
+                       "M": c.M, "N": c.N, "K": c.K, "tile": c.tile, "rows_per_step": nrows},
+            "cpu_baseline": {"value": round(value, 3), "unit": "GFLOP/s", "cores": oracle.max_threads(),
+                             "kind": "oracle",
+                             "sample": f"{nrows} random rows x {c.N} columns per step (K={c.K})"},
+            "e2e": {"value": round(value, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}: launch N>1 with torchrun")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    os.environ.pop("PDL_DRY_RUN", None)
+
+    c = W.CONFIGS[args.config]
+    M, N, K = c.M, c.N, c.K
+    np_dtype = np.float64 if args.dtype == "f64" else np.float32
+    tdt = torch.float64 if args.dtype == "f64" else torch.float32
+    es = 8 if args.dtype == "f64" else 4
+    A, B = host_inputs(args.config, np_dtype)
+
+    if world == 1:
+        pdl.load(pdl.descriptor_path(1))
+    else:
+        pdl.load(pdl.descriptor_path(world), rank=rank, nranks=world)
+    stream = torch.cuda.current_stream()
+    pdl.set_stream(stream)
+
+    wp = runtime.worker_plan(M, N, K, c.tile, rank)
+    flops_total = 2.0 * M * N * K
+    flops_worker = 2.0 * wp.rows * wp.cols * K
+
+    # ---- device-resident operands ----
+    if world == 1:
+        dA = torch.from_numpy(A).to(dev)
+        dB = torch.from_numpy(B).to(dev)
+        dC = torch.empty((M, N), dtype=tdt, device=dev)
+
+        def step():
+            pdl.task_matmul(dA, dB, dC, tile=c.tile)
+            pdl.run_async()
+    else:
+        grid = runtime.Grid(wp.Gr, wp.Gc, rank)
+        Ach, Bch = runtime.chunk_from_full(torch.from_numpy(A), torch.from_numpy(B), wp)
+        Ach, Bch = Ach.to(dev), Bch.to(dev)
+        bufs = runtime.PanelBuffers(wp, tdt, dev)
+        dC = torch.empty((wp.rows, wp.cols), dtype=tdt, device=dev)
+
+        def step():
+            Ap, Bp = runtime.exchange(Ach, Bch, wp, grid, bufs)
+            runtime.local_task(Ap, Bp, dC, wp, tile=c.tile)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(args.warmup):
+        step()
+    pdl.sync()
+    torch.cuda.synchronize()
+    st = pdl.query_json("stats")
+    launches_per_step = st["launches"]
+    pdl.kernel_times()   # clear
+
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    ms_total = e0.elapsed_time(e1)
+    ktimes = pdl.kernel_times()
+    clocks = clk.summary()
+    if world > 1:
+        t = torch.tensor([ms_total], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+    ms_step = ms_total / args.steps
+    value = flops_total * args.steps / (ms_total / 1e3) / 1e9   # GFLOP/s, whole job
+
+    # ---- roofline of the dominant kernel (K1, or K2 for FP32) ----
+    kavg = float(np.mean(ktimes)) if ktimes else None
+    peak_tf, peak_src = tensor_peak(args.dtype)
+    pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
+    achieved_tf = pipe_flops / (kavg / 1e3) / 1e12 if kavg else None
+    roofline = {"bound": "tensor", "achieved": round(achieved_tf, 2) if achieved_tf else None,
+                "peak": round(peak_tf, 1), "unit": "TFLOP/s",
+                "frac": round(achieved_tf / peak_tf, 4) if achieved_tf else None,
+                "traffic": ncu_traffic(args.dtype, args.config),
+                "kernel": "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_kernel (tcgen05)",
+                "kernel_ms": round(kavg, 3) if kavg else None,
+                "algorithmic_flops_per_launch": pipe_flops,
+                "peak_source": peak_src}
+    if args.dtype == "f32":
+        roofline["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
+
+    # ---- e2e: host pinned operands through the public API ----
+    e2e = None
+    if not args.no_e2e:
+        if world == 1:
+            hA = torch.from_numpy(A).pin_memory()
+            hB = torch.from_numpy(B).pin_memory()
+            hC = torch.empty((M, N), dtype=tdt).pin_memory()
+
+            def estep():
+                pdl.task_matmul(hA, hB, hC, tile=c.tile)
+                pdl.run_async()
+            h2d = (M * K + K * N) * es
+            d2h = M * N * es
+        else:
+            a0, a1 = wp.a_span
+            b0, b1 = wp.b_span
+            hAch, hBch = runtime.chunk_from_full(torch.from_numpy(A), torch.from_numpy(B), wp)
+            hAch, hBch = hAch.pin_memory(), hBch.pin_memory()
+            hCb = torch.empty((wp.rows, wp.cols), dtype=tdt).pin_memory()
+            dAch = torch.empty_like(hAch, device=dev)
+            dBch = torch.empty_like(hBch, device=dev)
+
+            def estep():
+                dAch.copy_(hAch, non_blocking=True)
+                dBch.copy_(hBch, non_blocking=True)
+                Ap, Bp = runtime.exchange(dAch, dBch, wp, grid, bufs)
+                runtime.local_task(Ap, Bp, dC, wp, tile=c.tile)
+                hCb.copy_(dC, non_blocking=True)
+            h2d = ((a1 - a0) * K + (b1 - b0) * wp.cols) * es
+            d2h = wp.rows * wp.cols * es
+        estep()
+        pdl.sync()
+        torch.cuda.synchronize()
+        barrier()
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for _ in range(args.e2e_steps):
+            estep()
+            pdl.sync()
+            torch.cuda.synchronize()   # the step's result is on the host
+        t1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ems = t0.elapsed_time(t1)
+        if world > 1:
+            t = torch.tensor([ems], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": round(flops_total * args.e2e_steps / (ems / 1e3) / 1e9, 1), "unit": "GFLOP/s",
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": round(ems / args.e2e_steps, 3)}
+        if world == 1:
+            del hA, hB, hC
+        pdl.kernel_times()
+
+    # ---- context: cuBLAS (torch.matmul) on the same device-resident operands ----
+    cublas = None
+    if world == 1 and not args.no_cublas:
+        torch.backends.cuda.matmul.allow_tf32 = False
+        torch.matmul(dA, dB, out=dC)
+        torch.cuda.synchronize()
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record()
+        for _ in range(3):
+            torch.matmul(dA, dB, out=dC)
+        t1.record()
+        torch.cuda.synchronize()
+        cublas = round(flops_total * 3 / (t0.elapsed_time(t1) / 1e3) / 1e9, 1)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(A, B, args.cpu_seconds)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 1), "unit": "GFLOP/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
+            "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} ({args.dtype})",
+            "config": {"workload": f"{args.config} {M}x{N}x{K} blocked matmul, task tile {c.tile}, "
+                                   f"PDL b200_x{world}",
+                       "M": M, "N": N, "K": K, "tile": c.tile, "parallelism": f"block2d {wp.Gr}x{wp.Gc}",
+                       "l2": "inputs larger than L2 (operands >> 126 MB), no flush needed"},
+            "pct_of_tensor_peak": round(100 * value / world / (peak_tf * 1e3) * (3 if args.dtype == "f32" else 1), 2),
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": int(launches_per_step * args.steps),
+            "clocks": clocks,
+        }
+        if cublas is not None:
+            line["cublas_gflops_same_operands"] = cublas
+        print(json.dumps(line), flush=True)
+    pdl.unload()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

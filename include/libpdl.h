@@ -1,0 +1,205 @@
+/*
+ * libpdl.h -- C ABI of the B200-native PDL-mapped blocked matmul.
+ *
+ * Paper: Sandrieser, Benkner, Pllana, "Explicit Platform Descriptions for
+ * Heterogeneous Many-Core Architectures", IPDPS 2011.  Citations "L<n>" are
+ * lines of /root/reference/PAPER.md (section in parentheses).
+ *
+ * The library is the run-time counterpart of the paper's PDL-parameterised,
+ * task-annotated program (SS IV): a PDL descriptor (SS III-B/C) is parsed into
+ * the hierarchical machine model (Master / Hybrid / Worker PUs, memory
+ * regions, interconnects, SS III-A L472-603); a `task` call records one
+ * DGEMM task C = A*B (the case-study kernel, SS IV-D L1402-1406); `pdl_run`
+ * maps the task's tile tasks onto the execution group's Worker PUs with a
+ * BLOCK distribution (SS IV-A L1199-1208, SS IV-B L1254-1281), stages operands
+ * along the interconnects (SS IV-C step 3, L1336-1341) and runs the sm_100a
+ * tile kernels.
+ *
+ * Conventions (readings R1-R6):
+ *  - C = A*B with alpha = 1, beta = 0: C has access mode `write` and is
+ *    overwritten (L1184-1186); A and B have access mode `read`.
+ *  - Row-major storage.  A is M x K, B is K x N, C is M x N.  Leading
+ *    dimensions are the number of columns unless given explicitly (_ex).
+ *    Column-major callers compute C^T = B^T A^T by swapping A<->B and M<->N.
+ *  - Pointers may be host memory (pageable or pinned; the Master's memory
+ *    region) or CUDA device memory (a Worker's memory region).
+ *  - Calls are not thread-safe: one Master thread drives the library
+ *    (Master PU = "starting point for execution of a program", L495-503).
+ *  - No CPU fallback exists.  If no usable B200 Worker is bound, pdl_run
+ *    fails with PDL_ENOWORKER / PDL_ECUDA.
+ *
+ * Ownership: the caller owns A, B, C.  They must stay valid (A, B unchanged,
+ * C untouched) from the task call until pdl_run/pdl_sync returns.  The
+ * library never frees or retains them.  Library-owned device buffers (Worker
+ * memory-region staging buffers, padded/split operand panels) are cached
+ * across runs and freed by pdl_unload.
+ *
+ * Errors: every entry point returns PDL_OK (0) or a negative code and sets a
+ * thread-local message readable with pdl_last_error().  After an error inside
+ * pdl_run the queue is cleared and C's contents are unspecified.
+ */
+#ifndef LIBPDL_H
+#define LIBPDL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Return codes. */
+#define PDL_OK            0
+#define PDL_EINVAL       -1  /* bad argument (null pointer with nonzero size, negative dim, overlap, unknown group/dist) */
+#define PDL_EPARSE       -2  /* malformed XML, or a structural rule of the machine model is broken */
+#define PDL_ENOWORKER    -3  /* no gpu Worker in the execution group, or more Workers than devices */
+#define PDL_ENOMEM       -4  /* device or host allocation failed */
+#define PDL_ECUDA        -5  /* a CUDA runtime/driver call failed */
+#define PDL_ENCCL        -6  /* reserved: collective failure (the exchange runs in the Python runtime) */
+#define PDL_ESTATE       -7  /* call out of order (task before load, load twice, ...) */
+#define PDL_EUNSUPPORTED -8  /* valid request this build does not implement */
+
+/* Element types of task_matmul_ex. */
+#define PDL_F64 0            /* the paper's precision: DGEMM (L1402-1406); FP64 DMMA tensor cores */
+#define PDL_F32 1            /* FP32 in/out; 3xTF32 split on tcgen05 tensor cores (north star (2)) */
+
+/* task_matmul_ex flags. */
+#define PDL_TASK_PANELS 1u   /* operands are this process's Worker panels (after the exchange):
+                                A = rows_w x K, B = K x cols_w, C = rows_w x cols_w block at
+                                the Worker's rectangle; see pdl_plan */
+
+/*
+ * pdl_load -- parse a PDL descriptor and build the machine model.
+ * descriptor: path to an XML file, or XML text if its first non-blank
+ *   character is '<'.  Entities: Master/Hybrid/Worker with PUDescriptor,
+ *   MemoryRegion(MRDescriptor), Interconnect(ICDescriptor),
+ *   LogicGroupAttribute; Descriptor -> Property(name, value) (L668-680);
+ *   prefixed tags (ocl:name) match by local name (L876-909).
+ * Rules checked (L495-531): >= 1 Master, Masters only at top level, Workers
+ *   are leaves controlled by a Master or Hybrid, Hybrids are controlled by a
+ *   Master or Hybrid, Interconnect endpoints exist, quantity >= 1, ids unique.
+ * Worker PUs with ARCHITECTURE (alias ARCH, value case-insensitive) = gpu are
+ *   bound to CUDA devices (DEVICE_ORDINAL property, else in document order)
+ *   and their unfixed properties are filled from the device (L737-747).
+ * This process is the single Master driving every Worker of the descriptor.
+ * Env: PDL_DRY_RUN=1 skips device binding (plans only; no device work);
+ *   PDL_ALLOW_OVERSUBSCRIBE=1 lets several Workers share a device.
+ * Errors: PDL_ESTATE if already loaded; PDL_EPARSE; PDL_ENOWORKER; PDL_ECUDA.
+ */
+int pdl_load(const char *descriptor);
+
+/*
+ * pdl_load_rank -- as pdl_load, for one process per GPU: `nranks` Masters
+ * co-exist ("Masters ... may co-exist with other Masters within the same
+ * system", L495-503) and process `rank` controls exactly Worker instance
+ * `rank` of the execution group, bound to the process's current CUDA device.
+ * nranks must equal the group's Worker count (checked at pdl_run).
+ * rank = 0, nranks = 1 is pdl_load.
+ */
+int pdl_load_rank(const char *descriptor, int rank, int nranks);
+
+/*
+ * task_matmul -- record one FP64 DGEMM task C = A*B (L1402-1406) with task
+ * tile edge `tile` (> 0: tile x tile tile tasks, the last row/column of tasks
+ * partial; 0: one task per Worker rectangle).  Access modes: A read, B read,
+ * C write (L1184-1186).  No device work happens here.
+ * Quick returns: M == 0 or N == 0 -> no-op; K == 0 -> C is zero-filled.
+ * Errors: PDL_ESTATE before pdl_load; PDL_EINVAL for negative sizes, null
+ *   pointers with nonzero sizes, C overlapping A or B.
+ */
+int task_matmul(const double *A, const double *B, double *C,
+                int64_t M, int64_t N, int64_t K, int64_t tile);
+
+/* task_matmul_f32 -- FP32 variant of the same task interface (3xTF32 tcgen05). */
+int task_matmul_f32(const float *A, const float *B, float *C,
+                    int64_t M, int64_t N, int64_t K, int64_t tile);
+
+/*
+ * task_matmul_ex -- general form.
+ * dtype: PDL_F64 | PDL_F32.  lda/ldb/ldc: leading dimensions in elements
+ *   (0 = dense: K, N, N; in PANELS mode 0 = K, cols_w, cols_w).
+ * group: LogicGroupAttribute naming the execution group (L1193-1199,
+ *   L1254-1261); NULL = every gpu Worker.
+ * dist: "BLOCK" (or NULL) -- the only distribution implemented
+ *   (L1200-1206); "CYCLIC"/"BLOCK-CYCLIC" -> PDL_EUNSUPPORTED.
+ * flags: 0 or PDL_TASK_PANELS.
+ */
+int task_matmul_ex(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb,
+                   void *C, int64_t ldc, int64_t M, int64_t N, int64_t K, int64_t tile,
+                   const char *group, const char *dist, unsigned flags);
+
+/*
+ * pdl_run -- map and execute all queued tasks in program order (access-mode
+ * dependencies reduce to queue order for one task type), then synchronise,
+ * harvest errors and clear the queue.  Blocks until C is written.
+ */
+int pdl_run(void);
+
+/* pdl_run_async -- as pdl_run without the final synchronisation; errors of
+ * the device work surface at the next pdl_sync.  The queue is cleared. */
+int pdl_run_async(void);
+
+/* pdl_sync -- wait for all device work issued by pdl_run_async. */
+int pdl_sync(void);
+
+/*
+ * pdl_set_stream -- launch this process's device work for Worker `worker`
+ * (local index, 0 in rank mode) on the given cudaStream_t (NULL = the
+ * library's own stream, which is a blocking stream, i.e. ordered with the
+ * legacy default stream; pass cudaStreamLegacy = (void*)1 for the legacy
+ * default stream itself).  Lets a caller order the library with its own
+ * stream and time it with its own events.
+ */
+int pdl_set_stream(int worker, void *stream);
+
+/*
+ * pdl_plan -- the BLOCK mapping of an M x N x K task with task edge `tile`
+ * onto the execution group (L1200-1206; SS IV-B static mapping L1254-1281).
+ * Writes PDL_PLAN_LEN int64 values to out[] (nout >= PDL_PLAN_LEN):
+ *   [0] G        Workers in the group        [1] Gr, [2] Gc  worker grid
+ *   [3] r, [4] c grid position of group Worker `worker` (w = r*Gc + c)
+ *   [5] row0, [6] row1, [7] col0, [8] col1   the Worker's C rectangle
+ *   [9] qa   rows per A chunk: the A row-panel (rows row0..row1) is split in
+ *            Gc chunks of qa rows; this Worker holds chunk c
+ *   [10] qb  K-rows per B chunk: the B column-panel (cols col0..col1) is
+ *            split in Gr chunks of qb K-rows; this Worker holds chunk r
+ *   [11] T_m, [12] T_n  task grid (ceil(M/tile) x ceil(N/tile))
+ *   [13] tr0, [14] tr1, [15] tc0, [16] tc1  the Worker's task rows / cols
+ *   [17] tile  effective task edge (0 in the request -> per-Worker blocks)
+ * Errors: PDL_ESTATE before pdl_load; PDL_EINVAL; PDL_ENOWORKER.
+ */
+#define PDL_PLAN_LEN 18
+int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group,
+             int worker, int64_t *out, int nout);
+
+/*
+ * pdl_query -- the "simple query API" over the loaded PDL (L935-937).
+ * Keys: "version", "masters", "workers", "groups", "model" (JSON),
+ *   "plan" (JSON of the last run's mappings), "stats" (JSON: launches,
+ *   kernel time of the last run), "worker/<i>/<PROPERTY>",
+ *   "worker/<i>/device", "worker/<i>/id", "pu/<id>/<PROPERTY>",
+ *   "interconnects" (JSON).
+ * Writes a NUL-terminated string (truncated to len-1) and returns the full
+ * length, or a negative code (PDL_EINVAL for an unknown key).
+ */
+int pdl_query(const char *key, char *out, size_t len);
+
+/*
+ * pdl_kernel_times -- device durations (ms, CUDA events on the launching
+ * stream) of the dominant tile-kernel launches (K1, or K2 for FP32) issued
+ * for local Worker `worker` since the previous call, in launch order.  Waits
+ * for those launches, writes min(count, n) values to ms[], clears the record
+ * and returns the count (at most 4096 are kept).
+ */
+int pdl_kernel_times(int worker, float *ms, int n);
+
+/* Message of the last error of this thread ("" if none). */
+const char *pdl_last_error(void);
+
+/* Free library-owned buffers and the model; the library can be loaded again. */
+void pdl_unload(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LIBPDL_H */

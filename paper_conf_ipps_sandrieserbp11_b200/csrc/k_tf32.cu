@@ -1,0 +1,347 @@
+// k_tf32.cu -- K3 (TF32 hi/lo split) and K2 (3xTF32 tile kernel on tcgen05).
+//
+// FP32 variant of the DGEMM task (same task interface, L1032-1039; the paper's
+// own task is FP64, L1402-1406; the FP32 variant follows the north star's
+// "if inputs are FP32, use split-TF32/3xTF32 ... so accuracy holds").
+//
+// Split (K3): x = hi + lo + r with hi = rna_tf32(x), lo = rna_tf32(x - hi)
+// (x - hi is exact in fp32), |r| <= 2^-22 |x|.  Product (K2):
+//   a*b ~= a_lo*b_hi + a_hi*b_lo + a_hi*b_hi     (a_lo*b_lo, ~2^-22, dropped)
+// The split is a pre-pass that also transposes B to K-major, so both UMMA
+// operands use the canonical K-major SWIZZLE_128B layout.
+//
+// K2 (v1, DESIGN.md SS Kernels/K2): CTA tile 128 x 128, BK = 32 fp32 (one
+// 128-byte swizzle atom), 3-stage TMA ring of {A_hi, A_lo, B_hi, B_lo};
+// warp 0 = TMA producer, warp 1 = TMEM allocator + single-thread tcgen05.mma
+// issuer (kind::tf32, M=128, N=128, K=8 per instruction, FP32 accumulator in
+// TMEM, 128 columns), warps 2..5 = epilogue (tcgen05.ld 32x32b -> registers
+// -> vectorised global stores).
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace pdlk {
+
+// ------------------------------------------------------------------------
+// K3: split pre-pass
+// ------------------------------------------------------------------------
+__device__ __forceinline__ float tf32_rna(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return __uint_as_float(r);
+}
+
+__global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int64_t M, int64_t K,
+                                  float *__restrict__ hi, float *__restrict__ lo, int64_t Kp) {
+    // one thread per 4 consecutive k of one row (Kp % 4 == 0)
+    const int64_t q = Kp >> 2;
+    const int64_t total = M * q;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = t / q, k0 = (t - i * q) << 2;
+        const float *src = A + i * lda;
+        float v[4], h[4], l[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) v[u] = (k0 + u < K) ? __ldg(src + k0 + u) : 0.0f;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            h[u] = tf32_rna(v[u]);
+            l[u] = tf32_rna(v[u] - h[u]);
+        }
+        *reinterpret_cast<float4 *>(hi + i * Kp + k0) = make_float4(h[0], h[1], h[2], h[3]);
+        *reinterpret_cast<float4 *>(lo + i * Kp + k0) = make_float4(l[0], l[1], l[2], l[3]);
+    }
+}
+
+// B (K x N) -> B^T split (N x Kp); 32 x 32 tiles through shared memory.
+__global__ void split_cols_t_kernel(const float *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
+                                    float *__restrict__ hi, float *__restrict__ lo, int64_t Kp) {
+    __shared__ float t[32][33];
+    const int64_t k0 = (int64_t)blockIdx.y * 32, n0 = (int64_t)blockIdx.x * 32;
+    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
+        const int64_t k = k0 + r, n = n0 + threadIdx.x;
+        t[r][threadIdx.x] = (k < K && n < N) ? __ldg(B + k * ldb + n) : 0.0f;
+    }
+    __syncthreads();
+    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
+        const int64_t n = n0 + r, k = k0 + threadIdx.x;
+        if (n < N && k < Kp) {
+            const float v = t[threadIdx.x][r];
+            const float h = tf32_rna(v);
+            hi[n * Kp + k] = h;
+            lo[n * Kp + k] = tf32_rna(v - h);
+        }
+    }
+}
+
+cudaError_t launch_split_rows(const float *A, int64_t lda, int64_t M, int64_t K, float *hi, float *lo, int64_t Kp,
+                              cudaStream_t s) {
+    if (M <= 0 || Kp <= 0) return cudaSuccess;
+    const int64_t total = M * (Kp >> 2);
+    int blocks = (int)((total + 255) / 256);
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, M, K, hi, lo, Kp);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t N, float *hi, float *lo, int64_t Kp,
+                                cudaStream_t s) {
+    if (N <= 0 || Kp <= 0) return cudaSuccess;
+    dim3 grid((unsigned)((N + 31) / 32), (unsigned)((Kp + 31) / 32));
+    split_cols_t_kernel<<<grid, dim3(32, 8), 0, s>>>(B, ldb, K, N, hi, lo, Kp);
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------
+// K2: 3xTF32 tcgen05 GEMM
+// ------------------------------------------------------------------------
+namespace k2 {
+constexpr int BM = 128, BN = 128, BK = K2_BK, STAGES = 3;
+constexpr int UMMA_K = 8;                           // tf32: 32 bytes of K per instruction
+constexpr int A_BYTES = BM * BK * 4;                // 16 KiB
+constexpr int B_BYTES = BN * BK * 4;                // 16 KiB
+constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;   // hi + lo of both operands
+constexpr int EPI_WARPS = 4;
+constexpr int THREADS = (2 + EPI_WARPS) * 32;
+constexpr int TMEM_COLS = 2 * BN;                   // double-buffered FP32 accumulator
+// K-chunk promotion (R16): the tensor cores accumulate a chunk of
+// KCB k-blocks (KCB*BK = 128 of K) in TMEM; the epilogue warps add each chunk
+// sum into an FP32 register accumulator with round-to-nearest while the MMA
+// warp fills the other TMEM buffer.  Measured on the B200 the TMEM
+// accumulation truncates (mean signed error -1.0e-8 * K for U[0,1) inputs),
+// so without promotion K >= 1024 breaks the 1e-5 bar.
+constexpr int KCB = 4;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+}  // namespace k2
+
+// UMMA shared-memory descriptor: K-major, SWIZZLE_128B, 8-row groups 1024 B apart.
+__device__ __forceinline__ uint64_t umma_desc_k_sw128(uint32_t saddr) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFFu);          // start address
+    d |= (uint64_t)(1u) << 16;                         // LBO (ignored for swizzled K-major)
+    d |= (uint64_t)(1024u >> 4) << 32;                 // SBO: 8 rows x 128 B
+    d |= (uint64_t)1u << 46;                           // descriptor version (sm_100)
+    d |= (uint64_t)2u << 61;                           // SWIZZLE_128B
+    return d;
+}
+
+// Instruction descriptor: kind::tf32, D = F32, A/B = TF32, both K-major.
+__host__ __device__ constexpr uint32_t idesc_tf32(int M, int N) {
+    return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ void umma_tf32(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+
+__device__ __forceinline__ void umma_commit(uint32_t bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar)
+                 : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+__global__ void __launch_bounds__(k2::THREADS, 1)
+    gemm_3xtf32_kernel(const __grid_constant__ CUtensorMap tAh, const __grid_constant__ CUtensorMap tAl,
+                       const __grid_constant__ CUtensorMap tBh, const __grid_constant__ CUtensorMap tBl,
+                       float *__restrict__ C, int64_t ldc, int M, int N, int Kp, int tiles_m, int tiles_n,
+                       int vec_ok) {
+    using namespace k2;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
+    const uint32_t bar_full = base + STAGES * STAGE_BYTES;      // STAGES x 8
+    const uint32_t bar_empty = bar_full + STAGES * 8;            // STAGES x 8
+    const uint32_t bar_tfull = bar_empty + STAGES * 8;           // 2 x 8: accumulator buffer ready
+    const uint32_t bar_tempty = bar_tfull + 16;                  // 2 x 8: accumulator buffer drained
+    const uint32_t tmem_slot = bar_tempty + 16;                  // 4 bytes
+    uint8_t *const gbase = smem_raw + (base - smem_u32(smem_raw));
+    volatile uint32_t *tmem_slot_ptr = reinterpret_cast<volatile uint32_t *>(gbase + (tmem_slot - base));
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    // grouped raster (16 tile rows per group)
+    const int bid = blockIdx.x;
+    const int per_group = 16 * tiles_n;
+    const int g = bid / per_group;
+    const int first_m = g * 16;
+    const int gsz = min(tiles_m - first_m, 16);
+    const int tm = first_m + (bid % per_group) % gsz;
+    const int tn = (bid % per_group) / gsz;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(bar_full + 8 * s, 1);
+            mbar_init(bar_empty + 8 * s, 1);
+        }
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(bar_tfull + 8 * b, 1);
+            mbar_init(bar_tempty + 8 * b, EPI_WARPS);
+        }
+        fence_barrier_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(tmem_slot),
+                     "n"(TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem_base = *tmem_slot_ptr;
+
+    const int nk = Kp / BK;
+    const int nchunks = (nk + KCB - 1) / KCB;
+
+    if (warp == 0) {
+        // ---------------- TMA producer ----------------
+        if (lane == 0) {
+            tma_prefetch_desc(&tAh);
+            tma_prefetch_desc(&tAl);
+            tma_prefetch_desc(&tBh);
+            tma_prefetch_desc(&tBl);
+            const int m0 = tm * BM, n0 = tn * BN;
+            for (int kb = 0; kb < nk; ++kb) {
+                const int s = kb % STAGES;
+                const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+                mbar_wait(bar_empty + 8 * s, ph ^ 1u);
+                const uint32_t fb = bar_full + 8 * s;
+                mbar_arrive_expect_tx(fb, STAGE_BYTES);
+                const uint32_t st = base + s * STAGE_BYTES;
+                tma_load_2d(st, &tAh, fb, kb * BK, m0);
+                tma_load_2d(st + A_BYTES, &tAl, fb, kb * BK, m0);
+                tma_load_2d(st + 2 * A_BYTES, &tBh, fb, kb * BK, n0);
+                tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBl, fb, kb * BK, n0);
+            }
+        }
+    } else if (warp == 1) {
+        // ---------------- MMA issuer (one thread) ----------------
+        if (lane == 0) {
+            constexpr uint32_t idesc = idesc_tf32(BM, BN);
+            for (int kb = 0; kb < nk; ++kb) {
+                const int chunk = kb / KCB, kin = kb - chunk * KCB;
+                const uint32_t buf = (uint32_t)chunk & 1u;
+                const uint32_t dtm = tmem_base + buf * BN;
+                if (kin == 0) {
+                    // wait until the epilogue drained this accumulator buffer (2 chunks ago)
+                    mbar_wait(bar_tempty + 8 * buf, ((uint32_t)(chunk >> 1) & 1u) ^ 1u);
+                    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                }
+                const int s = kb % STAGES;
+                const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+                mbar_wait(bar_full + 8 * s, ph);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                const uint32_t st = base + s * STAGE_BYTES;
+                const uint32_t ah = st, al = st + A_BYTES, bh = st + 2 * A_BYTES, bl = bh + B_BYTES;
+#pragma unroll
+                for (int kk = 0; kk < BK / UMMA_K; ++kk) {
+                    const uint32_t off = kk * UMMA_K * 4;   // 32 B per K step inside the swizzle atom
+                    const uint32_t acc0 = (kin == 0 && kk == 0) ? 0u : 1u;
+                    // small terms first: lo*hi, hi*lo, then hi*hi
+                    umma_tf32(dtm, umma_desc_k_sw128(al + off), umma_desc_k_sw128(bh + off), idesc, acc0);
+                    umma_tf32(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bl + off), idesc, 1u);
+                    umma_tf32(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bh + off), idesc, 1u);
+                }
+                umma_commit(bar_empty + 8 * s);                 // smem stage free when these MMAs finish
+                if (kin == KCB - 1 || kb == nk - 1) umma_commit(bar_tfull + 8 * buf);   // chunk sum ready
+            }
+        }
+        __syncwarp();
+    } else {
+        // ---------------- epilogue warps 2..5: promote chunks, then store ----------------
+        const int q = warp & 3;                         // TMEM lane quarter of this warp
+        const uint32_t tl = tmem_base + ((uint32_t)(q * 32) << 16);
+        float acc[BN];
+#pragma unroll
+        for (int j = 0; j < BN; ++j) acc[j] = 0.0f;
+        for (int chunk = 0; chunk < nchunks; ++chunk) {
+            const uint32_t buf = (uint32_t)chunk & 1u;
+            mbar_wait(bar_tfull + 8 * buf, (uint32_t)(chunk >> 1) & 1u);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll
+            for (int c0 = 0; c0 < BN; c0 += 32) {
+                uint32_t r[32];
+                tmem_ld32(tl + buf * BN + c0, r);
+#pragma unroll
+                for (int j = 0; j < 32; ++j) acc[c0 + j] += __uint_as_float(r[j]);   // RN fp32 promotion
+            }
+            asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+            __syncwarp();
+            if (lane == 0) mbar_arrive(bar_tempty + 8 * buf);
+        }
+        const int row = tm * BM + q * 32 + lane;
+        if (row < M) {
+            float *crow = C + (int64_t)row * ldc + (int64_t)tn * BN;
+            const int cbase = tn * BN;
+            if (vec_ok && cbase + BN <= N) {
+#pragma unroll
+                for (int j = 0; j < BN; j += 4)
+                    *reinterpret_cast<float4 *>(crow + j) = make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < BN; ++j)
+                    if (cbase + j < N) crow[j] = acc[j];
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(TMEM_COLS));
+    }
+}
+
+static bool map_f32(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_t Kp, uint64_t rows, uint32_t box_rows) {
+    cuuint64_t dims[2] = {Kp, rows};
+    cuuint64_t strides[1] = {Kp * 4};
+    cuuint32_t box[2] = {(cuuint32_t)k2::BK, box_rows};
+    cuuint32_t es[2] = {1, 1};
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
+                               const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
+                               cudaStream_t stream) {
+    using namespace k2;
+    if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
+    CUtensorMap tah, tal, tbh, tbl;
+    if (!map_f32(enc, &tah, Ahi, Kp, M, BM) || !map_f32(enc, &tal, Alo, Kp, M, BM) ||
+        !map_f32(enc, &tbh, Bhi, Kp, N, BN) || !map_f32(enc, &tbl, Blo, Kp, N, BN))
+        return cudaErrorInvalidValue;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static bool attr_done[64] = {false};
+    if (dev < 64 && !attr_done[dev]) {
+        cudaError_t e = cudaFuncSetAttribute(gemm_3xtf32_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+        if (e != cudaSuccess) return e;
+        attr_done[dev] = true;
+    }
+    const int tiles_m = (int)((M + BM - 1) / BM), tiles_n = (int)((N + BN - 1) / BN);
+    const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 3) == 0) ? 1 : 0;
+    gemm_3xtf32_kernel<<<tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(tah, tal, tbh, tbl, C, ldc, (int)M, (int)N,
+                                                                          (int)Kp, tiles_m, tiles_n, vec_ok);
+    return cudaGetLastError();
+}
+
+}  // namespace pdlk

@@ -1,0 +1,104 @@
+// pdl_map.cpp -- task decomposition and BLOCK mapping of tile tasks onto the
+// execution group's Workers.
+//
+// PAPER.md SS IV-A: distribution specifiers "hold references to input and
+// output parameter data-distributions (e.g., block, cyclic, block-cyclic) and
+// optional sizes ... for possible data-decomposition of data-parallel tasks"
+// (L1200-1208); example `(A:BLOCK:N, B:BLOCK:N)` (L1155-1156).  SS IV-B:
+// "From that generic model a compiler or run-time can further automatically
+// derive optimized mapping decisions to physical hardware elements"
+// (L1262-1266).  Readings R4-R6: C is cut into ceil(M/tile) x
+// ceil(N/tile) tile tasks; BLOCK distributes task rows / columns over a
+// Gr x Gc Worker grid; the Worker grid minimises exchanged operand bytes.
+#include <cmath>
+#include <limits>
+#include <sstream>
+
+#include "pdl_model.hpp"
+
+namespace pdl {
+
+static int64_t cdiv(int64_t a, int64_t b) { return b ? (a + b - 1) / b : 0; }
+
+Rect Plan::rect(int w) const {
+    int r = w / Gc, c = w % Gc;
+    return Rect{row[r], row[r + 1], col[c], col[c + 1]};
+}
+
+// A row-panel of Worker (r,c) split in Gc chunks of qa rows (ceil): chunk j =
+// panel rows [j*qa, min((j+1)*qa, rows)).  Gathering Gc chunks of qa rows
+// each leaves the panel contiguous in the first `rows` rows of the buffer.
+int64_t Plan::qa(int w) const {
+    Rect R = rect(w);
+    return cdiv(R.row1 - R.row0, Gc);
+}
+
+int64_t Plan::qb() const { return cdiv(K, Gr); }
+
+double Plan::exchanged_elems() const {
+    double tot = 0;
+    for (int w = 0; w < G; ++w) {
+        Rect R = rect(w);
+        double rows = double(R.row1 - R.row0), cols = double(R.col1 - R.col0);
+        tot += rows * K * (1.0 - 1.0 / Gc) + double(K) * cols * (1.0 - 1.0 / Gr);
+    }
+    return tot;
+}
+
+Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G) {
+    Plan p;
+    p.M = M; p.N = N; p.K = K; p.G = G;
+    // Worker grid: minimise per-Worker received elements, ties -> larger Gr.
+    double best = std::numeric_limits<double>::infinity();
+    for (int gr = G; gr >= 1; --gr) {
+        if (G % gr) continue;
+        int gc = G / gr;
+        double cost = (double(M) / gr) * double(K) * (1.0 - 1.0 / gc) +
+                      double(K) * (double(N) / gc) * (1.0 - 1.0 / gr);
+        if (cost < best * (1.0 - 1e-12)) { best = cost; p.Gr = gr; p.Gc = gc; }
+    }
+    if (tile > 0) {
+        p.tile = tile;
+        p.Tm = cdiv(M, tile);
+        p.Tn = cdiv(N, tile);
+    } else {
+        // tile = 0: one task per Worker rectangle (continuous BLOCK split).
+        p.tile = 0;
+        p.Tm = p.Gr;
+        p.Tn = p.Gc;
+    }
+    p.trow.resize(p.Gr + 1);
+    p.tcol.resize(p.Gc + 1);
+    p.row.resize(p.Gr + 1);
+    p.col.resize(p.Gc + 1);
+    for (int r = 0; r <= p.Gr; ++r) {
+        p.trow[r] = (int64_t)r * p.Tm / p.Gr;  // floor(r*Tm/Gr): remainder to higher rows
+        p.row[r] = p.tile ? std::min<int64_t>(p.trow[r] * p.tile, M) : (int64_t)r * M / p.Gr;
+    }
+    for (int c = 0; c <= p.Gc; ++c) {
+        p.tcol[c] = (int64_t)c * p.Tn / p.Gc;
+        p.col[c] = p.tile ? std::min<int64_t>(p.tcol[c] * p.tile, N) : (int64_t)c * N / p.Gc;
+    }
+    return p;
+}
+
+std::string Plan::to_json(const std::vector<int> &workers, const std::vector<std::string> &ids) const {
+    std::ostringstream o;
+    o << "{\"M\":" << M << ",\"N\":" << N << ",\"K\":" << K << ",\"tile\":" << tile << ",\"G\":" << G
+      << ",\"Gr\":" << Gr << ",\"Gc\":" << Gc << ",\"Tm\":" << Tm << ",\"Tn\":" << Tn
+      << ",\"qb\":" << qb() << ",\"exchanged_elems\":" << (int64_t)exchanged_elems() << ",\"workers\":[";
+    for (int w = 0; w < G; ++w) {
+        Rect R = rect(w);
+        int r = w / Gc, c = w % Gc;
+        if (w) o << ",";
+        o << "{\"w\":" << w << ",\"id\":\"" << (w < (int)ids.size() ? json_escape(ids[w]) : "") << "\""
+          << ",\"r\":" << r << ",\"c\":" << c << ",\"rows\":[" << R.row0 << "," << R.row1 << "],\"cols\":["
+          << R.col0 << "," << R.col1 << "],\"task_rows\":[" << trow[r] << "," << trow[r + 1]
+          << "],\"task_cols\":[" << tcol[c] << "," << tcol[c + 1] << "],\"qa\":" << qa(w) << "}";
+    }
+    (void)workers;
+    o << "]}";
+    return o.str();
+}
+
+}  // namespace pdl

@@ -1,0 +1,766 @@
+// pdl_runtime.cu -- the C ABI of libpdl.so (include/libpdl.h) and the task
+// runtime behind it: descriptor loading, device binding, task queue, BLOCK
+// mapping, operand staging along the interconnects, kernel launch, sync.
+//
+// PAPER.md SS IV-C step 3 "Output generation": "insertion of highly platform
+// specific code for data-partitioning, transfer and task invocations.  The
+// PDL allows us to derive data-transfer paths between memory-regions and
+// communication between processing-units via the explicitly specified
+// interconnect entity" (L1328-1341).  Here that step runs at run time:
+// pdl_run partitions C (pdl_map.cpp), moves operand panels from the Master's
+// memory region (host) to each Worker's memory region (HBM) over the Master->
+// Worker interconnect (PCIe), and invokes the Worker's task variant (K1 for
+// FP64, K3+K2 for FP32).  The Worker<->Worker exchange (NVLink) of the
+// one-process-per-GPU mode runs in the Python runtime over torch.distributed.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <fstream>
+#include <memory>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "../../include/libpdl.h"
+#include "kernels.h"
+#include "pdl_model.hpp"
+#include "pdl_xml.hpp"
+
+using namespace pdl;
+
+namespace {
+
+thread_local std::string g_err;
+
+int set_err(int code, const char *fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    if (getenv("PDL_LOG") && atoi(getenv("PDL_LOG")) > 0) fprintf(stderr, "[pdl] error %d: %s\n", code, buf);
+    return code;
+}
+
+void logf(int level, const char *fmt, ...) {
+    const char *e = getenv("PDL_LOG");
+    if (!e || atoi(e) < level) return;
+    va_list ap;
+    va_start(ap, fmt);
+    fprintf(stderr, "[pdl] ");
+    vfprintf(stderr, fmt, ap);
+    fprintf(stderr, "\n");
+    va_end(ap);
+}
+
+bool env_on(const char *name) {
+    const char *e = getenv(name);
+    return e && *e && strcmp(e, "0") != 0;
+}
+
+// A library-owned device buffer in a Worker's memory region, reused across runs.
+struct DevBuf {
+    void *ptr = nullptr;
+    size_t bytes = 0;
+};
+
+enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_COUNT };
+
+struct WorkerCtx {
+    int pu = -1;         // PU instance index in the model
+    int gw = -1;         // index in the default group order
+    int device = -1;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    DevBuf buf[BUF_COUNT];
+    cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr;   // around the dominant kernel of the last task
+    int launches = 0;                               // kernels launched in the last run
+    bool timed = false;
+    // event pairs around every dominant-kernel launch since the last pdl_kernel_times()
+    std::vector<cudaEvent_t> kt_ev;
+    size_t kt_n = 0;
+};
+
+constexpr size_t kMaxKernelTimes = 4096;
+
+// Record the start / end of a dominant-kernel launch on the worker's stream.
+int kt_mark(WorkerCtx &w, bool start) {
+    cudaEvent_t &last = start ? w.ev_k0 : w.ev_k1;
+    cudaError_t e = cudaEventRecord(last, w.stream);
+    if (e != cudaSuccess) return PDL_ECUDA;
+    if (w.kt_n >= kMaxKernelTimes) return PDL_OK;
+    size_t idx = 2 * w.kt_n + (start ? 0 : 1);
+    if (idx >= w.kt_ev.size()) {
+        cudaEvent_t ev;
+        if (cudaEventCreate(&ev) != cudaSuccess) return PDL_ECUDA;
+        w.kt_ev.push_back(ev);
+    }
+    if (cudaEventRecord(w.kt_ev[idx], w.stream) != cudaSuccess) return PDL_ECUDA;
+    if (!start) w.kt_n++;
+    return PDL_OK;
+}
+
+struct Task {
+    int dtype;
+    const void *A;
+    int64_t lda;
+    const void *B;
+    int64_t ldb;
+    void *C;
+    int64_t ldc;
+    int64_t M, N, K, tile;
+    bool has_group;
+    std::string group;
+    unsigned flags;
+};
+
+struct State {
+    bool loaded = false;
+    bool dry_run = false;
+    bool oversub = false;
+    int rank = 0, nranks = 1;
+    Model model;
+    std::vector<WorkerCtx> workers;   // one per bound gpu Worker (this process's)
+    std::vector<Task> queue;
+    std::string plan_json = "[]";
+    pdlk::EncodeTiledFn encode = nullptr;
+    int last_launches = 0;
+};
+
+State *g = nullptr;
+
+const char *kVersion = "libpdl 0.1.0 (sm_100a: K1 FP64 DMMA+TMA, K2 3xTF32 tcgen05+TMEM+TMA)";
+
+std::string read_descriptor(const char *d, bool *ok) {
+    *ok = true;
+    const char *p = d;
+    while (*p == ' ' || *p == '\t' || *p == '\n' || *p == '\r') ++p;
+    if (*p == '<') return std::string(d);
+    std::ifstream f(d, std::ios::binary);
+    if (!f) {
+        *ok = false;
+        return "";
+    }
+    std::stringstream ss;
+    ss << f.rdbuf();
+    return ss.str();
+}
+
+#define CUDA_TRY(call)                                                                                   \
+    do {                                                                                                 \
+        cudaError_t _e = (call);                                                                         \
+        if (_e != cudaSuccess) return set_err(PDL_ECUDA, "%s failed: %s", #call, cudaGetErrorString(_e)); \
+    } while (0)
+
+int get_encoder(pdlk::EncodeTiledFn *out) {
+    if (g->encode) {
+        *out = g->encode;
+        return PDL_OK;
+    }
+    void *fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+        return set_err(PDL_ECUDA, "cuTensorMapEncodeTiled unavailable (%s)", cudaGetErrorString(e));
+    g->encode = reinterpret_cast<pdlk::EncodeTiledFn>(fn);
+    *out = g->encode;
+    return PDL_OK;
+}
+
+// Fill unfixed Worker properties from the bound device (L737-747 "Values for
+// unfixed properties are marked to be editable by other tools ... later
+// instantiation by a runtime"), adding the standard set when absent.
+void fill_props(int pu, const cudaDeviceProp &p) {
+    auto set = [&](const char *name, const std::string &val, const char *unit) {
+        Property *q = g->model.prop_mut(pu, name);
+        if (q) {
+            if (!q->fixed) {
+                q->value = val;
+                q->unit = unit;
+            }
+            return;
+        }
+        Property np;
+        np.name = name;
+        np.key = norm_key(name);
+        np.value = val;
+        np.unit = unit;
+        np.fixed = false;
+        g->model.pus[pu].props.push_back(np);
+    };
+    set("DEVICE_NAME", p.name, "");
+    set("MAX_COMPUTE_UNITS", std::to_string(p.multiProcessorCount), "");
+    set("COMPUTE_CAPABILITY", std::to_string(p.major) + "." + std::to_string(p.minor), "");
+    set("GLOBAL_MEM_SIZE", std::to_string((unsigned long long)p.totalGlobalMem), "B");
+    set("LOCAL_MEM_SIZE", std::to_string((unsigned long long)p.sharedMemPerBlockOptin), "B");
+    set("L2_CACHE_SIZE", std::to_string(p.l2CacheSize), "B");
+    set("PCI_BUS_ID", std::to_string(p.pciBusID), "");
+    // memory region of the Worker: HBM size
+    auto &mrs = g->model.pus[pu].mrs;
+    if (mrs.empty()) {
+        MemoryRegion mr;
+        mr.id = "hbm";
+        mrs.push_back(mr);
+    }
+    bool found = false;
+    for (auto &q : mrs[0].props)
+        if (q.key == "SIZE") {
+            found = true;
+            if (!q.fixed) {
+                q.value = std::to_string((unsigned long long)p.totalGlobalMem);
+                q.unit = "B";
+            }
+        }
+    if (!found) {
+        Property np;
+        np.name = "SIZE";
+        np.key = "SIZE";
+        np.value = std::to_string((unsigned long long)p.totalGlobalMem);
+        np.unit = "B";
+        np.fixed = false;
+        mrs[0].props.push_back(np);
+    }
+}
+
+int bind_devices() {
+    std::vector<int> gw = g->model.all_gpu_workers();
+    if (g->dry_run) {
+        for (size_t i = 0; i < gw.size(); ++i) {
+            if (g->nranks > 1 && (int)i != g->rank) continue;
+            WorkerCtx w;
+            w.pu = gw[i];
+            w.gw = (int)i;
+            w.device = -1;
+            g->workers.push_back(w);
+        }
+        return PDL_OK;
+    }
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0)
+        return set_err(PDL_ENOWORKER, "no CUDA device available (%s): no CPU fallback exists",
+                       e == cudaSuccess ? "0 devices" : cudaGetErrorString(e));
+    if (gw.empty()) return set_err(PDL_ENOWORKER, "descriptor has no Worker with ARCHITECTURE=gpu");
+    int cur = 0;
+    cudaGetDevice(&cur);
+    std::vector<int> used(ndev, 0);
+    for (size_t i = 0; i < gw.size(); ++i) {
+        if (g->nranks > 1 && (int)i != g->rank) continue;
+        int dev;
+        const Property *ord = g->model.prop(gw[i], "DEVICE_ORDINAL");
+        if (g->nranks > 1) dev = cur;   // rank mode: the process's current device
+        else if (ord && !ord->value.empty()) dev = atoi(ord->value.c_str());
+        else dev = (int)i;
+        if (dev >= ndev) {
+            if (!g->oversub)
+                return set_err(PDL_ENOWORKER,
+                               "descriptor names %zu gpu Workers but only %d CUDA device(s) exist "
+                               "(set PDL_ALLOW_OVERSUBSCRIBE=1 to share devices)",
+                               gw.size(), ndev);
+            dev = dev % ndev;
+        }
+        if (used[dev] && !g->oversub)
+            return set_err(PDL_ENOWORKER, "two Workers bound to device %d (set PDL_ALLOW_OVERSUBSCRIBE=1)", dev);
+        used[dev]++;
+        cudaDeviceProp prop;
+        CUDA_TRY(cudaGetDeviceProperties(&prop, dev));
+        if (prop.major != 10)
+            return set_err(PDL_ENOWORKER, "device %d is sm_%d%d; this build targets sm_100a (B200) only", dev,
+                           prop.major, prop.minor);
+        WorkerCtx w;
+        w.pu = gw[i];
+        w.gw = (int)i;
+        w.device = dev;
+        CUDA_TRY(cudaSetDevice(dev));
+        // blocking stream: ordered with the legacy default stream callers often use
+        CUDA_TRY(cudaStreamCreate(&w.stream));
+        w.own_stream = true;
+        CUDA_TRY(cudaEventCreate(&w.ev_k0));
+        CUDA_TRY(cudaEventCreate(&w.ev_k1));
+        g->model.pus[gw[i]].device = dev;
+        fill_props(gw[i], prop);
+        g->workers.push_back(w);
+    }
+    cudaSetDevice(cur);
+    return PDL_OK;
+}
+
+void free_state() {
+    if (!g) return;
+    for (auto &w : g->workers) {
+        if (w.device >= 0) cudaSetDevice(w.device);
+        for (auto &b : w.buf)
+            if (b.ptr) cudaFree(b.ptr);
+        if (w.own_stream && w.stream) cudaStreamDestroy(w.stream);
+        if (w.ev_k0) cudaEventDestroy(w.ev_k0);
+        if (w.ev_k1) cudaEventDestroy(w.ev_k1);
+        for (auto ev : w.kt_ev) cudaEventDestroy(ev);
+    }
+    delete g;
+    g = nullptr;
+}
+
+int ensure_buf(WorkerCtx &w, int slot, size_t bytes, void **out) {
+    DevBuf &b = w.buf[slot];
+    if (b.bytes < bytes) {
+        if (b.ptr) {
+            cudaStreamSynchronize(w.stream);
+            cudaFree(b.ptr);
+            b.ptr = nullptr;
+            b.bytes = 0;
+        }
+        cudaError_t e = cudaMalloc(&b.ptr, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return set_err(PDL_ENOMEM, "cudaMalloc(%zu) on device %d failed: %s", bytes, w.device,
+                           cudaGetErrorString(e));
+        }
+        b.bytes = bytes;
+    }
+    *out = b.ptr;
+    return PDL_OK;
+}
+
+// Where a pointer lives: -1 host (Master memory region), else device ordinal.
+int locate(const void *p) {
+    cudaPointerAttributes a;
+    cudaError_t e = cudaPointerGetAttributes(&a, p);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return -1;
+    }
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return a.device;
+    return -1;
+}
+
+bool overlaps(const void *a, size_t an, const void *b, size_t bn) {
+    uintptr_t x = (uintptr_t)a, y = (uintptr_t)b;
+    return an && bn && x < y + bn && y < x + an;
+}
+
+int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
+
+// Make a rows x cols operand (elements of `es` bytes, leading dim ld) usable
+// by a TMA-fed kernel on worker w: device-resident on w.device, 16 B-aligned
+// base, pitch a multiple of 16 B.  Copies (H2D over the Master->Worker
+// interconnect, or D2D/peer) into a library buffer when needed.
+int stage_operand(WorkerCtx &w, int slot, const void *src, int64_t ld, int64_t rows, int64_t cols, int es,
+                  const void **out, int64_t *out_ld, bool need_tma_align) {
+    int loc = locate(src);
+    bool aligned = ((uintptr_t)src % 16 == 0) && ((ld * es) % 16 == 0);
+    if (loc == w.device && (aligned || !need_tma_align)) {
+        *out = src;
+        *out_ld = ld;
+        return PDL_OK;
+    }
+    int64_t pitch_el = round_up(std::max<int64_t>(cols, 1), 16 / es);
+    void *dst;
+    int rc = ensure_buf(w, slot, (size_t)(pitch_el * std::max<int64_t>(rows, 1) * es), &dst);
+    if (rc) return rc;
+    cudaError_t e = cudaMemcpy2DAsync(dst, (size_t)(pitch_el * es), src, (size_t)(ld * es), (size_t)(cols * es),
+                                      (size_t)rows, cudaMemcpyDefault, w.stream);
+    if (e != cudaSuccess) return set_err(PDL_ECUDA, "operand staging copy failed: %s", cudaGetErrorString(e));
+    *out = dst;
+    *out_ld = pitch_el;
+    return PDL_OK;
+}
+
+// Execute one task's rectangle on worker w.  A/B/C point at the rectangle's
+// panels (A: rows x K at ld lda; B: K x cols at ldb; C: rows x cols at ldc).
+int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
+    if (rows <= 0 || cols <= 0) return PDL_OK;
+    CUDA_TRY(cudaSetDevice(w.device));
+    const int es = t.dtype == PDL_F64 ? 8 : 4;
+    const int64_t K = t.K;
+    // C destination: in place when it is on this device, else a staging buffer
+    int cloc = locate(C);
+    void *Cd = C;
+    int64_t ldcd = t.ldc;
+    bool c_staged = false;
+    if (cloc != w.device) {
+        int64_t pitch = round_up(cols, 16 / es);
+        int rc = ensure_buf(w, BUF_C, (size_t)(pitch * rows * es), &Cd);
+        if (rc) return rc;
+        ldcd = pitch;
+        c_staged = true;
+    }
+    if (K == 0) {
+        // empty sum: C = 0 (BLAS convention)
+        CUDA_TRY(cudaMemset2DAsync(Cd, (size_t)(ldcd * es), 0, (size_t)(cols * es), (size_t)rows, w.stream));
+    } else if (t.dtype == PDL_F64) {
+        const void *Ad, *Bd;
+        int64_t lda, ldb;
+        int rc = stage_operand(w, BUF_A, A, t.lda, rows, K, 8, &Ad, &lda, true);
+        if (!rc) rc = stage_operand(w, BUF_B, B, t.ldb, K, cols, 8, &Bd, &ldb, true);
+        if (rc) return rc;
+        pdlk::EncodeTiledFn enc;
+        if ((rc = get_encoder(&enc))) return rc;
+        if (kt_mark(w, true)) return set_err(PDL_ECUDA, "event record failed");
+        cudaError_t e = pdlk::launch_dgemm_k1(enc, (const double *)Ad, lda, (const double *)Bd, ldb, (double *)Cd, ldcd,
+                                              rows, cols, K, w.stream);
+        if (e != cudaSuccess) return set_err(PDL_ECUDA, "K1 launch failed: %s", cudaGetErrorString(e));
+        if (kt_mark(w, false)) return set_err(PDL_ECUDA, "event record failed");
+        w.launches += 1;
+        w.timed = true;
+    } else {
+        // FP32: split pre-pass reads any device layout; host/other-device operands are staged first.
+        const void *Ad, *Bd;
+        int64_t lda, ldb;
+        int rc = stage_operand(w, BUF_A, A, t.lda, rows, K, 4, &Ad, &lda, false);
+        if (!rc) rc = stage_operand(w, BUF_B, B, t.ldb, K, cols, 4, &Bd, &ldb, false);
+        if (rc) return rc;
+        const int64_t Kp = round_up(K, pdlk::K2_BK);
+        void *ahi, *alo, *bhi, *blo;
+        if ((rc = ensure_buf(w, BUF_AHI, (size_t)(rows * Kp * 4), &ahi))) return rc;
+        if ((rc = ensure_buf(w, BUF_ALO, (size_t)(rows * Kp * 4), &alo))) return rc;
+        if ((rc = ensure_buf(w, BUF_BHI, (size_t)(cols * Kp * 4), &bhi))) return rc;
+        if ((rc = ensure_buf(w, BUF_BLO, (size_t)(cols * Kp * 4), &blo))) return rc;
+        cudaError_t e = pdlk::launch_split_rows((const float *)Ad, lda, rows, K, (float *)ahi, (float *)alo, Kp, w.stream);
+        if (e == cudaSuccess)
+            e = pdlk::launch_split_cols_t((const float *)Bd, ldb, K, cols, (float *)bhi, (float *)blo, Kp, w.stream);
+        if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
+        pdlk::EncodeTiledFn enc;
+        if ((rc = get_encoder(&enc))) return rc;
+        if (kt_mark(w, true)) return set_err(PDL_ECUDA, "event record failed");
+        e = pdlk::launch_gemm_3xtf32(enc, (const float *)ahi, (const float *)alo, (const float *)bhi, (const float *)blo,
+                                     Kp, (float *)Cd, ldcd, rows, cols, w.stream);
+        if (e != cudaSuccess) return set_err(PDL_ECUDA, "K2 launch failed: %s", cudaGetErrorString(e));
+        if (kt_mark(w, false)) return set_err(PDL_ECUDA, "event record failed");
+        w.launches += 3;
+        w.timed = true;
+    }
+    if (c_staged) {
+        cudaError_t e = cudaMemcpy2DAsync(C, (size_t)(t.ldc * es), Cd, (size_t)(ldcd * es), (size_t)(cols * es),
+                                          (size_t)rows, cudaMemcpyDefault, w.stream);
+        if (e != cudaSuccess) return set_err(PDL_ECUDA, "result gather copy failed: %s", cudaGetErrorString(e));
+    }
+    return PDL_OK;
+}
+
+int check_loaded() {
+    if (!g || !g->loaded) return set_err(PDL_ESTATE, "no platform loaded (call pdl_load first)");
+    return PDL_OK;
+}
+
+int do_load(const char *descriptor, int rank, int nranks) {
+    if (g && g->loaded) return set_err(PDL_ESTATE, "a platform is already loaded (call pdl_unload first)");
+    if (!descriptor) return set_err(PDL_EINVAL, "descriptor is NULL");
+    if (nranks < 1 || rank < 0 || rank >= nranks) return set_err(PDL_EINVAL, "bad rank %d of %d", rank, nranks);
+    bool ok;
+    std::string doc = read_descriptor(descriptor, &ok);
+    if (!ok) return set_err(PDL_EINVAL, "cannot read descriptor file '%s'", descriptor);
+    std::unique_ptr<State> st(new State());
+    try {
+        auto root = parse_xml(doc);
+        st->model = build_model(*root);
+    } catch (const XmlError &e) {
+        return set_err(PDL_EPARSE, "XML error at line %d: %s", e.line, e.msg.c_str());
+    } catch (const ModelError &e) {
+        return set_err(PDL_EPARSE, "PDL error at line %d: %s", e.line, e.msg.c_str());
+    }
+    st->dry_run = env_on("PDL_DRY_RUN");
+    st->oversub = env_on("PDL_ALLOW_OVERSUBSCRIBE");
+    st->rank = rank;
+    st->nranks = nranks;
+    g = st.release();
+    int rc = bind_devices();
+    if (rc) {
+        std::string msg = g_err;
+        free_state();
+        g_err = msg;
+        return rc;
+    }
+    g->loaded = true;
+    logf(1, "loaded: %zu PUs, %zu gpu Workers, rank %d/%d%s", g->model.pus.size(), g->model.all_gpu_workers().size(),
+         rank, nranks, g->dry_run ? " (dry run)" : "");
+    return PDL_OK;
+}
+
+int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, void *C, int64_t ldc, int64_t M,
+            int64_t N, int64_t K, int64_t tile, const char *group, const char *dist, unsigned flags) {
+    int rc = check_loaded();
+    if (rc) return rc;
+    if (dtype != PDL_F64 && dtype != PDL_F32) return set_err(PDL_EINVAL, "unknown dtype %d", dtype);
+    if (M < 0 || N < 0 || K < 0) return set_err(PDL_EINVAL, "negative size M=%lld N=%lld K=%lld", (long long)M,
+                                                (long long)N, (long long)K);
+    if (tile < 0) return set_err(PDL_EINVAL, "negative tile %lld", (long long)tile);
+    if (flags & ~PDL_TASK_PANELS) return set_err(PDL_EINVAL, "unknown flags 0x%x", flags);
+    if (dist && strcasecmp(dist, "BLOCK") != 0) {
+        if (!strcasecmp(dist, "CYCLIC") || !strcasecmp(dist, "BLOCK-CYCLIC") || !strcasecmp(dist, "BLOCK_CYCLIC"))
+            return set_err(PDL_EUNSUPPORTED, "distribution %s is not implemented (BLOCK only)", dist);
+        return set_err(PDL_EINVAL, "unknown distribution '%s' (L1200-1206 names block, cyclic, block-cyclic)", dist);
+    }
+    if (group && g->model.group_workers(group).empty())
+        return set_err(PDL_EINVAL, "execution group '%s' names no gpu Worker (LogicGroupAttribute)", group);
+    if (M == 0 || N == 0) return PDL_OK;   // nothing to write
+    const int es = dtype == PDL_F64 ? 8 : 4;
+    if (!C) return set_err(PDL_EINVAL, "C is NULL with M*N > 0");
+    if (K > 0 && (!A || !B)) return set_err(PDL_EINVAL, "A or B is NULL with K > 0");
+    // leading dimensions (0 = dense); in PANELS mode widths are the Worker's
+    int64_t lda_ = lda ? lda : K, ldb_ = ldb, ldc_ = ldc;
+    if (!(flags & PDL_TASK_PANELS)) {
+        if (!ldb_) ldb_ = N;
+        if (!ldc_) ldc_ = N;
+        if (lda_ < K || ldb_ < N || ldc_ < N) return set_err(PDL_EINVAL, "leading dimension smaller than the row width");
+        size_t an = (size_t)((M - 1) * lda_ + K) * es, bn = K ? (size_t)((K - 1) * ldb_ + N) * es : 0,
+               cn = (size_t)((M - 1) * ldc_ + N) * es;
+        if (K > 0 && (overlaps(C, cn, A, an) || overlaps(C, cn, B, bn)))
+            return set_err(PDL_EINVAL, "C overlaps A or B (C has access mode write, A/B read, L1184-1186)");
+    }
+    Task t{dtype, A, lda_, B, ldb_, C, ldc_, M, N, K, tile, group != nullptr, group ? group : "", flags};
+    g->queue.push_back(t);
+    return PDL_OK;
+}
+
+int execute(bool sync) {
+    int rc = check_loaded();
+    if (rc) return rc;
+    std::vector<Task> q;
+    q.swap(g->queue);   // the queue is cleared whatever happens
+    std::ostringstream pj;
+    pj << "[";
+    for (auto &w : g->workers) {
+        w.launches = 0;
+        w.timed = false;
+    }
+    for (size_t ti = 0; ti < q.size(); ++ti) {
+        const Task &t = q[ti];
+        std::vector<int> gw = g->model.group_workers(t.has_group ? t.group.c_str() : nullptr);
+        const int G = (int)gw.size();
+        if (G == 0) return set_err(PDL_ENOWORKER, "execution group has no gpu Worker");
+        if (g->nranks > 1 && G != g->nranks)
+            return set_err(PDL_ENOWORKER, "group has %d Workers but %d ranks co-exist: one process per Worker", G,
+                           g->nranks);
+        Plan plan = make_plan(t.M, t.N, t.K, t.tile, G);
+        std::vector<std::string> ids;
+        for (int x : gw) ids.push_back(g->model.pus[x].id);
+        if (ti) pj << ",";
+        pj << plan.to_json(gw, ids);
+        if (g->dry_run) continue;
+        const int es = t.dtype == PDL_F64 ? 8 : 4;
+        for (auto &w : g->workers) {
+            // group index of this bound Worker
+            int gi = -1;
+            for (int i = 0; i < G; ++i)
+                if (gw[i] == w.pu) gi = i;
+            if (gi < 0) continue;
+            Rect R = plan.rect(gi);
+            const int64_t rows = R.row1 - R.row0, cols = R.col1 - R.col0;
+            const char *A = (const char *)t.A, *B = (const char *)t.B;
+            char *C = (char *)t.C;
+            int64_t lda = t.lda, ldb = t.ldb, ldc = t.ldc;
+            if (t.flags & PDL_TASK_PANELS) {
+                if (!lda) lda = t.K;
+                if (!ldb) ldb = cols;
+                if (!ldc) ldc = cols;
+            } else {
+                A += (size_t)(R.row0 * lda) * es;
+                B += (size_t)R.col0 * es;
+                C += (size_t)(R.row0 * ldc + R.col0) * es;
+            }
+            Task tt = t;
+            tt.lda = lda;
+            tt.ldb = ldb;
+            tt.ldc = ldc;
+            rc = run_rect(w, tt, A, B, C, rows, cols);
+            if (rc) return rc;
+        }
+    }
+    pj << "]";
+    g->plan_json = pj.str();
+    if (sync) return pdl_sync();
+    return PDL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int pdl_load(const char *descriptor) { return do_load(descriptor, 0, 1); }
+
+int pdl_load_rank(const char *descriptor, int rank, int nranks) { return do_load(descriptor, rank, nranks); }
+
+int task_matmul(const double *A, const double *B, double *C, int64_t M, int64_t N, int64_t K, int64_t tile) {
+    return enqueue(PDL_F64, A, 0, B, 0, C, 0, M, N, K, tile, nullptr, nullptr, 0);
+}
+
+int task_matmul_f32(const float *A, const float *B, float *C, int64_t M, int64_t N, int64_t K, int64_t tile) {
+    return enqueue(PDL_F32, A, 0, B, 0, C, 0, M, N, K, tile, nullptr, nullptr, 0);
+}
+
+int task_matmul_ex(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, void *C, int64_t ldc, int64_t M,
+                   int64_t N, int64_t K, int64_t tile, const char *group, const char *dist, unsigned flags) {
+    if (lda < 0 || ldb < 0 || ldc < 0) return set_err(PDL_EINVAL, "negative leading dimension");
+    return enqueue(dtype, A, lda, B, ldb, C, ldc, M, N, K, tile, group, dist, flags);
+}
+
+int pdl_run(void) { return execute(true); }
+
+int pdl_run_async(void) { return execute(false); }
+
+int pdl_sync(void) {
+    int rc = check_loaded();
+    if (rc) return rc;
+    if (g->dry_run) return PDL_OK;
+    int launches = 0;
+    for (auto &w : g->workers) {
+        CUDA_TRY(cudaSetDevice(w.device));
+        cudaError_t e = cudaStreamSynchronize(w.stream);
+        if (e != cudaSuccess) return set_err(PDL_ECUDA, "device work failed on device %d: %s", w.device,
+                                             cudaGetErrorString(e));
+        launches += w.launches;
+    }
+    g->last_launches = launches;
+    return PDL_OK;
+}
+
+int pdl_set_stream(int worker, void *stream) {
+    int rc = check_loaded();
+    if (rc) return rc;
+    if (worker < 0 || worker >= (int)g->workers.size()) return set_err(PDL_EINVAL, "no local Worker %d", worker);
+    WorkerCtx &w = g->workers[worker];
+    if (g->dry_run) return PDL_OK;
+    CUDA_TRY(cudaSetDevice(w.device));
+    if (stream) {
+        if (w.own_stream && w.stream) {
+            cudaStreamSynchronize(w.stream);
+            cudaStreamDestroy(w.stream);
+        }
+        w.stream = (cudaStream_t)stream;
+        w.own_stream = false;
+    } else if (!w.own_stream) {
+        CUDA_TRY(cudaStreamCreate(&w.stream));
+        w.own_stream = true;
+    }
+    return PDL_OK;
+}
+
+int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group, int worker, int64_t *out, int nout) {
+    int rc = check_loaded();
+    if (rc) return rc;
+    if (M < 0 || N < 0 || K < 0 || tile < 0) return set_err(PDL_EINVAL, "negative size");
+    if (!out || nout < PDL_PLAN_LEN) return set_err(PDL_EINVAL, "out[] needs %d entries", PDL_PLAN_LEN);
+    std::vector<int> gw = g->model.group_workers(group);
+    if (gw.empty()) return set_err(PDL_ENOWORKER, "execution group has no gpu Worker");
+    const int G = (int)gw.size();
+    if (worker < 0 || worker >= G) return set_err(PDL_EINVAL, "worker %d outside the group of %d", worker, G);
+    Plan p = make_plan(M, N, K, tile, G);
+    Rect R = p.rect(worker);
+    const int r = worker / p.Gc, c = worker % p.Gc;
+    int64_t v[PDL_PLAN_LEN] = {G, p.Gr, p.Gc, r, c, R.row0, R.row1, R.col0, R.col1, p.qa(worker), p.qb(),
+                               p.Tm, p.Tn, p.trow[r], p.trow[r + 1], p.tcol[c], p.tcol[c + 1], p.tile};
+    for (int i = 0; i < PDL_PLAN_LEN; ++i) out[i] = v[i];
+    return PDL_OK;
+}
+
+int pdl_query(const char *key, char *out, size_t len) {
+    if (!key) return set_err(PDL_EINVAL, "key is NULL");
+    std::string k(key), res;
+    if (k == "version") {
+        res = kVersion;
+    } else {
+        int rc = check_loaded();
+        if (rc) return rc;
+        const Model &m = g->model;
+        if (k == "masters") res = std::to_string(m.masters.size());
+        else if (k == "workers") res = std::to_string(m.all_gpu_workers().size());
+        else if (k == "local_workers") res = std::to_string(g->workers.size());
+        else if (k == "model") res = m.to_json();
+        else if (k == "interconnects") res = m.ics_json();
+        else if (k == "plan") res = g->plan_json;
+        else if (k == "groups") {
+            std::vector<std::string> gs;
+            for (auto &p : m.pus)
+                for (auto &x : p.groups)
+                    if (std::find(gs.begin(), gs.end(), x) == gs.end()) gs.push_back(x);
+            res = "[";
+            for (size_t i = 0; i < gs.size(); ++i) res += (i ? ",\"" : "\"") + json_escape(gs[i]) + "\"";
+            res += "]";
+        } else if (k == "stats") {
+            std::ostringstream o;
+            o << "{\"launches\":" << g->last_launches << ",\"workers\":[";
+            bool first = true;
+            for (auto &w : g->workers) {
+                float ms = -1.f;
+                if (w.timed && !g->dry_run) {
+                    cudaSetDevice(w.device);
+                    if (cudaEventElapsedTime(&ms, w.ev_k0, w.ev_k1) != cudaSuccess) {
+                        cudaGetLastError();
+                        ms = -1.f;
+                    }
+                }
+                o << (first ? "" : ",") << "{\"id\":\"" << json_escape(m.pus[w.pu].id) << "\",\"device\":" << w.device
+                  << ",\"kernel_ms\":" << ms << ",\"launches\":" << w.launches << "}";
+                first = false;
+            }
+            o << "]}";
+            res = o.str();
+        } else if (k.rfind("worker/", 0) == 0 || k.rfind("pu/", 0) == 0) {
+            bool is_w = k[0] == 'w';
+            size_t s1 = k.find('/'), s2 = k.find('/', s1 + 1);
+            if (s2 == std::string::npos) return set_err(PDL_EINVAL, "bad key '%s'", key);
+            std::string who = k.substr(s1 + 1, s2 - s1 - 1), what = k.substr(s2 + 1);
+            int pu = -1;
+            if (is_w) {
+                std::vector<int> gw = m.all_gpu_workers();
+                char *end;
+                long i = strtol(who.c_str(), &end, 10);
+                if (*end || i < 0 || i >= (long)gw.size()) return set_err(PDL_EINVAL, "no gpu Worker %s", who.c_str());
+                pu = gw[i];
+            } else {
+                for (size_t i = 0; i < m.pus.size(); ++i)
+                    if (m.pus[i].id == who) pu = (int)i;
+                if (pu < 0) return set_err(PDL_EINVAL, "no PU with id '%s'", who.c_str());
+            }
+            if (what == "device") res = std::to_string(m.pus[pu].device);
+            else if (what == "id") res = m.pus[pu].id;
+            else if (what == "kind") res = kind_name(m.pus[pu].kind);
+            else {
+                const Property *p = m.prop(pu, what);
+                if (!p) return set_err(PDL_EINVAL, "PU %s has no property %s", m.pus[pu].id.c_str(), what.c_str());
+                res = p->value;
+            }
+        } else {
+            return set_err(PDL_EINVAL, "unknown query key '%s'", key);
+        }
+    }
+    if (out && len) {
+        size_t n = std::min(len - 1, res.size());
+        memcpy(out, res.data(), n);
+        out[n] = '\0';
+    }
+    return (int)res.size();
+}
+
+int pdl_kernel_times(int worker, float *ms, int n) {
+    int rc = check_loaded();
+    if (rc) return rc;
+    if (worker < 0 || worker >= (int)g->workers.size()) return set_err(PDL_EINVAL, "no local Worker %d", worker);
+    if (n < 0 || (n > 0 && !ms)) return set_err(PDL_EINVAL, "bad output buffer");
+    WorkerCtx &w = g->workers[worker];
+    if (g->dry_run) return 0;
+    CUDA_TRY(cudaSetDevice(w.device));
+    const int cnt = (int)w.kt_n;
+    for (int i = 0; i < cnt && i < n; ++i) {
+        CUDA_TRY(cudaEventSynchronize(w.kt_ev[2 * i + 1]));
+        CUDA_TRY(cudaEventElapsedTime(&ms[i], w.kt_ev[2 * i], w.kt_ev[2 * i + 1]));
+    }
+    w.kt_n = 0;
+    return cnt;
+}
+
+const char *pdl_last_error(void) { return g_err.c_str(); }
+
+void pdl_unload(void) {
+    free_state();
+    g_err.clear();
+}
+
+}  // extern "C"

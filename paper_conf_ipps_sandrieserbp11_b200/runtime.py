@@ -1,0 +1,160 @@
+"""One-process-per-GPU task runtime: the multi-Worker path of the DGEMM task.
+
+Each process is one co-existing Master controlling one Worker PU ("Masters
+... may co-exist with other Masters within the same system", PAPER.md
+L495-503), bound with ``pdl_load_rank``.  The BLOCK mapping (which C
+rectangle, which operand chunk each Worker holds) comes from libpdl's
+``pdl_plan`` (L1200-1208); this module only moves data between Workers:
+
+* initial ("unique chunk") layout -- Worker (r, c) of the Gr x Gc grid holds
+  chunk c of A's row-panel r (qa rows) and chunk r of B's column-panel c
+  (qb K-rows), so every operand byte lives on exactly one Worker;
+* exchange -- all-gather of the A chunks inside each grid row and of the B
+  chunks inside each grid column over torch.distributed (NCCL over NVLink 5 /
+  NVSwitch on the GPU box, gloo in the CPU tests).  This is the "derive
+  data-transfer paths ... via the explicitly specified interconnect entity"
+  step (L1336-1341) for the Worker<->Worker NVLink interconnect;
+* local task -- ``task_matmul_ex(..., PDL_TASK_PANELS)`` + ``pdl_run`` on the
+  gathered panels (libpdl, sm_100a kernels).
+
+There is no split-K, hence no reduction: each C element is produced by one
+Worker, and the result is bitwise identical for any Worker count (pin P7).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import torch
+import torch.distributed as dist
+
+from . import pdl
+
+
+@dataclass
+class WorkerPlan:
+    G: int
+    Gr: int
+    Gc: int
+    r: int
+    c: int
+    row0: int
+    row1: int
+    col0: int
+    col1: int
+    qa: int
+    qb: int
+    M: int
+    N: int
+    K: int
+
+    @property
+    def rows(self):
+        return self.row1 - self.row0
+
+    @property
+    def cols(self):
+        return self.col1 - self.col0
+
+    # this Worker's chunk of its A row-panel: panel rows [a0, a1)
+    @property
+    def a_span(self):
+        a0 = min(self.c * self.qa, self.rows)
+        return a0, min(a0 + self.qa, self.rows)
+
+    # this Worker's chunk of its B column-panel: K rows [b0, b1)
+    @property
+    def b_span(self):
+        b0 = min(self.r * self.qb, self.K)
+        return b0, min(b0 + self.qb, self.K)
+
+
+def worker_plan(M, N, K, tile, rank, group=None) -> WorkerPlan:
+    p = pdl.plan(M, N, K, tile, group=group, worker=rank)
+    return WorkerPlan(p["G"], p["Gr"], p["Gc"], p["r"], p["c"], p["row0"], p["row1"], p["col0"],
+                      p["col1"], p["qa"], p["qb"], M, N, K)
+
+
+class Grid:
+    """Row / column process groups of the Gr x Gc Worker grid (created
+    collectively: every rank creates every group in the same order)."""
+
+    def __init__(self, Gr, Gc, rank):
+        self.Gr, self.Gc, self.rank = Gr, Gc, rank
+        self.row_group = self.col_group = None
+        for r in range(Gr):
+            ranks = [r * Gc + c for c in range(Gc)]
+            g = dist.new_group(ranks) if Gc > 1 else None
+            if rank in ranks:
+                self.row_group = g
+        for c in range(Gc):
+            ranks = [r * Gc + c for r in range(Gr)]
+            g = dist.new_group(ranks) if Gr > 1 else None
+            if rank in ranks:
+                self.col_group = g
+
+
+def chunk_from_full(A, B, wp: WorkerPlan):
+    """Slice this Worker's unique chunks out of full A (M x K) and B (K x N),
+    zero-padded to qa x K and qb x cols (equal sizes for the all-gather)."""
+    a0, a1 = wp.a_span
+    b0, b1 = wp.b_span
+    Ach = torch.zeros((wp.qa, wp.K), dtype=A.dtype, device=A.device)
+    Bch = torch.zeros((wp.qb, wp.cols), dtype=B.dtype, device=B.device)
+    if a1 > a0:
+        Ach[: a1 - a0].copy_(A[wp.row0 + a0: wp.row0 + a1])
+    if b1 > b0 and wp.cols:
+        Bch[: b1 - b0].copy_(B[b0:b1, wp.col0: wp.col1])
+    return Ach, Bch
+
+
+class PanelBuffers:
+    def __init__(self, wp: WorkerPlan, dtype, device):
+        self.A = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dtype, device=device)
+        self.B = torch.empty((wp.Gr * wp.qb, wp.cols), dtype=dtype, device=device)
+
+
+def exchange(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers):
+    """All-gather the operand chunks: afterwards bufs.A[:rows] is the A
+    row-panel (rows x K) and bufs.B[:K] the B column-panel (K x cols)."""
+    if wp.Gc > 1:
+        dist.all_gather_into_tensor(bufs.A, Ach.contiguous(), group=grid.row_group)
+    else:
+        bufs.A.copy_(Ach)
+    if wp.Gr > 1:
+        dist.all_gather_into_tensor(bufs.B, Bch.contiguous(), group=grid.col_group)
+    else:
+        bufs.B.copy_(Bch)
+    return bufs.A[: wp.rows], bufs.B[: wp.K]
+
+
+def local_task(Apanel, Bpanel, Cblock, wp: WorkerPlan, tile=0, run=True):
+    """Run this Worker's rectangle through libpdl on the gathered panels."""
+    if wp.rows == 0 or wp.cols == 0:
+        return
+    pdl.task_matmul(Apanel, Bpanel, Cblock, M=wp.M, N=wp.N, K=wp.K, tile=tile,
+                    lda=Apanel.stride(0), ldb=Bpanel.stride(0), ldc=Cblock.stride(0), panels=True)
+    if run:
+        pdl.run_async()
+
+
+def distributed_matmul(A_full, B_full, C_full, tile=0, group=None):
+    """Public multi-Worker API: every rank passes the full (host or device)
+    A, B and its own C; rank r writes its rectangle of C.  Host operands are
+    copied chunk-wise to the Worker (PCIe), exchanged over NVLink, computed,
+    and the C block copied back (PCIe)."""
+    rank = dist.get_rank()
+    M, K = A_full.shape
+    N = B_full.shape[1]
+    wp = worker_plan(M, N, K, tile, rank, group)
+    grid = Grid(wp.Gr, wp.Gc, rank)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    Ach, Bch = chunk_from_full(A_full, B_full, wp)
+    Ach, Bch = Ach.to(dev, non_blocking=True), Bch.to(dev, non_blocking=True)
+    bufs = PanelBuffers(wp, A_full.dtype, dev)
+    Ap, Bp = exchange(Ach, Bch, wp, grid, bufs)
+    Cb = torch.empty((wp.rows, wp.cols), dtype=C_full.dtype, device=dev)
+    pdl.set_stream(torch.cuda.current_stream())
+    local_task(Ap, Bp, Cb, wp, tile)
+    pdl.sync()
+    C_full[wp.row0: wp.row1, wp.col0: wp.col1].copy_(Cb)
+    return wp

@@ -1,0 +1,83 @@
+"""N>1 path on CPU: world_size 2 and 4 processes over gloo.
+
+Each rank binds its Worker with pdl_load_rank (dry run: no device), takes its
+BLOCK plan from libpdl, slices its unique operand chunks, and runs the real
+exchange code (runtime.exchange: all-gather in grid rows / columns).  The
+gathered panels must equal the A row-panel and B column-panel of the Worker's
+C rectangle, and the rectangles of all ranks must tile C exactly once.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, shapes, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), PDL_DRY_RUN="1")
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime
+    import workloads as W
+    out = []
+    try:
+        pdl.load(pdl.descriptor_path(world), rank=rank, nranks=world)
+        assert pdl.query("local_workers") == "1"
+        for (M, N, K, tile) in shapes:
+            A = torch.from_numpy(W.signed((M, K), np.float64, 1))
+            B = torch.from_numpy(W.signed((K, N), np.float64, 2))
+            wp = runtime.worker_plan(M, N, K, tile, rank)
+            grid = runtime.Grid(wp.Gr, wp.Gc, rank)
+            Ach, Bch = runtime.chunk_from_full(A, B, wp)
+            bufs = runtime.PanelBuffers(wp, A.dtype, A.device)
+            Ap, Bp = runtime.exchange(Ach, Bch, wp, grid, bufs)
+            ok_a = torch.equal(Ap, A[wp.row0:wp.row1])
+            ok_b = torch.equal(Bp, B[:, wp.col0:wp.col1])
+            out.append((M, N, K, tile, wp.row0, wp.row1, wp.col0, wp.col1, wp.Gr, wp.Gc, ok_a, ok_b))
+        pdl.unload()
+        q.put((rank, out, None))
+    except Exception as e:  # pragma: no cover - reported to the parent
+        q.put((rank, out, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+SHAPES = [(64, 64, 64, 32), (100, 70, 30, 16), (37, 53, 19, 0), (129, 257, 65, 64), (3, 200, 7, 8)]
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_exchange_assembles_panels(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, SHAPES, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, out, err in res:
+        assert err is None, f"rank {rank}: {err}"
+        assert len(out) == len(SHAPES)
+    for si, (M, N, K, tile) in enumerate(SHAPES):
+        cover = np.zeros((M, N), dtype=int)
+        for rank, out, _ in res:
+            _, _, _, _, r0, r1, c0, c1, Gr, Gc, ok_a, ok_b = out[si]
+            assert ok_a and ok_b, (rank, SHAPES[si])
+            assert Gr * Gc == world
+            cover[r0:r1, c0:c1] += 1
+        assert np.all(cover == 1)
