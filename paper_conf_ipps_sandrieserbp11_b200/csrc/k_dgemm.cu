@@ -13,10 +13,12 @@
 //    4-stage shared-memory ring; mbarrier full/empty handshakes; eight DMMA
 //    warps (warp tile 64 x 32, 128 accumulator registers/thread), thread 0
 //    refilling each stage once all warps released it.
-//  * Bank-conflict-free fragment loads: within each 16-wide K block the four
-//    k4 MMA steps take k = {0,1,4,5}, {2,3,6,7}, {8,9,12,13}, {10,11,14,15}
-//    (same permutation for A and B), which with the 128B swizzle makes every
-//    64-bit fragment load exactly 2 shared-memory wavefronts.  The summation
+//  * Bank-conflict-free 16-byte fragment loads (ld.shared.v2.f64): within
+//    each 16-wide K block the four k4 MMA steps take k = {0,4,10,14},
+//    {1,5,11,15}, {2,6,8,12}, {3,7,9,13} (same permutation for A and B); with
+//    the 128B swizzle every quarter-warp hits 8 distinct bank groups, and one
+//    A load serves two steps, one B load two n8 tiles.  Fragments of the next
+//    step (and next K block) are prefetched before the current DMMAs.  The summation
 //    order per C element is fixed by this kernel alone, so results do not
 //    depend on the Worker rectangle or task tile (bitwise invariance, pin P7).
 //  * CTA tile 128 x 128, grouped rasterisation for L2 reuse, masked
@@ -49,10 +51,8 @@ __device__ __forceinline__ uint32_t swz128(uint32_t row, uint32_t j) {
     return row * 128u + ((((j >> 1) ^ (row & 7u)) << 4) | ((j & 1u) << 3));
 }
 
-__device__ __forceinline__ double lds64(uint32_t addr) {
-    double v;
-    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(addr));
-    return v;
+__device__ __forceinline__ void lds128(uint32_t addr, double &x, double &y) {
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(x), "=d"(y) : "r"(addr));
 }
 
 __device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b) {
@@ -114,10 +114,17 @@ __global__ void __launch_bounds__(k1::THREADS, 1)
     }
 
     // ---------------- DMMA consumers ----------------
+    // Fragment schedule (K1): each lane reads 16-byte chunks.  A: for
+    // row m the lane with MMA-k index p reads chunk cA(p) = {0,2,5,7}[p] (k =
+    // 2cA, 2cA+1: steps 0 and 1) and chunk cA(p)^1 (steps 2 and 3).  B: per step
+    // one 16 B load per 16-column pair gives the b operand of two n8 tiles
+    // (columns 2j and 2j+1).  The k order per 16-wide block is
+    // {0,4,10,14},{1,5,11,15},{2,6,8,12},{3,7,9,13}; with the 128B swizzle every
+    // quarter-warp of every ld.shared.v2.f64 hits 8 distinct bank groups.
     const int wm = warp >> 2, wn = warp & 3;   // 2 x 4 warps, warp tile 64 x 32
-    const uint32_t g4 = (uint32_t)lane >> 2;   // groupID
-    const uint32_t p = (uint32_t)lane & 3u;    // thread in group -> MMA k index
-    const uint32_t kperm = (p & 1u) + ((p >> 1) << 2);   // {0,1,4,5}
+    const uint32_t g4 = (uint32_t)lane >> 2;   // groupID (MMA row / B column pair)
+    const uint32_t p = (uint32_t)lane & 3u;    // thread in group (MMA k index)
+    const uint32_t cA = (0x7520u >> (4u * p)) & 0xFu;
 
     double acc[8][4][2];
 #pragma unroll
@@ -125,31 +132,59 @@ __global__ void __launch_bounds__(k1::THREADS, 1)
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
 
-    // per-lane constant parts of the fragment addresses
-    const uint32_t arow0 = 64u * wm + g4;              // + 8*mi
-    const uint32_t bcol0 = 32u * wn + g4;              // + 8*ni  (column inside the CTA tile)
+    const uint32_t rowA = 64u * wm + g4;
+    const uint32_t offA0 = rowA * 128u + ((cA ^ g4) << 4);           // + mi*1024, half 0
+    const uint32_t offA1 = rowA * 128u + (((cA ^ 1u) ^ g4) << 4);    // half 1
+    uint32_t offB[4];
+#pragma unroll
+    for (int st = 0; st < 4; ++st) {
+        const uint32_t k = 2u * (st < 2 ? cA : (cA ^ 1u)) + (uint32_t)(st & 1);
+        offB[st] = A_BYTES + (2u * wn) * B_SUB_BYTES + k * 128u + ((g4 ^ (k & 7u)) << 4);
+    }
 
+    double a[2][8][2];   // [half][mi][k of the two steps of that half]
+    double b[2][4];      // [step parity][ni]
+    auto load_a = [&](uint32_t st_base, int half) {
+        const uint32_t o = st_base + (half ? offA1 : offA0);
+#pragma unroll
+        for (int mi = 0; mi < 8; ++mi) lds128(o + mi * 1024u, a[half][mi][0], a[half][mi][1]);
+    };
+    auto load_b = [&](uint32_t st_base, int st) {
+        const uint32_t o = st_base + offB[st];
+        lds128(o, b[st & 1][0], b[st & 1][1]);                      // columns 16*pair + 2j, 2j+1, pair 0
+        lds128(o + B_SUB_BYTES, b[st & 1][2], b[st & 1][3]);        // pair 1
+    };
+
+    if (nk > 0) {
+        mbar_wait(bar_full, 0);
+        load_a(base, 0);
+        load_b(base, 0);
+    }
     for (int kb = 0; kb < nk; ++kb) {
         const int s = kb % STAGES;
         const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
-        mbar_wait(bar_full + 8 * s, ph);
         const uint32_t sa = base + s * STAGE_BYTES;
-        const uint32_t sb = sa + A_BYTES;
+        const int sn = (kb + 1) % STAGES;
+        const uint32_t san = base + sn * STAGE_BYTES;
 #pragma unroll
-        for (int step = 0; step < 4; ++step) {
-            const uint32_t k = (uint32_t)((step & 1) * 2 + (step >> 1) * 8) + kperm;
-            double a[8], b[4];
-#pragma unroll
-            for (int mi = 0; mi < 8; ++mi) a[mi] = lds64(sa + swz128(arow0 + 8u * mi, k));
-#pragma unroll
-            for (int ni = 0; ni < 4; ++ni) {
-                const uint32_t n = bcol0 + 8u * ni;
-                b[ni] = lds64(sb + (n >> 4) * B_SUB_BYTES + swz128(k, n & 15u));
+        for (int st = 0; st < 4; ++st) {
+            // prefetch the operands of the next step (next k-block for st == 3)
+            if (st == 0) load_a(sa, 1);
+            if (st == 2) {
+                if (kb + 1 < nk) mbar_wait(bar_full + 8 * sn, (uint32_t)((kb + 1) / STAGES) & 1u);
+                load_a(san, 0);
             }
+            if (st < 3) load_b(sa, st + 1);
+            else load_b(san, 0);
+            const int h = st >> 1, e = st & 1;
 #pragma unroll
             for (int mi = 0; mi < 8; ++mi)
 #pragma unroll
-                for (int ni = 0; ni < 4; ++ni) dmma(acc[mi][ni][0], acc[mi][ni][1], a[mi], b[ni]);
+                for (int ni = 0; ni < 4; ++ni) {
+                    // n8 tile ni uses columns 16*(ni>>1) + 2j + (ni&1) of the warp's 32
+                    const double bv = b[st & 1][(ni >> 1) * 2 + (ni & 1)];
+                    dmma(acc[mi][ni][0], acc[mi][ni][1], a[h][mi][e], bv);
+                }
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(bar_empty + 8 * s);
@@ -159,22 +194,28 @@ __global__ void __launch_bounds__(k1::THREADS, 1)
         }
     }
 
-    // ---------------- epilogue: registers -> global (masked, 16 B when aligned) ----------------
+    // ---------------- epilogue: registers -> global ----------------
+    // acc[mi][2q+e][h] is C[row][32wn + 16q + 4p + 2h + e]: each lane owns 4
+    // consecutive columns per 16-column pair -> two 16-byte stores.
     const int row_base = tm * BM + 64 * wm + (int)g4;
-    const int col_base = tn * BN + 32 * wn + 2 * (int)p;
 #pragma unroll
     for (int mi = 0; mi < 8; ++mi) {
         const int row = row_base + 8 * mi;
         if (row >= M) continue;
         double *crow = C + (int64_t)row * ldc;
 #pragma unroll
-        for (int ni = 0; ni < 4; ++ni) {
-            const int col = col_base + 8 * ni;
-            if (vec_ok && col + 1 < N) {
-                *reinterpret_cast<double2 *>(crow + col) = make_double2(acc[mi][ni][0], acc[mi][ni][1]);
+        for (int q = 0; q < 2; ++q) {
+            const int col = tn * BN + 32 * wn + 16 * q + 4 * (int)p;
+            const double v0 = acc[mi][2 * q][0], v1 = acc[mi][2 * q + 1][0];
+            const double v2 = acc[mi][2 * q][1], v3 = acc[mi][2 * q + 1][1];
+            if (vec_ok && col + 3 < N) {
+                *reinterpret_cast<double2 *>(crow + col) = make_double2(v0, v1);
+                *reinterpret_cast<double2 *>(crow + col + 2) = make_double2(v2, v3);
             } else {
-                if (col < N) crow[col] = acc[mi][ni][0];
-                if (col + 1 < N) crow[col + 1] = acc[mi][ni][1];
+                if (col < N) crow[col] = v0;
+                if (col + 1 < N) crow[col + 1] = v1;
+                if (col + 2 < N) crow[col + 2] = v2;
+                if (col + 3 < N) crow[col + 3] = v3;
             }
         }
     }
