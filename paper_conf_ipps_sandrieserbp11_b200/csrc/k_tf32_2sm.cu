@@ -1,0 +1,239 @@
+// k_tf32_2sm.cu -- K2 v3: 3xTF32 tile kernel on a CTA pair (tcgen05 cta_group::2).
+//
+// Same product as K2 v1 (k_tf32.cu; FP32 task variant, 3xTF32 split from K3,
+// K-chunk promotion of the truncating TMEM accumulation, R16) with
+// the B200's paired-SM tensor-core mode:
+//  * a cluster of 2 CTAs on one TPC computes a 256 x 256 tile: CTA r holds rows
+//    [128r, 128r+128) of A and rows [128r, 128r+128) of B^T (half of N) in its
+//    own shared memory; the leader CTA issues one
+//    tcgen05.mma.cta_group::2.kind::tf32 (M = 256, N = 256, K = 8) that reads
+//    the operands of both CTAs and writes each CTA's 128 x 256 FP32
+//    accumulator into that CTA's TMEM.  Per SM the tensor core reads half the
+//    shared-memory bytes of the 1-SM 128 x 256 shape and L2 traffic halves
+//    relative to 128 x 128 tiles;
+//  * both CTAs' TMA loads (.cta_group::2) complete on the leader's full
+//    barrier; MMA completion is multicast (tcgen05.commit ... multicast) to
+//    both CTAs' empty / accumulator-ready barriers; the peer's epilogue warps
+//    release accumulator buffers on the leader's barrier through mapa;
+//  * TMEM: 512 columns = 2 accumulator buffers x 256; 16 epilogue warps (4 per
+//    TMEM lane quarter, 64 columns each) promote every 128-wide K chunk into
+//    FP32 registers with round-to-nearest.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "kernels.h"
+#include "ptx.cuh"
+#include "tcgen05.cuh"
+
+namespace pdlk {
+
+namespace k2x {
+constexpr int BM = 128;                 // A rows per CTA (UMMA M = 256 over the pair)
+constexpr int BN = 256;                 // UMMA N (cluster tile columns)
+constexpr int BNH = BN / 2;             // B^T rows per CTA
+constexpr int BK = K2_BK, STAGES = 3, UMMA_K = 8;
+constexpr int A_BYTES = BM * BK * 4;    // 16 KiB
+constexpr int B_BYTES = BNH * BK * 4;   // 16 KiB
+constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;   // 64 KiB per CTA
+constexpr int EPI_WARPS = 16;
+constexpr int EPI_COLS = BN / (EPI_WARPS / 4);           // 64 columns per epilogue warp
+constexpr int FIRST_EPI_WARP = 2;   // warps 2..17: each TMEM lane quarter (warp % 4) gets 4 warps
+constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
+constexpr int TMEM_COLS = 512;
+constexpr int KCB = 4;                  // K chunk = KCB * BK = 128 (R16)
+constexpr int GROUP_M = 8;              // cluster-tile rows per raster group
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+}  // namespace k2x
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
+    gemm_3xtf32_2sm_kernel(const __grid_constant__ CUtensorMap tAh, const __grid_constant__ CUtensorMap tAl,
+                           const __grid_constant__ CUtensorMap tBh, const __grid_constant__ CUtensorMap tBl,
+                           float *__restrict__ C, int64_t ldc, int M, int N, int Kp, int tiles_m, int tiles_n,
+                           int vec_ok) {
+    using namespace k2x;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
+    const uint32_t bar_full = base + STAGES * STAGE_BYTES;   // STAGES x 8 (used in the leader)
+    const uint32_t bar_empty = bar_full + STAGES * 8;         // STAGES x 8 (both CTAs)
+    const uint32_t bar_tfull = bar_empty + STAGES * 8;        // 2 x 8 (both CTAs)
+    const uint32_t bar_tempty = bar_tfull + 16;               // 2 x 8 (leader: both CTAs' epilogues)
+    const uint32_t tmem_slot = bar_tempty + 16;
+    uint8_t *const gbase = smem_raw + (base - smem_u32(smem_raw));
+    volatile uint32_t *tmem_slot_ptr = reinterpret_cast<volatile uint32_t *>(gbase + (tmem_slot - base));
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = cluster_ctarank();
+
+    // grouped raster over 256 x 256 cluster tiles
+    const int cid = blockIdx.x >> 1;
+    const int per_group = GROUP_M * tiles_n;
+    const int g = cid / per_group;
+    const int first_m = g * GROUP_M;
+    const int gsz = min(tiles_m - first_m, GROUP_M);
+    const int tm = first_m + (cid % per_group) % gsz;
+    const int tn = (cid % per_group) / gsz;
+    const int m0 = tm * (2 * BM) + (int)rank * BM;   // this CTA's A rows
+    const int nb0 = tn * BN + (int)rank * BNH;       // this CTA's B^T rows
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(bar_full + 8 * s, 1);
+            mbar_init(bar_empty + 8 * s, 1);
+        }
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(bar_tfull + 8 * b, 1);
+            mbar_init(bar_tempty + 8 * b, 2 * EPI_WARPS);
+        }
+        fence_barrier_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(tmem_slot),
+                     "n"(TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    cluster_sync_all();   // barrier inits and TMEM allocation visible to both CTAs
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem_base = *tmem_slot_ptr;
+
+    const int nk = Kp / BK;
+    const int nchunks = (nk + KCB - 1) / KCB;
+
+    if (warp == 0) {
+        // ---------------- TMA producer (both CTAs) ----------------
+        if (lane == 0) {
+            tma_prefetch_desc(&tAh);
+            tma_prefetch_desc(&tAl);
+            tma_prefetch_desc(&tBh);
+            tma_prefetch_desc(&tBl);
+            for (int kb = 0; kb < nk; ++kb) {
+                const int s = kb % STAGES;
+                const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+                mbar_wait(bar_empty + 8 * s, ph ^ 1u);
+                const uint32_t fb_leader = mapa_shared(bar_full + 8 * s, 0);
+                if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * STAGE_BYTES);
+                const uint32_t st = base + s * STAGE_BYTES;
+                tma_load_2d_2sm(st, &tAh, fb_leader, kb * BK, m0);
+                tma_load_2d_2sm(st + A_BYTES, &tAl, fb_leader, kb * BK, m0);
+                tma_load_2d_2sm(st + 2 * A_BYTES, &tBh, fb_leader, kb * BK, nb0);
+                tma_load_2d_2sm(st + 2 * A_BYTES + B_BYTES, &tBl, fb_leader, kb * BK, nb0);
+            }
+        }
+    } else if (warp == 1) {
+        // ---------------- MMA issuer (leader CTA, one thread) ----------------
+        if (rank == 0 && lane == 0) {
+            constexpr uint32_t idesc = idesc_tf32(2 * BM, BN);
+            for (int kb = 0; kb < nk; ++kb) {
+                const int chunk = kb / KCB, kin = kb - chunk * KCB;
+                const uint32_t buf = (uint32_t)chunk & 1u;
+                const uint32_t dtm = tmem_base + buf * BN;
+                if (kin == 0) {
+                    mbar_wait(bar_tempty + 8 * buf, ((uint32_t)(chunk >> 1) & 1u) ^ 1u);
+                    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                }
+                const int s = kb % STAGES;
+                const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+                mbar_wait(bar_full + 8 * s, ph);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                const uint32_t st = base + s * STAGE_BYTES;
+                const uint32_t ah = st, al = st + A_BYTES, bh = st + 2 * A_BYTES, bl = bh + B_BYTES;
+#pragma unroll
+                for (int kk = 0; kk < BK / UMMA_K; ++kk) {
+                    const uint32_t off = kk * UMMA_K * 4;
+                    const uint32_t acc0 = (kin == 0 && kk == 0) ? 0u : 1u;
+                    umma_tf32_2sm(dtm, umma_desc_k_sw128(al + off), umma_desc_k_sw128(bh + off), idesc, acc0);
+                    umma_tf32_2sm(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bl + off), idesc, 1u);
+                    umma_tf32_2sm(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bh + off), idesc, 1u);
+                }
+                umma_commit_2sm(bar_empty + 8 * s);
+                if (kin == KCB - 1 || kb == nk - 1) umma_commit_2sm(bar_tfull + 8 * buf);
+            }
+        }
+        __syncwarp();
+    } else if (warp >= FIRST_EPI_WARP) {
+        // ---------------- epilogue: promote chunks (both CTAs) ----------------
+        const int e = warp - FIRST_EPI_WARP;
+        const int q = warp & 3;                      // TMEM lane quarter accessible to this warp
+        const int cg = e >> 2;                       // column group
+        const uint32_t tl = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(cg * EPI_COLS);
+        const uint32_t tempty_leader0 = mapa_shared(bar_tempty, 0);
+        float acc[EPI_COLS];
+#pragma unroll
+        for (int j = 0; j < EPI_COLS; ++j) acc[j] = 0.0f;
+        for (int chunk = 0; chunk < nchunks; ++chunk) {
+            const uint32_t buf = (uint32_t)chunk & 1u;
+            mbar_wait(bar_tfull + 8 * buf, (uint32_t)(chunk >> 1) & 1u);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll
+            for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
+                uint32_t r[16];
+                tmem_ld16(tl + buf * BN + c0, r);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) acc[c0 + j] += __uint_as_float(r[j]);
+            }
+            asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+            __syncwarp();
+            if (lane == 0) mbar_arrive_cluster(tempty_leader0 + 8 * buf);
+        }
+        const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
+        const int cbase = tn * BN + cg * EPI_COLS;
+        if (row < M) {
+            float *crow = C + (int64_t)row * ldc + cbase;
+            if (vec_ok && cbase + EPI_COLS <= N) {
+#pragma unroll
+                for (int j = 0; j < EPI_COLS; j += 4)
+                    *reinterpret_cast<float4 *>(crow + j) = make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < EPI_COLS; ++j)
+                    if (cbase + j < N) crow[j] = acc[j];
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    cluster_sync_all();   // both CTAs done with TMEM and with each other's shared memory
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(TMEM_COLS));
+    }
+}
+
+static bool map_f32_2sm(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_t Kp, uint64_t rows,
+                        uint32_t box_rows) {
+    cuuint64_t dims[2] = {Kp, rows};
+    cuuint64_t strides[1] = {Kp * 4};
+    cuuint32_t box[2] = {(cuuint32_t)k2x::BK, box_rows};
+    cuuint32_t es[2] = {1, 1};
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
+                                   const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
+                                   cudaStream_t stream) {
+    using namespace k2x;
+    if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
+    CUtensorMap tah, tal, tbh, tbl;
+    if (!map_f32_2sm(enc, &tah, Ahi, Kp, M, BM) || !map_f32_2sm(enc, &tal, Alo, Kp, M, BM) ||
+        !map_f32_2sm(enc, &tbh, Bhi, Kp, N, BNH) || !map_f32_2sm(enc, &tbl, Blo, Kp, N, BNH))
+        return cudaErrorInvalidValue;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static bool attr_done[64] = {false};
+    if (dev < 64 && !attr_done[dev]) {
+        cudaError_t e =
+            cudaFuncSetAttribute(gemm_3xtf32_2sm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+        if (e != cudaSuccess) return e;
+        attr_done[dev] = true;
+    }
+    const int tiles_m = (int)((M + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((N + BN - 1) / BN);
+    const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 3) == 0) ? 1 : 0;
+    gemm_3xtf32_2sm_kernel<<<2 * tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(
+        tah, tal, tbh, tbl, C, ldc, (int)M, (int)N, (int)Kp, tiles_m, tiles_n, vec_ok);
+    return cudaGetLastError();
+}
+
+}  // namespace pdlk

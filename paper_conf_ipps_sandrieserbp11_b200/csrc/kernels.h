@@ -34,5 +34,9 @@ cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t 
 cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
                                cudaStream_t stream);
+// K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
+cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
+                                   const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
+                                   cudaStream_t stream);
 
 }  // namespace pdlk

@@ -86,14 +86,17 @@ struct WorkerCtx {
     // event pairs around every dominant-kernel launch since the last pdl_kernel_times()
     std::vector<cudaEvent_t> kt_ev;
     size_t kt_n = 0;
+    // pipelined staging: copy-in, copy-out, second compute stream; reusable events
+    cudaStream_t aux[3] = {nullptr, nullptr, nullptr};
+    std::vector<cudaEvent_t> ev_pool;
 };
 
 constexpr size_t kMaxKernelTimes = 4096;
 
 // Record the start / end of a dominant-kernel launch on the worker's stream.
-int kt_mark(WorkerCtx &w, bool start) {
+int kt_mark(WorkerCtx &w, bool start, cudaStream_t st) {
     cudaEvent_t &last = start ? w.ev_k0 : w.ev_k1;
-    cudaError_t e = cudaEventRecord(last, w.stream);
+    cudaError_t e = cudaEventRecord(last, st);
     if (e != cudaSuccess) return PDL_ECUDA;
     if (w.kt_n >= kMaxKernelTimes) return PDL_OK;
     size_t idx = 2 * w.kt_n + (start ? 0 : 1);
@@ -102,7 +105,7 @@ int kt_mark(WorkerCtx &w, bool start) {
         if (cudaEventCreate(&ev) != cudaSuccess) return PDL_ECUDA;
         w.kt_ev.push_back(ev);
     }
-    if (cudaEventRecord(w.kt_ev[idx], w.stream) != cudaSuccess) return PDL_ECUDA;
+    if (cudaEventRecord(w.kt_ev[idx], st) != cudaSuccess) return PDL_ECUDA;
     if (!start) w.kt_n++;
     return PDL_OK;
 }
@@ -302,6 +305,9 @@ void free_state() {
         if (w.ev_k0) cudaEventDestroy(w.ev_k0);
         if (w.ev_k1) cudaEventDestroy(w.ev_k1);
         for (auto ev : w.kt_ev) cudaEventDestroy(ev);
+        for (auto ev : w.ev_pool) cudaEventDestroy(ev);
+        for (auto st : w.aux)
+            if (st) cudaStreamDestroy(st);
     }
     delete g;
     g = nullptr;
@@ -347,99 +353,227 @@ bool overlaps(const void *a, size_t an, const void *b, size_t bn) {
 
 int64_t round_up(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
 
-// Make a rows x cols operand (elements of `es` bytes, leading dim ld) usable
-// by a TMA-fed kernel on worker w: device-resident on w.device, 16 B-aligned
-// base, pitch a multiple of 16 B.  Copies (H2D over the Master->Worker
-// interconnect, or D2D/peer) into a library buffer when needed.
-int stage_operand(WorkerCtx &w, int slot, const void *src, int64_t ld, int64_t rows, int64_t cols, int es,
-                  const void **out, int64_t *out_ld, bool need_tma_align) {
-    int loc = locate(src);
-    bool aligned = ((uintptr_t)src % 16 == 0) && ((ld * es) % 16 == 0);
-    if (loc == w.device && (aligned || !need_tma_align)) {
-        *out = src;
-        *out_ld = ld;
-        return PDL_OK;
+// ---- pipelined execution of one Worker rectangle -------------------------
+//
+// The rectangle is cut into RB row bands x CP column panels of whole task
+// tiles.  Operands that live outside the Worker's memory region (host =
+// Master MR, or another device) are moved per band / panel on a copy-in
+// stream, each sub-rectangle's kernel waits only for its own A band and B
+// panel, and results leave on a copy-out stream as soon as their kernel ends,
+// so PCIe traffic overlaps the tile kernels (L1336-1341: "data-transfer paths
+// between memory-regions ... via the explicitly specified interconnect").
+// Sub-rectangle kernels alternate between two compute streams so one
+// kernel's last wave overlaps the next.  Device-resident operands take a
+// single launch (RB = CP = 1).  Every sub-kernel computes the same per-element
+// K order, so C is bitwise identical for any cut (R14).
+
+cudaEvent_t ev_get(WorkerCtx &w, size_t &next) {
+    if (next >= w.ev_pool.size()) {
+        cudaEvent_t e = nullptr;
+        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+        w.ev_pool.push_back(e);
     }
-    int64_t pitch_el = round_up(std::max<int64_t>(cols, 1), 16 / es);
-    void *dst;
-    int rc = ensure_buf(w, slot, (size_t)(pitch_el * std::max<int64_t>(rows, 1) * es), &dst);
-    if (rc) return rc;
-    cudaError_t e = cudaMemcpy2DAsync(dst, (size_t)(pitch_el * es), src, (size_t)(ld * es), (size_t)(cols * es),
-                                      (size_t)rows, cudaMemcpyDefault, w.stream);
-    if (e != cudaSuccess) return set_err(PDL_ECUDA, "operand staging copy failed: %s", cudaGetErrorString(e));
-    *out = dst;
-    *out_ld = pitch_el;
+    return w.ev_pool[next++];
+}
+
+int ensure_aux(WorkerCtx &w) {
+    for (int i = 0; i < 3; ++i)
+        if (!w.aux[i]) CUDA_TRY(cudaStreamCreateWithFlags(&w.aux[i], cudaStreamNonBlocking));
     return PDL_OK;
 }
 
-// Execute one task's rectangle on worker w.  A/B/C point at the rectangle's
-// panels (A: rows x K at ld lda; B: K x cols at ldb; C: rows x cols at ldc).
 int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
     if (rows <= 0 || cols <= 0) return PDL_OK;
     CUDA_TRY(cudaSetDevice(w.device));
     const int es = t.dtype == PDL_F64 ? 8 : 4;
+    const bool f64 = t.dtype == PDL_F64;
     const int64_t K = t.K;
-    // C destination: in place when it is on this device, else a staging buffer
-    int cloc = locate(C);
-    void *Cd = C;
-    int64_t ldcd = t.ldc;
-    bool c_staged = false;
-    if (cloc != w.device) {
-        int64_t pitch = round_up(cols, 16 / es);
-        int rc = ensure_buf(w, BUF_C, (size_t)(pitch * rows * es), &Cd);
-        if (rc) return rc;
-        ldcd = pitch;
-        c_staged = true;
+    const int64_t pe = 16 / es;   // elements per 16 bytes
+
+    // Where the operands live and whether they must be staged into this Worker's MR.
+    const bool a_st = K > 0 && (locate(A) != w.device || (f64 && (((uintptr_t)A % 16) || (t.lda * es) % 16)));
+    const bool b_st = K > 0 && (locate(B) != w.device || (f64 && (((uintptr_t)B % 16) || (t.ldb * es) % 16)));
+    const bool c_st = locate(C) != w.device;
+
+    // Cut: row bands / column panels aligned to 128 (a K1/K2 tile edge).
+    int RB = 1, CP = 1;
+    const char *pe_env = getenv("PDL_PIPELINE");
+    const bool force = pe_env && !strcmp(pe_env, "force");
+    const bool off = pe_env && !strcmp(pe_env, "0");
+    const double flops = 2.0 * rows * cols * (double)K;
+    if (!off && (a_st || b_st || c_st) && K > 0 && (force || flops >= 2e11)) {
+        RB = (int)std::min<int64_t>(8, std::max<int64_t>(1, rows / 2048));
+        CP = cols >= 8192 ? 2 : 1;
+        if (force) {
+            RB = (int)std::min<int64_t>(4, std::max<int64_t>(1, (rows + 127) / 128));
+            CP = (int)std::min<int64_t>(2, std::max<int64_t>(1, (cols + 127) / 128));
+        }
     }
-    if (K == 0) {
-        // empty sum: C = 0 (BLAS convention)
-        CUDA_TRY(cudaMemset2DAsync(Cd, (size_t)(ldcd * es), 0, (size_t)(cols * es), (size_t)rows, w.stream));
-    } else if (t.dtype == PDL_F64) {
-        const void *Ad, *Bd;
-        int64_t lda, ldb;
-        int rc = stage_operand(w, BUF_A, A, t.lda, rows, K, 8, &Ad, &lda, true);
-        if (!rc) rc = stage_operand(w, BUF_B, B, t.ldb, K, cols, 8, &Bd, &ldb, true);
-        if (rc) return rc;
-        pdlk::EncodeTiledFn enc;
-        if ((rc = get_encoder(&enc))) return rc;
-        if (kt_mark(w, true)) return set_err(PDL_ECUDA, "event record failed");
-        cudaError_t e = pdlk::launch_dgemm_k1(enc, (const double *)Ad, lda, (const double *)Bd, ldb, (double *)Cd, ldcd,
-                                              rows, cols, K, w.stream);
-        if (e != cudaSuccess) return set_err(PDL_ECUDA, "K1 launch failed: %s", cudaGetErrorString(e));
-        if (kt_mark(w, false)) return set_err(PDL_ECUDA, "event record failed");
-        w.launches += 1;
-        w.timed = true;
-    } else {
-        // FP32: split pre-pass reads any device layout; host/other-device operands are staged first.
-        const void *Ad, *Bd;
-        int64_t lda, ldb;
-        int rc = stage_operand(w, BUF_A, A, t.lda, rows, K, 4, &Ad, &lda, false);
-        if (!rc) rc = stage_operand(w, BUF_B, B, t.ldb, K, cols, 4, &Bd, &ldb, false);
-        if (rc) return rc;
-        const int64_t Kp = round_up(K, pdlk::K2_BK);
-        void *ahi, *alo, *bhi, *blo;
-        if ((rc = ensure_buf(w, BUF_AHI, (size_t)(rows * Kp * 4), &ahi))) return rc;
-        if ((rc = ensure_buf(w, BUF_ALO, (size_t)(rows * Kp * 4), &alo))) return rc;
-        if ((rc = ensure_buf(w, BUF_BHI, (size_t)(cols * Kp * 4), &bhi))) return rc;
-        if ((rc = ensure_buf(w, BUF_BLO, (size_t)(cols * Kp * 4), &blo))) return rc;
-        cudaError_t e = pdlk::launch_split_rows((const float *)Ad, lda, rows, K, (float *)ahi, (float *)alo, Kp, w.stream);
-        if (e == cudaSuccess)
-            e = pdlk::launch_split_cols_t((const float *)Bd, ldb, K, cols, (float *)bhi, (float *)blo, Kp, w.stream);
-        if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
-        pdlk::EncodeTiledFn enc;
-        if ((rc = get_encoder(&enc))) return rc;
-        if (kt_mark(w, true)) return set_err(PDL_ECUDA, "event record failed");
-        e = pdlk::launch_gemm_3xtf32(enc, (const float *)ahi, (const float *)alo, (const float *)bhi, (const float *)blo,
-                                     Kp, (float *)Cd, ldcd, rows, cols, w.stream);
-        if (e != cudaSuccess) return set_err(PDL_ECUDA, "K2 launch failed: %s", cudaGetErrorString(e));
-        if (kt_mark(w, false)) return set_err(PDL_ECUDA, "event record failed");
-        w.launches += 3;
-        w.timed = true;
+    std::vector<int64_t> rb(RB + 1), cp(CP + 1);
+    for (int i = 0; i <= RB; ++i) rb[i] = std::min<int64_t>(rows, round_up((int64_t)i * rows / RB, 128));
+    for (int j = 0; j <= CP; ++j) cp[j] = std::min<int64_t>(cols, round_up((int64_t)j * cols / CP, 128));
+    rb[RB] = rows;
+    cp[CP] = cols;
+    const bool piped = RB * CP > 1;
+    int rc;
+    if (piped && (rc = ensure_aux(w))) return rc;
+    cudaStream_t s_in = piped ? w.aux[0] : w.stream, s_out = piped ? w.aux[1] : w.stream;
+    cudaStream_t s_cmp[2] = {w.stream, piped ? w.aux[2] : w.stream};
+    size_t evn = 0;
+    cudaEvent_t ev_start = ev_get(w, evn);
+    if (!ev_start) return set_err(PDL_ECUDA, "event create failed");
+    if (piped) {
+        // side streams start after everything already queued on the Worker stream
+        CUDA_TRY(cudaEventRecord(ev_start, w.stream));
+        for (int i = 0; i < 3; ++i) CUDA_TRY(cudaStreamWaitEvent(w.aux[i], ev_start, 0));
     }
-    if (c_staged) {
-        cudaError_t e = cudaMemcpy2DAsync(C, (size_t)(t.ldc * es), Cd, (size_t)(ldcd * es), (size_t)(cols * es),
-                                          (size_t)rows, cudaMemcpyDefault, w.stream);
-        if (e != cudaSuccess) return set_err(PDL_ECUDA, "result gather copy failed: %s", cudaGetErrorString(e));
+
+    // Device views of the operands.
+    const char *Ad = (const char *)A, *Bd = (const char *)B;
+    char *Cd = (char *)C;
+    int64_t lda = t.lda, ldb = t.ldb, ldcd = t.ldc;
+    void *p;
+    if (a_st) {
+        lda = round_up(std::max<int64_t>(K, 1), pe);
+        if ((rc = ensure_buf(w, BUF_A, (size_t)(lda * rows * es), &p))) return rc;
+        Ad = (const char *)p;
+    }
+    if (b_st) {
+        ldb = round_up(cols, pe);
+        if ((rc = ensure_buf(w, BUF_B, (size_t)(ldb * K * es), &p))) return rc;
+        Bd = (const char *)p;
+    }
+    if (c_st) {
+        ldcd = round_up(cols, pe);
+        if ((rc = ensure_buf(w, BUF_C, (size_t)(ldcd * rows * es), &p))) return rc;
+        Cd = (char *)p;
+    }
+    // FP32 split buffers (K-major hi/lo of A rows and of B^T rows)
+    const int64_t Kp = round_up(std::max<int64_t>(K, 1), pdlk::K2_BK);
+    float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
+    if (!f64 && K > 0) {
+        if ((rc = ensure_buf(w, BUF_AHI, (size_t)(rows * Kp * 4), &p))) return rc;
+        ahi = (float *)p;
+        if ((rc = ensure_buf(w, BUF_ALO, (size_t)(rows * Kp * 4), &p))) return rc;
+        alo = (float *)p;
+        if ((rc = ensure_buf(w, BUF_BHI, (size_t)(cols * Kp * 4), &p))) return rc;
+        bhi = (float *)p;
+        if ((rc = ensure_buf(w, BUF_BLO, (size_t)(cols * Kp * 4), &p))) return rc;
+        blo = (float *)p;
+    }
+    pdlk::EncodeTiledFn enc = nullptr;
+    if (K > 0 && (rc = get_encoder(&enc))) return rc;
+    const char *k2v = getenv("PDL_K2");
+    const bool k2_1sm = k2v && !strcmp(k2v, "1sm");
+
+    std::vector<cudaEvent_t> ev_a(RB, nullptr), ev_b(CP, nullptr), ev_sa(RB, nullptr), ev_sb(CP, nullptr);
+    cudaEvent_t ev_last_out = nullptr, ev_last_cmp1 = nullptr;
+    int launch_idx = 0;
+    for (int i = 0; i < RB; ++i) {
+        const int64_t r0 = rb[i], nr = rb[i + 1] - rb[i];
+        if (nr <= 0) continue;
+        if (a_st) {
+            cudaError_t e = cudaMemcpy2DAsync(const_cast<char *>(Ad) + (size_t)(r0 * lda) * es, (size_t)(lda * es),
+                                              (const char *)A + (size_t)(r0 * t.lda) * es, (size_t)(t.lda * es),
+                                              (size_t)(K * es), (size_t)nr, cudaMemcpyDefault, s_in);
+            if (e != cudaSuccess) return set_err(PDL_ECUDA, "A staging copy failed: %s", cudaGetErrorString(e));
+            if (piped) {
+                ev_a[i] = ev_get(w, evn);
+                CUDA_TRY(cudaEventRecord(ev_a[i], s_in));
+            }
+        }
+        for (int j = 0; j < CP; ++j) {
+            const int64_t c0 = cp[j], nc = cp[j + 1] - cp[j];
+            if (nc <= 0) continue;
+            if (i == 0 && b_st) {
+                cudaError_t e = cudaMemcpy2DAsync(const_cast<char *>(Bd) + (size_t)c0 * es, (size_t)(ldb * es),
+                                                  (const char *)B + (size_t)c0 * es, (size_t)(t.ldb * es),
+                                                  (size_t)(nc * es), (size_t)K, cudaMemcpyDefault, s_in);
+                if (e != cudaSuccess) return set_err(PDL_ECUDA, "B staging copy failed: %s", cudaGetErrorString(e));
+                if (piped) {
+                    ev_b[j] = ev_get(w, evn);
+                    CUDA_TRY(cudaEventRecord(ev_b[j], s_in));
+                }
+            }
+            cudaStream_t cs = s_cmp[launch_idx & 1];
+            if (piped) {
+                if (ev_a[i]) CUDA_TRY(cudaStreamWaitEvent(cs, ev_a[i], 0));
+                if (ev_b[j]) CUDA_TRY(cudaStreamWaitEvent(cs, ev_b[j], 0));
+            }
+            char *Cs = Cd + (size_t)(r0 * ldcd + c0) * es;
+            cudaError_t e = cudaSuccess;
+            if (K == 0) {
+                e = cudaMemset2DAsync(Cs, (size_t)(ldcd * es), 0, (size_t)(nc * es), (size_t)nr, cs);
+            } else if (f64) {
+                if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
+                e = pdlk::launch_dgemm_k1(enc, (const double *)(Ad + (size_t)(r0 * lda) * es), lda,
+                                          (const double *)(Bd + (size_t)c0 * es), ldb, (double *)Cs, ldcd, nr, nc, K,
+                                          cs);
+                if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
+                w.launches += 1;
+            } else {
+                // K3 split of this band / panel once, shared by both compute streams
+                if (j == 0) {
+                    e = pdlk::launch_split_rows((const float *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K,
+                                                ahi + r0 * Kp, alo + r0 * Kp, Kp, cs);
+                    w.launches += 1;
+                    if (piped) {
+                        ev_sa[i] = ev_get(w, evn);
+                        CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
+                    }
+                } else if (ev_sa[i]) {
+                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
+                }
+                if (e == cudaSuccess && i == 0) {
+                    e = pdlk::launch_split_cols_t((const float *)(Bd + (size_t)c0 * es), ldb, K, nc, bhi + c0 * Kp,
+                                                  blo + c0 * Kp, Kp, cs);
+                    w.launches += 1;
+                    if (piped) {
+                        ev_sb[j] = ev_get(w, evn);
+                        CUDA_TRY(cudaEventRecord(ev_sb[j], cs));
+                    }
+                } else if (ev_sb[j]) {
+                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sb[j], 0));
+                }
+                if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
+                if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
+                if (k2_1sm)
+                    e = pdlk::launch_gemm_3xtf32(enc, ahi + r0 * Kp, alo + r0 * Kp, bhi + c0 * Kp, blo + c0 * Kp, Kp,
+                                                 (float *)Cs, ldcd, nr, nc, cs);
+                else
+                    e = pdlk::launch_gemm_3xtf32_2sm(enc, ahi + r0 * Kp, alo + r0 * Kp, bhi + c0 * Kp, blo + c0 * Kp,
+                                                     Kp, (float *)Cs, ldcd, nr, nc, cs);
+                if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
+                w.launches += 1;
+            }
+            if (e != cudaSuccess) return set_err(PDL_ECUDA, "tile kernel launch failed: %s", cudaGetErrorString(e));
+            w.timed = true;
+            if (piped && (launch_idx & 1)) {
+                ev_last_cmp1 = ev_get(w, evn);
+                CUDA_TRY(cudaEventRecord(ev_last_cmp1, cs));
+            }
+            if (c_st) {
+                if (piped) {
+                    cudaEvent_t ek = ev_get(w, evn);
+                    CUDA_TRY(cudaEventRecord(ek, cs));
+                    CUDA_TRY(cudaStreamWaitEvent(s_out, ek, 0));
+                }
+                e = cudaMemcpy2DAsync((char *)C + (size_t)(r0 * t.ldc + c0) * es, (size_t)(t.ldc * es), Cs,
+                                      (size_t)(ldcd * es), (size_t)(nc * es), (size_t)nr, cudaMemcpyDefault, s_out);
+                if (e != cudaSuccess) return set_err(PDL_ECUDA, "result gather copy failed: %s", cudaGetErrorString(e));
+            }
+            ++launch_idx;
+        }
+    }
+    if (piped) {
+        // join: the Worker stream completes after every side stream's work
+        ev_last_out = ev_get(w, evn);
+        CUDA_TRY(cudaEventRecord(ev_last_out, s_out));
+        CUDA_TRY(cudaStreamWaitEvent(w.stream, ev_last_out, 0));
+        if (ev_last_cmp1) CUDA_TRY(cudaStreamWaitEvent(w.stream, ev_last_cmp1, 0));
+        cudaEvent_t ein = ev_get(w, evn);
+        CUDA_TRY(cudaEventRecord(ein, s_in));
+        CUDA_TRY(cudaStreamWaitEvent(w.stream, ein, 0));
     }
     return PDL_OK;
 }
