@@ -117,14 +117,27 @@ def exchange(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers):
     """All-gather the operand chunks: afterwards bufs.A[:rows] is the A
     row-panel (rows x K) and bufs.B[:K] the B column-panel (K x cols)."""
     if wp.Gc > 1:
-        dist.all_gather_into_tensor(bufs.A, Ach.contiguous(), group=grid.row_group)
+        _all_gather(bufs.A, Ach, grid.row_group)
     else:
         bufs.A.copy_(Ach)
     if wp.Gr > 1:
-        dist.all_gather_into_tensor(bufs.B, Bch.contiguous(), group=grid.col_group)
+        _all_gather(bufs.B, Bch, grid.col_group)
     else:
         bufs.B.copy_(Bch)
     return bufs.A[: wp.rows], bufs.B[: wp.K]
+
+
+def _all_gather(out, chunk, group):
+    """NCCL all-gather into a contiguous buffer.  Under the gloo backend
+    (CPU tests; several ranks sharing one GPU in the 1-GPU validation run)
+    device tensors are staged through host memory, since gloo gathers host
+    tensors only."""
+    if out.is_cuda and dist.get_backend(group) == "gloo":
+        tmp = torch.empty(out.shape, dtype=out.dtype)
+        dist.all_gather_into_tensor(tmp, chunk.contiguous().cpu(), group=group)
+        out.copy_(tmp)
+    else:
+        dist.all_gather_into_tensor(out, chunk.contiguous(), group=group)
 
 
 def local_task(Apanel, Bpanel, Cblock, wp: WorkerPlan, tile=0, run=True):
