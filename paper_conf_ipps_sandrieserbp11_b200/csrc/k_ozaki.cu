@@ -1,0 +1,377 @@
+// k_ozaki.cu -- K4/K5: an FP64 DGEMM task variant on the INT8 tensor cores
+// (Ozaki scheme I), SURVEY.md SS8(f) NEXT-1.
+//
+// The paper's task model keeps one task interface with several implementation
+// variants, chosen from the platform description (task
+// repository and static pre-selection L1307-1326).  This file is the second
+// variant of the DGEMM task (the first is K1, FP64 DMMA); the runtime picks it
+// when the Worker's PDL property DGEMM_VARIANT is "ozaki" (K4).
+//
+// Method (error-free splitting into integer slices; Ozaki, Ogita, Oishi,
+// Rump 2012; here with 7-bit signed slices and exact INT32 accumulation):
+//   row scale   a_ik = 2^{e_i} a'_ik, |a'_ik| < 1      (e_i from frexp(max_k |a_ik|))
+//   col scale   b_kj = 2^{f_j} b'_kj, |b'_kj| < 1
+//   slices      a' = sum_{s<S} 2^{-7(s+1)} A_s,  A_s in [-127,127]  (truncation; exact FP64 ops)
+//   product     C_ij ~= 2^{e_i+f_j} sum_{d<S} 2^{-7(d+2)} [ sum_{s+t=d} A_s B_t ]_ij
+// Each diagonal d is ONE int8 GEMM with K' = (d+1) K: the slices are stored
+// concatenated along K ([A_0|A_1|...] and, for B^T, in reverse order
+// [...|B_1|B_0]), so [A_0..A_d] . [B_d..B_0]^T is a contiguous K' window of
+// both.  |sum| <= (d+1) K 127^2 < 2^31 for K chunks <= 16384 (S <= 8), so the
+// INT32 TMEM accumulation is exact; the epilogue scales by the exact power of
+// two and accumulates the S diagonals into the FP64 C (smallest first).
+// Representation error: |a - sum| < 2^{e_i - 7S}; with S = 7 the scaled error
+// versus D = |A||B| is <= ~2^-45 for data whose rows / columns do not span a
+// wide dynamic range (R19).  Inputs must be finite.
+//
+// GEMM kernel: the K2 v3 CTA-pair structure with tcgen05.mma.cta_group::2
+// .kind::i8 (M = 256, N = 256, K = 32 per instruction), 6-stage TMA ring of
+// 128-byte K blocks, INT32 accumulator in TMEM (256 columns), 16 epilogue
+// warps converting TMEM -> FP64 and read-modify-writing C.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdint>
+
+#include "kernels.h"
+#include "ptx.cuh"
+#include "tcgen05.cuh"
+
+namespace pdlk {
+
+// ------------------------------------------------------------------------
+// K5: slicing pre-pass
+// ------------------------------------------------------------------------
+
+// frexp exponent of a non-negative finite max: max < 2^e (0 -> 0).
+__device__ __forceinline__ int exp_of_max(double mx) {
+    if (!(mx > 0.0)) return 0;
+    int e;
+    frexp(mx, &e);
+    return e;
+}
+
+// Write S truncated 7-bit slices of v (|v| < 1).
+template <typename F>
+__device__ __forceinline__ void slice7(double v, int S, F &&store) {
+    for (int s = 0; s < S; ++s) {
+        v *= 128.0;
+        const double q = trunc(v);
+        v -= q;
+        store(s, (int8_t)(int)q);
+    }
+}
+
+// One CTA per row (grid-stride): A (M x K, lda) -> A8 rows [c][s][kk].
+__global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M, int64_t K, int S,
+                                     int64_t Kc, int nch, int8_t *__restrict__ A8, int64_t ld8,
+                                     int *__restrict__ ea) {
+    __shared__ double red[32];
+    const int64_t Kpad = (int64_t)nch * Kc;
+    for (int64_t i = blockIdx.x; i < M; i += gridDim.x) {
+        const double *row = A + i * lda;
+        double mx = 0.0;
+        for (int64_t k = threadIdx.x; k < K; k += blockDim.x) mx = fmax(mx, fabs(row[k]));
+        for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = mx;
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            mx = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : 0.0;
+            for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+            if (threadIdx.x == 0) red[0] = mx;
+        }
+        __syncthreads();
+        const int e = exp_of_max(red[0]);
+        if (threadIdx.x == 0) ea[i] = e;
+        int8_t *out = A8 + i * ld8;
+        for (int64_t k = threadIdx.x; k < Kpad; k += blockDim.x) {
+            const double v = k < K ? ldexp(row[k], -e) : 0.0;
+            const int64_t c = k / Kc, kk = k - c * Kc;
+            int8_t *o = out + (c * S) * Kc + kk;
+            slice7(v, S, [&](int s, int8_t q) { o[(int64_t)s * Kc] = q; });
+        }
+        __syncthreads();
+    }
+}
+
+// Column max |b| of B (K x N): bits of the non-negative max via atomicMax.
+__global__ void oz_colmax_kernel(const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
+                                 unsigned long long *__restrict__ bmax) {
+    const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (n >= N) return;
+    const int64_t k0 = (int64_t)blockIdx.y * 256, k1 = min(K, k0 + 256);
+    double mx = 0.0;
+    for (int64_t k = k0; k < k1; ++k) mx = fmax(mx, fabs(B[k * ldb + n]));
+    atomicMax(bmax + n, (unsigned long long)__double_as_longlong(mx));
+}
+
+// B (K x N) -> Bt8 (N rows of [c][S-1-s][kk]) through a 32 x 32 smem transpose.
+__global__ void oz_split_cols_t_kernel(const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S,
+                                       int64_t Kc, int nch, const unsigned long long *__restrict__ bmax,
+                                       int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb) {
+    __shared__ double t[32][33];
+    const int64_t k0 = (int64_t)blockIdx.y * 32, n0 = (int64_t)blockIdx.x * 32;
+    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
+        const int64_t k = k0 + r, n = n0 + threadIdx.x;
+        t[r][threadIdx.x] = (k < K && n < N) ? B[k * ldb + n] : 0.0;
+    }
+    __syncthreads();
+    const int64_t Kpad = (int64_t)nch * Kc;
+    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
+        const int64_t n = n0 + r, k = k0 + threadIdx.x;
+        if (n >= N || k >= Kpad) continue;
+        const int f = exp_of_max(__longlong_as_double((long long)bmax[n]));
+        if (blockIdx.y == 0 && threadIdx.x == 0) fb[n] = f;
+        const double v = ldexp(t[threadIdx.x][r], -f);
+        const int64_t c = k / Kc, kk = k - c * Kc;
+        int8_t *o = Bt8 + n * ld8 + (c * S) * Kc + kk;
+        slice7(v, S, [&](int s, int8_t q) { o[(int64_t)(S - 1 - s) * Kc] = q; });
+    }
+}
+
+// ------------------------------------------------------------------------
+// K4: int8 CTA-pair GEMM of one diagonal, FP64 epilogue
+// ------------------------------------------------------------------------
+namespace koz {
+constexpr int BM = 128, BN = 256, BNH = 128;
+constexpr int BK = 128, STAGES = 6, UMMA_K = 32;
+constexpr int A_BYTES = BM * BK;        // 16 KiB
+constexpr int B_BYTES = BNH * BK;       // 16 KiB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int EPI_WARPS = 16, EPI_COLS = 64, FIRST_EPI_WARP = 2;
+constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
+constexpr int TMEM_COLS = 256;
+constexpr int GROUP_M = 8;
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+}  // namespace koz
+
+__host__ __device__ constexpr uint32_t idesc_i8(int M, int N) {
+    return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ void umma_i8_2sm(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                            uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::i8 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
+    oz_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
+                       double *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
+                       const int *__restrict__ fb, int scale_exp, int accumulate, int tiles_m, int tiles_n,
+                       int vec_ok) {
+    using namespace koz;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
+    const uint32_t bar_full = base + STAGES * STAGE_BYTES;
+    const uint32_t bar_empty = bar_full + STAGES * 8;
+    const uint32_t bar_tfull = bar_empty + STAGES * 8;
+    const uint32_t tmem_slot = bar_tfull + 8;
+    uint8_t *const gbase = smem_raw + (base - smem_u32(smem_raw));
+    volatile uint32_t *tmem_slot_ptr = reinterpret_cast<volatile uint32_t *>(gbase + (tmem_slot - base));
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = cluster_ctarank();
+    const int cid = blockIdx.x >> 1;
+    const int per_group = GROUP_M * tiles_n;
+    const int g = cid / per_group;
+    const int first_m = g * GROUP_M;
+    const int gsz = min(tiles_m - first_m, GROUP_M);
+    const int tm = first_m + (cid % per_group) % gsz;
+    const int tn = (cid % per_group) / gsz;
+    const int m0 = tm * (2 * BM) + (int)rank * BM;
+    const int nb0 = tn * BN + (int)rank * BNH;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(bar_full + 8 * s, 1);
+            mbar_init(bar_empty + 8 * s, 1);
+        }
+        mbar_init(bar_tfull, 1);
+        fence_barrier_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(tmem_slot),
+                     "n"(TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    cluster_sync_all();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem_base = *tmem_slot_ptr;
+    const int nk = Kd / BK;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            tma_prefetch_desc(&tA);
+            tma_prefetch_desc(&tB);
+            for (int kb = 0; kb < nk; ++kb) {
+                const int s = kb % STAGES;
+                const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+                mbar_wait(bar_empty + 8 * s, ph ^ 1u);
+                const uint32_t fb_leader = mapa_shared(bar_full + 8 * s, 0);
+                if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * STAGE_BYTES);
+                const uint32_t st = base + s * STAGE_BYTES;
+                tma_load_2d_2sm(st, &tA, fb_leader, kb * BK, m0);
+                tma_load_2d_2sm(st + A_BYTES, &tB, fb_leader, kb * BK, nb0);
+            }
+        }
+    } else if (warp == 1) {
+        if (rank == 0 && lane == 0) {
+            constexpr uint32_t idesc = idesc_i8(2 * BM, BN);
+            for (int kb = 0; kb < nk; ++kb) {
+                const int s = kb % STAGES;
+                const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
+                mbar_wait(bar_full + 8 * s, ph);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                const uint32_t st = base + s * STAGE_BYTES;
+#pragma unroll
+                for (int kk = 0; kk < BK / UMMA_K; ++kk) {
+                    const uint32_t off = kk * UMMA_K;   // 32 bytes of K per instruction
+                    umma_i8_2sm(tmem_base, umma_desc_k_sw128(st + off), umma_desc_k_sw128(st + A_BYTES + off), idesc,
+                                (kb | kk) ? 1u : 0u);
+                }
+                umma_commit_2sm(bar_empty + 8 * s);
+            }
+            umma_commit_2sm(bar_tfull);
+        }
+        __syncwarp();
+    } else {
+        const int e = warp - FIRST_EPI_WARP;
+        const int q = warp & 3;
+        const int cg = e >> 2;
+        const uint32_t tl = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(cg * EPI_COLS);
+        mbar_wait(bar_tfull, 0);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
+        const int cbase = tn * BN + cg * EPI_COLS;
+        const int er = row < M ? ea[row] + scale_exp : 0;
+        double *crow = C + (int64_t)row * ldc + cbase;
+#pragma unroll
+        for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
+            uint32_t r[16];
+            tmem_ld16(tl + c0, r);
+            if (row < M) {
+                double v[16];
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    const int col = cbase + c0 + j;
+                    const int f = col < N ? fb[col] : 0;
+                    v[j] = ldexp((double)(int32_t)r[j], er + f);   // exact: int32 -> f64, power-of-two scale
+                }
+                if (vec_ok && cbase + c0 + 16 <= N) {
+#pragma unroll
+                    for (int j = 0; j < 16; j += 2) {
+                        double2 *p = reinterpret_cast<double2 *>(crow + c0 + j);
+                        double2 o = accumulate ? *p : make_double2(0.0, 0.0);
+                        *p = make_double2(o.x + v[j], o.y + v[j + 1]);
+                    }
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 16; ++j)
+                        if (cbase + c0 + j < N) crow[c0 + j] = (accumulate ? crow[c0 + j] : 0.0) + v[j];
+                }
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    cluster_sync_all();
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(TMEM_COLS));
+    }
+}
+
+// ------------------------------------------------------------------------
+// host side
+// ------------------------------------------------------------------------
+OzakiLayout ozaki_layout(int64_t rows, int64_t cols, int64_t K, int S) {
+    OzakiLayout L;
+    L.S = S;
+    L.nch = (int)((K + OZ_KC_MAX - 1) / OZ_KC_MAX);
+    if (L.nch < 1) L.nch = 1;
+    const int64_t per = (K + L.nch - 1) / L.nch;
+    L.Kc = ((per + koz::BK - 1) / koz::BK) * koz::BK;
+    L.ld8 = (int64_t)L.nch * S * L.Kc;
+    L.a8_bytes = (size_t)rows * L.ld8;
+    L.b8_bytes = (size_t)cols * L.ld8;
+    return L;
+}
+
+cudaError_t launch_ozaki_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
+                                 int8_t *A8, int *ea, cudaStream_t s) {
+    if (rows <= 0) return cudaSuccess;
+    int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
+    oz_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, L.S, L.Kc, L.nch, A8, L.ld8, ea);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
+                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s) {
+    if (cols <= 0) return cudaSuccess;
+    cudaError_t e = cudaMemsetAsync(bmax, 0, (size_t)cols * sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+    if (K > 0) {
+        dim3 g1((unsigned)((cols + 255) / 256), (unsigned)((K + 255) / 256));
+        oz_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
+    }
+    const int64_t Kpad = (int64_t)L.nch * L.Kc;
+    dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 31) / 32));
+    oz_split_cols_t_kernel<<<g2, dim3(32, 8), 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb);
+    return cudaGetLastError();
+}
+
+static bool map_i8(EncodeTiledFn enc, CUtensorMap *m, const int8_t *ptr, uint64_t kd, uint64_t rows, uint64_t ld,
+                   uint32_t box_rows) {
+    cuuint64_t dims[2] = {kd, rows};
+    cuuint64_t strides[1] = {ld};
+    cuuint32_t box[2] = {(cuuint32_t)koz::BK, box_rows};
+    cuuint32_t es[2] = {1, 1};
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<int8_t *>(ptr), dims, strides, box, es,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// All diagonals and K chunks of one rectangle: S * nch int8 GEMM launches,
+// smallest diagonal first; the first launch overwrites C.
+cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
+                              const OzakiLayout &L, double *C, int64_t ldc, int64_t rows, int64_t cols,
+                              cudaStream_t stream, int *launches) {
+    using namespace koz;
+    if (rows <= 0 || cols <= 0) return cudaSuccess;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static bool attr_done[64] = {false};
+    if (dev < 64 && !attr_done[dev]) {
+        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+        if (e != cudaSuccess) return e;
+        attr_done[dev] = true;
+    }
+    const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + BN - 1) / BN);
+    const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
+    int first = 1;
+    for (int c = 0; c < L.nch; ++c) {
+        for (int d = L.S - 1; d >= 0; --d) {
+            const int64_t kd = (int64_t)(d + 1) * L.Kc;
+            const int8_t *a = A8 + (int64_t)c * L.S * L.Kc;
+            const int8_t *b = Bt8 + ((int64_t)c * L.S + (L.S - 1 - d)) * L.Kc;
+            CUtensorMap ta, tb;
+            if (!map_i8(enc, &ta, a, (uint64_t)kd, (uint64_t)rows, (uint64_t)L.ld8, BM) ||
+                !map_i8(enc, &tb, b, (uint64_t)kd, (uint64_t)cols, (uint64_t)L.ld8, BNH))
+                return cudaErrorInvalidValue;
+            oz_gemm_2sm_kernel<<<2 * tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(
+                ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m, tiles_n,
+                vec_ok);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return e;
+            first = 0;
+            if (launches) ++*launches;
+        }
+    }
+    return cudaSuccess;
+}
+
+}  // namespace pdlk

@@ -34,6 +34,25 @@ cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t 
 cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
                                cudaStream_t stream);
+// K4/K5 -- FP64 DGEMM variant on INT8 tensor cores (Ozaki scheme, k_ozaki.cu).
+// Slices: A8 = rows x ld8 int8, row layout [chunk][slice][Kc]; Bt8 = cols x ld8
+// int8, row layout [chunk][S-1-slice][Kc]; ea/fb = per-row / per-column
+// power-of-two exponents; bmax = cols x u64 scratch.
+constexpr int64_t OZ_KC_MAX = 16384;   // (d+1)*Kc*127^2 < 2^31 for S <= 8
+struct OzakiLayout {
+    int S = 7, nch = 1;
+    int64_t Kc = 0, ld8 = 0;
+    size_t a8_bytes = 0, b8_bytes = 0;
+};
+OzakiLayout ozaki_layout(int64_t rows, int64_t cols, int64_t K, int S);
+cudaError_t launch_ozaki_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
+                                 int8_t *A8, int *ea, cudaStream_t s);
+cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
+                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s);
+cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
+                              const OzakiLayout &L, double *C, int64_t ldc, int64_t rows, int64_t cols,
+                              cudaStream_t stream, int *launches);
+
 // K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                    const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,

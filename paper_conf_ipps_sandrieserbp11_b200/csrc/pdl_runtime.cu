@@ -71,7 +71,7 @@ struct DevBuf {
     size_t bytes = 0;
 };
 
-enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_COUNT };
+enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_OZA, BUF_OZB, BUF_OZE, BUF_COUNT };
 
 struct WorkerCtx {
     int pu = -1;         // PU instance index in the model
@@ -382,6 +382,21 @@ int ensure_aux(WorkerCtx &w) {
     return PDL_OK;
 }
 
+// FP64 task variant of a Worker: PDL property DGEMM_VARIANT ("dmma" default |
+// "ozaki") and OZAKI_SLICES (2..8, default 7); env PDL_DGEMM_VARIANT /
+// PDL_OZAKI_SLICES override the descriptor (tests, bench).
+bool worker_ozaki(const WorkerCtx &w, int *slices) {
+    std::string v;
+    if (const char *e = getenv("PDL_DGEMM_VARIANT")) v = e;
+    else if (const Property *p = g->model.prop(w.pu, "DGEMM_VARIANT")) v = p->value;
+    if (lower(trim(v)) != "ozaki") return false;
+    int s = 7;
+    if (const char *e = getenv("PDL_OZAKI_SLICES")) s = atoi(e);
+    else if (const Property *p = g->model.prop(w.pu, "OZAKI_SLICES")) s = atoi(p->value.c_str());
+    *slices = std::max(2, std::min(8, s));
+    return true;
+}
+
 int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
     if (rows <= 0 || cols <= 0) return PDL_OK;
     CUDA_TRY(cudaSetDevice(w.device));
@@ -466,6 +481,27 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     const char *k2v = getenv("PDL_K2");
     const bool k2_1sm = k2v && !strcmp(k2v, "1sm");
 
+    // DGEMM task variant of this Worker, pre-selected from its PDL properties
+    // (task repository + static pre-selection, L1307-1326): K1 (DMMA) or K4 (Ozaki).
+    int oz_slices = 0;
+    const bool ozaki = f64 && K > 0 && worker_ozaki(w, &oz_slices);
+    pdlk::OzakiLayout OL;
+    int8_t *a8 = nullptr, *b8 = nullptr;
+    int *oz_ea = nullptr, *oz_fb = nullptr;
+    unsigned long long *oz_bmax = nullptr;
+    if (ozaki) {
+        OL = pdlk::ozaki_layout(rows, cols, K, oz_slices);
+        if ((rc = ensure_buf(w, BUF_OZA, OL.a8_bytes, &p))) return rc;
+        a8 = (int8_t *)p;
+        if ((rc = ensure_buf(w, BUF_OZB, OL.b8_bytes, &p))) return rc;
+        b8 = (int8_t *)p;
+        const size_t eb = (size_t)round_up(rows, 2) * 4 + (size_t)round_up(cols, 2) * 4 + (size_t)cols * 8;
+        if ((rc = ensure_buf(w, BUF_OZE, eb, &p))) return rc;
+        oz_bmax = (unsigned long long *)p;
+        oz_ea = (int *)(oz_bmax + cols);
+        oz_fb = oz_ea + round_up(rows, 2);
+    }
+
     std::vector<cudaEvent_t> ev_a(RB, nullptr), ev_b(CP, nullptr), ev_sa(RB, nullptr), ev_sb(CP, nullptr);
     cudaEvent_t ev_last_out = nullptr, ev_last_cmp1 = nullptr;
     int launch_idx = 0;
@@ -504,6 +540,37 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             cudaError_t e = cudaSuccess;
             if (K == 0) {
                 e = cudaMemset2DAsync(Cs, (size_t)(ldcd * es), 0, (size_t)(nc * es), (size_t)nr, cs);
+            } else if (ozaki) {
+                // K5 slicing of this band / panel once, shared by both compute streams
+                if (j == 0) {
+                    e = pdlk::launch_ozaki_split_a((const double *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K, OL,
+                                                   a8 + r0 * OL.ld8, oz_ea + r0, cs);
+                    w.launches += 1;
+                    if (piped) {
+                        ev_sa[i] = ev_get(w, evn);
+                        CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
+                    }
+                } else if (ev_sa[i]) {
+                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
+                }
+                if (e == cudaSuccess && i == 0) {
+                    e = pdlk::launch_ozaki_split_b((const double *)(Bd + (size_t)c0 * es), ldb, K, nc, OL,
+                                                   b8 + c0 * OL.ld8, oz_fb + c0, oz_bmax + c0, cs);
+                    w.launches += 2;
+                    if (piped) {
+                        ev_sb[j] = ev_get(w, evn);
+                        CUDA_TRY(cudaEventRecord(ev_sb[j], cs));
+                    }
+                } else if (ev_sb[j]) {
+                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sb[j], 0));
+                }
+                if (e != cudaSuccess) return set_err(PDL_ECUDA, "K5 slicing launch failed: %s", cudaGetErrorString(e));
+                if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
+                int nl = 0;
+                e = pdlk::launch_ozaki_gemm(enc, a8 + r0 * OL.ld8, b8 + c0 * OL.ld8, oz_ea + r0, oz_fb + c0, OL,
+                                            (double *)Cs, ldcd, nr, nc, cs, &nl);
+                if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
+                w.launches += nl;
             } else if (f64) {
                 if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
                 e = pdlk::launch_dgemm_k1(enc, (const double *)(Ad + (size_t)(r0 * lda) * es), lda,
