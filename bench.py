@@ -49,6 +49,7 @@ FP64_DMMA_PEAK_TFLOPS = 37.0
 # tcgen05 kind::tf32 issue rate (M=256 N=256 cta_group::2 and M=128 N=256
 # cta_group::1, 148 SMs, no memory traffic): profiles/r01_tc_microbench.json.
 TF32_TCGEN05_PEAK_TFLOPS = 1107.0
+INT8_TCGEN05_PEAK_TOPS = 4571.0
 
 
 def parse():
@@ -64,6 +65,9 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cublas", action="store_true")
+    p.add_argument("--variant", choices=("dmma", "ozaki"), default="dmma",
+                   help="FP64 DGEMM task variant (PDL DGEMM_VARIANT): K1 DMMA or K4 Ozaki INT8")
+    p.add_argument("--slices", type=int, default=7, help="OZAKI_SLICES for --variant ozaki")
     p.add_argument("--dist-backend", choices=("nccl", "gloo"), default="nccl",
                    help="gloo only to validate the N>1 flow with ranks sharing one GPU")
     return p.parse_args()
@@ -88,6 +92,10 @@ def tensor_peak(dtype):
     the conservative denominator.
     """
     pk, src = peaks()
+    if dtype == "i8":
+        return INT8_TCGEN05_PEAK_TOPS, ("INT8 tcgen05 issue rate measured (tools/tc_microbench; "
+                                        "profiles/r01_tc_microbench.json)"), \
+            {"peak": round(pk["bf16_tflops"] * 2, 1), "source": f"{src} bf16 burst x nominal 4.5/2.25"}
     if dtype == "f64":
         return FP64_DMMA_PEAK_TFLOPS, "FP64 DMMA.8x8x4 issue rate measured (tools/microbench; profiles/r01_microbench.json)", None
     alt = pk["bf16_tflops"] * 1.1 / 2.25
@@ -262,10 +270,14 @@ def main():
     es = 8 if args.dtype == "f64" else 4
     A, B = host_inputs(args.config, np_dtype)
 
+    ozaki = args.dtype == "f64" and args.variant == "ozaki"
+    # the DGEMM task variant is pre-selected through the Worker's PDL properties (L1316-1326)
+    desc = pdl.descriptor_xml(world, args.variant if args.dtype == "f64" else None,
+                              args.slices if ozaki else None)
     if world == 1:
-        pdl.load(pdl.descriptor_path(1))
+        pdl.load(desc)
     else:
-        pdl.load(pdl.descriptor_path(world), rank=rank, nranks=world)
+        pdl.load(desc, rank=rank, nranks=world)
     stream = torch.cuda.current_stream()
     pdl.set_stream(stream)
 
@@ -328,14 +340,22 @@ def main():
 
     # ---- roofline of the dominant kernel (K1, or K2 for FP32) ----
     kavg = float(np.mean(ktimes)) if ktimes else None
-    peak_tf, peak_src, peak_alt = tensor_peak(args.dtype)
-    pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
+    peak_tf, peak_src, peak_alt = tensor_peak("i8" if ozaki else args.dtype)
+    if ozaki:
+        # int8 tensor ops of the S slice diagonals: sum_d 2*rows*cols*(d+1)*Kc per K chunk
+        nch = max(1, -(-K // 16384))
+        kc = -(-(-(-K // nch)) // 128) * 128
+        pipe_flops = 2.0 * wp.rows * wp.cols * kc * nch * args.slices * (args.slices + 1) / 2
+        kname = f"K4 oz_gemm_2sm_kernel x {args.slices * nch} slice-diagonal launches (tcgen05 kind::i8)"
+    else:
+        pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
+        kname = "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_2sm_kernel (tcgen05)"
     achieved_tf = pipe_flops / (kavg / 1e3) / 1e12 if kavg else None
     roofline = {"bound": "tensor", "achieved": round(achieved_tf, 2) if achieved_tf else None,
                 "peak": round(peak_tf, 1), "unit": "TFLOP/s",
                 "frac": round(achieved_tf / peak_tf, 4) if achieved_tf else None,
-                "traffic": ncu_traffic(args.dtype, args.config),
-                "kernel": "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_kernel (tcgen05)",
+                "traffic": ncu_traffic("ozaki" if ozaki else args.dtype, args.config),
+                "kernel": kname,
                 "kernel_ms": round(kavg, 3) if kavg else None,
                 "algorithmic_flops_per_launch": pipe_flops,
                 "peak_source": peak_src}
@@ -343,6 +363,9 @@ def main():
         roofline["peak_alt"] = peak_alt
     if args.dtype == "f32":
         roofline["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
+    if ozaki:
+        roofline["note"] = ("achieved counts int8 tensor ops (S(S+1)/2 slice products, 2 ops per MAC); "
+                            "useful FP64 FLOP = 2MNK")
 
     # ---- e2e: host pinned operands through the public API ----
     e2e = None
@@ -423,13 +446,16 @@ def main():
         line = {
             "metric": METRIC, "value": round(value, 1), "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": f"f64-ozaki-i8x{args.slices}" if ozaki else args.dtype,
             "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} ({args.dtype})",
             "config": {"workload": f"{args.config} {M}x{N}x{K} blocked matmul, task tile {c.tile}, "
                                    f"PDL b200_x{world}",
                        "M": M, "N": N, "K": K, "tile": c.tile, "parallelism": f"block2d {wp.Gr}x{wp.Gc}",
+                       "task_variant": (f"ozaki (K4/K5, {args.slices} int8 slices)" if ozaki else
+                                        ("dmma (K1)" if args.dtype == "f64" else "3xtf32 (K3+K2)")),
                        "l2": "inputs larger than L2 (operands >> 126 MB), no flush needed"},
-            "pct_of_tensor_peak": round(100 * value / world / (peak_tf * 1e3) * (3 if args.dtype == "f32" else 1), 2),
+            "pct_of_tensor_peak": round(100 * (pipe_flops / flops_worker) * value / world / (peak_tf * 1e3), 2),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": int(launches_per_step * args.steps),
             "clocks": clocks,
