@@ -68,6 +68,7 @@ def parse():
     p.add_argument("--variant", choices=("dmma", "ozaki"), default="dmma",
                    help="FP64 DGEMM task variant (PDL DGEMM_VARIANT): K1 DMMA or K4 Ozaki INT8")
     p.add_argument("--slices", type=int, default=7, help="OZAKI_SLICES for --variant ozaki")
+    p.add_argument("--no-alt", action="store_true", help="skip timing the other FP64 variant")
     p.add_argument("--dist-backend", choices=("nccl", "gloo"), default="nccl",
                    help="gloo only to validate the N>1 flow with ranks sharing one GPU")
     return p.parse_args()
@@ -168,6 +169,15 @@ def ncu_traffic(dtype, cfg):
         return d.get(f"{dtype}/{cfg}")
     except (OSError, ValueError):
         return None
+
+
+def ozaki_ops(rows, cols, K, S):
+    """INT8 tensor ops of the Ozaki variant: S slice diagonals, diagonal d is a
+    GEMM with K' = (d+1) Kc per K chunk (k_ozaki.cu)."""
+    nch = max(1, -(-K // 16384))
+    kc = -(-(-(-K // nch)) // 128) * 128
+    ops = 2.0 * rows * cols * kc * nch * S * (S + 1) / 2
+    return ops, f"K4 oz_gemm_2sm_kernel x {S * nch} slice-diagonal launches (tcgen05 kind::i8)"
 
 
 def host_inputs(cfg, np_dtype):
@@ -342,11 +352,7 @@ def main():
     kavg = float(np.mean(ktimes)) if ktimes else None
     peak_tf, peak_src, peak_alt = tensor_peak("i8" if ozaki else args.dtype)
     if ozaki:
-        # int8 tensor ops of the S slice diagonals: sum_d 2*rows*cols*(d+1)*Kc per K chunk
-        nch = max(1, -(-K // 16384))
-        kc = -(-(-(-K // nch)) // 128) * 128
-        pipe_flops = 2.0 * wp.rows * wp.cols * kc * nch * args.slices * (args.slices + 1) / 2
-        kname = f"K4 oz_gemm_2sm_kernel x {args.slices * nch} slice-diagonal launches (tcgen05 kind::i8)"
+        pipe_flops, kname = ozaki_ops(wp.rows, wp.cols, K, args.slices)
     else:
         pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
         kname = "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_2sm_kernel (tcgen05)"
@@ -438,6 +444,42 @@ def main():
         torch.cuda.synchronize()
         cublas = round(flops_total * 3 / (t0.elapsed_time(t1) / 1e3) / 1e9, 1)
 
+    # ---- the other FP64 task variant on the same resident operands (PDL-selected) ----
+    alt = None
+    if world == 1 and args.dtype == "f64" and args.variant == "dmma" and not args.no_alt:
+        pdl.unload()
+        pdl.load(pdl.descriptor_xml(1, "ozaki", args.slices))
+        pdl.set_stream(stream)
+        for _ in range(2):
+            step()
+        pdl.sync()
+        torch.cuda.synchronize()
+        pdl.kernel_times()
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        with ClockSampler(local) as clk2:
+            t0.record(stream)
+            for _ in range(args.steps):
+                step()
+            t1.record(stream)
+            torch.cuda.synchronize()
+        ams = t0.elapsed_time(t1)
+        akt = pdl.kernel_times()
+        aops, akname = ozaki_ops(M, N, K, args.slices)
+        apeak, apsrc, _ = tensor_peak("i8")
+        aach = aops / (float(np.mean(akt)) / 1e3) / 1e12 if akt else None
+        alt = {"variant": f"ozaki: FP64 DGEMM on INT8 tcgen05 ({args.slices} slices, K4/K5)",
+               "dtype": f"f64-ozaki-i8x{args.slices}",
+               "value": round(flops_total * args.steps / (ams / 1e3) / 1e9, 1), "unit": "GFLOP/s",
+               "ms_per_step": round(ams / args.steps, 3),
+               "parity": "max scaled err <= 1e-12 vs oracle (tests/test_gpu_ozaki.py, incl. C4 sampled rows)",
+               "roofline": {"bound": "tensor", "achieved": round(aach, 1) if aach else None,
+                            "peak": apeak, "unit": "TFLOP/s", "frac": round(aach / apeak, 4) if aach else None,
+                            "traffic": ncu_traffic("ozaki", args.config), "kernel": akname,
+                            "kernel_ms": round(float(np.mean(akt)), 3) if akt else None,
+                            "peak_source": apsrc},
+               "clocks": clk2.summary()}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(A, B, args.cpu_seconds)
@@ -462,6 +504,8 @@ def main():
         }
         if cublas is not None:
             line["cublas_gflops_same_operands"] = cublas
+        if alt is not None:
+            line["alt_variant"] = alt
         print(json.dumps(line), flush=True)
     pdl.unload()
     if world > 1:
