@@ -84,11 +84,25 @@ __global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, 
         const int e = exp_of_max(red[0]);
         if (threadIdx.x == 0) ea[i] = e;
         int8_t *out = A8 + i * ld8;
-        for (int64_t k = threadIdx.x; k < Kpad; k += blockDim.x) {
-            const double v = k < K ? ldexp(row[k], -e) : 0.0;
-            const int64_t c = k / Kc, kk = k - c * Kc;
+        // groups of 8 consecutive k (Kc % 128 == 0: a group never straddles a chunk);
+        // one 8-byte store per slice per group
+        for (int64_t k8 = (int64_t)threadIdx.x * 8; k8 < Kpad; k8 += (int64_t)blockDim.x * 8) {
+            double v[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? ldexp(row[k8 + j], -e) : 0.0;
+            const int64_t c = k8 / Kc, kk = k8 - c * Kc;
             int8_t *o = out + (c * S) * Kc + kk;
-            slice7(v, S, [&](int s, int8_t q) { o[(int64_t)s * Kc] = q; });
+            for (int s = 0; s < S; ++s) {
+                uint64_t pk = 0;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    v[j] *= 128.0;
+                    const double q = trunc(v[j]);
+                    v[j] -= q;
+                    pk |= (uint64_t)(uint8_t)(int8_t)(int)q << (8 * j);
+                }
+                *reinterpret_cast<uint64_t *>(o + (int64_t)s * Kc) = pk;
+            }
         }
         __syncthreads();
     }
@@ -106,26 +120,40 @@ __global__ void oz_colmax_kernel(const double *__restrict__ B, int64_t ldb, int6
 }
 
 // B (K x N) -> Bt8 (N rows of [c][S-1-s][kk]) through a 32 x 32 smem transpose.
-__global__ void oz_split_cols_t_kernel(const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S,
-                                       int64_t Kc, int nch, const unsigned long long *__restrict__ bmax,
-                                       int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb) {
-    __shared__ double t[32][33];
-    const int64_t k0 = (int64_t)blockIdx.y * 32, n0 = (int64_t)blockIdx.x * 32;
-    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
-        const int64_t k = k0 + r, n = n0 + threadIdx.x;
-        t[r][threadIdx.x] = (k < K && n < N) ? B[k * ldb + n] : 0.0;
+// Tile of 64 k x 32 n: coalesced loads along n into shared memory, then each
+// thread slices 8 consecutive k of one column -> one 8-byte store per slice.
+__global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
+    const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S, int64_t Kc, int nch,
+    const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb) {
+    __shared__ double t[64][33];
+    const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;   // 32 x 8
+    for (int r = ty; r < 64; r += 8) {
+        const int64_t k = k0 + r, n = n0 + tx;
+        t[r][tx] = (k < K && n < N) ? B[k * ldb + n] : 0.0;
     }
     __syncthreads();
     const int64_t Kpad = (int64_t)nch * Kc;
-    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
-        const int64_t n = n0 + r, k = k0 + threadIdx.x;
-        if (n >= N || k >= Kpad) continue;
-        const int f = exp_of_max(__longlong_as_double((long long)bmax[n]));
-        if (blockIdx.y == 0 && threadIdx.x == 0) fb[n] = f;
-        const double v = ldexp(t[threadIdx.x][r], -f);
-        const int64_t c = k / Kc, kk = k - c * Kc;
-        int8_t *o = Bt8 + n * ld8 + (c * S) * Kc + kk;
-        slice7(v, S, [&](int s, int8_t q) { o[(int64_t)(S - 1 - s) * Kc] = q; });
+    const int nl = threadIdx.x >> 3, g = threadIdx.x & 7;    // column, group of 8 k
+    const int64_t n = n0 + nl, k8 = k0 + 8 * g;
+    if (n >= N || k8 >= Kpad) return;
+    const int f = exp_of_max(__longlong_as_double((long long)bmax[n]));
+    if (blockIdx.y == 0 && g == 0) fb[n] = f;
+    double v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = ldexp(t[8 * g + j][nl], -f);
+    const int64_t c = k8 / Kc, kk = k8 - c * Kc;
+    int8_t *o = Bt8 + n * ld8 + (c * S) * Kc + kk;
+    for (int s = 0; s < S; ++s) {
+        uint64_t pk = 0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            v[j] *= 128.0;
+            const double q = trunc(v[j]);
+            v[j] -= q;
+            pk |= (uint64_t)(uint8_t)(int8_t)(int)q << (8 * j);
+        }
+        *reinterpret_cast<uint64_t *>(o + (int64_t)(S - 1 - s) * Kc) = pk;
     }
 }
 
@@ -162,7 +190,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
     oz_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
                        double *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
                        const int *__restrict__ fb, int scale_exp, int accumulate, int tiles_m, int tiles_n,
-                       int vec_ok) {
+                       int group_m, int vec_ok) {
     using namespace koz;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
@@ -175,13 +203,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t rank = cluster_ctarank();
-    const int cid = blockIdx.x >> 1;
-    const int per_group = GROUP_M * tiles_n;
-    const int g = cid / per_group;
-    const int first_m = g * GROUP_M;
-    const int gsz = min(tiles_m - first_m, GROUP_M);
-    const int tm = first_m + (cid % per_group) % gsz;
-    const int tn = (cid % per_group) / gsz;
+    int tm, tn;
+    raster_tile(blockIdx.x >> 1, tiles_m, tiles_n, group_m, &tm, &tn);
     const int m0 = tm * (2 * BM) + (int)rank * BM;
     const int nb0 = tn * BN + (int)rank * BNH;
 
@@ -319,8 +342,8 @@ cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_
         oz_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
     }
     const int64_t Kpad = (int64_t)L.nch * L.Kc;
-    dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 31) / 32));
-    oz_split_cols_t_kernel<<<g2, dim3(32, 8), 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb);
+    dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 63) / 64));
+    oz_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb);
     return cudaGetLastError();
 }
 
@@ -364,7 +387,7 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
                 return cudaErrorInvalidValue;
             oz_gemm_2sm_kernel<<<2 * tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(
                 ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m, tiles_n,
-                vec_ok);
+                raster_group_m(GROUP_M), vec_ok);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             first = 0;

@@ -417,8 +417,10 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     const bool off = pe_env && !strcmp(pe_env, "0");
     const double flops = 2.0 * rows * cols * (double)K;
     if (!off && (a_st || b_st || c_st) && K > 0 && (force || flops >= 2e11)) {
+        // first sub-kernel waits for one A band + one B panel only: smaller
+        // panels start compute sooner; >= 2048 x 4096 keeps each launch >= 1.7 waves
         RB = (int)std::min<int64_t>(8, std::max<int64_t>(1, rows / 2048));
-        CP = cols >= 8192 ? 2 : 1;
+        CP = (int)std::min<int64_t>(4, std::max<int64_t>(1, cols / 4096));
         if (force) {
             RB = (int)std::min<int64_t>(4, std::max<int64_t>(1, (rows + 127) / 128));
             CP = (int)std::min<int64_t>(2, std::max<int64_t>(1, (cols + 127) / 128));

@@ -2,6 +2,7 @@
 #pragma once
 #include <cuda.h>
 #include <cstdint>
+#include <cstdlib>
 
 namespace pdlk {
 
@@ -58,6 +59,25 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
           "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
         : "r"(taddr));
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+// Grouped rasterisation of cluster tiles: group_m tile rows sweep the tile
+// columns together (column-major inside a group), so the clusters resident
+// at one time share A and B panels in L2.
+__device__ __forceinline__ void raster_tile(int cid, int tiles_m, int tiles_n, int group_m, int *tm, int *tn) {
+    const int per_group = group_m * tiles_n;
+    const int g = cid / per_group;
+    const int first_m = g * group_m;
+    const int gsz = min(tiles_m - first_m, group_m);
+    *tm = first_m + (cid % per_group) % gsz;
+    *tn = (cid % per_group) / gsz;
+}
+
+// Raster group size: compiled default, PDL_GROUP_M env override (tuning).
+inline int raster_group_m(int dflt) {
+    const char *e = getenv("PDL_GROUP_M");
+    int v = e ? atoi(e) : dflt;
+    return v > 0 ? v : dflt;
 }
 
 // ---- CTA pair (cta_group::2) ----
