@@ -169,7 +169,7 @@ constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int EPI_WARPS = 16, EPI_COLS = 64, FIRST_EPI_WARP = 2;
 constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
 constexpr int TMEM_COLS = 256;
-constexpr int GROUP_M = 8;
+constexpr int GROUP_M = 4;   // raster sweep (tools/sweep_group.sh): 4 best of {2,4,8,16,32}
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
 }  // namespace koz
 

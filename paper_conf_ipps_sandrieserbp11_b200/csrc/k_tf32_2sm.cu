@@ -43,7 +43,7 @@ constexpr int FIRST_EPI_WARP = 2;   // warps 2..17: each TMEM lane quarter (warp
 constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
 constexpr int TMEM_COLS = 512;
 constexpr int KCB = 4;                  // K chunk = KCB * BK = 128 (R16)
-constexpr int GROUP_M = 8;              // cluster-tile rows per raster group
+constexpr int GROUP_M = 4;              // cluster-tile rows per raster group (sweep: 4 best)
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
 }  // namespace k2x
 
