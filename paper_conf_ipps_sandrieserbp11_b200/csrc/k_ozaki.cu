@@ -43,29 +43,31 @@ namespace pdlk {
 // K5: slicing pre-pass
 // ------------------------------------------------------------------------
 
-// frexp exponent of a non-negative finite max: max < 2^e (0 -> 0).
-__device__ __forceinline__ int exp_of_max(double mx) {
+// Scale exponent of a row / column from its non-negative finite max:
+// max < 2^e (0 -> 0).  Round-to-nearest slicing (rn) additionally needs
+// 128 * max * 2^-e < 127.5 so the first rint() stays within [-127, 127].
+__device__ __forceinline__ int exp_of_max(double mx, int rn) {
     if (!(mx > 0.0)) return 0;
     int e;
-    frexp(mx, &e);
+    const double m = frexp(mx, &e);
+    if (rn && m * 128.0 >= 127.5) ++e;
     return e;
 }
 
-// Write S truncated 7-bit slices of v (|v| < 1).
-template <typename F>
-__device__ __forceinline__ void slice7(double v, int S, F &&store) {
-    for (int s = 0; s < S; ++s) {
-        v *= 128.0;
-        const double q = trunc(v);
-        v -= q;
-        store(s, (int8_t)(int)q);
-    }
+// One slicing step: v <- 128 v, q = round(v) (trunc or nearest), v <- v - q
+// (all exact in FP64).  trunc: |q| <= 127, remainders in (-1,1); nearest:
+// |q| <= 127 for the first slice, <= 64 after, remainders in [-1/2, 1/2].
+__device__ __forceinline__ double slice_q(double &v, int rn) {
+    v *= 128.0;
+    const double q = rn ? rint(v) : trunc(v);
+    v -= q;
+    return q;
 }
 
 // One CTA per row (grid-stride): A (M x K, lda) -> A8 rows [c][s][kk].
 __global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M, int64_t K, int S,
                                      int64_t Kc, int nch, int8_t *__restrict__ A8, int64_t ld8,
-                                     int *__restrict__ ea) {
+                                     int *__restrict__ ea, int rn) {
     __shared__ double red[32];
     const int64_t Kpad = (int64_t)nch * Kc;
     for (int64_t i = blockIdx.x; i < M; i += gridDim.x) {
@@ -81,7 +83,7 @@ __global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, 
             if (threadIdx.x == 0) red[0] = mx;
         }
         __syncthreads();
-        const int e = exp_of_max(red[0]);
+        const int e = exp_of_max(red[0], rn);
         if (threadIdx.x == 0) ea[i] = e;
         int8_t *out = A8 + i * ld8;
         // groups of 8 consecutive k (Kc % 128 == 0: a group never straddles a chunk);
@@ -96,9 +98,7 @@ __global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, 
                 uint64_t pk = 0;
 #pragma unroll
                 for (int j = 0; j < 8; ++j) {
-                    v[j] *= 128.0;
-                    const double q = trunc(v[j]);
-                    v[j] -= q;
+                    const double q = slice_q(v[j], rn);
                     pk |= (uint64_t)(uint8_t)(int8_t)(int)q << (8 * j);
                 }
                 *reinterpret_cast<uint64_t *>(o + (int64_t)s * Kc) = pk;
@@ -124,7 +124,8 @@ __global__ void oz_colmax_kernel(const double *__restrict__ B, int64_t ldb, int6
 // thread slices 8 consecutive k of one column -> one 8-byte store per slice.
 __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
     const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S, int64_t Kc, int nch,
-    const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb) {
+    const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
+    int rn) {
     __shared__ double t[64][33];
     const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
     const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;   // 32 x 8
@@ -137,7 +138,7 @@ __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
     const int nl = threadIdx.x >> 3, g = threadIdx.x & 7;    // column, group of 8 k
     const int64_t n = n0 + nl, k8 = k0 + 8 * g;
     if (n >= N || k8 >= Kpad) return;
-    const int f = exp_of_max(__longlong_as_double((long long)bmax[n]));
+    const int f = exp_of_max(__longlong_as_double((long long)bmax[n]), rn);
     if (blockIdx.y == 0 && g == 0) fb[n] = f;
     double v[8];
 #pragma unroll
@@ -148,9 +149,7 @@ __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
         uint64_t pk = 0;
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-            v[j] *= 128.0;
-            const double q = trunc(v[j]);
-            v[j] -= q;
+            const double q = slice_q(v[j], rn);
             pk |= (uint64_t)(uint8_t)(int8_t)(int)q << (8 * j);
         }
         *reinterpret_cast<uint64_t *>(o + (int64_t)(S - 1 - s) * Kc) = pk;
@@ -328,7 +327,7 @@ cudaError_t launch_ozaki_split_a(const double *A, int64_t lda, int64_t rows, int
                                  int8_t *A8, int *ea, cudaStream_t s) {
     if (rows <= 0) return cudaSuccess;
     int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
-    oz_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, L.S, L.Kc, L.nch, A8, L.ld8, ea);
+    oz_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, L.S, L.Kc, L.nch, A8, L.ld8, ea, L.rn);
     return cudaGetLastError();
 }
 
@@ -343,7 +342,7 @@ cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_
     }
     const int64_t Kpad = (int64_t)L.nch * L.Kc;
     dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 63) / 64));
-    oz_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb);
+    oz_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb, L.rn);
     return cudaGetLastError();
 }
 

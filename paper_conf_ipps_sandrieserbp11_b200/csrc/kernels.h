@@ -41,6 +41,7 @@ cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float 
 constexpr int64_t OZ_KC_MAX = 16384;   // (d+1)*Kc*127^2 < 2^31 for S <= 8
 struct OzakiLayout {
     int S = 7, nch = 1;
+    int rn = 0;          // slice rounding: 0 = truncation, 1 = round-to-nearest
     int64_t Kc = 0, ld8 = 0;
     size_t a8_bytes = 0, b8_bytes = 0;
 };

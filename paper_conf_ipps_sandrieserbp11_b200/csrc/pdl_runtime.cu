@@ -385,7 +385,7 @@ int ensure_aux(WorkerCtx &w) {
 // FP64 task variant of a Worker: PDL property DGEMM_VARIANT ("dmma" default |
 // "ozaki") and OZAKI_SLICES (2..8, default 7); env PDL_DGEMM_VARIANT /
 // PDL_OZAKI_SLICES override the descriptor (tests, bench).
-bool worker_ozaki(const WorkerCtx &w, int *slices) {
+bool worker_ozaki(const WorkerCtx &w, int *slices, int *rn) {
     std::string v;
     if (const char *e = getenv("PDL_DGEMM_VARIANT")) v = e;
     else if (const Property *p = g->model.prop(w.pu, "DGEMM_VARIANT")) v = p->value;
@@ -394,6 +394,11 @@ bool worker_ozaki(const WorkerCtx &w, int *slices) {
     if (const char *e = getenv("PDL_OZAKI_SLICES")) s = atoi(e);
     else if (const Property *p = g->model.prop(w.pu, "OZAKI_SLICES")) s = atoi(p->value.c_str());
     *slices = std::max(2, std::min(8, s));
+    // OZAKI_ROUNDING: "trunc" (default) | "nearest"
+    std::string r;
+    if (const char *e = getenv("PDL_OZAKI_ROUNDING")) r = e;
+    else if (const Property *p = g->model.prop(w.pu, "OZAKI_ROUNDING")) r = p->value;
+    *rn = lower(trim(r)) == "nearest" ? 1 : 0;
     return true;
 }
 
@@ -486,13 +491,15 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     // DGEMM task variant of this Worker, pre-selected from its PDL properties
     // (task repository + static pre-selection, L1307-1326): K1 (DMMA) or K4 (Ozaki).
     int oz_slices = 0;
-    const bool ozaki = f64 && K > 0 && worker_ozaki(w, &oz_slices);
+    int oz_rn = 0;
+    const bool ozaki = f64 && K > 0 && worker_ozaki(w, &oz_slices, &oz_rn);
     pdlk::OzakiLayout OL;
     int8_t *a8 = nullptr, *b8 = nullptr;
     int *oz_ea = nullptr, *oz_fb = nullptr;
     unsigned long long *oz_bmax = nullptr;
     if (ozaki) {
         OL = pdlk::ozaki_layout(rows, cols, K, oz_slices);
+        OL.rn = oz_rn;
         if ((rc = ensure_buf(w, BUF_OZA, OL.a8_bytes, &p))) return rc;
         a8 = (int8_t *)p;
         if ((rc = ensure_buf(w, BUF_OZB, OL.b8_bytes, &p))) return rc;
