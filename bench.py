@@ -67,7 +67,8 @@ def parse():
     p.add_argument("--no-cublas", action="store_true")
     p.add_argument("--variant", choices=("dmma", "ozaki"), default="dmma",
                    help="FP64 DGEMM task variant (PDL DGEMM_VARIANT): K1 DMMA or K4 Ozaki INT8")
-    p.add_argument("--slices", type=int, default=7, help="OZAKI_SLICES for --variant ozaki")
+    p.add_argument("--slices", type=int, default=6,
+                   help="OZAKI_SLICES for --variant ozaki (round-to-nearest slices)")
     p.add_argument("--no-alt", action="store_true", help="skip timing the other FP64 variant")
     p.add_argument("--dist-backend", choices=("nccl", "gloo"), default="nccl",
                    help="gloo only to validate the N>1 flow with ranks sharing one GPU")

@@ -288,8 +288,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
 #pragma unroll
                     for (int j = 0; j < 16; j += 2) {
                         double2 *p = reinterpret_cast<double2 *>(crow + c0 + j);
-                        double2 o = accumulate ? *p : make_double2(0.0, 0.0);
-                        *p = make_double2(o.x + v[j], o.y + v[j + 1]);
+                        // streaming (evict-first) C traffic keeps the slice panels in L2
+                        double2 o = accumulate ? __ldcs(p) : make_double2(0.0, 0.0);
+                        __stcs(p, make_double2(o.x + v[j], o.y + v[j + 1]));
                     }
                 } else {
 #pragma unroll

@@ -179,7 +179,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
             if (vec_ok && cbase + EPI_COLS <= N) {
 #pragma unroll
                 for (int j = 0; j < EPI_COLS; j += 4)
-                    *reinterpret_cast<float4 *>(crow + j) = make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]);
+                    __stcs(reinterpret_cast<float4 *>(crow + j), make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]));
             } else {
 #pragma unroll
                 for (int j = 0; j < EPI_COLS; ++j)

@@ -29,8 +29,9 @@ def _env(monkeypatch):
     pdl.unload()
 
 
-def oz_matmul(A, B, tile=0, workers=1, host=False, slices=7):
-    pdl.load(pdl.descriptor_xml(workers, "ozaki", slices))
+def oz_matmul(A, B, tile=0, workers=1, host=False, slices=None, rounding=None):
+    """Default slicing = the library's default (6 round-to-nearest slices)."""
+    pdl.load(pdl.descriptor_xml(workers, "ozaki", slices, rounding))
     try:
         M, K = A.shape
         N = B.shape[1]
@@ -125,11 +126,15 @@ def test_wide_exponent_rows_columns():
     check(oz_matmul(A, B), A, B)
 
 
-@pytest.mark.parametrize("slices,tol", [(6, 1e-10), (8, 1e-13)])
-def test_slice_count_accuracy(slices, tol):
+@pytest.mark.parametrize("slices,rounding,tol", [(6, "nearest", 1e-13), (7, "trunc", 1e-13),
+                                                (5, "nearest", 1e-10), (6, "trunc", 1e-10),
+                                                (8, "nearest", 1e-14)])
+def test_slice_count_accuracy(slices, rounding, tol):
+    """Measured error versus slice count and rounding (R19): truncation biases
+    the error (U[0,1) data), round-to-nearest slices are unbiased."""
     A = W.uniform((256, 4096), np.float64, 41)
     B = W.uniform((4096, 256), np.float64, 42)
-    check(oz_matmul(A, B, slices=slices), A, B, tol=tol)
+    check(oz_matmul(A, B, slices=slices, rounding=rounding), A, B, tol=tol)
 
 
 @pytest.mark.slow
