@@ -132,8 +132,16 @@ struct Parser {
         return v;
     }
 
+    int depth = 0;
+    static constexpr int kMaxDepth = 1024;   // recursion bound (descriptors are shallow trees)
+
     std::unique_ptr<XmlNode> element() {
         if (peek() != '<') fail("expected '<'");
+        if (++depth > kMaxDepth) fail("element nesting deeper than 1024");
+        struct DepthGuard {
+            int &d;
+            ~DepthGuard() { --d; }
+        } guard{depth};
         auto n = std::make_unique<XmlNode>();
         n->line = line;
         adv();
