@@ -67,6 +67,14 @@ extern "C" {
 #define PDL_TASK_PANELS 1u   /* operands are this process's Worker panels (after the exchange):
                                 A = rows_w x K, B = K x cols_w, C = rows_w x cols_w block at
                                 the Worker's rectangle; see pdl_plan */
+#define PDL_TASK_LOCAL 2u    /* the whole M x N x K task is one tile task of this process's
+                                (first) Worker: no mapping over the group.  The multi-rank
+                                runtime uses it to compute a Worker rectangle chunk by chunk
+                                while the exchange of the next chunk is in flight */
+#define PDL_TASK_REUSE_B 4u  /* B (same pointer, ldb, K, N) is unchanged since the previous task
+                                of this Worker: reuse its prepared form (FP32 split / Ozaki
+                                slices) instead of recomputing it; ignored when no matching
+                                prepared B exists */
 
 /*
  * pdl_load -- parse a PDL descriptor and build the machine model.

@@ -89,6 +89,18 @@ struct WorkerCtx {
     // pipelined staging: copy-in, copy-out, second compute stream; reusable events
     cudaStream_t aux[3] = {nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> ev_pool;
+    // identity of the B operand whose prepared form (FP32 split / Ozaki slices)
+    // sits in the B-side buffers (PDL_TASK_REUSE_B)
+    struct BSig {
+        bool valid = false;
+        const void *B = nullptr;
+        int64_t ldb = 0, K = 0, cols = 0;
+        int dtype = -1, oz = 0, S = 0, rn = 0;
+        bool operator==(const BSig &o) const {
+            return valid && o.valid && B == o.B && ldb == o.ldb && K == o.K && cols == o.cols && dtype == o.dtype &&
+                   oz == o.oz && S == o.S && rn == o.rn;
+        }
+    } bsig;
 };
 
 constexpr size_t kMaxKernelTimes = 4096;
@@ -135,6 +147,7 @@ struct State {
     std::string plan_json = "[]";
     pdlk::EncodeTiledFn encode = nullptr;
     int last_launches = 0;
+    long long total_launches = 0;   // every kernel launched since pdl_load
 };
 
 State *g = nullptr;
@@ -329,6 +342,7 @@ int ensure_buf(WorkerCtx &w, int slot, size_t bytes, void **out) {
                            cudaGetErrorString(e));
         }
         b.bytes = bytes;
+        if (slot == BUF_BHI || slot == BUF_BLO || slot == BUF_OZB || slot == BUF_OZE) w.bsig.valid = false;
     }
     *out = b.ptr;
     return PDL_OK;
@@ -509,10 +523,26 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         b8 = (int8_t *)p;
         const size_t eb = (size_t)round_up(rows, 2) * 4 + (size_t)round_up(cols, 2) * 4 + (size_t)cols * 8;
         if ((rc = ensure_buf(w, BUF_OZE, eb, &p))) return rc;
+        // [bmax: cols u64][fb: cols int][ea: rows int] -- the B-side part does not
+        // move with `rows`, so a prepared B survives row-chunk tasks (REUSE_B)
         oz_bmax = (unsigned long long *)p;
-        oz_ea = (int *)(oz_bmax + cols);
-        oz_fb = oz_ea + round_up(rows, 2);
+        oz_fb = (int *)(oz_bmax + cols);
+        oz_ea = oz_fb + round_up(cols, 2);
     }
+
+    // B prepared by a previous task of this Worker (PDL_TASK_REUSE_B)?
+    WorkerCtx::BSig want;
+    want.valid = true;
+    want.B = B;
+    want.ldb = t.ldb;
+    want.K = K;
+    want.cols = cols;
+    want.dtype = t.dtype;
+    want.oz = ozaki ? 1 : 0;
+    want.S = ozaki ? OL.S : 0;
+    want.rn = ozaki ? OL.rn : 0;
+    const bool prep_b = K > 0 && (ozaki || !f64);
+    const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
 
     std::vector<cudaEvent_t> ev_a(RB, nullptr), ev_b(CP, nullptr), ev_sa(RB, nullptr), ev_sb(CP, nullptr);
     cudaEvent_t ev_last_out = nullptr, ev_last_cmp1 = nullptr;
@@ -565,7 +595,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 } else if (ev_sa[i]) {
                     CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
                 }
-                if (e == cudaSuccess && i == 0) {
+                if (e == cudaSuccess && i == 0 && !b_ready) {
                     e = pdlk::launch_ozaki_split_b((const double *)(Bd + (size_t)c0 * es), ldb, K, nc, OL,
                                                    b8 + c0 * OL.ld8, oz_fb + c0, oz_bmax + c0, cs);
                     w.launches += 2;
@@ -603,7 +633,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 } else if (ev_sa[i]) {
                     CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
                 }
-                if (e == cudaSuccess && i == 0) {
+                if (e == cudaSuccess && i == 0 && !b_ready) {
                     e = pdlk::launch_split_cols_t((const float *)(Bd + (size_t)c0 * es), ldb, K, nc, bhi + c0 * Kp,
                                                   blo + c0 * Kp, Kp, cs);
                     w.launches += 1;
@@ -643,6 +673,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             }
             ++launch_idx;
         }
+    }
+    if (prep_b) {
+        // the B-side buffers now hold this task's prepared B (whole panel only when unpiped)
+        w.bsig = want;
+        w.bsig.valid = !piped && !b_st;
     }
     if (piped) {
         // join: the Worker stream completes after every side stream's work
@@ -704,7 +739,10 @@ int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, v
     if (M < 0 || N < 0 || K < 0) return set_err(PDL_EINVAL, "negative size M=%lld N=%lld K=%lld", (long long)M,
                                                 (long long)N, (long long)K);
     if (tile < 0) return set_err(PDL_EINVAL, "negative tile %lld", (long long)tile);
-    if (flags & ~PDL_TASK_PANELS) return set_err(PDL_EINVAL, "unknown flags 0x%x", flags);
+    if (flags & ~(PDL_TASK_PANELS | PDL_TASK_LOCAL | PDL_TASK_REUSE_B))
+        return set_err(PDL_EINVAL, "unknown flags 0x%x", flags);
+    if ((flags & PDL_TASK_PANELS) && (flags & PDL_TASK_LOCAL))
+        return set_err(PDL_EINVAL, "PDL_TASK_PANELS and PDL_TASK_LOCAL are exclusive");
     if (dist && strcasecmp(dist, "BLOCK") != 0) {
         if (!strcasecmp(dist, "CYCLIC") || !strcasecmp(dist, "BLOCK-CYCLIC") || !strcasecmp(dist, "BLOCK_CYCLIC"))
             return set_err(PDL_EUNSUPPORTED, "distribution %s is not implemented (BLOCK only)", dist);
@@ -745,6 +783,16 @@ int execute(bool sync) {
     }
     for (size_t ti = 0; ti < q.size(); ++ti) {
         const Task &t = q[ti];
+        if (t.flags & PDL_TASK_LOCAL) {
+            // one tile task of this process's (first) Worker, no mapping
+            if (ti) pj << ",";
+            pj << "{\"local\":true,\"M\":" << t.M << ",\"N\":" << t.N << ",\"K\":" << t.K << "}";
+            if (g->dry_run) continue;
+            if (g->workers.empty()) return set_err(PDL_ENOWORKER, "no Worker bound to this process");
+            rc = run_rect(g->workers[0], t, t.A, t.B, t.C, t.M, t.N);
+            if (rc) return rc;
+            continue;
+        }
         std::vector<int> gw = g->model.group_workers(t.has_group ? t.group.c_str() : nullptr);
         const int G = (int)gw.size();
         if (G == 0) return set_err(PDL_ENOWORKER, "execution group has no gpu Worker");
@@ -788,6 +836,7 @@ int execute(bool sync) {
     }
     pj << "]";
     g->plan_json = pj.str();
+    for (auto &w : g->workers) g->total_launches += w.launches;
     if (sync) return pdl_sync();
     return PDL_OK;
 }
@@ -898,7 +947,8 @@ int pdl_query(const char *key, char *out, size_t len) {
             res += "]";
         } else if (k == "stats") {
             std::ostringstream o;
-            o << "{\"launches\":" << g->last_launches << ",\"workers\":[";
+            o << "{\"launches\":" << g->last_launches << ",\"total_launches\":" << g->total_launches
+              << ",\"workers\":[";
             bool first = true;
             for (auto &w : g->workers) {
                 float ms = -1.f;

@@ -81,6 +81,7 @@ class Grid:
     def __init__(self, Gr, Gc, rank):
         self.Gr, self.Gc, self.rank = Gr, Gc, rank
         self.row_group = self.col_group = None
+        self.row_ranks = [rank // Gc * Gc + c for c in range(Gc)]   # global ranks of my grid row
         for r in range(Gr):
             ranks = [r * Gc + c for c in range(Gc)]
             g = dist.new_group(ranks) if Gc > 1 else None
@@ -140,6 +141,73 @@ def _all_gather(out, chunk, group):
         dist.all_gather_into_tensor(out, chunk.contiguous(), group=group)
 
 
+class _Done:
+    def wait(self):
+        pass
+
+
+def _broadcast(t, src, group):
+    """Asynchronous broadcast of one A chunk inside the grid row (NCCL);
+    host-staged and synchronous under gloo (see _all_gather)."""
+    if t.is_cuda and dist.get_backend(group) == "gloo":
+        tmp = t.cpu() if dist.get_rank() == src else torch.empty(t.shape, dtype=t.dtype)
+        dist.broadcast(tmp, src=src, group=group)
+        t.copy_(tmp)
+        return _Done()
+    return dist.broadcast(t, src=src, group=group, async_op=True)
+
+
+def chunk_rows(wp: WorkerPlan, j):
+    """Rows [lo, hi) of the A row-panel (and of the C block) held by chunk j."""
+    lo = min(j * wp.qa, wp.rows)
+    return lo, min(lo + wp.qa, wp.rows)
+
+
+def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers, compute):
+    """Exchange with the A transfer overlapped by compute.
+
+    The B column-panel is all-gathered first (every C row needs it).  The A
+    row-panel then arrives as Gc asynchronous broadcasts inside the grid row,
+    one per owner; `compute(j, lo, hi, Apanel_rows, Bpanel, first)` runs on
+    the Worker's own chunk first, then on chunk j as soon as its broadcast has
+    landed (the stream waits on the NCCL work, the host does not), so the
+    remaining (Gc-1)/Gc of the A traffic hides behind the kernels.  Results are
+    bitwise identical to the non-overlapped path (R14)."""
+    if wp.Gr > 1:
+        _all_gather(bufs.B, Bch, grid.col_group)
+    else:
+        bufs.B.copy_(Bch)
+    Bp = bufs.B[: wp.K]
+    qa, c = wp.qa, wp.c
+    bufs.A[c * qa:(c + 1) * qa].copy_(Ach)
+    works = {}
+    if wp.Gc > 1:
+        for j in range(wp.Gc):   # same order on every rank of the row
+            works[j] = _broadcast(bufs.A[j * qa:(j + 1) * qa], grid.row_ranks[j], grid.row_group)
+    first = True
+    for j in [c] + [x for x in range(wp.Gc) if x != c]:
+        lo, hi = chunk_rows(wp, j)
+        if j != c and j in works:
+            works[j].wait()
+        if hi > lo and wp.cols > 0:
+            compute(j, lo, hi, bufs.A[lo:hi], Bp, first)
+            first = False
+    for w in works.values():
+        w.wait()
+    return bufs.A[: wp.rows], Bp
+
+
+def chunk_task(Cblock, wp: WorkerPlan, tile=0):
+    """compute() for exchange_overlapped: one PDL_TASK_LOCAL task per A chunk
+    on this process's Worker; the prepared B panel is reused after the first."""
+    def compute(j, lo, hi, Arows, Bp, first):
+        Cv = Cblock[lo:hi]
+        pdl.task_matmul(Arows, Bp, Cv, M=hi - lo, N=wp.cols, K=wp.K, tile=tile,
+                        lda=Arows.stride(0), ldb=Bp.stride(0), ldc=Cv.stride(0), local=True, reuse_b=not first)
+        pdl.run_async()
+    return compute
+
+
 def local_task(Apanel, Bpanel, Cblock, wp: WorkerPlan, tile=0, run=True):
     """Run this Worker's rectangle through libpdl on the gathered panels."""
     if wp.rows == 0 or wp.cols == 0:
@@ -150,11 +218,12 @@ def local_task(Apanel, Bpanel, Cblock, wp: WorkerPlan, tile=0, run=True):
         pdl.run_async()
 
 
-def distributed_matmul(A_full, B_full, C_full, tile=0, group=None):
+def distributed_matmul(A_full, B_full, C_full, tile=0, group=None, overlap=True):
     """Public multi-Worker API: every rank passes the full (host or device)
     A, B and its own C; rank r writes its rectangle of C.  Host operands are
-    copied chunk-wise to the Worker (PCIe), exchanged over NVLink, computed,
-    and the C block copied back (PCIe)."""
+    copied chunk-wise to the Worker (PCIe), exchanged over NVLink (overlapped
+    with the tile kernels unless overlap=False), computed, and the C block
+    copied back (PCIe)."""
     rank = dist.get_rank()
     M, K = A_full.shape
     N = B_full.shape[1]
@@ -164,10 +233,13 @@ def distributed_matmul(A_full, B_full, C_full, tile=0, group=None):
     Ach, Bch = chunk_from_full(A_full, B_full, wp)
     Ach, Bch = Ach.to(dev, non_blocking=True), Bch.to(dev, non_blocking=True)
     bufs = PanelBuffers(wp, A_full.dtype, dev)
-    Ap, Bp = exchange(Ach, Bch, wp, grid, bufs)
     Cb = torch.empty((wp.rows, wp.cols), dtype=C_full.dtype, device=dev)
     pdl.set_stream(torch.cuda.current_stream())
-    local_task(Ap, Bp, Cb, wp, tile)
+    if overlap:
+        exchange_overlapped(Ach, Bch, wp, grid, bufs, chunk_task(Cb, wp, tile))
+    else:
+        Ap, Bp = exchange(Ach, Bch, wp, grid, bufs)
+        local_task(Ap, Bp, Cb, wp, tile)
     pdl.sync()
     C_full[wp.row0: wp.row1, wp.col0: wp.col1].copy_(Cb)
     return wp

@@ -47,6 +47,23 @@ def _worker(rank, world, port, shapes, q):
             Ap, Bp = runtime.exchange(Ach, Bch, wp, grid, bufs)
             ok_a = torch.equal(Ap, A[wp.row0:wp.row1])
             ok_b = torch.equal(Bp, B[:, wp.col0:wp.col1])
+            # overlapped exchange: every chunk handed to compute() must already
+            # hold its rows; own chunk first; rows covered exactly once
+            bufs2 = runtime.PanelBuffers(wp, A.dtype, A.device)
+            seen = []
+
+            def compute(j, lo, hi, Arows, Bp2, first):
+                seen.append((j, lo, hi, first))
+                assert torch.equal(Arows, A[wp.row0 + lo: wp.row0 + hi])
+                assert torch.equal(Bp2, B[:, wp.col0:wp.col1])
+
+            Ap2, Bp2 = runtime.exchange_overlapped(Ach, Bch, wp, grid, bufs2, compute)
+            ok_a = ok_a and torch.equal(Ap2, A[wp.row0:wp.row1]) and torch.equal(Bp2, Bp)
+            lo_c, hi_c = runtime.chunk_rows(wp, wp.c)
+            if seen:
+                ok_a = ok_a and seen[0][3] and not any(s[3] for s in seen[1:])
+                ok_a = ok_a and (hi_c == lo_c or seen[0][0] == wp.c)
+            ok_a = ok_a and sum(s[2] - s[1] for s in seen) == (wp.rows if wp.cols else 0)
             out.append((M, N, K, tile, wp.row0, wp.row1, wp.col0, wp.col1, wp.Gr, wp.Gc, ok_a, ok_b))
         pdl.unload()
         q.put((rank, out, None))
