@@ -201,6 +201,21 @@ int pdl_query(const char *key, char *out, size_t len);
  */
 int pdl_kernel_times(int worker, float *ms, int n);
 
+/*
+ * pdl_describe -- generate a PDL descriptor of this machine (
+ * the analogue of Listing 2, "Generated from OpenCL run-time libraries",
+ * L869-917): one Master PU for the host (ARCHITECTURE from the build target,
+ * host memory region size), one Worker PU per CUDA device (ARCHITECTURE gpu,
+ * DEVICE_ORDINAL fixed; DEVICE_NAME, MAX_COMPUTE_UNITS, COMPUTE_CAPABILITY,
+ * GLOBAL_MEM_SIZE, LOCAL_MEM_SIZE, L2_CACHE_SIZE, CLOCK_RATE, PCI_BUS_ID as
+ * unfixed properties; LogicGroupAttribute "gpus"), a PCIe
+ * Interconnect Master -> each Worker, and an NVLink Interconnect between every
+ * pair of Workers with peer access (cudaDeviceCanAccessPeer).  Needs no
+ * pdl_load.  Writes NUL-terminated XML (truncated to len-1) and returns its
+ * full length; PDL_ENOWORKER if no CUDA device is visible.
+ */
+int pdl_describe(char *out, size_t len);
+
 /* Message of the last error of this thread ("" if none). */
 const char *pdl_last_error(void);
 

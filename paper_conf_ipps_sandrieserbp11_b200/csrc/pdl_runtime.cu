@@ -27,6 +27,8 @@
 #include <string>
 #include <vector>
 
+#include <unistd.h>
+
 #include "../../include/libpdl.h"
 #include "kernels.h"
 #include "pdl_model.hpp"
@@ -152,7 +154,8 @@ struct State {
 
 State *g = nullptr;
 
-const char *kVersion = "libpdl 0.1.0 (sm_100a: K1 FP64 DMMA+TMA, K2 3xTF32 tcgen05+TMEM+TMA)";
+const char *kVersion =
+    "libpdl 0.2.0 (sm_100a: K1 FP64 DMMA+TMA, K2 3xTF32 tcgen05 CTA-pair, K4 FP64 Ozaki on INT8 tcgen05)";
 
 std::string read_descriptor(const char *d, bool *ok) {
     *ok = true;
@@ -1017,6 +1020,86 @@ int pdl_kernel_times(int worker, float *ms, int n) {
     }
     w.kt_n = 0;
     return cnt;
+}
+
+int pdl_describe(char *out, size_t len) {
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return set_err(PDL_ENOWORKER, "no CUDA device visible (%s)",
+                       e == cudaSuccess ? "0 devices" : cudaGetErrorString(e));
+    }
+#if defined(__x86_64__)
+    const char *arch = "x86";
+#elif defined(__aarch64__)
+    const char *arch = "arm";
+#else
+    const char *arch = "unknown";
+#endif
+    const long long host_bytes = (long long)sysconf(_SC_PHYS_PAGES) * (long long)sysconf(_SC_PAGE_SIZE);
+    auto prop = [](std::ostringstream &o, const char *name, const std::string &val, const char *unit, bool fixed) {
+        o << "      <Property fixed=\"" << (fixed ? "true" : "false") << "\"><name>" << name << "</name><value";
+        if (unit && *unit) o << " unit=\"" << unit << "\"";
+        std::string x;
+        for (char ch : val) {
+            switch (ch) {
+                case '&': x += "&amp;"; break;
+                case '<': x += "&lt;"; break;
+                case '>': x += "&gt;"; break;
+                default: x += ch;
+            }
+        }
+        o << ">" << x << "</value></Property>\n";
+    };
+    std::ostringstream o;
+    o << "<?xml version=\"1.0\"?>\n<!-- generated by pdl_describe (" << kVersion << ") -->\n";
+    o << "<Master id=\"0\" quantity=\"1\">\n  <PUDescriptor>\n";
+    prop(o, "ARCHITECTURE", arch, "", true);
+    o << "  </PUDescriptor>\n  <MemoryRegion id=\"host\"><MRDescriptor>\n";
+    prop(o, "SIZE", std::to_string(host_bytes), "B", false);
+    o << "  </MRDescriptor></MemoryRegion>\n";
+    for (int d = 0; d < ndev; ++d) {
+        cudaDeviceProp p;
+        if (cudaGetDeviceProperties(&p, d) != cudaSuccess) {
+            cudaGetLastError();
+            return set_err(PDL_ECUDA, "cudaGetDeviceProperties(%d) failed", d);
+        }
+        o << "  <Worker id=\"gpu" << d << "\" quantity=\"1\">\n    <PUDescriptor>\n";
+        prop(o, "ARCHITECTURE", "gpu", "", true);
+        prop(o, "DEVICE_ORDINAL", std::to_string(d), "", true);
+        prop(o, "DEVICE_NAME", p.name, "", false);
+        prop(o, "MAX_COMPUTE_UNITS", std::to_string(p.multiProcessorCount), "", false);
+        prop(o, "COMPUTE_CAPABILITY", std::to_string(p.major) + "." + std::to_string(p.minor), "", false);
+        prop(o, "GLOBAL_MEM_SIZE", std::to_string((unsigned long long)p.totalGlobalMem), "B", false);
+        prop(o, "LOCAL_MEM_SIZE", std::to_string((unsigned long long)p.sharedMemPerBlockOptin), "B", false);
+        prop(o, "L2_CACHE_SIZE", std::to_string(p.l2CacheSize), "B", false);
+        int clk = 0;
+        cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, d);
+        prop(o, "CLOCK_RATE", std::to_string(clk), "kHz", false);
+        prop(o, "PCI_BUS_ID", std::to_string(p.pciBusID), "", false);
+        o << "    </PUDescriptor>\n    <MemoryRegion id=\"hbm\"><MRDescriptor>\n";
+        prop(o, "SIZE", std::to_string((unsigned long long)p.totalGlobalMem), "B", false);
+        o << "    </MRDescriptor></MemoryRegion>\n    <LogicGroupAttribute>gpus</LogicGroupAttribute>\n  </Worker>\n";
+    }
+    for (int d = 0; d < ndev; ++d) o << "  <Interconnect type=\"PCIe\" from=\"0\" to=\"gpu" << d << "\" scheme=\"\"/>\n";
+    for (int a = 0; a < ndev; ++a)
+        for (int b = a + 1; b < ndev; ++b) {
+            int can = 0;
+            if (cudaDeviceCanAccessPeer(&can, a, b) != cudaSuccess) {
+                cudaGetLastError();
+                can = 0;
+            }
+            if (can) o << "  <Interconnect type=\"NVLink\" from=\"gpu" << a << "\" to=\"gpu" << b << "\" scheme=\"p2p\"/>\n";
+        }
+    o << "</Master>\n";
+    const std::string res = o.str();
+    if (out && len) {
+        size_t n = std::min(len - 1, res.size());
+        memcpy(out, res.data(), n);
+        out[n] = '\0';
+    }
+    return (int)res.size();
 }
 
 const char *pdl_last_error(void) { return g_err.c_str(); }
