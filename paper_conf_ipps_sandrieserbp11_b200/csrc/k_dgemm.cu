@@ -27,6 +27,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 
 #include "kernels.h"
 #include "ptx.cuh"
@@ -64,7 +65,7 @@ __device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b)
 __global__ void __launch_bounds__(k1::THREADS, 1)
     dgemm_k1_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     double *__restrict__ C, int64_t ldc, int M, int N, int K, int tiles_m, int tiles_n,
-                    int vec_ok) {
+                    int group_m, int vec_ok) {
     using namespace k1;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
@@ -73,12 +74,12 @@ __global__ void __launch_bounds__(k1::THREADS, 1)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-    // grouped raster: GROUP_M tile rows sweep the tile columns together
+    // grouped raster: group_m tile rows sweep the tile columns together
     const int bid = blockIdx.x;
-    const int per_group = GROUP_M * tiles_n;
+    const int per_group = group_m * tiles_n;
     const int g = bid / per_group;
-    const int first_m = g * GROUP_M;
-    const int gsz = min(tiles_m - first_m, GROUP_M);
+    const int first_m = g * group_m;
+    const int gsz = min(tiles_m - first_m, group_m);
     const int tm = first_m + (bid % per_group) % gsz;
     const int tn = (bid % per_group) / gsz;
 
@@ -258,8 +259,10 @@ cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, con
     }
     const int tiles_m = (int)((M + BM - 1) / BM), tiles_n = (int)((N + BN - 1) / BN);
     const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
+    const char *gm = getenv("PDL_GROUP_M_K1");   // raster tuning knob
+    const int group_m = gm && atoi(gm) > 0 ? atoi(gm) : GROUP_M;
     dgemm_k1_kernel<<<tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(ta, tb, C, ldc, (int)M, (int)N, (int)K,
-                                                                        tiles_m, tiles_n, vec_ok);
+                                                                        tiles_m, tiles_n, group_m, vec_ok);
     return cudaGetLastError();
 }
 
