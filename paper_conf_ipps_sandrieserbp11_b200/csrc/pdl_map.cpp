@@ -10,7 +10,10 @@
 // (L1262-1266).  Readings R4-R6: C is cut into ceil(M/tile) x
 // ceil(N/tile) tile tasks; BLOCK distributes task rows / columns over a
 // Gr x Gc Worker grid; the Worker grid minimises exchanged operand bytes.
+#include <algorithm>
+#include <cctype>
 #include <cmath>
+#include <cstdlib>
 #include <limits>
 #include <sstream>
 
@@ -45,9 +48,70 @@ double Plan::exchanged_elems() const {
     return tot;
 }
 
-Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G) {
+bool parse_dist(const char *s, DistSpec *out) {
+    DistSpec d;
+    if (!s) {
+        *out = d;
+        return true;
+    }
+    std::string v;
+    for (const char *c = s; *c; ++c) v += (char)std::toupper((unsigned char)*c);
+    std::string name = v, size;
+    size_t colon = v.find(':');
+    if (colon != std::string::npos) {
+        name = v.substr(0, colon);
+        size = v.substr(colon + 1);
+    }
+    for (auto &ch : name)
+        if (ch == '_') ch = '-';
+    if (name == "BLOCK") {
+        d.kind = Dist::Block;   // BLOCK:N -- N (L1155) is the element count, implied by the task
+    } else if (name == "CYCLIC" || name == "BLOCK-CYCLIC") {
+        d.kind = name == "CYCLIC" ? Dist::Cyclic : Dist::BlockCyclic;
+        d.b = 1;
+        if (!size.empty() && name == "BLOCK-CYCLIC") {
+            char *end = nullptr;
+            long long b = std::strtoll(size.c_str(), &end, 10);
+            if (!end || *end || b < 1) return false;
+            d.b = b;
+        }
+    } else {
+        return false;
+    }
+    *out = d;
+    return true;
+}
+
+// Element segments of grid index g (of Gx) over T tasks of edge `tile` along a
+// dimension of length L, merged when adjacent.
+static std::vector<Seg> segs_of(const Plan &p, int g, int Gx, int64_t T, int64_t L, const std::vector<int64_t> &bnd) {
+    std::vector<Seg> out;
+    if (p.dist.kind == Dist::Block) {
+        if (bnd[g + 1] > bnd[g]) out.push_back(Seg{bnd[g], bnd[g + 1]});
+        return out;
+    }
+    const int64_t edge = p.tile ? p.tile : 1;
+    const int64_t b = p.dist.b;
+    for (int64_t q = g; q * b < T; q += Gx) {
+        const int64_t lo = std::min(q * b * edge, L), hi = std::min((q + 1) * b * edge, L);
+        if (hi <= lo) continue;
+        if (!out.empty() && out.back().hi == lo) out.back().hi = hi;
+        else out.push_back(Seg{lo, hi});
+    }
+    return out;
+}
+
+std::vector<Seg> Plan::row_segs(int r) const { return segs_of(*this, r, Gr, Tm, M, row); }
+std::vector<Seg> Plan::col_segs(int c) const { return segs_of(*this, c, Gc, Tn, N, col); }
+
+Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec dist) {
     Plan p;
     p.M = M; p.N = N; p.K = K; p.G = G;
+    p.dist = dist;
+    if (dist.kind != Dist::Block && tile <= 0) {
+        // cyclic over single elements is meaningless for tile tasks: use 128-wide tasks
+        tile = 128;
+    }
     // Worker grid: minimise per-Worker received elements, ties -> larger Gr.
     double best = std::numeric_limits<double>::infinity();
     for (int gr = G; gr >= 1; --gr) {
@@ -86,7 +150,9 @@ std::string Plan::to_json(const std::vector<int> &workers, const std::vector<std
     std::ostringstream o;
     o << "{\"M\":" << M << ",\"N\":" << N << ",\"K\":" << K << ",\"tile\":" << tile << ",\"G\":" << G
       << ",\"Gr\":" << Gr << ",\"Gc\":" << Gc << ",\"Tm\":" << Tm << ",\"Tn\":" << Tn
-      << ",\"qb\":" << qb() << ",\"exchanged_elems\":" << (int64_t)exchanged_elems() << ",\"workers\":[";
+      << ",\"qb\":" << qb() << ",\"exchanged_elems\":" << (int64_t)exchanged_elems() << ",\"dist\":\""
+      << (dist.kind == Dist::Block ? "BLOCK" : dist.kind == Dist::Cyclic ? "CYCLIC" : "BLOCK-CYCLIC") << "\",\"dist_b\":"
+      << dist.b << ",\"workers\":[";
     for (int w = 0; w < G; ++w) {
         Rect R = rect(w);
         int r = w / Gc, c = w % Gc;
@@ -94,7 +160,16 @@ std::string Plan::to_json(const std::vector<int> &workers, const std::vector<std
         o << "{\"w\":" << w << ",\"id\":\"" << (w < (int)ids.size() ? json_escape(ids[w]) : "") << "\""
           << ",\"r\":" << r << ",\"c\":" << c << ",\"rows\":[" << R.row0 << "," << R.row1 << "],\"cols\":["
           << R.col0 << "," << R.col1 << "],\"task_rows\":[" << trow[r] << "," << trow[r + 1]
-          << "],\"task_cols\":[" << tcol[c] << "," << tcol[c + 1] << "],\"qa\":" << qa(w) << "}";
+          << "],\"task_cols\":[" << tcol[c] << "," << tcol[c + 1] << "],\"qa\":" << qa(w);
+        if (dist.kind != Dist::Block) {
+            o << ",\"row_segs\":[";
+            auto rs = row_segs(r), cs = col_segs(c);
+            for (size_t i = 0; i < rs.size(); ++i) o << (i ? "," : "") << "[" << rs[i].lo << "," << rs[i].hi << "]";
+            o << "],\"col_segs\":[";
+            for (size_t i = 0; i < cs.size(); ++i) o << (i ? "," : "") << "[" << cs[i].lo << "," << cs[i].hi << "]";
+            o << "]";
+        }
+        o << "}";
     }
     (void)workers;
     o << "]}";

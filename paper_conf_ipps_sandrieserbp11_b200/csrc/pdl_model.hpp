@@ -97,23 +97,43 @@ struct Rect {
     int64_t row0 = 0, row1 = 0, col0 = 0, col1 = 0;
 };
 
+// Data distributions of the execute annotation (L1200-1206: "block, cyclic,
+// block-cyclic ... and optional sizes").
+enum class Dist { Block, Cyclic, BlockCyclic };
+struct DistSpec {
+    Dist kind = Dist::Block;
+    int64_t b = 1;   // tasks per cyclic block (CYCLIC = BLOCK-CYCLIC:1)
+};
+// Parse "BLOCK", "CYCLIC", "BLOCK-CYCLIC[:b]" (case-insensitive; NULL = BLOCK).
+// Returns false for an unknown name or a bad size.
+bool parse_dist(const char *s, DistSpec *out);
+
+struct Seg {
+    int64_t lo = 0, hi = 0;   // element range [lo, hi)
+};
+
 struct Plan {
     int64_t M = 0, N = 0, K = 0, tile = 0;   // tile: effective task edge (0 = per-Worker blocks)
     int G = 0, Gr = 0, Gc = 0;
+    DistSpec dist;
     int64_t Tm = 0, Tn = 0;                  // task grid
-    std::vector<int64_t> trow, tcol;         // task-row / task-col boundaries per grid row / col (Gr+1, Gc+1)
-    std::vector<int64_t> row, col;           // element boundaries (Gr+1, Gc+1)
-    Rect rect(int w) const;                  // w = r*Gc + c
+    std::vector<int64_t> trow, tcol;         // BLOCK: task-row / task-col boundaries per grid row / col
+    std::vector<int64_t> row, col;           // BLOCK: element boundaries (Gr+1, Gc+1)
+    Rect rect(int w) const;                  // BLOCK: the Worker's rectangle, w = r*Gc + c
     int64_t qa(int w) const;                 // rows per A chunk for Worker w
     int64_t qb() const;                      // K-rows per B chunk
     double exchanged_elems() const;          // received by all Workers (A + B)
+    // any distribution: the Worker's C row / column segments (merged when adjacent)
+    std::vector<Seg> row_segs(int r) const;
+    std::vector<Seg> col_segs(int c) const;
     std::string to_json(const std::vector<int> &workers, const std::vector<std::string> &ids) const;
 };
 
 // Choose Gr x Gc = G minimising received operand elements
 //   (M/Gr)*K*(1 - 1/Gc) + K*(N/Gc)*(1 - 1/Gr)   per Worker;
-// ties -> larger Gr.  Then BLOCK-distribute task rows / cols (L1200-1206):
-// grid row r gets task rows [floor(r*Tm/Gr), floor((r+1)*Tm/Gr)).
-Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G);
+// ties -> larger Gr.  BLOCK distributes task rows / cols (L1200-1206): grid row
+// r gets task rows [floor(r*Tm/Gr), floor((r+1)*Tm/Gr)); CYCLIC / BLOCK-CYCLIC:b
+// give grid row r the b-task blocks q with q % Gr == r (columns likewise).
+Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec dist = DistSpec());
 
 }  // namespace pdl

@@ -136,6 +136,7 @@ struct Task {
     bool has_group;
     std::string group;
     unsigned flags;
+    DistSpec dist;
 };
 
 struct State {
@@ -746,11 +747,13 @@ int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, v
         return set_err(PDL_EINVAL, "unknown flags 0x%x", flags);
     if ((flags & PDL_TASK_PANELS) && (flags & PDL_TASK_LOCAL))
         return set_err(PDL_EINVAL, "PDL_TASK_PANELS and PDL_TASK_LOCAL are exclusive");
-    if (dist && strcasecmp(dist, "BLOCK") != 0) {
-        if (!strcasecmp(dist, "CYCLIC") || !strcasecmp(dist, "BLOCK-CYCLIC") || !strcasecmp(dist, "BLOCK_CYCLIC"))
-            return set_err(PDL_EUNSUPPORTED, "distribution %s is not implemented (BLOCK only)", dist);
-        return set_err(PDL_EINVAL, "unknown distribution '%s' (L1200-1206 names block, cyclic, block-cyclic)", dist);
-    }
+    DistSpec ds;
+    if (!parse_dist(dist, &ds))
+        return set_err(PDL_EINVAL, "unknown distribution '%s' (L1200-1206: BLOCK, CYCLIC, BLOCK-CYCLIC[:b])", dist);
+    if (ds.kind != Dist::Block && ((flags & PDL_TASK_PANELS) || g->nranks > 1))
+        return set_err(PDL_EUNSUPPORTED,
+                       "distribution %s needs one process driving the Workers (the multi-rank panel exchange is BLOCK)",
+                       dist);
     if (group && g->model.group_workers(group).empty())
         return set_err(PDL_EINVAL, "execution group '%s' names no gpu Worker (LogicGroupAttribute)", group);
     if (M == 0 || N == 0) return PDL_OK;   // nothing to write
@@ -768,7 +771,7 @@ int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, v
         if (K > 0 && (overlaps(C, cn, A, an) || overlaps(C, cn, B, bn)))
             return set_err(PDL_EINVAL, "C overlaps A or B (C has access mode write, A/B read, L1184-1186)");
     }
-    Task t{dtype, A, lda_, B, ldb_, C, ldc_, M, N, K, tile, group != nullptr, group ? group : "", flags};
+    Task t{dtype, A, lda_, B, ldb_, C, ldc_, M, N, K, tile, group != nullptr, group ? group : "", flags, ds};
     g->queue.push_back(t);
     return PDL_OK;
 }
@@ -802,7 +805,7 @@ int execute(bool sync) {
         if (g->nranks > 1 && G != g->nranks)
             return set_err(PDL_ENOWORKER, "group has %d Workers but %d ranks co-exist: one process per Worker", G,
                            g->nranks);
-        Plan plan = make_plan(t.M, t.N, t.K, t.tile, G);
+        Plan plan = make_plan(t.M, t.N, t.K, t.tile, G, t.dist);
         std::vector<std::string> ids;
         for (int x : gw) ids.push_back(g->model.pus[x].id);
         if (ti) pj << ",";
@@ -815,6 +818,20 @@ int execute(bool sync) {
             for (int i = 0; i < G; ++i)
                 if (gw[i] == w.pu) gi = i;
             if (gi < 0) continue;
+            if (t.dist.kind != Dist::Block) {
+                // CYCLIC / BLOCK-CYCLIC: the Worker's tasks form row segments x column
+                // segments; each product is one sub-rectangle (same per-element K
+                // order, so C is bitwise the BLOCK result, R14)
+                for (const Seg &rs : plan.row_segs(gi / plan.Gc))
+                    for (const Seg &cs : plan.col_segs(gi % plan.Gc)) {
+                        const char *A = (const char *)t.A + (size_t)(rs.lo * t.lda) * es;
+                        const char *B = (const char *)t.B + (size_t)cs.lo * es;
+                        char *C = (char *)t.C + (size_t)(rs.lo * t.ldc + cs.lo) * es;
+                        rc = run_rect(w, t, A, B, C, rs.hi - rs.lo, cs.hi - cs.lo);
+                        if (rc) return rc;
+                    }
+                continue;
+            }
             Rect R = plan.rect(gi);
             const int64_t rows = R.row1 - R.row0, cols = R.col1 - R.col0;
             const char *A = (const char *)t.A, *B = (const char *)t.B;
