@@ -104,7 +104,21 @@ static std::vector<Seg> segs_of(const Plan &p, int g, int Gx, int64_t T, int64_t
 std::vector<Seg> Plan::row_segs(int r) const { return segs_of(*this, r, Gr, Tm, M, row); }
 std::vector<Seg> Plan::col_segs(int c) const { return segs_of(*this, c, Gc, Tn, N, col); }
 
-Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec dist) {
+std::vector<double> worker_speeds(const Model &m, const std::vector<int> &workers) {
+    std::vector<double> s;
+    for (int w : workers) {
+        double v = 1.0;
+        if (const Property *p = m.prop(w, "RELATIVE_SPEED")) {
+            char *end = nullptr;
+            double x = std::strtod(p->value.c_str(), &end);
+            if (end && !*end && x > 0 && std::isfinite(x)) v = x;
+        }
+        s.push_back(v);
+    }
+    return s;
+}
+
+Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec dist, const std::vector<double> *speeds) {
     Plan p;
     p.M = M; p.N = N; p.K = K; p.G = G;
     p.dist = dist;
@@ -112,6 +126,9 @@ Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec di
         // cyclic over single elements is meaningless for tile tasks: use 128-wide tasks
         tile = 128;
     }
+    bool hetero = false;
+    if (speeds && (int)speeds->size() == G && dist.kind == Dist::Block)
+        for (double s : *speeds) hetero |= (s != (*speeds)[0]);
     // Worker grid: minimise per-Worker received elements, ties -> larger Gr.
     double best = std::numeric_limits<double>::infinity();
     for (int gr = G; gr >= 1; --gr) {
@@ -120,6 +137,10 @@ Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec di
         double cost = (double(M) / gr) * double(K) * (1.0 - 1.0 / gc) +
                       double(K) * (double(N) / gc) * (1.0 - 1.0 / gr);
         if (cost < best * (1.0 - 1e-12)) { best = cost; p.Gr = gr; p.Gc = gc; }
+    }
+    if (hetero) {
+        p.Gr = G;
+        p.Gc = 1;
     }
     if (tile > 0) {
         p.tile = tile;
@@ -135,9 +156,24 @@ Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec di
     p.tcol.resize(p.Gc + 1);
     p.row.resize(p.Gr + 1);
     p.col.resize(p.Gc + 1);
-    for (int r = 0; r <= p.Gr; ++r) {
-        p.trow[r] = (int64_t)r * p.Tm / p.Gr;  // floor(r*Tm/Gr): remainder to higher rows
-        p.row[r] = p.tile ? std::min<int64_t>(p.trow[r] * p.tile, M) : (int64_t)r * M / p.Gr;
+    if (hetero) {
+        // task rows proportional to speed: boundary r = round(Tm * sum_{i<r} s_i / sum s)
+        // (tile = 0: rows of C instead of task rows)
+        double tot = 0;
+        for (double s : *speeds) tot += s;
+        const int64_t units = p.tile ? p.Tm : M;
+        double acc = 0;
+        for (int r = 0; r <= p.Gr; ++r) {
+            const int64_t b = r == p.Gr ? units : (int64_t)std::llround(units * acc / tot);
+            p.trow[r] = p.tile ? b : r;
+            p.row[r] = p.tile ? std::min<int64_t>(b * p.tile, M) : b;
+            if (r < p.Gr) acc += (*speeds)[r];
+        }
+    } else {
+        for (int r = 0; r <= p.Gr; ++r) {
+            p.trow[r] = (int64_t)r * p.Tm / p.Gr;  // floor(r*Tm/Gr): remainder to higher rows
+            p.row[r] = p.tile ? std::min<int64_t>(p.trow[r] * p.tile, M) : (int64_t)r * M / p.Gr;
+        }
     }
     for (int c = 0; c <= p.Gc; ++c) {
         p.tcol[c] = (int64_t)c * p.Tn / p.Gc;

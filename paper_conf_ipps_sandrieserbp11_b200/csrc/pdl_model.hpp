@@ -134,6 +134,15 @@ struct Plan {
 // ties -> larger Gr.  BLOCK distributes task rows / cols (L1200-1206): grid row
 // r gets task rows [floor(r*Tm/Gr), floor((r+1)*Tm/Gr)); CYCLIC / BLOCK-CYCLIC:b
 // give grid row r the b-task blocks q with q % Gr == r (columns likewise).
-Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec dist = DistSpec());
+//
+// Heterogeneous Workers (the paper's GTX480 + GTX285 box,
+// L1398-1402): when `speeds` (PDL property RELATIVE_SPEED of each Worker) are
+// not all equal, BLOCK becomes a 1-D row split (Gr = G, Gc = 1) with task rows
+// proportional to speed (cumulative rounding), so every Worker finishes together.
+Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec dist = DistSpec(),
+               const std::vector<double> *speeds = nullptr);
+
+// RELATIVE_SPEED of the group's Workers (1 when absent or invalid).
+std::vector<double> worker_speeds(const Model &m, const std::vector<int> &workers);
 
 }  // namespace pdl

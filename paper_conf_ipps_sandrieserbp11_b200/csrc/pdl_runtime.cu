@@ -805,7 +805,8 @@ int execute(bool sync) {
         if (g->nranks > 1 && G != g->nranks)
             return set_err(PDL_ENOWORKER, "group has %d Workers but %d ranks co-exist: one process per Worker", G,
                            g->nranks);
-        Plan plan = make_plan(t.M, t.N, t.K, t.tile, G, t.dist);
+        const std::vector<double> speeds = worker_speeds(g->model, gw);
+        Plan plan = make_plan(t.M, t.N, t.K, t.tile, G, t.dist, &speeds);
         std::vector<std::string> ids;
         for (int x : gw) ids.push_back(g->model.pus[x].id);
         if (ti) pj << ",";
@@ -933,7 +934,8 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group, i
     if (gw.empty()) return set_err(PDL_ENOWORKER, "execution group has no gpu Worker");
     const int G = (int)gw.size();
     if (worker < 0 || worker >= G) return set_err(PDL_EINVAL, "worker %d outside the group of %d", worker, G);
-    Plan p = make_plan(M, N, K, tile, G);
+    const std::vector<double> speeds = worker_speeds(g->model, gw);
+    Plan p = make_plan(M, N, K, tile, G, DistSpec(), &speeds);
     Rect R = p.rect(worker);
     const int r = worker / p.Gc, c = worker % p.Gc;
     int64_t v[PDL_PLAN_LEN] = {G, p.Gr, p.Gc, r, c, R.row0, R.row1, R.col0, R.col1, p.qa(worker), p.qb(),
