@@ -128,8 +128,14 @@ int task_matmul_f32(const float *A, const float *B, float *C,
  *   (0 = dense: K, N, N; in PANELS mode 0 = K, cols_w, cols_w).
  * group: LogicGroupAttribute naming the execution group (L1193-1199,
  *   L1254-1261); NULL = every gpu Worker.
- * dist: "BLOCK" (or NULL) -- the only distribution implemented
- *   (L1200-1206); "CYCLIC"/"BLOCK-CYCLIC" -> PDL_EUNSUPPORTED.
+ * dist: data distribution of C's tile tasks over the group (L1200-1206:
+ *   "block, cyclic, block-cyclic ... and optional sizes"): "BLOCK" (or NULL;
+ *   "BLOCK:N" accepted, N implied), "CYCLIC", "BLOCK-CYCLIC:b" (b tasks per
+ *   block, default 1), case-insensitive.  CYCLIC / BLOCK-CYCLIC need one
+ *   process driving the Workers (pdl_load): with PDL_TASK_PANELS or
+ *   pdl_load_rank they return PDL_EUNSUPPORTED.  Unknown names -> PDL_EINVAL.
+ *   Workers whose PDL property RELATIVE_SPEED differs get a speed-weighted
+ *   1-D BLOCK split (heterogeneous platforms, L1398-1402).
  * flags: 0 or PDL_TASK_PANELS.
  */
 int task_matmul_ex(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb,
