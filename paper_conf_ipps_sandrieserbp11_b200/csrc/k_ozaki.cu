@@ -160,16 +160,24 @@ __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
 // K4: int8 CTA-pair GEMM of one diagonal, FP64 epilogue
 // ------------------------------------------------------------------------
 namespace koz {
-constexpr int BM = 128, BN = 256, BNH = 128;
-constexpr int BK = 128, STAGES = 6, UMMA_K = 32;
+// NSUB N=256 sub-tiles per cluster: NSUB = 2 gives 256 x 512 cluster tiles
+// (two MMAs per K step into TMEM columns [0,256) and [256,512)), halving the
+// A-panel traffic per output element; NSUB = 1 for narrow problems.
+constexpr int BM = 128, BN1 = 256, BNH = 128;
+constexpr int BK = 128, UMMA_K = 32;
 constexpr int A_BYTES = BM * BK;        // 16 KiB
-constexpr int B_BYTES = BNH * BK;       // 16 KiB
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int EPI_WARPS = 16, EPI_COLS = 64, FIRST_EPI_WARP = 2;
+constexpr int B_BYTES = BNH * BK;       // 16 KiB per N=256 sub-tile
+constexpr int EPI_WARPS = 16, FIRST_EPI_WARP = 2;
 constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
-constexpr int TMEM_COLS = 256;
 constexpr int GROUP_M = 4;   // raster sweep (tools/sweep_group.sh): 4 best of {2,4,8,16,32}
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+template <int NSUB> struct Cfg {
+    static constexpr int BN = BN1 * NSUB;
+    static constexpr int STAGE_BYTES = A_BYTES + NSUB * B_BYTES;
+    static constexpr int STAGES = (6 * (A_BYTES + B_BYTES)) / STAGE_BYTES;   // 6 or 4
+    static constexpr int EPI_COLS = 64 * NSUB;
+    static constexpr int TMEM_COLS = 256 * NSUB;
+    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+};
 }  // namespace koz
 
 __host__ __device__ constexpr uint32_t idesc_i8(int M, int N) {
@@ -185,12 +193,15 @@ __device__ __forceinline__ void umma_i8_2sm(uint32_t tmem_d, uint64_t adesc, uin
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
 }
 
+template <int NSUB>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
     oz_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
                        double *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
                        const int *__restrict__ fb, int scale_exp, int accumulate, int tiles_m, int tiles_n,
                        int group_m, int vec_ok) {
     using namespace koz;
+    constexpr int BN = Cfg<NSUB>::BN, STAGES = Cfg<NSUB>::STAGES, STAGE_BYTES = Cfg<NSUB>::STAGE_BYTES;
+    constexpr int EPI_COLS = Cfg<NSUB>::EPI_COLS, TMEM_COLS = Cfg<NSUB>::TMEM_COLS;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
     const uint32_t bar_full = base + STAGES * STAGE_BYTES;
@@ -205,7 +216,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
     int tm, tn;
     raster_tile(blockIdx.x >> 1, tiles_m, tiles_n, group_m, &tm, &tn);
     const int m0 = tm * (2 * BM) + (int)rank * BM;
-    const int nb0 = tn * BN + (int)rank * BNH;
+    const int nb0 = tn * BN + (int)rank * BNH;   // + j * 256 for sub-tile j
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
@@ -238,12 +249,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
                 if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * STAGE_BYTES);
                 const uint32_t st = base + s * STAGE_BYTES;
                 tma_load_2d_2sm(st, &tA, fb_leader, kb * BK, m0);
-                tma_load_2d_2sm(st + A_BYTES, &tB, fb_leader, kb * BK, nb0);
+#pragma unroll
+                for (int j = 0; j < NSUB; ++j)
+                    tma_load_2d_2sm(st + A_BYTES + j * B_BYTES, &tB, fb_leader, kb * BK, nb0 + j * BN1);
             }
         }
     } else if (warp == 1) {
         if (rank == 0 && lane == 0) {
-            constexpr uint32_t idesc = idesc_i8(2 * BM, BN);
+            constexpr uint32_t idesc = idesc_i8(2 * BM, BN1);
             for (int kb = 0; kb < nk; ++kb) {
                 const int s = kb % STAGES;
                 const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
@@ -253,8 +266,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
 #pragma unroll
                 for (int kk = 0; kk < BK / UMMA_K; ++kk) {
                     const uint32_t off = kk * UMMA_K;   // 32 bytes of K per instruction
-                    umma_i8_2sm(tmem_base, umma_desc_k_sw128(st + off), umma_desc_k_sw128(st + A_BYTES + off), idesc,
-                                (kb | kk) ? 1u : 0u);
+#pragma unroll
+                    for (int j = 0; j < NSUB; ++j)
+                        umma_i8_2sm(tmem_base + j * BN1, umma_desc_k_sw128(st + off),
+                                    umma_desc_k_sw128(st + A_BYTES + j * B_BYTES + off), idesc, (kb | kk) ? 1u : 0u);
                 }
                 umma_commit_2sm(bar_empty + 8 * s);
             }
@@ -369,10 +384,19 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
     cudaGetDevice(&dev);
     static bool attr_done[64] = {false};
     if (dev < 64 && !attr_done[dev]) {
-        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             Cfg<1>::SMEM_BYTES);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     Cfg<2>::SMEM_BYTES);
         if (e != cudaSuccess) return e;
         attr_done[dev] = true;
     }
+    // 256 x 512 cluster tiles unless the rectangle is narrow (PDL_OZ_NSUB=1|2 overrides).
+    // Exact INT32 sums: the tile shape does not change a bit of C.
+    int nsub = cols > 256 ? 2 : 1;
+    if (const char *e = getenv("PDL_OZ_NSUB")) nsub = atoi(e) == 1 ? 1 : 2;
+    const int BN = nsub == 2 ? Cfg<2>::BN : Cfg<1>::BN;
     const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + BN - 1) / BN);
     const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
     int first = 1;
@@ -385,9 +409,14 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
             if (!map_i8(enc, &ta, a, (uint64_t)kd, (uint64_t)rows, (uint64_t)L.ld8, BM) ||
                 !map_i8(enc, &tb, b, (uint64_t)kd, (uint64_t)cols, (uint64_t)L.ld8, BNH))
                 return cudaErrorInvalidValue;
-            oz_gemm_2sm_kernel<<<2 * tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(
-                ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m, tiles_n,
-                raster_group_m(GROUP_M), vec_ok);
+            if (nsub == 2)
+                oz_gemm_2sm_kernel<2><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
+                    ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
+                    tiles_n, raster_group_m(GROUP_M), vec_ok);
+            else
+                oz_gemm_2sm_kernel<1><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
+                    ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
+                    tiles_n, raster_group_m(GROUP_M), vec_ok);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             first = 0;
