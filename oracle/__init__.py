@@ -48,8 +48,9 @@ def build(force: bool = False) -> str:
 def _load():
     global _lib
     if _lib is None:
-        build()
-        lib = ctypes.CDLL(_LIB)
+        # ORACLE_LIB: load another build of oracle.c (mutation tests only)
+        path = os.environ.get("ORACLE_LIB") or build()
+        lib = ctypes.CDLL(path)
         i64 = ctypes.c_int64
         vp = ctypes.c_void_p
         lib.oracle_matmul_rows.argtypes = [ctypes.c_int, vp, vp, i64, i64, i64,
