@@ -65,15 +65,17 @@ __device__ __forceinline__ double slice_q(double &v, int rn) {
 }
 
 // One CTA per row (grid-stride): A (M x K, lda) -> A8 rows [c][s][kk].
-__global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M, int64_t K, int S,
+// T = double (FP64 task) or float (FP32 task; promoted exactly to double).
+template <typename T>
+__global__ void oz_split_rows_kernel(const T *__restrict__ A, int64_t lda, int64_t M, int64_t K, int S,
                                      int64_t Kc, int nch, int8_t *__restrict__ A8, int64_t ld8,
                                      int *__restrict__ ea, int rn) {
     __shared__ double red[32];
     const int64_t Kpad = (int64_t)nch * Kc;
     for (int64_t i = blockIdx.x; i < M; i += gridDim.x) {
-        const double *row = A + i * lda;
+        const T *row = A + i * lda;
         double mx = 0.0;
-        for (int64_t k = threadIdx.x; k < K; k += blockDim.x) mx = fmax(mx, fabs(row[k]));
+        for (int64_t k = threadIdx.x; k < K; k += blockDim.x) mx = fmax(mx, fabs((double)row[k]));
         for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
         if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = mx;
         __syncthreads();
@@ -91,7 +93,7 @@ __global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, 
         for (int64_t k8 = (int64_t)threadIdx.x * 8; k8 < Kpad; k8 += (int64_t)blockDim.x * 8) {
             double v[8];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? ldexp(row[k8 + j], -e) : 0.0;
+            for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? ldexp((double)row[k8 + j], -e) : 0.0;
             const int64_t c = k8 / Kc, kk = k8 - c * Kc;
             int8_t *o = out + (c * S) * Kc + kk;
             for (int s = 0; s < S; ++s) {
@@ -109,21 +111,23 @@ __global__ void oz_split_rows_kernel(const double *__restrict__ A, int64_t lda, 
 }
 
 // Column max |b| of B (K x N): bits of the non-negative max via atomicMax.
-__global__ void oz_colmax_kernel(const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
+template <typename T>
+__global__ void oz_colmax_kernel(const T *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
                                  unsigned long long *__restrict__ bmax) {
     const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (n >= N) return;
     const int64_t k0 = (int64_t)blockIdx.y * 256, k1 = min(K, k0 + 256);
     double mx = 0.0;
-    for (int64_t k = k0; k < k1; ++k) mx = fmax(mx, fabs(B[k * ldb + n]));
+    for (int64_t k = k0; k < k1; ++k) mx = fmax(mx, fabs((double)B[k * ldb + n]));
     atomicMax(bmax + n, (unsigned long long)__double_as_longlong(mx));
 }
 
 // B (K x N) -> Bt8 (N rows of [c][S-1-s][kk]) through a 32 x 32 smem transpose.
 // Tile of 64 k x 32 n: coalesced loads along n into shared memory, then each
 // thread slices 8 consecutive k of one column -> one 8-byte store per slice.
+template <typename T>
 __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
-    const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S, int64_t Kc, int nch,
+    const T *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S, int64_t Kc, int nch,
     const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
     int rn) {
     __shared__ double t[64][33];
@@ -131,7 +135,7 @@ __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
     const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;   // 32 x 8
     for (int r = ty; r < 64; r += 8) {
         const int64_t k = k0 + r, n = n0 + tx;
-        t[r][tx] = (k < K && n < N) ? B[k * ldb + n] : 0.0;
+        t[r][tx] = (k < K && n < N) ? (double)B[k * ldb + n] : 0.0;
     }
     __syncthreads();
     const int64_t Kpad = (int64_t)nch * Kc;
@@ -193,10 +197,10 @@ __device__ __forceinline__ void umma_i8_2sm(uint32_t tmem_d, uint64_t adesc, uin
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
 }
 
-template <int NSUB>
+template <int NSUB, typename TC>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
     oz_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
-                       double *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
+                       TC *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
                        const int *__restrict__ fb, int scale_exp, int accumulate, int tiles_m, int tiles_n,
                        int group_m, int vec_ok) {
     using namespace koz;
@@ -286,7 +290,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
         const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
         const int cbase = tn * BN + cg * EPI_COLS;
         const int er = row < M ? ea[row] + scale_exp : 0;
-        double *crow = C + (int64_t)row * ldc + cbase;
+        TC *crow = C + (int64_t)row * ldc + cbase;
 #pragma unroll
         for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
             uint32_t r[16];
@@ -300,17 +304,29 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
                     v[j] = ldexp((double)(int32_t)r[j], er + f);   // exact: int32 -> f64, power-of-two scale
                 }
                 if (vec_ok && cbase + c0 + 16 <= N) {
+                    if constexpr (sizeof(TC) == 8) {
 #pragma unroll
-                    for (int j = 0; j < 16; j += 2) {
-                        double2 *p = reinterpret_cast<double2 *>(crow + c0 + j);
-                        // streaming (evict-first) C traffic keeps the slice panels in L2
-                        double2 o = accumulate ? __ldcs(p) : make_double2(0.0, 0.0);
-                        __stcs(p, make_double2(o.x + v[j], o.y + v[j + 1]));
+                        for (int j = 0; j < 16; j += 2) {
+                            double2 *p = reinterpret_cast<double2 *>(crow + c0 + j);
+                            // streaming (evict-first) C traffic keeps the slice panels in L2
+                            double2 o = accumulate ? __ldcs(p) : make_double2(0.0, 0.0);
+                            __stcs(p, make_double2(o.x + v[j], o.y + v[j + 1]));
+                        }
+                    } else {
+                        // FP32 task: each diagonal adds in double and rounds once to float
+#pragma unroll
+                        for (int j = 0; j < 16; j += 4) {
+                            float4 *p = reinterpret_cast<float4 *>(crow + c0 + j);
+                            float4 o = accumulate ? __ldcs(p) : make_float4(0.f, 0.f, 0.f, 0.f);
+                            __stcs(p, make_float4((float)((double)o.x + v[j]), (float)((double)o.y + v[j + 1]),
+                                                  (float)((double)o.z + v[j + 2]), (float)((double)o.w + v[j + 3])));
+                        }
                     }
                 } else {
 #pragma unroll
                     for (int j = 0; j < 16; ++j)
-                        if (cbase + c0 + j < N) crow[c0 + j] = (accumulate ? crow[c0 + j] : 0.0) + v[j];
+                        if (cbase + c0 + j < N)
+                            crow[c0 + j] = (TC)((accumulate ? (double)crow[c0 + j] : 0.0) + v[j]);
                 }
             }
         }
@@ -339,27 +355,46 @@ OzakiLayout ozaki_layout(int64_t rows, int64_t cols, int64_t K, int S) {
     return L;
 }
 
-cudaError_t launch_ozaki_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
-                                 int8_t *A8, int *ea, cudaStream_t s) {
+template <typename T>
+static cudaError_t split_a_impl(const T *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L, int8_t *A8,
+                                int *ea, cudaStream_t s) {
     if (rows <= 0) return cudaSuccess;
     int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
-    oz_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, L.S, L.Kc, L.nch, A8, L.ld8, ea, L.rn);
+    oz_split_rows_kernel<T><<<blocks, 256, 0, s>>>(A, lda, rows, K, L.S, L.Kc, L.nch, A8, L.ld8, ea, L.rn);
     return cudaGetLastError();
 }
 
-cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
-                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s) {
+template <typename T>
+static cudaError_t split_b_impl(const T *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L, int8_t *Bt8,
+                                int *fb, unsigned long long *bmax, cudaStream_t s) {
     if (cols <= 0) return cudaSuccess;
     cudaError_t e = cudaMemsetAsync(bmax, 0, (size_t)cols * sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
     if (K > 0) {
         dim3 g1((unsigned)((cols + 255) / 256), (unsigned)((K + 255) / 256));
-        oz_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
+        oz_colmax_kernel<T><<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
     }
     const int64_t Kpad = (int64_t)L.nch * L.Kc;
     dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 63) / 64));
-    oz_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb, L.rn);
+    oz_split_cols_t_kernel<T><<<g2, 256, 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb, L.rn);
     return cudaGetLastError();
+}
+
+cudaError_t launch_ozaki_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
+                                 int8_t *A8, int *ea, cudaStream_t s) {
+    return split_a_impl(A, lda, rows, K, L, A8, ea, s);
+}
+cudaError_t launch_ozaki_split_a(const float *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
+                                 int8_t *A8, int *ea, cudaStream_t s) {
+    return split_a_impl(A, lda, rows, K, L, A8, ea, s);
+}
+cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
+                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s) {
+    return split_b_impl(B, ldb, K, cols, L, Bt8, fb, bmax, s);
+}
+cudaError_t launch_ozaki_split_b(const float *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
+                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s) {
+    return split_b_impl(B, ldb, K, cols, L, Bt8, fb, bmax, s);
 }
 
 static bool map_i8(EncodeTiledFn enc, CUtensorMap *m, const int8_t *ptr, uint64_t kd, uint64_t rows, uint64_t ld,
@@ -375,19 +410,20 @@ static bool map_i8(EncodeTiledFn enc, CUtensorMap *m, const int8_t *ptr, uint64_
 
 // All diagonals and K chunks of one rectangle: S * nch int8 GEMM launches,
 // smallest diagonal first; the first launch overwrites C.
-cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
-                              const OzakiLayout &L, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                              cudaStream_t stream, int *launches) {
+template <typename TC>
+static cudaError_t gemm_impl(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
+                             const OzakiLayout &L, TC *C, int64_t ldc, int64_t rows, int64_t cols, cudaStream_t stream,
+                             int *launches) {
     using namespace koz;
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     int dev = 0;
     cudaGetDevice(&dev);
     static bool attr_done[64] = {false};
     if (dev < 64 && !attr_done[dev]) {
-        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1, TC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              Cfg<1>::SMEM_BYTES);
         if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<2, TC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      Cfg<2>::SMEM_BYTES);
         if (e != cudaSuccess) return e;
         attr_done[dev] = true;
@@ -398,7 +434,7 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
     if (const char *e = getenv("PDL_OZ_NSUB")) nsub = atoi(e) == 1 ? 1 : 2;
     const int BN = nsub == 2 ? Cfg<2>::BN : Cfg<1>::BN;
     const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + BN - 1) / BN);
-    const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
+    const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && ((ldc * sizeof(TC)) & 15) == 0) ? 1 : 0;
     int first = 1;
     for (int c = 0; c < L.nch; ++c) {
         for (int d = L.S - 1; d >= 0; --d) {
@@ -410,11 +446,11 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
                 !map_i8(enc, &tb, b, (uint64_t)kd, (uint64_t)cols, (uint64_t)L.ld8, BNH))
                 return cudaErrorInvalidValue;
             if (nsub == 2)
-                oz_gemm_2sm_kernel<2><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
+                oz_gemm_2sm_kernel<2, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
                     ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
                     tiles_n, raster_group_m(GROUP_M), vec_ok);
             else
-                oz_gemm_2sm_kernel<1><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
+                oz_gemm_2sm_kernel<1, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
                     ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
                     tiles_n, raster_group_m(GROUP_M), vec_ok);
             cudaError_t e = cudaGetLastError();
@@ -424,6 +460,17 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
         }
     }
     return cudaSuccess;
+}
+
+cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
+                              const OzakiLayout &L, double *C, int64_t ldc, int64_t rows, int64_t cols,
+                              cudaStream_t stream, int *launches) {
+    return gemm_impl(enc, A8, Bt8, ea, fb, L, C, ldc, rows, cols, stream, launches);
+}
+cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
+                              const OzakiLayout &L, float *C, int64_t ldc, int64_t rows, int64_t cols,
+                              cudaStream_t stream, int *launches) {
+    return gemm_impl(enc, A8, Bt8, ea, fb, L, C, ldc, rows, cols, stream, launches);
 }
 
 }  // namespace pdlk

@@ -53,6 +53,15 @@ cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_
 cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
                               const OzakiLayout &L, double *C, int64_t ldc, int64_t rows, int64_t cols,
                               cudaStream_t stream, int *launches);
+// FP32 task variant on the same machinery: FP32 inputs promoted exactly, each
+// diagonal added in double and rounded once into the FP32 C.
+cudaError_t launch_ozaki_split_a(const float *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
+                                 int8_t *A8, int *ea, cudaStream_t s);
+cudaError_t launch_ozaki_split_b(const float *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
+                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s);
+cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
+                              const OzakiLayout &L, float *C, int64_t ldc, int64_t rows, int64_t cols,
+                              cudaStream_t stream, int *launches);
 
 // K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,

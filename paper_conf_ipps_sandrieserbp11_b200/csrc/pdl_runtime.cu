@@ -400,20 +400,24 @@ int ensure_aux(WorkerCtx &w) {
     return PDL_OK;
 }
 
-// FP64 task variant of a Worker: PDL property DGEMM_VARIANT ("dmma" default |
-// "ozaki") and OZAKI_SLICES (2..8, default 7); env PDL_DGEMM_VARIANT /
-// PDL_OZAKI_SLICES override the descriptor (tests, bench).
-bool worker_ozaki(const WorkerCtx &w, int *slices, int *rn) {
+// Task variant of a Worker (task repository + static pre-selection, L1307-1326):
+//   FP64: PDL property DGEMM_VARIANT ("dmma" default | "ozaki"), OZAKI_SLICES (default 6)
+//   FP32: PDL property SGEMM_VARIANT ("3xtf32" default | "ozaki"), OZAKI_SLICES_F32 (default 4)
+// OZAKI_ROUNDING ("nearest" default | "trunc") for both; env PDL_<NAME> overrides
+// the descriptor (tests, bench).
+bool worker_ozaki(const WorkerCtx &w, bool f64, int *slices, int *rn) {
+    const char *vname = f64 ? "DGEMM_VARIANT" : "SGEMM_VARIANT";
+    const char *sname = f64 ? "OZAKI_SLICES" : "OZAKI_SLICES_F32";
     std::string v;
-    if (const char *e = getenv("PDL_DGEMM_VARIANT")) v = e;
-    else if (const Property *p = g->model.prop(w.pu, "DGEMM_VARIANT")) v = p->value;
+    if (const char *e = getenv((std::string("PDL_") + vname).c_str())) v = e;
+    else if (const Property *p = g->model.prop(w.pu, vname)) v = p->value;
     if (lower(trim(v)) != "ozaki") return false;
-    // Defaults from the measured accuracy sweep (profiles/r01_ozaki_accuracy.txt,
-    // K = 16384): round-to-nearest slices, S = 6 -> max scaled error 3.7e-14
+    // Defaults from the measured accuracy sweeps (profiles/r01_ozaki_accuracy*.txt,
+    // K = 16384): FP64 -- round-to-nearest slices, S = 6 -> max scaled error 3.7e-14
     // (truncation needs S = 7 for 3.0e-14; truncation S = 6 gives 1.6e-12).
-    int s = 6;
-    if (const char *e = getenv("PDL_OZAKI_SLICES")) s = atoi(e);
-    else if (const Property *p = g->model.prop(w.pu, "OZAKI_SLICES")) s = atoi(p->value.c_str());
+    int s = f64 ? 6 : 4;
+    if (const char *e = getenv((std::string("PDL_") + sname).c_str())) s = atoi(e);
+    else if (const Property *p = g->model.prop(w.pu, sname)) s = atoi(p->value.c_str());
     *slices = std::max(2, std::min(8, s));
     // OZAKI_ROUNDING: "nearest" (default) | "trunc"
     std::string r;
@@ -491,10 +495,16 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         if ((rc = ensure_buf(w, BUF_C, (size_t)(ldcd * rows * es), &p))) return rc;
         Cd = (char *)p;
     }
+    // Task variant of this Worker, pre-selected from its PDL properties (task
+    // repository + static pre-selection, L1307-1326): FP64 K1 (DMMA) or K4
+    // (Ozaki), FP32 K3+K2 (3xTF32) or K4 (Ozaki).
+    int oz_slices = 0;
+    int oz_rn = 0;
+    const bool ozaki = K > 0 && worker_ozaki(w, f64, &oz_slices, &oz_rn);
     // FP32 split buffers (K-major hi/lo of A rows and of B^T rows)
     const int64_t Kp = round_up(std::max<int64_t>(K, 1), pdlk::K2_BK);
     float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
-    if (!f64 && K > 0) {
+    if (!f64 && K > 0 && !ozaki) {
         if ((rc = ensure_buf(w, BUF_AHI, (size_t)(rows * Kp * 4), &p))) return rc;
         ahi = (float *)p;
         if ((rc = ensure_buf(w, BUF_ALO, (size_t)(rows * Kp * 4), &p))) return rc;
@@ -509,11 +519,6 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     const char *k2v = getenv("PDL_K2");
     const bool k2_1sm = k2v && !strcmp(k2v, "1sm");
 
-    // DGEMM task variant of this Worker, pre-selected from its PDL properties
-    // (task repository + static pre-selection, L1307-1326): K1 (DMMA) or K4 (Ozaki).
-    int oz_slices = 0;
-    int oz_rn = 0;
-    const bool ozaki = f64 && K > 0 && worker_ozaki(w, &oz_slices, &oz_rn);
     pdlk::OzakiLayout OL;
     int8_t *a8 = nullptr, *b8 = nullptr;
     int *oz_ea = nullptr, *oz_fb = nullptr;
@@ -589,8 +594,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             } else if (ozaki) {
                 // K5 slicing of this band / panel once, shared by both compute streams
                 if (j == 0) {
-                    e = pdlk::launch_ozaki_split_a((const double *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K, OL,
-                                                   a8 + r0 * OL.ld8, oz_ea + r0, cs);
+                    const char *Ab = Ad + (size_t)(r0 * lda) * es;
+                    e = f64 ? pdlk::launch_ozaki_split_a((const double *)Ab, lda, nr, K, OL, a8 + r0 * OL.ld8,
+                                                         oz_ea + r0, cs)
+                            : pdlk::launch_ozaki_split_a((const float *)Ab, lda, nr, K, OL, a8 + r0 * OL.ld8,
+                                                         oz_ea + r0, cs);
                     w.launches += 1;
                     if (piped) {
                         ev_sa[i] = ev_get(w, evn);
@@ -600,8 +608,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                     CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
                 }
                 if (e == cudaSuccess && i == 0 && !b_ready) {
-                    e = pdlk::launch_ozaki_split_b((const double *)(Bd + (size_t)c0 * es), ldb, K, nc, OL,
-                                                   b8 + c0 * OL.ld8, oz_fb + c0, oz_bmax + c0, cs);
+                    const char *Bp = Bd + (size_t)c0 * es;
+                    e = f64 ? pdlk::launch_ozaki_split_b((const double *)Bp, ldb, K, nc, OL, b8 + c0 * OL.ld8,
+                                                         oz_fb + c0, oz_bmax + c0, cs)
+                            : pdlk::launch_ozaki_split_b((const float *)Bp, ldb, K, nc, OL, b8 + c0 * OL.ld8,
+                                                         oz_fb + c0, oz_bmax + c0, cs);
                     w.launches += 2;
                     if (piped) {
                         ev_sb[j] = ev_get(w, evn);
@@ -613,8 +624,10 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (e != cudaSuccess) return set_err(PDL_ECUDA, "K5 slicing launch failed: %s", cudaGetErrorString(e));
                 if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
                 int nl = 0;
-                e = pdlk::launch_ozaki_gemm(enc, a8 + r0 * OL.ld8, b8 + c0 * OL.ld8, oz_ea + r0, oz_fb + c0, OL,
-                                            (double *)Cs, ldcd, nr, nc, cs, &nl);
+                e = f64 ? pdlk::launch_ozaki_gemm(enc, a8 + r0 * OL.ld8, b8 + c0 * OL.ld8, oz_ea + r0, oz_fb + c0,
+                                                  OL, (double *)Cs, ldcd, nr, nc, cs, &nl)
+                        : pdlk::launch_ozaki_gemm(enc, a8 + r0 * OL.ld8, b8 + c0 * OL.ld8, oz_ea + r0, oz_fb + c0,
+                                                  OL, (float *)Cs, ldcd, nr, nc, cs, &nl);
                 if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
                 w.launches += nl;
             } else if (f64) {

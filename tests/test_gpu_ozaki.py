@@ -137,6 +137,58 @@ def test_slice_count_accuracy(slices, rounding, tol):
     check(oz_matmul(A, B, slices=slices, rounding=rounding), A, B, tol=tol)
 
 
+def oz32_matmul(A, B, tile=0, workers=1, host=False, slices=None):
+    props = {"SGEMM_VARIANT": "ozaki"}
+    if slices:
+        props["OZAKI_SLICES_F32"] = slices
+    pdl.load(pdl.descriptor_xml(workers, props=props))
+    try:
+        M, N = A.shape[0], B.shape[1]
+        if host:
+            C = np.full((M, N), np.nan, dtype=np.float32)
+            pdl.task_matmul(A, B, C, tile=tile)
+            pdl.run()
+            return C
+        dA, dB = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+        dC = torch.full((M, N), float("nan"), dtype=torch.float32, device="cuda")
+        pdl.task_matmul(dA, dB, dC, tile=tile)
+        pdl.run()
+        return dC.cpu().numpy()
+    finally:
+        pdl.unload()
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3"])
+def test_fp32_ozaki_configs(name):
+    """FP32 task variant SGEMM_VARIANT = ozaki (INT8 slices of the FP32
+    inputs, FP32 C) at the 1e-5 bar."""
+    c = W.CONFIGS[name]
+    A, B = W.config_inputs(name, np.float32)
+    C = oz32_matmul(A, B, tile=c.tile)
+    rows = None if c.M <= 1024 else W.sampled_rows(c.M, (), c.tile, n_random=32)
+    check(C, A, B, rows=rows, tol=1e-5)
+
+
+@pytest.mark.parametrize("slices,tol", [(3, 1e-5), (4, 2e-6)])
+def test_fp32_ozaki_k_sweep(slices, tol, capsys):
+    for K in (256, 4096, 16384):
+        A = W.uniform((128, K), np.float32, 71)
+        B = W.signed((K, 192), np.float32, 72)
+        err = check(oz32_matmul(A, B, slices=slices), A, B, tol=tol)
+        with capsys.disabled():
+            print(f"\n[fp32 ozaki S={slices}] K={K} max_err={err:.3e}")
+
+
+def test_fp32_ozaki_invariance_bitwise(monkeypatch):
+    A = W.uniform((700, 390), np.float32, 81)
+    B = W.uniform((390, 333), np.float32, 82)
+    ref = oz32_matmul(A, B)
+    check(ref, A, B, tol=1e-5)
+    assert np.array_equal(oz32_matmul(A, B, tile=64, workers=4), ref)
+    monkeypatch.setenv("PDL_PIPELINE", "force")
+    assert np.array_equal(oz32_matmul(A, B, host=True), ref)
+
+
 @pytest.mark.slow
 def test_c4_full_size_sampled():
     c = W.CONFIGS["C4"]
