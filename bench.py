@@ -65,10 +65,11 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cublas", action="store_true")
-    p.add_argument("--variant", choices=("dmma", "ozaki"), default="dmma",
-                   help="FP64 DGEMM task variant (PDL DGEMM_VARIANT): K1 DMMA or K4 Ozaki INT8")
-    p.add_argument("--slices", type=int, default=6,
-                   help="OZAKI_SLICES for --variant ozaki (round-to-nearest slices)")
+    p.add_argument("--variant", choices=("default", "ozaki"), default="default",
+                   help="task variant pinned in the PDL descriptor: default (FP64 K1 DMMA / FP32 K3+K2 3xTF32) "
+                        "or ozaki (K4/K5 INT8 slices; DGEMM_VARIANT / SGEMM_VARIANT)")
+    p.add_argument("--slices", type=int, default=None,
+                   help="Ozaki slices (default 6 for FP64, 3 for FP32; round-to-nearest)")
     p.add_argument("--no-alt", action="store_true", help="skip timing the other FP64 variant")
     p.add_argument("--dist-backend", choices=("nccl", "gloo"), default="nccl",
                    help="gloo only to validate the N>1 flow with ranks sharing one GPU")
@@ -170,6 +171,15 @@ def ncu_traffic(dtype, cfg):
         return d.get(f"{dtype}/{cfg}")
     except (OSError, ValueError):
         return None
+
+
+def variant_descriptor(pdl, world, dtype, ozaki, S):
+    """PDL descriptor XML with the task variant pinned as Worker properties."""
+    if not ozaki:
+        return pdl.descriptor_xml(world)
+    if dtype == "f64":
+        return pdl.descriptor_xml(world, "ozaki", S)
+    return pdl.descriptor_xml(world, props={"SGEMM_VARIANT": "ozaki", "OZAKI_SLICES_F32": S})
 
 
 def ozaki_ops(rows, cols, K, S):
@@ -281,10 +291,11 @@ def main():
     es = 8 if args.dtype == "f64" else 4
     A, B = host_inputs(args.config, np_dtype)
 
-    ozaki = args.dtype == "f64" and args.variant == "ozaki"
-    # the DGEMM task variant is pre-selected through the Worker's PDL properties (L1316-1326)
-    desc = pdl.descriptor_xml(world, args.variant if args.dtype == "f64" else None,
-                              args.slices if ozaki else None)
+    ozaki = args.variant == "ozaki"
+    S = args.slices or (6 if args.dtype == "f64" else 3)
+    args.slices = S
+    # the task variant is pre-selected through the Worker's PDL properties (L1316-1326)
+    desc = variant_descriptor(pdl, world, args.dtype, ozaki, S)
     if world == 1:
         pdl.load(desc)
     else:
@@ -365,7 +376,8 @@ def main():
     roofline = {"bound": "tensor", "achieved": round(achieved_tf, 2) if achieved_tf else None,
                 "peak": round(peak_tf, 1), "unit": "TFLOP/s",
                 "frac": round(achieved_tf / peak_tf, 4) if achieved_tf else None,
-                "traffic": ncu_traffic("ozaki" if ozaki else args.dtype, args.config),
+                "traffic": ncu_traffic(("ozaki" if args.dtype == "f64" else "ozaki32") if ozaki else args.dtype,
+                                       args.config),
                 "kernel": kname,
                 "kernel_ms": round(kavg, 3) if kavg else None,
                 "algorithmic_flops_per_launch": pipe_flops,
@@ -448,11 +460,11 @@ def main():
         torch.cuda.synchronize()
         cublas = round(flops_total * 3 / (t0.elapsed_time(t1) / 1e3) / 1e9, 1)
 
-    # ---- the other FP64 task variant on the same resident operands (PDL-selected) ----
+    # ---- the Ozaki task variant on the same resident operands (PDL-selected) ----
     alt = None
-    if world == 1 and args.dtype == "f64" and args.variant == "dmma" and not args.no_alt:
+    if world == 1 and not ozaki and not args.no_alt:
         pdl.unload()
-        pdl.load(pdl.descriptor_xml(1, "ozaki", args.slices))
+        pdl.load(variant_descriptor(pdl, 1, args.dtype, True, args.slices))
         pdl.set_stream(stream)
         for _ in range(2):
             step()
@@ -472,14 +484,16 @@ def main():
         aops, akname = ozaki_ops(M, N, K, args.slices)
         apeak, apsrc, _ = tensor_peak("i8")
         aach = aops / (float(np.mean(akt)) / 1e3) / 1e12 if akt else None
-        alt = {"variant": f"ozaki: FP64 DGEMM on INT8 tcgen05 ({args.slices} slices, K4/K5)",
-               "dtype": f"f64-ozaki-i8x{args.slices}",
+        tol = "1e-12" if args.dtype == "f64" else "1e-5"
+        alt = {"variant": f"ozaki: {args.dtype.upper()} matmul on INT8 tcgen05 ({args.slices} slices, K4/K5)",
+               "dtype": f"{args.dtype}-ozaki-i8x{args.slices}",
                "value": round(flops_total * args.steps / (ams / 1e3) / 1e9, 1), "unit": "GFLOP/s",
                "ms_per_step": round(ams / args.steps, 3),
-               "parity": "max scaled err <= 1e-12 vs oracle (tests/test_gpu_ozaki.py, incl. C4 sampled rows)",
+               "parity": f"max scaled err <= {tol} vs oracle (tests/test_gpu_ozaki.py)",
                "roofline": {"bound": "tensor", "achieved": round(aach, 1) if aach else None,
                             "peak": apeak, "unit": "TFLOP/s", "frac": round(aach / apeak, 4) if aach else None,
-                            "traffic": ncu_traffic("ozaki", args.config), "kernel": akname,
+                            "traffic": ncu_traffic("ozaki" if args.dtype == "f64" else "ozaki32", args.config),
+                            "kernel": akname,
                             "kernel_ms": round(float(np.mean(akt)), 3) if akt else None,
                             "peak_source": apsrc},
                "clocks": clk2.summary()}
@@ -493,7 +507,7 @@ def main():
             "metric": METRIC, "value": round(value, 1), "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-            "dtype": f"f64-ozaki-i8x{args.slices}" if ozaki else args.dtype,
+            "dtype": f"{args.dtype}-ozaki-i8x{args.slices}" if ozaki else args.dtype,
             "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} ({args.dtype})",
             "config": {"workload": f"{args.config} {M}x{N}x{K} blocked matmul, task tile {c.tile}, "
                                    f"PDL b200_x{world}",

@@ -402,7 +402,7 @@ int ensure_aux(WorkerCtx &w) {
 
 // Task variant of a Worker (task repository + static pre-selection, L1307-1326):
 //   FP64: PDL property DGEMM_VARIANT ("dmma" default | "ozaki"), OZAKI_SLICES (default 6)
-//   FP32: PDL property SGEMM_VARIANT ("3xtf32" default | "ozaki"), OZAKI_SLICES_F32 (default 4)
+//   FP32: PDL property SGEMM_VARIANT ("3xtf32" default | "ozaki"), OZAKI_SLICES_F32 (default 3)
 // OZAKI_ROUNDING ("nearest" default | "trunc") for both; env PDL_<NAME> overrides
 // the descriptor (tests, bench).
 bool worker_ozaki(const WorkerCtx &w, bool f64, int *slices, int *rn) {
@@ -412,10 +412,11 @@ bool worker_ozaki(const WorkerCtx &w, bool f64, int *slices, int *rn) {
     if (const char *e = getenv((std::string("PDL_") + vname).c_str())) v = e;
     else if (const Property *p = g->model.prop(w.pu, vname)) v = p->value;
     if (lower(trim(v)) != "ozaki") return false;
-    // Defaults from the measured accuracy sweeps (profiles/r01_ozaki_accuracy*.txt,
-    // K = 16384): FP64 -- round-to-nearest slices, S = 6 -> max scaled error 3.7e-14
-    // (truncation needs S = 7 for 3.0e-14; truncation S = 6 gives 1.6e-12).
-    int s = f64 ? 6 : 4;
+    // Defaults from the measured accuracy sweeps (profiles/r01_ozaki_accuracy*.txt):
+    // FP64 -- round-to-nearest slices, S = 6 -> max scaled error 3.7e-14 at K = 16384
+    // (truncation needs S = 7 for 3.0e-14; truncation S = 6 gives 1.6e-12);
+    // FP32 -- S = 3 (8+7+7 bits) -> max 3.3e-7 (K = 256) .. 4.3e-8 (K = 16384), 1e-5 bar.
+    int s = f64 ? 6 : 3;
     if (const char *e = getenv((std::string("PDL_") + sname).c_str())) s = atoi(e);
     else if (const Property *p = g->model.prop(w.pu, sname)) s = atoi(p->value.c_str());
     *slices = std::max(2, std::min(8, s));
