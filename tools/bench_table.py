@@ -24,10 +24,19 @@ import workloads as W  # noqa: E402
 from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
 
 ROWS = [("C1", "f64", 1, None), ("C1", "f32", 1, None), ("C2", "f64", 1, None), ("C2", "f32", 1, None),
-        ("C2", "f64", 1, "ozaki"), ("C3", "f64", 2, None), ("C3", "f64", 4, None), ("C3", "f32", 4, None),
-        ("C3", "f64", 4, "ozaki"), ("C0", "f64", 1, None), ("C0", "f64", 2, None), ("C0", "f64", 2, "ozaki"),
-        ("C4", "f64", 1, None), ("C4", "f32", 1, None), ("C4", "f64", 1, "ozaki"),
-        ("C5", "f64", 8, None), ("C5", "f32", 8, None), ("C5", "f64", 8, "ozaki")]
+        ("C2", "f64", 1, "ozaki"), ("C2", "f32", 1, "ozaki"), ("C3", "f64", 2, None), ("C3", "f64", 4, None),
+        ("C3", "f32", 4, None), ("C3", "f64", 4, "ozaki"), ("C3", "f32", 4, "ozaki"), ("C0", "f64", 1, None),
+        ("C0", "f64", 2, None), ("C0", "f64", 2, "ozaki"),
+        ("C4", "f64", 1, None), ("C4", "f32", 1, None), ("C4", "f64", 1, "ozaki"), ("C4", "f32", 1, "ozaki"),
+        ("C5", "f64", 8, None), ("C5", "f32", 8, None), ("C5", "f64", 8, "ozaki"), ("C5", "f32", 8, "ozaki")]
+
+
+def descriptor(G, dt, variant):
+    if variant != "ozaki":
+        return pdl.descriptor_xml(G)
+    if dt == "f64":
+        return pdl.descriptor_xml(G, "ozaki")
+    return pdl.descriptor_xml(G, props={"SGEMM_VARIANT": "ozaki"})
 
 
 def timed(fn, steps, stream):
@@ -48,7 +57,7 @@ def run_row(cfg, dt, G, variant, steps):
     A, B = W.config_inputs(cfg, npdt)
     flops = 2.0 * c.M * c.N * c.K
     os.environ["PDL_ALLOW_OVERSUBSCRIBE"] = "1"
-    pdl.load(pdl.descriptor_xml(G, variant))
+    pdl.load(descriptor(G, dt, variant))
     stream = torch.cuda.current_stream()
     pdl.set_stream(stream)
     try:
