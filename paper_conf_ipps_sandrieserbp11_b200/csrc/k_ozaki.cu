@@ -430,7 +430,10 @@ static cudaError_t gemm_impl(EncodeTiledFn enc, const int8_t *A8, const int8_t *
     }
     // 256 x 512 cluster tiles unless the rectangle is narrow (PDL_OZ_NSUB=1|2 overrides).
     // Exact INT32 sums: the tile shape does not change a bit of C.
-    int nsub = cols > 256 ? 2 : 1;
+    // 256 x 512 only when it still gives >= 2 waves of CTA pairs (148 clusters);
+    // small rectangles keep 256 x 256 for parallelism
+    const int64_t clusters512 = ((rows + 2 * BM - 1) / (2 * BM)) * ((cols + 511) / 512);
+    int nsub = (cols > 256 && clusters512 >= 148) ? 2 : 1;
     if (const char *e = getenv("PDL_OZ_NSUB")) nsub = atoi(e) == 1 ? 1 : 2;
     const int BN = nsub == 2 ? Cfg<2>::BN : Cfg<1>::BN;
     const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + BN - 1) / BN);
