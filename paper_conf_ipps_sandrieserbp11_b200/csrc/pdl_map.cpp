@@ -129,14 +129,30 @@ Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec di
     bool hetero = false;
     if (speeds && (int)speeds->size() == G && dist.kind == Dist::Block)
         for (double s : *speeds) hetero |= (s != (*speeds)[0]);
-    // Worker grid: minimise per-Worker received elements, ties -> larger Gr.
-    double best = std::numeric_limits<double>::infinity();
-    for (int gr = G; gr >= 1; --gr) {
+    // Worker grid for the overlapped exchange (runtime.exchange_overlapped): the B
+    // column-panel all-gather is exposed, the A chunks stream in behind the
+    // Worker's own chunk.  Choose Gr x Gc = G with Gc <= 4 (the own chunk is >= 1/4
+    // of the Worker's work, enough to hide the other A chunks) minimising the
+    // received B elements K*(N/Gc)*(1 - 1/Gr); ties -> fewer received elements in
+    // total, then smaller Gr.  (G = 2: 1x2, 4: 1x4, 8: 2x4.)
+    double best_b = std::numeric_limits<double>::infinity(), best_tot = best_b;
+    for (int gr = 1; gr <= G; ++gr) {
         if (G % gr) continue;
-        int gc = G / gr;
-        double cost = (double(M) / gr) * double(K) * (1.0 - 1.0 / gc) +
-                      double(K) * (double(N) / gc) * (1.0 - 1.0 / gr);
-        if (cost < best * (1.0 - 1e-12)) { best = cost; p.Gr = gr; p.Gc = gc; }
+        const int gc = G / gr;
+        if (gc > 4 && gr < G) {
+            bool alt = false;   // only skip if some grid with gc <= 4 exists
+            for (int g2 = gr + 1; g2 <= G; ++g2)
+                if (G % g2 == 0 && G / g2 <= 4) alt = true;
+            if (alt) continue;
+        }
+        const double b = double(K) * (double(N) / gc) * (1.0 - 1.0 / gr);
+        const double tot = (double(M) / gr) * double(K) * (1.0 - 1.0 / gc) + b;
+        if (b < best_b * (1.0 - 1e-12) || (b <= best_b * (1.0 + 1e-12) && tot < best_tot * (1.0 - 1e-12))) {
+            best_b = b;
+            best_tot = tot;
+            p.Gr = gr;
+            p.Gc = gc;
+        }
     }
     if (hetero) {
         p.Gr = G;

@@ -129,9 +129,9 @@ struct Plan {
     std::string to_json(const std::vector<int> &workers, const std::vector<std::string> &ids) const;
 };
 
-// Choose Gr x Gc = G minimising received operand elements
-//   (M/Gr)*K*(1 - 1/Gc) + K*(N/Gc)*(1 - 1/Gr)   per Worker;
-// ties -> larger Gr.  BLOCK distributes task rows / cols (L1200-1206): grid row
+// Choose Gr x Gc = G (Gc <= 4) minimising the exposed exchange, the received B
+// elements K*(N/Gc)*(1 - 1/Gr) (the A chunks overlap the kernels); ties -> fewer
+// received elements in total, then smaller Gr.  BLOCK distributes task rows / cols (L1200-1206): grid row
 // r gets task rows [floor(r*Tm/Gr), floor((r+1)*Tm/Gr)); CYCLIC / BLOCK-CYCLIC:b
 // give grid row r the b-task blocks q with q % Gr == r (columns likewise).
 //

@@ -169,10 +169,11 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
     The B column-panel is all-gathered first (every C row needs it).  The A
     row-panel then arrives as Gc asynchronous broadcasts inside the grid row,
     one per owner; `compute(j, lo, hi, Apanel_rows, Bpanel, first)` runs on
-    the Worker's own chunk first, then on chunk j as soon as its broadcast has
+    the Worker's own chunk first (no wait), then on the chunks before it and
+    the chunks after it, each group as one launch once its broadcasts have
     landed (the stream waits on the NCCL work, the host does not), so the
-    remaining (Gc-1)/Gc of the A traffic hides behind the kernels.  Results are
-    bitwise identical to the non-overlapped path (R14)."""
+    other (Gc-1)/Gc of the A traffic hides behind the own-chunk kernel.
+    Results are bitwise identical to the non-overlapped path (R14)."""
     if wp.Gr > 1:
         _all_gather(bufs.B, Bch, grid.col_group)
     else:
@@ -184,13 +185,20 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
     if wp.Gc > 1:
         for j in range(wp.Gc):   # same order on every rank of the row
             works[j] = _broadcast(bufs.A[j * qa:(j + 1) * qa], grid.row_ranks[j], grid.row_group)
+    # Compute in at most three launches so each stays wave-efficient: the own
+    # chunk at once, then the chunks before it (broadcast first, so they land
+    # first), then the chunks after it.
+    groups = [[c], list(range(0, c)), list(range(c + 1, wp.Gc))]
     first = True
-    for j in [c] + [x for x in range(wp.Gc) if x != c]:
-        lo, hi = chunk_rows(wp, j)
-        if j != c and j in works:
-            works[j].wait()
+    for grp in groups:
+        if not grp:
+            continue
+        for j in grp:
+            if j != c and j in works:
+                works[j].wait()
+        lo, hi = chunk_rows(wp, grp[0])[0], chunk_rows(wp, grp[-1])[1]
         if hi > lo and wp.cols > 0:
-            compute(j, lo, hi, bufs.A[lo:hi], Bp, first)
+            compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first)
             first = False
     for w in works.values():
         w.wait()

@@ -190,6 +190,26 @@ def test_fp32_ozaki_invariance_bitwise(monkeypatch):
 
 
 @pytest.mark.slow
+def test_fp32_c4_full_size_sampled():
+    c = W.CONFIGS["C4"]
+    A, B = W.config_inputs("C4", np.float32)
+    C = oz32_matmul(A, B, tile=c.tile)
+    check(C, A, B, rows=W.sampled_rows(c.M, (), c.tile, n_random=12), tol=1e-5)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("dt", ["f64", "f32"])
+def test_c5_ragged_8_workers(dt):
+    """C5 ragged (10000x7000x3000, tile 128) on 8 oversubscribed Workers."""
+    c = W.CONFIGS["C5"]
+    npdt = np.float64 if dt == "f64" else np.float32
+    A, B = W.config_inputs("C5", npdt)
+    C = oz_matmul(A, B, tile=c.tile, workers=8) if dt == "f64" else oz32_matmul(A, B, tile=c.tile, workers=8)
+    rows = W.sampled_rows(c.M, (1248, 2496, 3744, 5008, 6256, 7504, 8752), c.tile, n_random=24)
+    check(C, A, B, rows=rows, tol=1e-12 if dt == "f64" else 1e-5)
+
+
+@pytest.mark.slow
 def test_c4_full_size_sampled():
     c = W.CONFIGS["C4"]
     A, B = W.config_inputs("C4", np.float64)

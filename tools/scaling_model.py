@@ -1,0 +1,68 @@
+"""Strong-scaling model of the multi-Worker path (NVLink scaling is not
+measurable with one GPU per gpurun call; this predicts it from measured parts).
+
+Per Worker (plan from libpdl, dry run): compute time = its FLOPs / the measured
+single-B200 rate of the task variant (profiles/r01_bench_table.jsonl, C4);
+exchange = B column-panel all-gather (exposed) + A-chunk broadcasts overlapped
+with the chunk kernels (exposed only if a chunk transfer outlasts the previous
+chunk's compute).  NVLink: 770 GB/s per direction per GPU (the measured peer
+copy bandwidth quoted in /opt/skills/guides/B200_PROFILING.md), all-gather
+received bytes at that rate.
+
+    python tools/scaling_model.py   -> markdown table on stdout
+"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+os.environ["PDL_DRY_RUN"] = "1"
+from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
+
+NVLINK = 770e9
+
+
+def rates():
+    r = {}
+    with open(os.path.join(ROOT, "profiles", "r01_bench_table.jsonl")) as f:
+        for line in f:
+            d = json.loads(line)
+            if d["config"] == "C4":
+                r[(d["dtype"], d["variant"])] = d["gflops"] * 1e9
+    return r
+
+
+def model(M, N, K, tile, G, rate, es):
+    pdl.unload()
+    pdl.load(pdl.descriptor_path(G))
+    worst = 0.0
+    for w in range(G):
+        p = pdl.plan(M, N, K, tile, worker=w)
+        rows, cols = p["row1"] - p["row0"], p["col1"] - p["col0"]
+        t_comp = 2.0 * rows * cols * K / rate
+        b_bytes = K * cols * es * (1 - 1 / p["Gr"])            # received B chunks
+        a_chunk = p["qa"] * K * es                              # one A chunk
+        t_b = b_bytes / NVLINK
+        # the own chunk (1/Gc of the work) computes while the other Gc-1 chunks arrive
+        t_own = t_comp / p["Gc"]
+        t_a_exposed = max(0.0, (p["Gc"] - 1) * a_chunk / NVLINK - t_own)
+        worst = max(worst, t_b + t_a_exposed + t_comp)
+    pdl.unload()
+    return worst
+
+
+def main():
+    r = rates()
+    M = N = K = 16384
+    rows = ["| variant | G=1 ms | G=2 | G=4 | G=8 | predicted S_8 |", "|---|---|---|---|---|---|"]
+    for (dt, var), rate in sorted(r.items()):
+        es = 8 if dt == "f64" else 4
+        ts = [model(M, N, K, 1024, G, rate, es) for G in (1, 2, 4, 8)]
+        rows.append(f"| {dt} {var} | {ts[0] * 1e3:.1f} | {ts[1] * 1e3:.1f} | {ts[2] * 1e3:.1f} | "
+                    f"{ts[3] * 1e3:.1f} | {ts[0] / ts[3]:.2f} |")
+    print("\n".join(rows))
+
+
+if __name__ == "__main__":
+    main()
