@@ -557,10 +557,23 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     std::vector<cudaEvent_t> ev_a(RB, nullptr), ev_b(CP, nullptr), ev_sa(RB, nullptr), ev_sb(CP, nullptr);
     cudaEvent_t ev_last_out = nullptr, ev_last_cmp1 = nullptr;
     int launch_idx = 0;
-    for (int i = 0; i < RB; ++i) {
+    // Sub-rectangle order: the inner loop runs over the operand whose chunks are
+    // smaller, so while the first outer chunk computes, the inner chunks stream in
+    // at least as fast as the kernels consume them and only one A band + one B
+    // panel precede the first kernel (C4 host-staged: A bands of 2048 x K = 268 MB
+    // inner, B panels of K x 4096 = 537 MB outer).  Copies and the K3 / K5
+    // operand preparation happen at a chunk's first use.
+    const bool col_outer = piped && (rows / RB) * K <= K * (cols / CP);
+    std::vector<char> a_in(RB, 0), b_in(CP, 0), a_prep(RB, 0), b_prep(CP, 0);
+    const int n_outer = col_outer ? CP : RB, n_inner = col_outer ? RB : CP;
+    for (int o = 0; o < n_outer; ++o) {
+      for (int q = 0; q < n_inner; ++q) {
+        const int i = col_outer ? q : o, j = col_outer ? o : q;
         const int64_t r0 = rb[i], nr = rb[i + 1] - rb[i];
-        if (nr <= 0) continue;
-        if (a_st) {
+        const int64_t c0 = cp[j], nc = cp[j + 1] - cp[j];
+        if (nr <= 0 || nc <= 0) continue;
+        if (a_st && !a_in[i]) {
+            a_in[i] = 1;
             cudaError_t e = cudaMemcpy2DAsync(const_cast<char *>(Ad) + (size_t)(r0 * lda) * es, (size_t)(lda * es),
                                               (const char *)A + (size_t)(r0 * t.lda) * es, (size_t)(t.lda * es),
                                               (size_t)(K * es), (size_t)nr, cudaMemcpyDefault, s_in);
@@ -570,10 +583,9 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 CUDA_TRY(cudaEventRecord(ev_a[i], s_in));
             }
         }
-        for (int j = 0; j < CP; ++j) {
-            const int64_t c0 = cp[j], nc = cp[j + 1] - cp[j];
-            if (nc <= 0) continue;
-            if (i == 0 && b_st) {
+        {
+            if (b_st && !b_in[j]) {
+                b_in[j] = 1;
                 cudaError_t e = cudaMemcpy2DAsync(const_cast<char *>(Bd) + (size_t)c0 * es, (size_t)(ldb * es),
                                                   (const char *)B + (size_t)c0 * es, (size_t)(t.ldb * es),
                                                   (size_t)(nc * es), (size_t)K, cudaMemcpyDefault, s_in);
@@ -594,7 +606,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 e = cudaMemset2DAsync(Cs, (size_t)(ldcd * es), 0, (size_t)(nc * es), (size_t)nr, cs);
             } else if (ozaki) {
                 // K5 slicing of this band / panel once, shared by both compute streams
-                if (j == 0) {
+                if (!a_prep[i]) {
+                    a_prep[i] = 1;
                     const char *Ab = Ad + (size_t)(r0 * lda) * es;
                     e = f64 ? pdlk::launch_ozaki_split_a((const double *)Ab, lda, nr, K, OL, a8 + r0 * OL.ld8,
                                                          oz_ea + r0, cs)
@@ -608,7 +621,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 } else if (ev_sa[i]) {
                     CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
                 }
-                if (e == cudaSuccess && i == 0 && !b_ready) {
+                if (e == cudaSuccess && !b_prep[j] && !b_ready) {
+                    b_prep[j] = 1;
                     const char *Bp = Bd + (size_t)c0 * es;
                     e = f64 ? pdlk::launch_ozaki_split_b((const double *)Bp, ldb, K, nc, OL, b8 + c0 * OL.ld8,
                                                          oz_fb + c0, oz_bmax + c0, cs)
@@ -640,7 +654,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 w.launches += 1;
             } else {
                 // K3 split of this band / panel once, shared by both compute streams
-                if (j == 0) {
+                if (!a_prep[i]) {
+                    a_prep[i] = 1;
                     e = pdlk::launch_split_rows((const float *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K,
                                                 ahi + r0 * Kp, alo + r0 * Kp, Kp, cs);
                     w.launches += 1;
@@ -651,7 +666,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 } else if (ev_sa[i]) {
                     CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
                 }
-                if (e == cudaSuccess && i == 0 && !b_ready) {
+                if (e == cudaSuccess && !b_prep[j] && !b_ready) {
+                    b_prep[j] = 1;
                     e = pdlk::launch_split_cols_t((const float *)(Bd + (size_t)c0 * es), ldb, K, nc, bhi + c0 * Kp,
                                                   blo + c0 * Kp, Kp, cs);
                     w.launches += 1;
@@ -691,6 +707,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             }
             ++launch_idx;
         }
+      }
     }
     if (prep_b) {
         // the B-side buffers now hold this task's prepared B (whole panel only when unpiped)
