@@ -65,7 +65,7 @@ __device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b)
 __global__ void __launch_bounds__(k1::THREADS, 1)
     dgemm_k1_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     double *__restrict__ C, int64_t ldc, int M, int N, int K, int tiles_m, int tiles_n,
-                    int group_m, int vec_ok) {
+                    int group_m, int vec_ok, int *dyn_next, int *dyn_mine) {
     using namespace k1;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
@@ -74,8 +74,14 @@ __global__ void __launch_bounds__(k1::THREADS, 1)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-    // grouped raster: group_m tile rows sweep the tile columns together
-    const int bid = blockIdx.x;
+    // grouped raster: group_m tile rows sweep the tile columns together.  Under
+    // the DYNAMIC distribution the raster index is claimed from the counter all
+    // Workers share instead of taken from blockIdx (CTAs left over exit).
+    int bid = blockIdx.x;
+    if (dyn_next) {
+        bid = cta_claim_tile(dyn_next, dyn_mine, tiles_m * tiles_n);
+        if (bid >= tiles_m * tiles_n) return;
+    }
     const int per_group = group_m * tiles_n;
     const int g = bid / per_group;
     const int first_m = g * group_m;
@@ -239,7 +245,8 @@ int k1_smem_bytes() { return k1::SMEM_BYTES; }
 // Host launcher.  A: rows x K (lda), B: K x cols (ldb), both device-resident,
 // 16 B aligned base, lda*8 and ldb*8 multiples of 16 (checked by the runtime).
 cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
-                            double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream) {
+                            double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream,
+                            int *dyn_next, int *dyn_mine) {
     using namespace k1;
     if (M <= 0 || N <= 0) return cudaSuccess;
     CUtensorMap ta, tb;
@@ -262,7 +269,8 @@ cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, con
     const char *gm = getenv("PDL_GROUP_M_K1");   // raster tuning knob
     const int group_m = gm && atoi(gm) > 0 ? atoi(gm) : GROUP_M;
     dgemm_k1_kernel<<<tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(ta, tb, C, ldc, (int)M, (int)N, (int)K,
-                                                                        tiles_m, tiles_n, group_m, vec_ok);
+                                                                        tiles_m, tiles_n, group_m, vec_ok, dyn_next,
+                                                                        dyn_mine);
     return cudaGetLastError();
 }
 

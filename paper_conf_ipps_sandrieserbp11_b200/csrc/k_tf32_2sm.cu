@@ -51,7 +51,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
     gemm_3xtf32_2sm_kernel(const __grid_constant__ CUtensorMap tAh, const __grid_constant__ CUtensorMap tAl,
                            const __grid_constant__ CUtensorMap tBh, const __grid_constant__ CUtensorMap tBl,
                            float *__restrict__ C, int64_t ldc, int M, int N, int Kp, int tiles_m, int tiles_n,
-                           int group_m, int vec_ok) {
+                           int group_m, int vec_ok, int *dyn_next, int *dyn_mine) {
     using namespace k2x;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
@@ -66,9 +66,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t rank = cluster_ctarank();
 
-    // grouped raster over 256 x 256 cluster tiles
+    // grouped raster over 256 x 256 cluster tiles; DYNAMIC: the pair claims its
+    // raster index from the counter all Workers share (pairs left over exit)
+    int cid = blockIdx.x >> 1;
+    if (dyn_next) {
+        cid = cluster_claim_tile(dyn_next, dyn_mine, tiles_m * tiles_n);
+        if (cid >= tiles_m * tiles_n) return;
+    }
     int tm, tn;
-    raster_tile(blockIdx.x >> 1, tiles_m, tiles_n, group_m, &tm, &tn);
+    raster_tile(cid, tiles_m, tiles_n, group_m, &tm, &tn);
     const int m0 = tm * (2 * BM) + (int)rank * BM;   // this CTA's A rows
     const int nb0 = tn * BN + (int)rank * BNH;       // this CTA's B^T rows
 
@@ -208,7 +214,7 @@ static bool map_f32_2sm(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uin
 
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                    const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                                   cudaStream_t stream) {
+                                   cudaStream_t stream, int *dyn_next, int *dyn_mine) {
     using namespace k2x;
     if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
     CUtensorMap tah, tal, tbh, tbl;
@@ -227,7 +233,8 @@ cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const fl
     const int tiles_m = (int)((M + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((N + BN - 1) / BN);
     const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 3) == 0) ? 1 : 0;
     gemm_3xtf32_2sm_kernel<<<2 * tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(
-        tah, tal, tbh, tbl, C, ldc, (int)M, (int)N, (int)Kp, tiles_m, tiles_n, raster_group_m(GROUP_M), vec_ok);
+        tah, tal, tbh, tbl, C, ldc, (int)M, (int)N, (int)Kp, tiles_m, tiles_n, raster_group_m(GROUP_M), vec_ok, dyn_next,
+        dyn_mine);
     return cudaGetLastError();
 }
 

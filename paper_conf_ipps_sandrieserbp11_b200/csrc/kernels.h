@@ -17,7 +17,10 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t
 // K1 -- FP64 DMMA tile kernel.  Requirements (checked by the caller):
 // A, B device pointers, 16 B aligned, lda*8 % 16 == 0, ldb*8 % 16 == 0.
 cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
-                            double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream);
+                            double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream,
+                            int *dyn_next = nullptr, int *dyn_mine = nullptr);
+// dyn_next / dyn_mine (K1, K2): DYNAMIC distribution -- CTAs claim raster tiles
+// from the shared counter *dyn_next and count their claims in *dyn_mine.
 int k1_smem_bytes();
 
 // K3 -- TF32 hi/lo split pre-pass.  Kp = K rounded up to K2's BK (32).
@@ -66,6 +69,6 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
 // K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                    const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                                   cudaStream_t stream);
+                                   cudaStream_t stream, int *dyn_next = nullptr, int *dyn_mine = nullptr);
 
 }  // namespace pdlk

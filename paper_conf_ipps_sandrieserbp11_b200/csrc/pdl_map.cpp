@@ -66,6 +66,8 @@ bool parse_dist(const char *s, DistSpec *out) {
         if (ch == '_') ch = '-';
     if (name == "BLOCK") {
         d.kind = Dist::Block;   // BLOCK:N -- N (L1155) is the element count, implied by the task
+    } else if (name == "DYNAMIC" && size.empty()) {
+        d.kind = Dist::Dynamic;
     } else if (name == "CYCLIC" || name == "BLOCK-CYCLIC") {
         d.kind = name == "CYCLIC" ? Dist::Cyclic : Dist::BlockCyclic;
         d.b = 1;
@@ -203,12 +205,18 @@ std::string Plan::to_json(const std::vector<int> &workers, const std::vector<std
     o << "{\"M\":" << M << ",\"N\":" << N << ",\"K\":" << K << ",\"tile\":" << tile << ",\"G\":" << G
       << ",\"Gr\":" << Gr << ",\"Gc\":" << Gc << ",\"Tm\":" << Tm << ",\"Tn\":" << Tn
       << ",\"qb\":" << qb() << ",\"exchanged_elems\":" << (int64_t)exchanged_elems() << ",\"dist\":\""
-      << (dist.kind == Dist::Block ? "BLOCK" : dist.kind == Dist::Cyclic ? "CYCLIC" : "BLOCK-CYCLIC") << "\",\"dist_b\":"
+      << (dist.kind == Dist::Block ? "BLOCK" : dist.kind == Dist::Cyclic ? "CYCLIC"
+          : dist.kind == Dist::Dynamic ? "DYNAMIC" : "BLOCK-CYCLIC") << "\",\"dist_b\":"
       << dist.b << ",\"workers\":[";
     for (int w = 0; w < G; ++w) {
         Rect R = rect(w);
         int r = w / Gc, c = w % Gc;
         if (w) o << ",";
+        if (dist.kind == Dist::Dynamic) {   // no static rectangle: tiles are claimed at run time
+            o << "{\"w\":" << w << ",\"id\":\"" << (w < (int)ids.size() ? json_escape(ids[w]) : "")
+              << "\",\"rows\":[0," << M << "],\"cols\":[0," << N << "],\"dynamic\":true}";
+            continue;
+        }
         o << "{\"w\":" << w << ",\"id\":\"" << (w < (int)ids.size() ? json_escape(ids[w]) : "") << "\""
           << ",\"r\":" << r << ",\"c\":" << c << ",\"rows\":[" << R.row0 << "," << R.row1 << "],\"cols\":["
           << R.col0 << "," << R.col1 << "],\"task_rows\":[" << trow[r] << "," << trow[r + 1]

@@ -99,12 +99,14 @@ struct Rect {
 
 // Data distributions of the execute annotation (L1200-1206: "block, cyclic,
 // block-cyclic ... and optional sizes").
-enum class Dist { Block, Cyclic, BlockCyclic };
+// DYNAMIC (the paper's future-work dynamic scheduler, L1556-1562):
+// no static assignment -- the Workers' kernels claim tiles from a shared counter.
+enum class Dist { Block, Cyclic, BlockCyclic, Dynamic };
 struct DistSpec {
     Dist kind = Dist::Block;
     int64_t b = 1;   // tasks per cyclic block (CYCLIC = BLOCK-CYCLIC:1)
 };
-// Parse "BLOCK", "CYCLIC", "BLOCK-CYCLIC[:b]" (case-insensitive; NULL = BLOCK).
+// Parse "BLOCK", "CYCLIC", "BLOCK-CYCLIC[:b]", "DYNAMIC" (case-insensitive; NULL = BLOCK).
 // Returns false for an unknown name or a bad size.
 bool parse_dist(const char *s, DistSpec *out);
 

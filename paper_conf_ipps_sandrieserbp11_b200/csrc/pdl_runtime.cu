@@ -81,6 +81,11 @@ struct WorkerCtx {
     int device = -1;
     cudaStream_t stream = nullptr;
     bool own_stream = false;
+    // SM partition (PDL Worker property SM_LIMIT): a green context owning
+    // sm_limit SMs of the device; the Worker's compute streams belong to it
+    int sm_limit = 0;
+    CUgreenCtx gctx = nullptr;
+    cudaEvent_t ev_legacy = nullptr;   // orders the non-blocking green stream with the legacy stream
     DevBuf buf[BUF_COUNT];
     cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr;   // around the dominant kernel of the last task
     int launches = 0;                               // kernels launched in the last run
@@ -151,6 +156,12 @@ struct State {
     pdlk::EncodeTiledFn encode = nullptr;
     int last_launches = 0;
     long long total_launches = 0;   // every kernel launched since pdl_load
+    // DYNAMIC distribution: [0] next tile, [1 + i] tiles claimed by group Worker i
+    int *dyn = nullptr;
+    int dyn_dev = -1;
+    int dyn_n = 0;                  // Workers of the last DYNAMIC task
+    long long dyn_tiles = 0;        // its tile count
+    std::string dyn_kernel;
 };
 
 State *g = nullptr;
@@ -191,6 +202,116 @@ int get_encoder(pdlk::EncodeTiledFn *out) {
         return set_err(PDL_ECUDA, "cuTensorMapEncodeTiled unavailable (%s)", cudaGetErrorString(e));
     g->encode = reinterpret_cast<pdlk::EncodeTiledFn>(fn);
     *out = g->encode;
+    return PDL_OK;
+}
+
+// Driver entry points for green contexts (SM partitions of one device), loaded
+// through the runtime so libpdl does not link libcuda directly.
+struct GreenApi {
+    CUresult (*dev_get)(CUdevice *, int) = nullptr;
+    CUresult (*get_resource)(CUdevice, CUdevResource *, CUdevResourceType) = nullptr;
+    CUresult (*split)(CUdevResource *, unsigned *, const CUdevResource *, CUdevResource *, unsigned,
+                      unsigned) = nullptr;
+    CUresult (*gen_desc)(CUdevResourceDesc *, CUdevResource *, unsigned) = nullptr;
+    CUresult (*create)(CUgreenCtx *, CUdevResourceDesc, CUdevice, unsigned) = nullptr;
+    CUresult (*stream_create)(CUstream *, CUgreenCtx, unsigned, int) = nullptr;
+    CUresult (*destroy)(CUgreenCtx) = nullptr;
+};
+
+const GreenApi *green_api() {
+    static GreenApi a;
+    static int state = 0;   // 0 untried, 1 ok, -1 unavailable
+    if (state == 0) {
+        auto get = [](const char *name, void **fn) {
+            cudaDriverEntryPointQueryResult q;
+            return cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q) == cudaSuccess &&
+                   q == cudaDriverEntryPointSuccess && *fn;
+        };
+        bool ok = get("cuDeviceGet", (void **)&a.dev_get) &&
+                  get("cuDeviceGetDevResource", (void **)&a.get_resource) &&
+                  get("cuDevSmResourceSplitByCount", (void **)&a.split) &&
+                  get("cuDevResourceGenerateDesc", (void **)&a.gen_desc) &&
+                  get("cuGreenCtxCreate", (void **)&a.create) &&
+                  get("cuGreenCtxStreamCreate", (void **)&a.stream_create) &&
+                  get("cuGreenCtxDestroy", (void **)&a.destroy);
+        cudaGetLastError();
+        state = ok ? 1 : -1;
+    }
+    return state == 1 ? &a : nullptr;
+}
+
+// A compute stream of the Worker: in its green context when it has an SM partition.
+int worker_stream(const WorkerCtx &w, cudaStream_t *out, bool blocking) {
+    if (w.gctx) {
+        CUstream s = nullptr;
+        if (green_api()->stream_create(&s, w.gctx, CU_STREAM_NON_BLOCKING, 0) != CUDA_SUCCESS)
+            return set_err(PDL_ECUDA, "cuGreenCtxStreamCreate failed on device %d", w.device);
+        *out = (cudaStream_t)s;
+        return PDL_OK;
+    }
+    cudaError_t e = blocking ? cudaStreamCreate(out) : cudaStreamCreateWithFlags(out, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return set_err(PDL_ECUDA, "stream create failed: %s", cudaGetErrorString(e));
+    return PDL_OK;
+}
+
+int gcd_int(int a, int b) { return b ? gcd_int(b, a % b) : a; }
+
+// SM partitions (heterogeneous Workers emulated on one B200).
+// Workers carrying the PDL property SM_LIMIT = n run on a green context of n
+// SMs (rounded up to the partition granularity of 8 on sm_90+).  Workers that
+// share a device get disjoint partitions: the device's SMs are split into
+// groups of gcd(n_i) SMs and each Worker takes n_i / gcd consecutive groups.
+int make_partitions() {
+    std::vector<int> devs;
+    for (auto &w : g->workers)
+        if (w.sm_limit > 0 && std::find(devs.begin(), devs.end(), w.device) == devs.end()) devs.push_back(w.device);
+    for (int dev : devs) {
+        const GreenApi *api = green_api();
+        if (!api) return set_err(PDL_EUNSUPPORTED, "SM_LIMIT needs green contexts (driver API unavailable)");
+        CUDA_TRY(cudaSetDevice(dev));
+        CUDA_TRY(cudaFree(nullptr));   // primary context active before the green contexts retain it
+        CUdevice cd;
+        CUdevResource full;
+        if (api->dev_get(&cd, dev) != CUDA_SUCCESS || api->get_resource(cd, &full, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS)
+            return set_err(PDL_ECUDA, "cannot query the SM resource of device %d", dev);
+        std::vector<WorkerCtx *> ws;
+        int unit = 0, need = 0;
+        for (auto &w : g->workers)
+            if (w.device == dev && w.sm_limit > 0) {
+                w.sm_limit = (w.sm_limit + 7) / 8 * 8;
+                unit = gcd_int(unit, w.sm_limit);
+                need += w.sm_limit;
+                ws.push_back(&w);
+            }
+        if (need > (int)full.sm.smCount)
+            return set_err(PDL_EINVAL, "SM_LIMIT of the Workers on device %d sums to %d SMs; the device has %u", dev, need,
+                           full.sm.smCount);
+        unsigned n = full.sm.smCount / unit;
+        std::vector<CUdevResource> parts(n);
+        CUdevResource rem;
+        if (api->split(parts.data(), &n, &full, &rem, 0, unit) != CUDA_SUCCESS)
+            return set_err(PDL_ECUDA, "cuDevSmResourceSplitByCount(%d) failed on device %d", unit, dev);
+        unsigned next = 0;
+        for (WorkerCtx *w : ws) {
+            const unsigned k = w->sm_limit / unit;
+            if (next + k > n) return set_err(PDL_EINVAL, "device %d cannot be split into SM_LIMIT partitions", dev);
+            CUdevResourceDesc desc;
+            if (api->gen_desc(&desc, &parts[next], k) != CUDA_SUCCESS ||
+                api->create(&w->gctx, desc, cd, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS)
+                return set_err(PDL_ECUDA, "green context of %u SMs failed on device %d", k * unit, dev);
+            unsigned sms = 0;
+            for (unsigned i = 0; i < k; ++i) sms += parts[next + i].sm.smCount;
+            next += k;
+            w->sm_limit = (int)sms;
+            if (w->own_stream && w->stream) cudaStreamDestroy(w->stream);
+            int rc = worker_stream(*w, &w->stream, false);
+            if (rc) return rc;
+            w->own_stream = true;
+            // runtime instantiation of the unfixed compute-unit property (L737-747)
+            Property *q = g->model.prop_mut(w->pu, "MAX_COMPUTE_UNITS");
+            if (q && !q->fixed) q->value = std::to_string(sms);
+        }
+    }
     return PDL_OK;
 }
 
@@ -270,7 +391,7 @@ int bind_devices() {
     if (gw.empty()) return set_err(PDL_ENOWORKER, "descriptor has no Worker with ARCHITECTURE=gpu");
     int cur = 0;
     cudaGetDevice(&cur);
-    std::vector<int> used(ndev, 0);
+    std::vector<int> used(ndev, 0), limited(ndev, 0);
     for (size_t i = 0; i < gw.size(); ++i) {
         if (g->nranks > 1 && (int)i != g->rank) continue;
         int dev;
@@ -286,9 +407,22 @@ int bind_devices() {
                                gw.size(), ndev);
             dev = dev % ndev;
         }
-        if (used[dev] && !g->oversub)
-            return set_err(PDL_ENOWORKER, "two Workers bound to device %d (set PDL_ALLOW_OVERSUBSCRIBE=1)", dev);
+        // SM_LIMIT: the Worker owns a partition of the device's SMs (green context);
+        // Workers that all carry it may share a device without oversubscription
+        int sm_limit = 0;
+        if (const Property *sl = g->model.prop(gw[i], "SM_LIMIT")) {
+            char *end = nullptr;
+            long v = std::strtol(sl->value.c_str(), &end, 10);
+            if (!end || *end || v < 1)
+                return set_err(PDL_EINVAL, "Worker %s: SM_LIMIT '%s' is not a positive integer",
+                               g->model.pus[gw[i]].id.c_str(), sl->value.c_str());
+            sm_limit = (int)v;
+        }
+        if (used[dev] && !g->oversub && !(sm_limit > 0 && limited[dev] == used[dev]))
+            return set_err(PDL_ENOWORKER, "two Workers bound to device %d (set PDL_ALLOW_OVERSUBSCRIBE=1, "
+                           "or give each an SM_LIMIT partition)", dev);
         used[dev]++;
+        if (sm_limit > 0) limited[dev]++;
         cudaDeviceProp prop;
         CUDA_TRY(cudaGetDeviceProperties(&prop, dev));
         if (prop.major != 10)
@@ -298,6 +432,7 @@ int bind_devices() {
         w.pu = gw[i];
         w.gw = (int)i;
         w.device = dev;
+        w.sm_limit = sm_limit;
         CUDA_TRY(cudaSetDevice(dev));
         // blocking stream: ordered with the legacy default stream callers often use
         CUDA_TRY(cudaStreamCreate(&w.stream));
@@ -308,8 +443,9 @@ int bind_devices() {
         fill_props(gw[i], prop);
         g->workers.push_back(w);
     }
+    int rc = make_partitions();
     cudaSetDevice(cur);
-    return PDL_OK;
+    return rc;
 }
 
 void free_state() {
@@ -321,10 +457,16 @@ void free_state() {
         if (w.own_stream && w.stream) cudaStreamDestroy(w.stream);
         if (w.ev_k0) cudaEventDestroy(w.ev_k0);
         if (w.ev_k1) cudaEventDestroy(w.ev_k1);
+        if (w.ev_legacy) cudaEventDestroy(w.ev_legacy);
         for (auto ev : w.kt_ev) cudaEventDestroy(ev);
         for (auto ev : w.ev_pool) cudaEventDestroy(ev);
         for (auto st : w.aux)
             if (st) cudaStreamDestroy(st);
+        if (w.gctx) green_api()->destroy(w.gctx);
+    }
+    if (g->dyn) {
+        cudaSetDevice(g->dyn_dev);
+        cudaFree(g->dyn);
     }
     delete g;
     g = nullptr;
@@ -395,8 +537,10 @@ cudaEvent_t ev_get(WorkerCtx &w, size_t &next) {
 }
 
 int ensure_aux(WorkerCtx &w) {
-    for (int i = 0; i < 3; ++i)
+    // copy-in, copy-out: plain streams; aux[2] computes, so it joins the Worker's partition
+    for (int i = 0; i < 2; ++i)
         if (!w.aux[i]) CUDA_TRY(cudaStreamCreateWithFlags(&w.aux[i], cudaStreamNonBlocking));
+    if (!w.aux[2]) return worker_stream(w, &w.aux[2], false);
     return PDL_OK;
 }
 
@@ -727,6 +871,156 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     return PDL_OK;
 }
 
+// ---- DYNAMIC distribution (dynamic schedulers, L1556-1562) ----
+//
+// Every Worker of the group launches the whole tile grid of its task variant
+// (K1 128 x 128 tiles, K2 256 x 256 pair tiles); each CTA (pair) claims the next
+// raster tile from one counter in the first Worker's memory region (system-scope
+// atomics; NVLink peer memory for Workers on other devices), so a faster Worker
+// (more SMs, higher clocks, less competing work) takes more tiles and all
+// finish together, without a speed model.  A tile's computation is the static
+// one, so C is bitwise the BLOCK result (R14).  Operands are used in place when
+// resident on the Worker's device, else staged whole into its memory region.
+// C is written in place by every Worker (peer access when it lives on another
+// device) or, for a host C, into a staging buffer on the first Worker and copied
+// out once every Worker is done.
+constexpr int kMaxDynWorkers = 64;
+
+int enable_peer(int from, int to) {
+    if (from == to) return PDL_OK;
+    int can = 0;
+    CUDA_TRY(cudaDeviceCanAccessPeer(&can, from, to));
+    if (!can) return set_err(PDL_EUNSUPPORTED, "DYNAMIC: device %d cannot access device %d's memory (no P2P)", from, to);
+    CUDA_TRY(cudaSetDevice(from));
+    cudaError_t e = cudaDeviceEnablePeerAccess(to, 0);
+    if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+    else if (e != cudaSuccess) return set_err(PDL_ECUDA, "peer access %d -> %d: %s", from, to, cudaGetErrorString(e));
+    return PDL_OK;
+}
+
+int run_dynamic(const Task &t, const std::vector<int> &gw) {
+    std::vector<WorkerCtx *> ws;
+    for (int pu : gw)
+        for (auto &w : g->workers)
+            if (w.pu == pu) ws.push_back(&w);
+    if (ws.empty()) return set_err(PDL_ENOWORKER, "no Worker of the group is bound to this process");
+    if ((int)ws.size() > kMaxDynWorkers) return set_err(PDL_EINVAL, "DYNAMIC supports %d Workers", kMaxDynWorkers);
+    const bool f64 = t.dtype == PDL_F64;
+    const int es = f64 ? 8 : 4;
+    const int64_t M = t.M, N = t.N, K = t.K, pe = 16 / es;
+    for (auto *w : ws) {
+        int sl, rn;
+        if (K > 0 && worker_ozaki(*w, f64, &sl, &rn))
+            return set_err(PDL_EUNSUPPORTED,
+                           "DYNAMIC needs a single-launch task variant (dmma / 3xtf32); Worker %s runs Ozaki "
+                           "(S diagonal launches updating C)",
+                           g->model.pus[w->pu].id.c_str());
+    }
+    WorkerCtx &own = *ws[0];
+    int rc;
+    size_t evn_own = 0;
+    // C destination
+    const int cdev = locate(t.C);
+    char *Cd = (char *)t.C;
+    int64_t ldc = t.ldc;
+    void *p;
+    if (cdev < 0) {
+        ldc = round_up(N, pe);
+        if ((rc = ensure_buf(own, BUF_C, (size_t)(ldc * M * es), &p))) return rc;
+        Cd = (char *)p;
+    }
+    const int c_home = cdev >= 0 ? cdev : own.device;
+    if (K == 0) {
+        CUDA_TRY(cudaSetDevice(c_home));
+        CUDA_TRY(cudaMemset2DAsync(Cd, (size_t)(ldc * es), 0, (size_t)(N * es), (size_t)M, own.stream));
+    } else {
+        // shared claim counters in the first Worker's memory region
+        if (g->dyn && g->dyn_dev != own.device) {
+            CUDA_TRY(cudaSetDevice(g->dyn_dev));
+            CUDA_TRY(cudaDeviceSynchronize());
+            cudaFree(g->dyn);
+            g->dyn = nullptr;
+        }
+        CUDA_TRY(cudaSetDevice(own.device));
+        if (!g->dyn) {
+            CUDA_TRY(cudaMalloc(&g->dyn, (1 + kMaxDynWorkers) * sizeof(int)));
+            g->dyn_dev = own.device;
+        }
+        CUDA_TRY(cudaMemsetAsync(g->dyn, 0, (1 + kMaxDynWorkers) * sizeof(int), own.stream));
+        cudaEvent_t ev_reset = ev_get(own, evn_own);
+        if (!ev_reset) return set_err(PDL_ECUDA, "event create failed");
+        CUDA_TRY(cudaEventRecord(ev_reset, own.stream));
+        pdlk::EncodeTiledFn enc = nullptr;
+        if ((rc = get_encoder(&enc))) return rc;
+        const int64_t Kp = round_up(K, pdlk::K2_BK);
+        for (size_t i = 0; i < ws.size(); ++i) {
+            WorkerCtx &w = *ws[i];
+            if ((rc = enable_peer(w.device, g->dyn_dev)) || (rc = enable_peer(w.device, c_home))) return rc;
+            CUDA_TRY(cudaSetDevice(w.device));
+            if (&w != &own) CUDA_TRY(cudaStreamWaitEvent(w.stream, ev_reset, 0));
+            // operands readable by this Worker
+            const char *Ad = (const char *)t.A, *Bd = (const char *)t.B;
+            int64_t lda = t.lda, ldb = t.ldb;
+            if (locate(t.A) != w.device || (f64 && (((uintptr_t)t.A % 16) || (t.lda * es) % 16))) {
+                lda = round_up(K, pe);
+                if ((rc = ensure_buf(w, BUF_A, (size_t)(lda * M * es), &p))) return rc;
+                CUDA_TRY(cudaMemcpy2DAsync(p, (size_t)(lda * es), t.A, (size_t)(t.lda * es), (size_t)(K * es),
+                                           (size_t)M, cudaMemcpyDefault, w.stream));
+                Ad = (const char *)p;
+            }
+            if (locate(t.B) != w.device || (f64 && (((uintptr_t)t.B % 16) || (t.ldb * es) % 16))) {
+                ldb = round_up(N, pe);
+                if ((rc = ensure_buf(w, BUF_B, (size_t)(ldb * K * es), &p))) return rc;
+                CUDA_TRY(cudaMemcpy2DAsync(p, (size_t)(ldb * es), t.B, (size_t)(t.ldb * es), (size_t)(N * es),
+                                           (size_t)K, cudaMemcpyDefault, w.stream));
+                Bd = (const char *)p;
+            }
+            int *mine = g->dyn + 1 + i;
+            cudaError_t e;
+            if (f64) {
+                if (kt_mark(w, true, w.stream)) return set_err(PDL_ECUDA, "event record failed");
+                e = pdlk::launch_dgemm_k1(enc, (const double *)Ad, lda, (const double *)Bd, ldb, (double *)Cd, ldc, M,
+                                          N, K, w.stream, g->dyn, mine);
+                w.launches += 1;
+            } else {
+                float *buf4[4];
+                const int slots[4] = {BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO};
+                for (int b = 0; b < 4; ++b) {
+                    if ((rc = ensure_buf(w, slots[b], (size_t)((b < 2 ? M : N) * Kp * 4), &p))) return rc;
+                    buf4[b] = (float *)p;
+                }
+                w.bsig.valid = false;
+                e = pdlk::launch_split_rows((const float *)Ad, lda, M, K, buf4[0], buf4[1], Kp, w.stream);
+                if (e == cudaSuccess)
+                    e = pdlk::launch_split_cols_t((const float *)Bd, ldb, K, N, buf4[2], buf4[3], Kp, w.stream);
+                if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
+                if (kt_mark(w, true, w.stream)) return set_err(PDL_ECUDA, "event record failed");
+                e = pdlk::launch_gemm_3xtf32_2sm(enc, buf4[0], buf4[1], buf4[2], buf4[3], Kp, (float *)Cd, ldc, M, N,
+                                                 w.stream, g->dyn, mine);
+                w.launches += 3;
+            }
+            if (e != cudaSuccess) return set_err(PDL_ECUDA, "tile kernel launch failed: %s", cudaGetErrorString(e));
+            if (kt_mark(w, false, w.stream)) return set_err(PDL_ECUDA, "event record failed");
+            w.timed = true;
+            if (&w != &own) {
+                size_t evn_w = 0;
+                cudaEvent_t done = ev_get(w, evn_w);
+                if (!done) return set_err(PDL_ECUDA, "event create failed");
+                CUDA_TRY(cudaEventRecord(done, w.stream));
+                CUDA_TRY(cudaStreamWaitEvent(own.stream, done, 0));   // join on the first Worker
+            }
+        }
+        g->dyn_n = (int)ws.size();
+        g->dyn_kernel = f64 ? "K1 dgemm_k1_kernel" : "K2 gemm_3xtf32_2sm_kernel";
+    }
+    if (cdev < 0) {
+        CUDA_TRY(cudaSetDevice(own.device));
+        CUDA_TRY(cudaMemcpy2DAsync(t.C, (size_t)(t.ldc * es), Cd, (size_t)(ldc * es), (size_t)(N * es), (size_t)M,
+                                   cudaMemcpyDefault, own.stream));
+    }
+    return PDL_OK;
+}
+
 int check_loaded() {
     if (!g || !g->loaded) return set_err(PDL_ESTATE, "no platform loaded (call pdl_load first)");
     return PDL_OK;
@@ -818,6 +1112,17 @@ int execute(bool sync) {
         w.launches = 0;
         w.timed = false;
     }
+    // Green-context streams are non-blocking: give them the ordering of the
+    // blocking Worker streams (after the legacy default stream's prior work,
+    // and the legacy stream after them -- see the end of this function).
+    if (!g->dry_run)
+        for (auto &w : g->workers)
+            if (w.gctx && w.own_stream) {
+                CUDA_TRY(cudaSetDevice(w.device));
+                if (!w.ev_legacy) CUDA_TRY(cudaEventCreateWithFlags(&w.ev_legacy, cudaEventDisableTiming));
+                CUDA_TRY(cudaEventRecord(w.ev_legacy, cudaStreamLegacy));
+                CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_legacy, 0));
+            }
     for (size_t ti = 0; ti < q.size(); ++ti) {
         const Task &t = q[ti];
         if (t.flags & PDL_TASK_LOCAL) {
@@ -843,6 +1148,11 @@ int execute(bool sync) {
         if (ti) pj << ",";
         pj << plan.to_json(gw, ids);
         if (g->dry_run) continue;
+        if (t.dist.kind == Dist::Dynamic) {
+            rc = run_dynamic(t, gw);
+            if (rc) return rc;
+            continue;
+        }
         const int es = t.dtype == PDL_F64 ? 8 : 4;
         for (auto &w : g->workers) {
             // group index of this bound Worker
@@ -889,6 +1199,13 @@ int execute(bool sync) {
     pj << "]";
     g->plan_json = pj.str();
     for (auto &w : g->workers) g->total_launches += w.launches;
+    if (!g->dry_run)
+        for (auto &w : g->workers)
+            if (w.gctx && w.own_stream) {
+                CUDA_TRY(cudaSetDevice(w.device));
+                CUDA_TRY(cudaEventRecord(w.ev_legacy, w.stream));
+                CUDA_TRY(cudaStreamWaitEvent(cudaStreamLegacy, w.ev_legacy, 0));
+            }
     if (sync) return pdl_sync();
     return PDL_OK;
 }
@@ -950,7 +1267,8 @@ int pdl_set_stream(int worker, void *stream) {
         w.stream = (cudaStream_t)stream;
         w.own_stream = false;
     } else if (!w.own_stream) {
-        CUDA_TRY(cudaStreamCreate(&w.stream));
+        int rc2 = worker_stream(w, &w.stream, true);
+        if (rc2) return rc2;
         w.own_stream = true;
     }
     return PDL_OK;
@@ -1013,10 +1331,26 @@ int pdl_query(const char *key, char *out, size_t len) {
                     }
                 }
                 o << (first ? "" : ",") << "{\"id\":\"" << json_escape(m.pus[w.pu].id) << "\",\"device\":" << w.device
-                  << ",\"kernel_ms\":" << ms << ",\"launches\":" << w.launches << "}";
+                  << ",\"kernel_ms\":" << ms << ",\"launches\":" << w.launches << ",\"sm_limit\":" << w.sm_limit
+                  << "}";
                 first = false;
             }
-            o << "]}";
+            o << "]";
+            // tiles each Worker claimed in the last DYNAMIC task (valid after pdl_sync)
+            if (g->dyn_n > 0 && g->dyn && !g->dry_run) {
+                std::vector<int> claims(g->dyn_n + 1, 0);
+                cudaSetDevice(g->dyn_dev);
+                if (cudaMemcpy(claims.data(), g->dyn, claims.size() * sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess)
+                    cudaGetLastError();
+                long long tot = 0;
+                o << ",\"dynamic\":{\"kernel\":\"" << g->dyn_kernel << "\",\"tiles\":[";
+                for (int i = 0; i < g->dyn_n; ++i) {
+                    o << (i ? "," : "") << claims[1 + i];
+                    tot += claims[1 + i];
+                }
+                o << "],\"total\":" << tot << "}";
+            }
+            o << "}";
             res = o.str();
         } else if (k.rfind("worker/", 0) == 0 || k.rfind("pu/", 0) == 0) {
             bool is_w = k[0] == 'w';

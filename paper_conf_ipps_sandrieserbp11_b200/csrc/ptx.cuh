@@ -71,4 +71,19 @@ __device__ __forceinline__ uint32_t elect_one() {
     return pred;
 }
 
+// Dynamic tile claim for one CTA (DYNAMIC distribution): thread
+// 0 takes the next tile index from the counter shared by every Worker
+// (system-scope atomic: it may sit in a peer GPU's memory) and counts it for
+// its Worker.  Returns the claimed index (>= ntiles: nothing left, exit).
+__device__ __forceinline__ int cta_claim_tile(int *next, int *mine, int ntiles) {
+    __shared__ int s_claim;
+    if (threadIdx.x == 0) {
+        const int t = atomicAdd_system(next, 1);
+        if (t < ntiles) atomicAdd_system(mine, 1);
+        s_claim = t;
+    }
+    __syncthreads();
+    return s_claim;
+}
+
 }  // namespace pdlk

@@ -123,4 +123,22 @@ __device__ __forceinline__ void umma_commit_2sm(uint32_t bar) {
         : "memory");
 }
 
+// Dynamic tile claim for a CTA pair (DYNAMIC distribution): CTA
+// rank 0 takes the next tile index from the counter shared by every Worker
+// (system-scope atomic: the counter may sit in a peer GPU's memory), counts it
+// for its Worker, and hands it to both CTAs through distributed shared memory.
+// Returns the claimed index (>= ntiles: nothing left, the pair exits).
+__device__ __forceinline__ int cluster_claim_tile(int *next, int *mine, int ntiles) {
+    __shared__ int s_claim;
+    if (cluster_ctarank() == 0 && threadIdx.x == 0) {
+        const int t = atomicAdd_system(next, 1);
+        if (t < ntiles) atomicAdd_system(mine, 1);
+        const uint32_t local = smem_u32(&s_claim);
+        asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(mapa_shared(local, 0)), "r"(t) : "memory");
+        asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(mapa_shared(local, 1)), "r"(t) : "memory");
+    }
+    cluster_sync_all();
+    return *reinterpret_cast<volatile int *>(&s_claim);
+}
+
 }  // namespace pdlk
