@@ -89,6 +89,11 @@ extern "C" {
  * Worker PUs with ARCHITECTURE (alias ARCH, value case-insensitive) = gpu are
  *   bound to CUDA devices (DEVICE_ORDINAL property, else in document order)
  *   and their unfixed properties are filled from the device (L737-747).
+ *   A Worker property SM_LIMIT = n (n >= 1, rounded up to a multiple of 8)
+ *   runs the Worker on a green context of n SMs; Workers that all carry it may
+ *   share a device, and get disjoint partitions (the device is split into groups
+ *   of gcd(n_i) SMs; PDL_EINVAL when the device cannot supply enough groups or
+ *   the sum exceeds its SMs).  This emulates heterogeneous Workers on one GPU.
  * This process is the single Master driving every Worker of the descriptor.
  * Env: PDL_DRY_RUN=1 skips device binding (plans only; no device work);
  *   PDL_ALLOW_OVERSUBSCRIBE=1 lets several Workers share a device.
@@ -131,7 +136,14 @@ int task_matmul_f32(const float *A, const float *B, float *C,
  * dist: data distribution of C's tile tasks over the group (L1200-1206:
  *   "block, cyclic, block-cyclic ... and optional sizes"): "BLOCK" (or NULL;
  *   "BLOCK:N" accepted, N implied), "CYCLIC", "BLOCK-CYCLIC:b" (b tasks per
- *   block, default 1), case-insensitive.  CYCLIC / BLOCK-CYCLIC need one
+ *   block, default 1), "DYNAMIC" (no static assignment: every Worker launches
+ *   the whole tile grid and its CTAs claim tiles from one counter in the first
+ *   Worker's memory -- the dynamic scheduling of the paper's future work,
+ *   L1556-1562; operands must be device-resident on, or are staged whole to,
+ *   every Worker; C must be host memory or reachable by peer access; the
+ *   single-launch variants only: Ozaki Workers -> PDL_EUNSUPPORTED at pdl_run;
+ *   tiles claimed per Worker in pdl_query("stats")["dynamic"]),
+ *   case-insensitive.  Non-BLOCK distributions need one
  *   process driving the Workers (pdl_load): with PDL_TASK_PANELS or
  *   pdl_load_rank they return PDL_EUNSUPPORTED.  Unknown names -> PDL_EINVAL.
  *   Workers whose PDL property RELATIVE_SPEED differs get a speed-weighted
@@ -190,7 +202,9 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group,
  * pdl_query -- the "simple query API" over the loaded PDL (L935-937).
  * Keys: "version", "masters", "workers", "groups", "model" (JSON),
  *   "plan" (JSON of the last run's mappings), "stats" (JSON: launches,
- *   kernel time of the last run), "worker/<i>/<PROPERTY>",
+ *   kernel time and SM partition per Worker of the last run; "dynamic": tiles
+ *   each Worker claimed in the last DYNAMIC task -- read after pdl_sync),
+ *   "worker/<i>/<PROPERTY>",
  *   "worker/<i>/device", "worker/<i>/id", "pu/<id>/<PROPERTY>",
  *   "interconnects" (JSON).
  * Writes a NUL-terminated string (truncated to len-1) and returns the full

@@ -259,8 +259,11 @@ int gcd_int(int a, int b) { return b ? gcd_int(b, a % b) : a; }
 // SM partitions (heterogeneous Workers emulated on one B200).
 // Workers carrying the PDL property SM_LIMIT = n run on a green context of n
 // SMs (rounded up to the partition granularity of 8 on sm_90+).  Workers that
-// share a device get disjoint partitions: the device's SMs are split into
-// groups of gcd(n_i) SMs and each Worker takes n_i / gcd consecutive groups.
+// share a device get disjoint partitions: the device's SMs are split once into
+// groups of u = gcd(n_i) SMs and Worker i takes n_i / u of them.  (A split's
+// remainder cannot be split again -- CUDA_ERROR_INVALID_RESOURCE_CONFIGURATION
+// on B200 -- and groups never straddle the GPC structure, so e.g. 8-SM groups
+// cover only 120 of the 148 SMs; profiles/r01_green_probe.json.)
 int make_partitions() {
     std::vector<int> devs;
     for (auto &w : g->workers)
@@ -291,10 +294,13 @@ int make_partitions() {
         CUdevResource rem;
         if (api->split(parts.data(), &n, &full, &rem, 0, unit) != CUDA_SUCCESS)
             return set_err(PDL_ECUDA, "cuDevSmResourceSplitByCount(%d) failed on device %d", unit, dev);
+        if ((int)n * unit < need)
+            return set_err(PDL_EINVAL,
+                           "device %d yields only %u disjoint groups of %d SMs (gcd of the SM_LIMITs); %d SMs requested",
+                           dev, n, unit, need);
         unsigned next = 0;
         for (WorkerCtx *w : ws) {
             const unsigned k = w->sm_limit / unit;
-            if (next + k > n) return set_err(PDL_EINVAL, "device %d cannot be split into SM_LIMIT partitions", dev);
             CUdevResourceDesc desc;
             if (api->gen_desc(&desc, &parts[next], k) != CUDA_SUCCESS ||
                 api->create(&w->gctx, desc, cd, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS)
