@@ -188,6 +188,19 @@ __host__ __device__ constexpr uint32_t idesc_i8(int M, int N) {
     return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
 
+// x * 2^E for an int32 x, correctly rounded (as ldexp): one DMUL by the power
+// of two built from its bits when 2^E is a normal double; otherwise an exact
+// first step to the edge of the normal range, then one rounding multiply.
+__device__ __forceinline__ double pow2_normal(int E) {   // E in [-1022, 1023]
+    return __longlong_as_double((long long)(1023 + E) << 52);
+}
+__device__ __forceinline__ double scale_pow2(int32_t x, int E) {
+    if (E >= -1022 && E <= 1023) return (double)x * pow2_normal(E);
+    const int E1 = E < 0 ? -1022 : 1023;
+    const int E2 = max(-1022, min(1023, E - E1));
+    return ((double)x * pow2_normal(E1)) * pow2_normal(E2);
+}
+
 __device__ __forceinline__ void umma_i8_2sm(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
                                             uint32_t accumulate) {
     asm volatile(
@@ -287,48 +300,79 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
         const uint32_t tl = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(cg * EPI_COLS);
         mbar_wait(bar_tfull, 0);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
+        // TMEM lane = C row: each thread converts its own row (exact power-of-two
+        // scaling), then the warp transposes 32 rows x 16 columns through shared
+        // memory (the operand ring is idle once bar_tfull fired) so that the C
+        // read-modify-write is row-contiguous: 8 lanes x 16 B per row, 4 rows per
+        // instruction.  128B XOR swizzle: both phases are bank-conflict free.
+        const int row0 = tm * (2 * BM) + (int)rank * BM + q * 32;   // first row of this warp
+        const int row = row0 + lane;
         const int cbase = tn * BN + cg * EPI_COLS;
         const int er = row < M ? ea[row] + scale_exp : 0;
-        TC *crow = C + (int64_t)row * ldc + cbase;
-#pragma unroll
+        const uint32_t stg = base + (uint32_t)e * 4096u;               // 32 x 128 B per warp
+        const int rsub = lane >> 3, kch = lane & 7;                    // read phase: row in 4, 16 B chunk
+        const bool vec = vec_ok != 0;
+#pragma unroll 1
         for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
             uint32_t r[16];
             tmem_ld16(tl + c0, r);
-            if (row < M) {
-                double v[16];
 #pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const int col = cbase + c0 + j;
-                    const int f = col < N ? fb[col] : 0;
-                    v[j] = ldexp((double)(int32_t)r[j], er + f);   // exact: int32 -> f64, power-of-two scale
+            for (int k = 0; k < 8; ++k) {
+                double v0 = 0.0, v1 = 0.0;
+                if (row < M) {
+                    const int col = cbase + c0 + 2 * k;
+                    v0 = scale_pow2((int32_t)r[2 * k], er + (col < N ? fb[col] : 0));   // exact
+                    v1 = scale_pow2((int32_t)r[2 * k + 1], er + (col + 1 < N ? fb[col + 1] : 0));
                 }
-                if (vec_ok && cbase + c0 + 16 <= N) {
-                    if constexpr (sizeof(TC) == 8) {
+                const uint32_t a = stg + (uint32_t)lane * 128u + (((uint32_t)k ^ ((uint32_t)lane & 7u)) << 4);
+                asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(v0), "d"(v1) : "memory");
+            }
+            __syncwarp();
+            // the C loads of four rows are issued before their stores (two DRAM
+            // round trips per 32 x 16 chunk instead of eight dependent ones)
+            const int col = cbase + c0 + 2 * kch;
+            const bool vcol = vec && col + 1 < N;
 #pragma unroll
-                        for (int j = 0; j < 16; j += 2) {
-                            double2 *p = reinterpret_cast<double2 *>(crow + c0 + j);
-                            // streaming (evict-first) C traffic keeps the slice panels in L2
-                            double2 o = accumulate ? __ldcs(p) : make_double2(0.0, 0.0);
-                            __stcs(p, make_double2(o.x + v[j], o.y + v[j + 1]));
-                        }
-                    } else {
-                        // FP32 task: each diagonal adds in double and rounds once to float
+            for (int h = 0; h < 2; ++h) {
+                double2 val[4], old[4];
 #pragma unroll
-                        for (int j = 0; j < 16; j += 4) {
-                            float4 *p = reinterpret_cast<float4 *>(crow + c0 + j);
-                            float4 o = accumulate ? __ldcs(p) : make_float4(0.f, 0.f, 0.f, 0.f);
-                            __stcs(p, make_float4((float)((double)o.x + v[j]), (float)((double)o.y + v[j + 1]),
-                                                  (float)((double)o.z + v[j + 2]), (float)((double)o.w + v[j + 3])));
+                for (int u = 0; u < 4; ++u) {
+                    const int rr = 4 * (4 * h + u) + rsub;             // row within the warp's 32
+                    const uint32_t a = stg + (uint32_t)rr * 128u + (((uint32_t)kch ^ ((uint32_t)rr & 7u)) << 4);
+                    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(val[u].x), "=d"(val[u].y) : "r"(a) : "memory");
+                    old[u] = make_double2(0.0, 0.0);
+                    const int grow = row0 + rr;
+                    if (accumulate && vcol && grow < M) {
+                        const TC *cp = C + (int64_t)grow * ldc + col;
+                        if constexpr (sizeof(TC) == 8) {
+                            old[u] = __ldcs(reinterpret_cast<const double2 *>(cp));
+                        } else {
+                            const float2 o = __ldcs(reinterpret_cast<const float2 *>(cp));
+                            old[u] = make_double2((double)o.x, (double)o.y);
                         }
                     }
-                } else {
+                }
 #pragma unroll
-                    for (int j = 0; j < 16; ++j)
-                        if (cbase + c0 + j < N)
-                            crow[c0 + j] = (TC)((accumulate ? (double)crow[c0 + j] : 0.0) + v[j]);
+                for (int u = 0; u < 4; ++u) {
+                    const int grow = row0 + 4 * (4 * h + u) + rsub;
+                    if (grow >= M) continue;
+                    TC *cp = C + (int64_t)grow * ldc + col;
+                    const double v0 = val[u].x, v1 = val[u].y;
+                    if (vcol) {
+                        // streaming (evict-first) C traffic keeps the slice panels in L2;
+                        // FP32 task: each diagonal adds in double and rounds once to float
+                        if constexpr (sizeof(TC) == 8)
+                            __stcs(reinterpret_cast<double2 *>(cp), make_double2(old[u].x + v0, old[u].y + v1));
+                        else
+                            __stcs(reinterpret_cast<float2 *>(cp),
+                                   make_float2((float)(old[u].x + v0), (float)(old[u].y + v1)));
+                    } else {
+                        if (col < N) cp[0] = (TC)((accumulate ? (double)cp[0] : 0.0) + v0);
+                        if (col + 1 < N) cp[1] = (TC)((accumulate ? (double)cp[1] : 0.0) + v1);
+                    }
                 }
             }
+            __syncwarp();
         }
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
