@@ -65,12 +65,13 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cublas", action="store_true")
-    p.add_argument("--variant", choices=("default", "ozaki"), default="default",
-                   help="task variant pinned in the PDL descriptor: default (FP64 K1 DMMA / FP32 K3+K2 3xTF32) "
-                        "or ozaki (K4/K5 INT8 slices; DGEMM_VARIANT / SGEMM_VARIANT)")
+    p.add_argument("--variant", choices=("default", "ozaki", "ozaki2"), default="default",
+                   help="task variant pinned in the PDL descriptor: default (FP64 K1 DMMA / FP32 K3+K2 3xTF32), "
+                        "ozaki (K4/K5 INT8 slices; DGEMM_VARIANT / SGEMM_VARIANT) or ozaki2 (FP64 only: "
+                        "K6/K7 Ozaki scheme II, INT8 residue GEMMs + CRT)")
     p.add_argument("--slices", type=int, default=None,
                    help="Ozaki slices (default 6 for FP64, 3 for FP32; round-to-nearest)")
-    p.add_argument("--no-alt", action="store_true", help="skip timing the other FP64 variant")
+    p.add_argument("--no-alt", action="store_true", help="skip timing the other task variants")
     p.add_argument("--dist-backend", choices=("nccl", "gloo"), default="nccl",
                    help="gloo only to validate the N>1 flow with ranks sharing one GPU")
     return p.parse_args()
@@ -173,10 +174,12 @@ def ncu_traffic(dtype, cfg):
         return None
 
 
-def variant_descriptor(pdl, world, dtype, ozaki, S):
+def variant_descriptor(pdl, world, dtype, variant, S):
     """PDL descriptor XML with the task variant pinned as Worker properties."""
-    if not ozaki:
+    if variant == "default":
         return pdl.descriptor_xml(world)
+    if variant == "ozaki2":
+        return pdl.descriptor_xml(world, props={"DGEMM_VARIANT": "ozaki2"})
     if dtype == "f64":
         return pdl.descriptor_xml(world, "ozaki", S)
     return pdl.descriptor_xml(world, props={"SGEMM_VARIANT": "ozaki", "OZAKI_SLICES_F32": S})
@@ -189,6 +192,41 @@ def ozaki_ops(rows, cols, K, S):
     kc = -(-(-(-K // nch)) // 128) * 128
     ops = 2.0 * rows * cols * kc * nch * S * (S + 1) / 2
     return ops, f"K4 oz_gemm_2sm_kernel x {S * nch} slice-diagonal launches (tcgen05 kind::i8)"
+
+
+OZ2_MODULI = (256, 255, 253, 251, 247, 241, 239, 233, 229, 227, 223, 217, 211, 199)
+
+
+def ozaki2_moduli(K, bits=43):
+    """Moduli count and scaling bits of ozaki2_plan (k_ozaki2.cu): the fewest
+    moduli whose product M admits p >= bits with 2^(2p+1+ceil(log2 Kc)) < M."""
+    nch = max(1, -(-K // 65536))
+    kc = max(128, -(-(-(-K // nch)) // 128) * 128)
+    lk = (kc - 1).bit_length()
+    M = 1
+    for n, m in enumerate(OZ2_MODULI, 1):
+        M *= m
+        p = max([q for q in range(1, 53) if (1 << (2 * q + 1 + lk)) < M] or [0])
+        if p >= bits:
+            break
+    return n, p, nch, kc
+
+
+def ozaki2_ops(rows, cols, K):
+    n, p, nch, kc = ozaki2_moduli(K)
+    ops = 2.0 * rows * cols * kc * nch * n
+    return ops, f"K6 oz_gemm_2sm_kernel<uint8> x {n * nch} residue GEMMs (tcgen05 kind::i8, p = {p}) + CRT pass"
+
+
+def variant_ops(variant, rows, cols, K, S):
+    return ozaki2_ops(rows, cols, K) if variant == "ozaki2" else ozaki_ops(rows, cols, K, S)
+
+
+def variant_label(variant, dtype, S, K):
+    if variant == "ozaki2":
+        n = ozaki2_moduli(K)[0]
+        return f"{dtype}-ozaki2-i8x{n}", f"ozaki2 (K6/K7, {n} moduli, CRT)"
+    return f"{dtype}-ozaki-i8x{S}", f"ozaki (K4/K5, {S} int8 slices)"
 
 
 def host_inputs(cfg, np_dtype):
@@ -291,11 +329,13 @@ def main():
     es = 8 if args.dtype == "f64" else 4
     A, B = host_inputs(args.config, np_dtype)
 
-    ozaki = args.variant == "ozaki"
+    if args.variant == "ozaki2" and args.dtype != "f64":
+        sys.exit("--variant ozaki2 is an FP64 task variant")
+    ozaki = args.variant in ("ozaki", "ozaki2")
     S = args.slices or (6 if args.dtype == "f64" else 3)
     args.slices = S
     # the task variant is pre-selected through the Worker's PDL properties (L1316-1326)
-    desc = variant_descriptor(pdl, world, args.dtype, ozaki, S)
+    desc = variant_descriptor(pdl, world, args.dtype, args.variant, S)
     if world == 1:
         pdl.load(desc)
     else:
@@ -368,7 +408,7 @@ def main():
     kavg = float(np.sum(ktimes)) / args.steps if ktimes else None
     peak_tf, peak_src, peak_alt = tensor_peak("i8" if ozaki else args.dtype)
     if ozaki:
-        pipe_flops, kname = ozaki_ops(wp.rows, wp.cols, K, args.slices)
+        pipe_flops, kname = variant_ops(args.variant, wp.rows, wp.cols, K, args.slices)
     else:
         pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
         kname = "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_2sm_kernel (tcgen05)"
@@ -376,7 +416,7 @@ def main():
     roofline = {"bound": "tensor", "achieved": round(achieved_tf, 2) if achieved_tf else None,
                 "peak": round(peak_tf, 1), "unit": "TFLOP/s",
                 "frac": round(achieved_tf / peak_tf, 4) if achieved_tf else None,
-                "traffic": ncu_traffic(("ozaki" if args.dtype == "f64" else "ozaki32") if ozaki else args.dtype,
+                "traffic": ncu_traffic((args.variant if args.dtype == "f64" else "ozaki32") if ozaki else args.dtype,
                                        args.config),
                 "kernel": kname,
                 "kernel_ms": round(kavg, 3) if kavg else None,
@@ -460,11 +500,12 @@ def main():
         torch.cuda.synchronize()
         cublas = round(flops_total * 3 / (t0.elapsed_time(t1) / 1e3) / 1e9, 1)
 
-    # ---- the Ozaki task variant on the same resident operands (PDL-selected) ----
-    alt = None
-    if world == 1 and not ozaki and not args.no_alt:
+    # ---- the other task variants on the same resident operands (PDL-selected) ----
+    alts = []
+    others = [v for v in (("ozaki", "ozaki2") if args.dtype == "f64" else ("ozaki",)) if v != args.variant]
+    for av in (others if world == 1 and not args.no_alt else []):
         pdl.unload()
-        pdl.load(variant_descriptor(pdl, 1, args.dtype, True, args.slices))
+        pdl.load(variant_descriptor(pdl, 1, args.dtype, av, args.slices))
         pdl.set_stream(stream)
         for _ in range(2):
             step()
@@ -481,22 +522,24 @@ def main():
             torch.cuda.synchronize()
         ams = t0.elapsed_time(t1)
         akt = pdl.kernel_times()
-        aops, akname = ozaki_ops(M, N, K, args.slices)
+        aops, akname = variant_ops(av, M, N, K, args.slices)
         apeak, apsrc, _ = tensor_peak("i8")
         aach = aops / (float(np.mean(akt)) / 1e3) / 1e12 if akt else None
         tol = "1e-12" if args.dtype == "f64" else "1e-5"
-        alt = {"variant": f"ozaki: {args.dtype.upper()} matmul on INT8 tcgen05 ({args.slices} slices, K4/K5)",
-               "dtype": f"{args.dtype}-ozaki-i8x{args.slices}",
-               "value": round(flops_total * args.steps / (ams / 1e3) / 1e9, 1), "unit": "GFLOP/s",
-               "ms_per_step": round(ams / args.steps, 3),
-               "parity": f"max scaled err <= {tol} vs oracle (tests/test_gpu_ozaki.py)",
-               "roofline": {"bound": "tensor", "achieved": round(aach, 1) if aach else None,
-                            "peak": apeak, "unit": "TFLOP/s", "frac": round(aach / apeak, 4) if aach else None,
-                            "traffic": ncu_traffic("ozaki" if args.dtype == "f64" else "ozaki32", args.config),
-                            "kernel": akname,
-                            "kernel_ms": round(float(np.mean(akt)), 3) if akt else None,
-                            "peak_source": apsrc},
-               "clocks": clk2.summary()}
+        adt, alabel = variant_label(av, args.dtype, args.slices, K)
+        alts.append({"variant": f"{alabel}: {args.dtype.upper()} matmul on INT8 tcgen05",
+                     "dtype": adt,
+                     "value": round(flops_total * args.steps / (ams / 1e3) / 1e9, 1), "unit": "GFLOP/s",
+                     "ms_per_step": round(ams / args.steps, 3),
+                     "parity": f"max scaled err <= {tol} vs oracle (tests/test_gpu_{av}.py)",
+                     "roofline": {"bound": "tensor", "achieved": round(aach, 1) if aach else None,
+                                  "peak": apeak, "unit": "TFLOP/s",
+                                  "frac": round(aach / apeak, 4) if aach else None,
+                                  "traffic": ncu_traffic(av if args.dtype == "f64" else "ozaki32", args.config),
+                                  "kernel": akname,
+                                  "kernel_ms": round(float(np.mean(akt)), 3) if akt else None,
+                                  "peak_source": apsrc},
+                     "clocks": clk2.summary()})
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -507,12 +550,12 @@ def main():
             "metric": METRIC, "value": round(value, 1), "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-            "dtype": f"{args.dtype}-ozaki-i8x{args.slices}" if ozaki else args.dtype,
+            "dtype": variant_label(args.variant, args.dtype, args.slices, K)[0] if ozaki else args.dtype,
             "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} ({args.dtype})",
             "config": {"workload": f"{args.config} {M}x{N}x{K} blocked matmul, task tile {c.tile}, "
                                    f"PDL b200_x{world}",
                        "M": M, "N": N, "K": K, "tile": c.tile, "parallelism": f"block2d {wp.Gr}x{wp.Gc}",
-                       "task_variant": (f"ozaki (K4/K5, {args.slices} int8 slices)" if ozaki else
+                       "task_variant": (variant_label(args.variant, args.dtype, args.slices, K)[1] if ozaki else
                                         ("dmma (K1)" if args.dtype == "f64" else "3xtf32 (K3+K2)")),
                        "l2": "inputs larger than L2 (operands >> 126 MB), no flush needed"},
             "pct_of_tensor_peak": round(100 * (pipe_flops / flops_worker) * value / world / (peak_tf * 1e3), 2),
@@ -522,8 +565,8 @@ def main():
         }
         if cublas is not None:
             line["cublas_gflops_same_operands"] = cublas
-        if alt is not None:
-            line["alt_variant"] = alt
+        if alts:
+            line["alt_variants"] = alts
         print(json.dumps(line), flush=True)
     pdl.unload()
     if world > 1:

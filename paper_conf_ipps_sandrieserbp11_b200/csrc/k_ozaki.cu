@@ -215,7 +215,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
     oz_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
                        TC *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
                        const int *__restrict__ fb, int scale_exp, int accumulate, int tiles_m, int tiles_n,
-                       int group_m, int vec_ok) {
+                       int group_m, int vec_ok, int modulus, float inv_mod) {
     using namespace koz;
     constexpr int BN = Cfg<NSUB>::BN, STAGES = Cfg<NSUB>::STAGES, STAGE_BYTES = Cfg<NSUB>::STAGE_BYTES;
     constexpr int EPI_COLS = Cfg<NSUB>::EPI_COLS, TMEM_COLS = Cfg<NSUB>::TMEM_COLS;
@@ -300,6 +300,43 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
         const uint32_t tl = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(cg * EPI_COLS);
         mbar_wait(bar_tfull, 0);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        if constexpr (sizeof(TC) == 1) {
+            // Ozaki-II (K6): the exact INT32 sum reduced mod m into a byte plane
+            // (C = plane, ldc = its row pitch, 16-byte aligned).  Each thread owns
+            // its TMEM lane = row and stores 16 consecutive residues per step.
+            const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
+            const int cbase = tn * BN + cg * EPI_COLS;
+            uint8_t *prow = reinterpret_cast<uint8_t *>(C) + (int64_t)row * ldc + cbase;
+#pragma unroll 1
+            for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
+                uint32_t r[16];
+                tmem_ld16(tl + c0, r);
+                if (row >= M) continue;
+                uint32_t pk[4];
+#pragma unroll
+                for (int w4 = 0; w4 < 4; ++w4) {
+                    uint32_t word = 0;
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) {
+                        const int x = (int)r[4 * w4 + b];
+                        int res = x - __float2int_rn((float)x * inv_mod) * modulus;   // |q error| <= 1
+                        res += res < 0 ? modulus : 0;
+                        res += res < 0 ? modulus : 0;
+                        res -= res >= modulus ? modulus : 0;
+                        res -= res >= modulus ? modulus : 0;
+                        word |= (uint32_t)res << (8 * b);
+                    }
+                    pk[w4] = word;
+                }
+                if (cbase + c0 + 16 <= N) {
+                    *reinterpret_cast<uint4 *>(prow + c0) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                } else {
+#pragma unroll
+                    for (int jj = 0; jj < 16; ++jj)
+                        if (cbase + c0 + jj < N) prow[c0 + jj] = (uint8_t)(pk[jj >> 2] >> (8 * (jj & 3)));
+                }
+            }
+        } else {
         // TMEM lane = C row: each thread converts its own row (exact power-of-two
         // scaling), then the warp transposes 32 rows x 16 columns through shared
         // memory (the operand ring is idle once bar_tfull fired) so that the C
@@ -373,6 +410,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
                 }
             }
             __syncwarp();
+        }
         }
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -495,11 +533,11 @@ static cudaError_t gemm_impl(EncodeTiledFn enc, const int8_t *A8, const int8_t *
             if (nsub == 2)
                 oz_gemm_2sm_kernel<2, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
                     ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
-                    tiles_n, raster_group_m(GROUP_M), vec_ok);
+                    tiles_n, raster_group_m(GROUP_M), vec_ok, 0, 0.f);
             else
                 oz_gemm_2sm_kernel<1, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
                     ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
-                    tiles_n, raster_group_m(GROUP_M), vec_ok);
+                    tiles_n, raster_group_m(GROUP_M), vec_ok, 0, 0.f);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             first = 0;
@@ -518,6 +556,56 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
                               const OzakiLayout &L, float *C, int64_t ldc, int64_t rows, int64_t cols,
                               cudaStream_t stream, int *launches) {
     return gemm_impl(enc, A8, Bt8, ea, fb, L, C, ldc, rows, cols, stream, launches);
+}
+
+// Ozaki-II (K6): one INT8 GEMM per modulus and K chunk, each writing its byte
+// plane of residues (k_ozaki2.cu builds the operands and rebuilds C).
+cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
+                               uint8_t *R, int64_t ldr, int64_t plane, int64_t rows, int64_t cols, cudaStream_t stream,
+                               int *launches) {
+    using namespace koz;
+    if (rows <= 0 || cols <= 0) return cudaSuccess;
+    if ((reinterpret_cast<uintptr_t>(R) & 15u) || (ldr & 15) || (plane & 15)) return cudaErrorInvalidValue;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static bool attr_done[64] = {false};
+    if (dev < 64 && !attr_done[dev]) {
+        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1, uint8_t>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<1>::SMEM_BYTES);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<2, uint8_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     Cfg<2>::SMEM_BYTES);
+        if (e != cudaSuccess) return e;
+        attr_done[dev] = true;
+    }
+    const int64_t clusters512 = ((rows + 2 * BM - 1) / (2 * BM)) * ((cols + 511) / 512);
+    int nsub = (cols > 256 && clusters512 >= 148) ? 2 : 1;
+    if (const char *e = getenv("PDL_OZ_NSUB")) nsub = atoi(e) == 1 ? 1 : 2;
+    const int BN = nsub == 2 ? Cfg<2>::BN : Cfg<1>::BN;
+    const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + BN - 1) / BN);
+    for (int c = 0; c < P.nch; ++c) {
+        for (int t = 0; t < P.n; ++t) {
+            const int64_t off = ((int64_t)c * P.n + t) * P.Kc;
+            CUtensorMap ta, tb;
+            if (!map_i8(enc, &ta, A8 + off, (uint64_t)P.Kc, (uint64_t)rows, (uint64_t)P.ld8, BM) ||
+                !map_i8(enc, &tb, Bt8 + off, (uint64_t)P.Kc, (uint64_t)cols, (uint64_t)P.ld8, BNH))
+                return cudaErrorInvalidValue;
+            uint8_t *Rp = R + ((int64_t)c * P.n + t) * plane;
+            const float inv = 1.0f / (float)P.m[t];
+            if (nsub == 2)
+                oz_gemm_2sm_kernel<2, uint8_t><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
+                    ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, nullptr, nullptr, 0, 0, tiles_m, tiles_n,
+                    raster_group_m(GROUP_M), 1, P.m[t], inv);
+            else
+                oz_gemm_2sm_kernel<1, uint8_t><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
+                    ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, nullptr, nullptr, 0, 0, tiles_m, tiles_n,
+                    raster_group_m(GROUP_M), 1, P.m[t], inv);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return e;
+            if (launches) ++*launches;
+        }
+    }
+    return cudaSuccess;
 }
 
 }  // namespace pdlk

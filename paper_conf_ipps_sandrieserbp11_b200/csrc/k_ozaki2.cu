@@ -1,0 +1,362 @@
+// k_ozaki2.cu -- K6/K7: the FP64 DGEMM task variant "ozaki2" on the INT8 tensor
+// cores (Ozaki scheme II: integer scaling + Chinese remainder theorem),
+// SURVEY.md SS8(f) NEXT-1, a third implementation variant of the DGEMM task
+// (task repository / static pre-selection, PAPER.md L1033-1039, L1307-1326;
+// PDL property DGEMM_VARIANT = "ozaki2").
+//
+// Method (Ozaki, Uchino, Imamura 2025, "Ozaki scheme II"; K6):
+//   scaling   A'_ik = rint(A_ik 2^{p-e_i}),  B'_kj = rint(B_kj 2^{p-f_j})   (|.| <= 2^p)
+//             e_i: max_k |A_ik| < 2^{e_i};  f_j likewise for columns of B
+//   residues  for pairwise-coprime m_t <= 256: a_t = A' mod m_t in [-128, 127]
+//   GEMMs     X_t = sum_k a_t b_t  (exact INT32 on tcgen05 kind::i8), u_t = X_t mod m_t
+//   CRT       X = A'B' is the unique integer in (-M/2, M/2] with X = u_t (mod m_t),
+//             M = prod m_t; exact because |X| <= K 2^{2p} < M/2 by the choice of p
+//   result    C_ij = X_ij 2^{e_i + f_j - 2p}
+// The only rounding is the scaling of A and B to p-bit integers (|err| <= 2^{e_i-p-1}
+// per element) and the final conversion of X to double; n moduli replace the
+// S(S+1)/2 slice products of scheme I (13 GEMMs instead of 21 at K = 16384 for
+// p = 43).  Inputs must be finite (R15).
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdint>
+
+#include "kernels.h"
+
+namespace pdlk {
+
+// Pairwise-coprime moduli <= 256 (2^8, 3*5*17, 11*23, 251, 13*19, primes, 7*31, ...),
+// largest first: residues in [-128, 127] fit int8 and products sum exactly in INT32.
+static const int kModuli[OZ2_MAX_MODULI] = {256, 255, 253, 251, 247, 241, 239, 233, 229, 227, 223, 217, 211, 199};
+
+__constant__ double c_oz2_m[OZ2_MAX_MODULI];
+__constant__ double c_oz2_inv[OZ2_MAX_MODULI];
+
+// ------------------------------------------------------------------------
+// plan (host): moduli count, scaling bits, CRT constants
+// ------------------------------------------------------------------------
+typedef unsigned __int128 u128;
+
+static int inv_mod(int a, int m) {   // a^-1 mod m (gcd(a, m) = 1)
+    int t = 0, nt = 1, r = m, nr = a % m;
+    while (nr) {
+        const int q = r / nr;
+        int x = t - q * nt;
+        t = nt;
+        nt = x;
+        x = r - q * nr;
+        r = nr;
+        nr = x;
+    }
+    return t < 0 ? t + m : t;
+}
+
+static int ilog2_ceil(int64_t x) {
+    int b = 0;
+    while (((int64_t)1 << b) < x) ++b;
+    return b;
+}
+
+// Largest p <= 52 with 2^(2p+1) * 2^ceil(log2 Kc) < M (so |X| <= Kc 2^(2p) < M/2).
+static int bits_for(u128 M, int64_t Kc) {
+    const int lk = ilog2_ceil(Kc < 1 ? 1 : Kc);
+    int p = 0;
+    for (int q = 1; q <= 52; ++q)
+        if (2 * q + 1 + lk < 127 && ((u128)1 << (2 * q + 1 + lk)) < M) p = q;
+    return p;
+}
+
+Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits) {
+    Ozaki2Plan P;
+    P.nch = (int)((K + OZ2_KC_MAX - 1) / OZ2_KC_MAX);
+    if (P.nch < 1) P.nch = 1;
+    const int64_t per = (K + P.nch - 1) / P.nch;
+    P.Kc = ((per + 127) / 128) * 128;   // whole 128-byte K blocks (BK of the INT8 GEMM)
+    if (P.Kc < 128) P.Kc = 128;
+    int n = nmod > 0 ? (nmod > OZ2_MAX_MODULI ? OZ2_MAX_MODULI : (nmod < 2 ? 2 : nmod)) : 0;
+    if (n == 0) {   // fewest moduli reaching the requested scaling bits
+        u128 M = 1;
+        for (n = 1; n <= OZ2_MAX_MODULI; ++n) {
+            M *= (u128)kModuli[n - 1];
+            if (bits_for(M, P.Kc) >= bits) break;
+        }
+        if (n > OZ2_MAX_MODULI) n = OZ2_MAX_MODULI;
+    }
+    P.n = n;
+    u128 M = 1;
+    for (int t = 0; t < n; ++t) {
+        P.m[t] = kModuli[t];
+        M *= (u128)kModuli[t];
+    }
+    P.p = bits_for(M, P.Kc);
+    for (int t = 0; t < n; ++t) {
+        const u128 Mt = M / (u128)P.m[t];
+        const int r = (int)(Mt % (u128)P.m[t]);
+        const u128 W = (Mt * (u128)inv_mod(r, P.m[t])) % M;
+        P.W[t][0] = (unsigned long long)W;
+        P.W[t][1] = (unsigned long long)(W >> 64);
+    }
+    P.Mw[0] = (unsigned long long)M;
+    P.Mw[1] = (unsigned long long)(M >> 64);
+    const u128 H = M / 2;
+    P.Hw[0] = (unsigned long long)H;
+    P.Hw[1] = (unsigned long long)(H >> 64);
+    P.Md = (double)P.Mw[1] * 18446744073709551616.0 + (double)P.Mw[0];
+    P.ld8 = (int64_t)P.nch * n * P.Kc;
+    P.a8_bytes = (size_t)rows * P.ld8;
+    P.b8_bytes = (size_t)cols * P.ld8;
+    return P;
+}
+
+// ------------------------------------------------------------------------
+// K7: scaling + residues (pre-pass)
+// ------------------------------------------------------------------------
+__device__ __forceinline__ double pow2d(int E) {   // 2^E, E in [-1022, 1023]
+    return __longlong_as_double((long long)(1023 + E) << 52);
+}
+// x 2^E exactly as ldexp would round it (two exact-operand steps off the normal range)
+__device__ __forceinline__ double scale2(double x, int E) {
+    if (E >= -1022 && E <= 1023) return x * pow2d(E);
+    const int E1 = E < 0 ? -1022 : 1023;
+    return (x * pow2d(E1)) * pow2d(max(-1022, min(1023, E - E1)));
+}
+__device__ __forceinline__ int exp_of_max2(double mx) {   // mx < 2^e (0 -> 0)
+    if (!(mx > 0.0)) return 0;
+    int e;
+    frexp(mx, &e);
+    return e;
+}
+// v (an integer, |v| <= 2^52) mod m as a representative in [-128, 127]
+__device__ __forceinline__ int res8(double v, int t) {
+    const double m = c_oz2_m[t];
+    double r = fma(-rint(v * c_oz2_inv[t]), m, v);   // exact: |q m| < 2^53
+    if (r > 127.0) r -= m;
+    if (r < -128.0) r += m;
+    return (int)r;
+}
+
+// One CTA per row (grid-stride): A (rows x K) -> A8 rows [c][t][kk].
+__global__ void oz2_split_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M, int64_t K, int n,
+                                      int p, int64_t Kc, int nch, int8_t *__restrict__ A8, int64_t ld8,
+                                      int *__restrict__ ea) {
+    __shared__ double red[32];
+    const int64_t Kpad = (int64_t)nch * Kc;
+    for (int64_t i = blockIdx.x; i < M; i += gridDim.x) {
+        const double *row = A + i * lda;
+        double mx = 0.0;
+        for (int64_t k = threadIdx.x; k < K; k += blockDim.x) mx = fmax(mx, fabs(row[k]));
+        for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = mx;
+        __syncthreads();
+        if (threadIdx.x < 32) {
+            mx = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : 0.0;
+            for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+            if (threadIdx.x == 0) red[0] = mx;
+        }
+        __syncthreads();
+        const int e = exp_of_max2(red[0]);
+        if (threadIdx.x == 0) ea[i] = e;
+        int8_t *out = A8 + i * ld8;
+        for (int64_t k8 = (int64_t)threadIdx.x * 8; k8 < Kpad; k8 += (int64_t)blockDim.x * 8) {
+            double v[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? rint(scale2(row[k8 + j], p - e)) : 0.0;
+            const int64_t c = k8 / Kc, kk = k8 - c * Kc;
+            int8_t *o = out + (c * n) * Kc + kk;
+            for (int t = 0; t < n; ++t) {
+                uint64_t pk = 0;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) pk |= (uint64_t)(uint8_t)(int8_t)res8(v[j], t) << (8 * j);
+                *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pk;
+            }
+        }
+        __syncthreads();
+    }
+}
+
+__global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
+                                  unsigned long long *__restrict__ bmax) {
+    const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (n >= N) return;
+    const int64_t k0 = (int64_t)blockIdx.y * 256, k1 = min(K, k0 + 256);
+    double mx = 0.0;
+    for (int64_t k = k0; k < k1; ++k) mx = fmax(mx, fabs(B[k * ldb + n]));
+    atomicMax(bmax + n, (unsigned long long)__double_as_longlong(mx));
+}
+
+// B (K x N) -> Bt8 (N rows of [c][t][kk]) through a 64 k x 32 n shared tile.
+__global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
+    const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int n, int p, int64_t Kc, int nch,
+    const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb) {
+    __shared__ double tl[64][33];
+    const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    for (int r = ty; r < 64; r += 8) {
+        const int64_t k = k0 + r, nn = n0 + tx;
+        tl[r][tx] = (k < K && nn < N) ? B[k * ldb + nn] : 0.0;
+    }
+    __syncthreads();
+    const int64_t Kpad = (int64_t)nch * Kc;
+    const int nl = threadIdx.x >> 3, g = threadIdx.x & 7;
+    const int64_t col = n0 + nl, k8 = k0 + 8 * g;
+    if (col >= N || k8 >= Kpad) return;
+    const int f = exp_of_max2(__longlong_as_double((long long)bmax[col]));
+    if (blockIdx.y == 0 && g == 0) fb[col] = f;
+    double v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = rint(scale2(tl[8 * g + j][nl], p - f));
+    const int64_t c = k8 / Kc, kk = k8 - c * Kc;
+    int8_t *o = Bt8 + col * ld8 + (c * n) * Kc + kk;
+    for (int t = 0; t < n; ++t) {
+        uint64_t pk = 0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) pk |= (uint64_t)(uint8_t)(int8_t)res8(v[j], t) << (8 * j);
+        *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pk;
+    }
+}
+
+// ------------------------------------------------------------------------
+// K6 epilogue pass: CRT reconstruction of X from the residue planes
+// ------------------------------------------------------------------------
+struct Oz2Crt {
+    int n, nch, p;
+    unsigned long long W[OZ2_MAX_MODULI][2];
+    unsigned long long Mw[2], Hw[2];
+    double Md;
+};
+
+// 8 consecutive columns per thread: 8 bytes from each plane, 8 doubles out.
+__global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__restrict__ R, int64_t ldr,
+                                                              int64_t plane, const int *__restrict__ ea,
+                                                              const int *__restrict__ fb, const Oz2Crt crt,
+                                                              double *__restrict__ C, int64_t ldc, int64_t rows,
+                                                              int64_t cols) {
+    const int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y;
+    const int64_t c8 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
+    if (row >= rows || c8 >= cols) return;
+    const u128 M = ((u128)crt.Mw[1] << 64) | crt.Mw[0];
+    const u128 H = ((u128)crt.Hw[1] << 64) | crt.Hw[0];
+    double acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    for (int c = 0; c < crt.nch; ++c) {
+        // S = sum_t u_t W_t in two 64-bit words per column (u_t < 2^8, W_t < M < 2^111:
+        // S < 14 * 2^119 < 2^128)
+        uint64_t slo[8], shi[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) slo[j] = shi[j] = 0;
+        for (int t = 0; t < crt.n; ++t) {
+            const uint8_t *pr = R + ((int64_t)c * crt.n + t) * plane + row * ldr + c8;
+            const uint64_t u8x8 = *reinterpret_cast<const uint64_t *>(pr);   // ldr, c8 multiples of 8
+            const uint64_t wl = crt.W[t][0], wh = crt.W[t][1];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                const uint64_t u = (u8x8 >> (8 * j)) & 0xffu;
+                const uint64_t pl = u * wl;
+                const uint64_t ph = __umul64hi(u, wl) + u * wh;
+                slo[j] += pl;
+                shi[j] += ph + (slo[j] < pl ? 1u : 0u);
+            }
+        }
+        u128 S[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) S[j] = ((u128)shi[j] << 64) | slo[j];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            // X = S mod M, then the balanced representative in (-M/2, M/2]
+            const double Sd = (double)(uint64_t)(S[j] >> 64) * 18446744073709551616.0 + (double)(uint64_t)S[j];
+            const uint64_t q = (uint64_t)floor(Sd / crt.Md);
+            __int128 X = (__int128)S[j] - (__int128)((u128)q * M);
+            if (X < 0) X += (__int128)M;
+            if (X < 0) X += (__int128)M;
+            if (X >= (__int128)M) X -= (__int128)M;
+            if (X >= (__int128)M) X -= (__int128)M;
+            if (X > (__int128)H) X -= (__int128)M;
+            const long long hi = (long long)(X >> 64);
+            const uint64_t lo = (uint64_t)X;
+            acc[j] += (double)hi * 18446744073709551616.0 + (double)lo;
+        }
+    }
+    const int er = ea[row] - 2 * crt.p;
+    double *crow = C + row * ldc + c8;
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+        if (c8 + j < cols) crow[j] = scale2(acc[j], er + fb[c8 + j]);
+}
+
+// ------------------------------------------------------------------------
+// host launchers
+// ------------------------------------------------------------------------
+static cudaError_t upload_moduli(const Ozaki2Plan &P) {
+    // identical for every plan (the moduli table is fixed); cheap synchronous copy
+    static bool done = false;
+    static int dev_done[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (done && dev < 64 && dev_done[dev]) return cudaSuccess;
+    double m[OZ2_MAX_MODULI], inv[OZ2_MAX_MODULI];
+    for (int t = 0; t < OZ2_MAX_MODULI; ++t) {
+        m[t] = (double)kModuli[t];
+        inv[t] = 1.0 / (double)kModuli[t];
+    }
+    cudaError_t e = cudaMemcpyToSymbol(c_oz2_m, m, sizeof m);
+    if (e == cudaSuccess) e = cudaMemcpyToSymbol(c_oz2_inv, inv, sizeof inv);
+    if (e == cudaSuccess && dev < 64) {
+        dev_done[dev] = 1;
+        done = true;
+    }
+    (void)P;
+    return e;
+}
+
+cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
+                                  int8_t *A8, int *ea, cudaStream_t s) {
+    if (rows <= 0) return cudaSuccess;
+    cudaError_t e = upload_moduli(P);
+    if (e != cudaSuccess) return e;
+    const int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
+    oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
+                                  int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s) {
+    if (cols <= 0) return cudaSuccess;
+    cudaError_t e = upload_moduli(P);
+    if (e != cudaSuccess) return e;
+    e = cudaMemsetAsync(bmax, 0, (size_t)cols * sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+    if (K > 0) {
+        dim3 g1((unsigned)((cols + 255) / 256), (unsigned)((K + 255) / 256));
+        oz2_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
+    }
+    const int64_t Kpad = (int64_t)P.nch * P.Kc;
+    dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 63) / 64));
+    oz2_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, P.n, P.p, P.Kc, P.nch, bmax, Bt8, P.ld8, fb);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
+                                      const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
+                                      cudaStream_t s) {
+    if (rows <= 0 || cols <= 0) return cudaSuccess;
+    if ((reinterpret_cast<uintptr_t>(R) & 7u) || (ldr & 7) || (plane & 7)) return cudaErrorInvalidValue;
+    Oz2Crt crt;
+    crt.n = P.n;
+    crt.nch = P.nch;
+    crt.p = P.p;
+    for (int t = 0; t < OZ2_MAX_MODULI; ++t) {
+        crt.W[t][0] = P.W[t][0];
+        crt.W[t][1] = P.W[t][1];
+    }
+    crt.Mw[0] = P.Mw[0];
+    crt.Mw[1] = P.Mw[1];
+    crt.Hw[0] = P.Hw[0];
+    crt.Hw[1] = P.Hw[1];
+    crt.Md = P.Md;
+    dim3 block(32, 8);
+    dim3 grid((unsigned)((cols + 255) / 256), (unsigned)((rows + 7) / 8));
+    oz2_reconstruct_kernel<<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, crt, C, ldc, rows, cols);
+    return cudaGetLastError();
+}
+
+}  // namespace pdlk

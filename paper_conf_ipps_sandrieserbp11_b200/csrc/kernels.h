@@ -66,6 +66,40 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
                               const OzakiLayout &L, float *C, int64_t ldc, int64_t rows, int64_t cols,
                               cudaStream_t stream, int *launches);
 
+// K6/K7 -- FP64 DGEMM variant "ozaki2" (Ozaki scheme II: integer scaling and the
+// Chinese remainder theorem over INT8 GEMMs, k_ozaki2.cu).  A' = rint(A 2^(p-e_i))
+// row-wise, B' = rint(B 2^(p-f_j)) column-wise (|A'|, |B'| <= 2^p); for each of n
+// pairwise-coprime moduli m_t <= 256 one INT8 GEMM of the residues (exact INT32)
+// reduced mod m_t into a byte plane; X = A'B' is rebuilt from the n planes by CRT
+// (exact: |X| < M/2, M = prod m_t) and C = X 2^(e_i + f_j - 2p).
+// Residues: A8 = rows x ld8, row layout [chunk][modulus][Kc]; Bt8 = cols x ld8 the
+// same for B^T.  Planes: R + (c n + t) * plane, rows x ldr bytes each.
+constexpr int OZ2_MAX_MODULI = 14;        // sum_t u_t W_t < 2^128 (u_t < 256, W_t < M < 2^111)
+constexpr int64_t OZ2_KC_MAX = 65536;     // |sum r_a r_b| <= Kc 2^14 < 2^31
+struct Ozaki2Plan {
+    int n = 0;                            // moduli in use
+    int p = 0;                            // integer scaling bits
+    int nch = 1;
+    int64_t Kc = 0, ld8 = 0;
+    size_t a8_bytes = 0, b8_bytes = 0;
+    int m[OZ2_MAX_MODULI] = {};
+    unsigned long long W[OZ2_MAX_MODULI][2] = {};   // CRT weights (lo, hi words)
+    unsigned long long Mw[2] = {}, Hw[2] = {};      // M and floor(M / 2)
+    double Md = 0.0;
+};
+// nmod = 0: the fewest moduli that give p >= bits for this K chunk.
+Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits);
+cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
+                                  int8_t *A8, int *ea, cudaStream_t s);
+cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
+                                  int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s);
+cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
+                               uint8_t *R, int64_t ldr, int64_t plane, int64_t rows, int64_t cols, cudaStream_t s,
+                               int *launches);
+cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
+                                      const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
+                                      cudaStream_t s);
+
 // K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                    const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,

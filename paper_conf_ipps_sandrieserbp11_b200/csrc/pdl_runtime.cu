@@ -73,7 +73,7 @@ struct DevBuf {
     size_t bytes = 0;
 };
 
-enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_OZA, BUF_OZB, BUF_OZE, BUF_COUNT };
+enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_OZA, BUF_OZB, BUF_OZE, BUF_OZR, BUF_COUNT };
 
 struct WorkerCtx {
     int pu = -1;         // PU instance index in the model
@@ -578,6 +578,32 @@ bool worker_ozaki(const WorkerCtx &w, bool f64, int *slices, int *rn) {
     return true;
 }
 
+// FP64 variant "ozaki2" (Ozaki scheme II, K6/K7): DGEMM_VARIANT = "ozaki2";
+// OZAKI2_MODULI (default 0 = the fewest giving OZAKI2_BITS), OZAKI2_BITS (default
+// 43: |scaling error| <= 2^-44 of the row / column max; max scaled error at C4
+// in profiles/r01_ozaki2_accuracy.txt).  env PDL_<NAME> overrides.
+bool worker_ozaki2(const WorkerCtx &w, int *nmod, int *bits) {
+    std::string v;
+    if (const char *e = getenv("PDL_DGEMM_VARIANT")) v = e;
+    else if (const Property *p = g->model.prop(w.pu, "DGEMM_VARIANT")) v = p->value;
+    if (lower(trim(v)) != "ozaki2") return false;
+    *nmod = 0;
+    *bits = 43;
+    if (const char *e = getenv("PDL_OZAKI2_MODULI")) *nmod = atoi(e);
+    else if (const Property *p = g->model.prop(w.pu, "OZAKI2_MODULI")) *nmod = atoi(p->value.c_str());
+    if (const char *e = getenv("PDL_OZAKI2_BITS")) *bits = atoi(e);
+    else if (const Property *p = g->model.prop(w.pu, "OZAKI2_BITS")) *bits = atoi(p->value.c_str());
+    *bits = std::max(8, std::min(52, *bits));
+    return true;
+}
+
+bool worker_sgemm_ozaki2(const WorkerCtx &w) {
+    std::string v;
+    if (const char *e = getenv("PDL_SGEMM_VARIANT")) v = e;
+    else if (const Property *p = g->model.prop(w.pu, "SGEMM_VARIANT")) v = p->value;
+    return lower(trim(v)) == "ozaki2";
+}
+
 int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
     if (rows <= 0 || cols <= 0) return PDL_OK;
     CUDA_TRY(cudaSetDevice(w.device));
@@ -651,7 +677,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     // (Ozaki), FP32 K3+K2 (3xTF32) or K4 (Ozaki).
     int oz_slices = 0;
     int oz_rn = 0;
-    const bool ozaki = K > 0 && worker_ozaki(w, f64, &oz_slices, &oz_rn);
+    int oz2_nmod = 0, oz2_bits = 0;
+    if (!f64 && K > 0 && worker_sgemm_ozaki2(w))
+        return set_err(PDL_EUNSUPPORTED, "SGEMM_VARIANT ozaki2: Ozaki scheme II is an FP64 variant (use ozaki)");
+    const bool ozaki2 = K > 0 && f64 && worker_ozaki2(w, &oz2_nmod, &oz2_bits);
+    const bool ozaki = K > 0 && !ozaki2 && worker_ozaki(w, f64, &oz_slices, &oz_rn);
     // FP32 split buffers (K-major hi/lo of A rows and of B^T rows)
     const int64_t Kp = round_up(std::max<int64_t>(K, 1), pdlk::K2_BK);
     float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
@@ -690,6 +720,26 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         oz_ea = oz_fb + round_up(cols, 2);
     }
 
+    pdlk::Ozaki2Plan P2;
+    uint8_t *oz2_R = nullptr;
+    int64_t oz2_ldr = 0, oz2_plane = 0;
+    if (ozaki2) {
+        P2 = pdlk::ozaki2_plan(rows, cols, K, oz2_nmod, oz2_bits);
+        if ((rc = ensure_buf(w, BUF_OZA, P2.a8_bytes, &p))) return rc;
+        a8 = (int8_t *)p;
+        if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
+        b8 = (int8_t *)p;
+        const size_t eb = (size_t)round_up(rows, 2) * 4 + (size_t)round_up(cols, 2) * 4 + (size_t)cols * 8;
+        if ((rc = ensure_buf(w, BUF_OZE, eb, &p))) return rc;
+        oz_bmax = (unsigned long long *)p;
+        oz_fb = (int *)(oz_bmax + cols);
+        oz_ea = oz_fb + round_up(cols, 2);
+        oz2_ldr = round_up(cols, 16);
+        oz2_plane = oz2_ldr * rows;
+        if ((rc = ensure_buf(w, BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
+        oz2_R = (uint8_t *)p;
+    }
+
     // B prepared by a previous task of this Worker (PDL_TASK_REUSE_B)?
     WorkerCtx::BSig want;
     want.valid = true;
@@ -698,10 +748,10 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     want.K = K;
     want.cols = cols;
     want.dtype = t.dtype;
-    want.oz = ozaki ? 1 : 0;
-    want.S = ozaki ? OL.S : 0;
-    want.rn = ozaki ? OL.rn : 0;
-    const bool prep_b = K > 0 && (ozaki || !f64);
+    want.oz = ozaki ? 1 : ozaki2 ? 2 : 0;
+    want.S = ozaki ? OL.S : ozaki2 ? P2.n : 0;
+    want.rn = ozaki ? OL.rn : ozaki2 ? P2.p : 0;
+    const bool prep_b = K > 0 && (ozaki || ozaki2 || !f64);
     const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
 
     std::vector<cudaEvent_t> ev_a(RB, nullptr), ev_b(CP, nullptr), ev_sa(RB, nullptr), ev_sb(CP, nullptr);
@@ -754,6 +804,43 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             cudaError_t e = cudaSuccess;
             if (K == 0) {
                 e = cudaMemset2DAsync(Cs, (size_t)(ldcd * es), 0, (size_t)(nc * es), (size_t)nr, cs);
+            } else if (ozaki2) {
+                // K7 scaling + residues of this band / panel once, shared by both compute streams
+                if (!a_prep[i]) {
+                    a_prep[i] = 1;
+                    e = pdlk::launch_ozaki2_split_a((const double *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K, P2,
+                                                    a8 + r0 * P2.ld8, oz_ea + r0, cs);
+                    w.launches += 1;
+                    if (piped) {
+                        ev_sa[i] = ev_get(w, evn);
+                        CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
+                    }
+                } else if (ev_sa[i]) {
+                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
+                }
+                if (e == cudaSuccess && !b_prep[j] && !b_ready) {
+                    b_prep[j] = 1;
+                    e = pdlk::launch_ozaki2_split_b((const double *)(Bd + (size_t)c0 * es), ldb, K, nc, P2,
+                                                    b8 + c0 * P2.ld8, oz_fb + c0, oz_bmax + c0, cs);
+                    w.launches += 2;
+                    if (piped) {
+                        ev_sb[j] = ev_get(w, evn);
+                        CUDA_TRY(cudaEventRecord(ev_sb[j], cs));
+                    }
+                } else if (ev_sb[j]) {
+                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sb[j], 0));
+                }
+                if (e != cudaSuccess) return set_err(PDL_ECUDA, "K7 residue launch failed: %s", cudaGetErrorString(e));
+                if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
+                int nl = 0;
+                uint8_t *Rs = oz2_R + r0 * oz2_ldr + c0;
+                e = pdlk::launch_ozaki2_gemm(enc, a8 + r0 * P2.ld8, b8 + c0 * P2.ld8, P2, Rs, oz2_ldr, oz2_plane, nr,
+                                             nc, cs, &nl);
+                if (e == cudaSuccess)
+                    e = pdlk::launch_ozaki2_reconstruct(Rs, oz2_ldr, oz2_plane, oz_ea + r0, oz_fb + c0, P2,
+                                                        (double *)Cs, ldcd, nr, nc, cs);
+                if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
+                w.launches += nl + 1;
             } else if (ozaki) {
                 // K5 slicing of this band / panel once, shared by both compute streams
                 if (!a_prep[i]) {
@@ -916,7 +1003,8 @@ int run_dynamic(const Task &t, const std::vector<int> &gw) {
     const int64_t M = t.M, N = t.N, K = t.K, pe = 16 / es;
     for (auto *w : ws) {
         int sl, rn;
-        if (K > 0 && worker_ozaki(*w, f64, &sl, &rn))
+        int n2, b2;
+        if (K > 0 && (worker_ozaki(*w, f64, &sl, &rn) || (f64 && worker_ozaki2(*w, &n2, &b2))))
             return set_err(PDL_EUNSUPPORTED,
                            "DYNAMIC needs a single-launch task variant (dmma / 3xtf32); Worker %s runs Ozaki "
                            "(S diagonal launches updating C)",

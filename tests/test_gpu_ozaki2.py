@@ -1,0 +1,183 @@
+"""GPU parity of the FP64 task variant "ozaki2" (K6/K7: Ozaki scheme II --
+integer scaling, INT8 residue GEMMs on tcgen05 for pairwise-coprime moduli,
+CRT reconstruction) against the CPU oracle.
+
+Selected through the Worker's PDL properties (DGEMM_VARIANT = ozaki2,
+OZAKI2_MODULI, OZAKI2_BITS).  Tolerance: the 1e-12 FP64
+bar of K1 (scaled by D = |A||B|, R13).  Inputs that are integers of
+at most p bits (after the power-of-two row / column scaling) are represented
+exactly, and the CRT rebuilds their product exactly, so those results are
+compared bitwise.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
+
+
+@pytest.fixture(autouse=True)
+def _env(monkeypatch):
+    for k in ("PDL_DRY_RUN", "PDL_DGEMM_VARIANT", "PDL_OZAKI2_MODULI", "PDL_OZAKI2_BITS"):
+        monkeypatch.delenv(k, raising=False)
+    monkeypatch.setenv("PDL_ALLOW_OVERSUBSCRIBE", "1")
+    pdl.unload()
+    yield
+    pdl.unload()
+
+
+def oz2_matmul(A, B, tile=0, workers=1, host=False, moduli=None, bits=None):
+    props = {"DGEMM_VARIANT": "ozaki2"}
+    if moduli:
+        props["OZAKI2_MODULI"] = moduli
+    if bits:
+        props["OZAKI2_BITS"] = bits
+    pdl.load(pdl.descriptor_xml(workers, props=props))
+    try:
+        M, N = A.shape[0], B.shape[1]
+        if host:
+            C = np.full((M, N), np.nan)
+            pdl.task_matmul(A, B, C, tile=tile)
+            pdl.run()
+            return C
+        dA, dB = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+        dC = torch.full((M, N), float("nan"), dtype=torch.float64, device="cuda")
+        pdl.task_matmul(dA, dB, dC, tile=tile)
+        pdl.run()
+        return dC.cpu().numpy()
+    finally:
+        pdl.unload()
+
+
+def check(C, A, B, rows=None, tol=1e-12):
+    Cref, D = oracle.matmul(A, B, rows=rows)
+    err = oracle.scaled_error(C if rows is None else C[rows], Cref, D)
+    assert np.isfinite(err).all()
+    assert err.max() <= tol, f"max scaled err {err.max():.3e} > {tol:g}"
+    return float(err.max())
+
+
+def test_variant_selected_and_launch_count():
+    """13 moduli at the default 43 scaling bits for K <= 16384: split A +
+    (colmax, split B) + 13 residue GEMMs + the CRT pass."""
+    pdl.load(pdl.descriptor_xml(1, props={"DGEMM_VARIANT": "ozaki2"}))
+    assert pdl.query("worker/0/DGEMM_VARIANT") == "ozaki2"
+    A = W.uniform((300, 200), np.float64, 1)
+    B = W.uniform((200, 100), np.float64, 2)
+    dA, dB = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+    dC = torch.empty((300, 100), dtype=torch.float64, device="cuda")
+    pdl.task_matmul(dA, dB, dC)
+    pdl.run()
+    n = pdl.query_json("stats")["launches"] - 4
+    assert 11 <= n <= 13, n       # fewer moduli suffice for K = 200
+    check(dC.cpu().numpy(), A, B)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3"])
+def test_configs_parity(name):
+    c = W.CONFIGS[name]
+    A, B = W.config_inputs(name, np.float64)
+    C = oz2_matmul(A, B, tile=c.tile)
+    rows = None if c.M <= 1024 else W.sampled_rows(c.M, (), c.tile, n_random=32)
+    check(C, A, B, rows=rows)
+
+
+@pytest.mark.parametrize("M,N,K", [(1, 1, 1), (3, 5, 7), (33, 31, 32), (127, 129, 128), (129, 255, 257),
+                                   (257, 130, 33), (200, 17, 1000), (300, 530, 4100)])
+def test_signed_shapes(M, N, K):
+    A = W.signed((M, K), np.float64, 100 + M)
+    B = W.signed((K, N), np.float64, 200 + N)
+    check(oz2_matmul(A, B, tile=32), A, B)
+    check(oz2_matmul(A, B, host=True), A, B)
+
+
+def test_integer_identity_rank1_bitwise():
+    """Small integers (and their power-of-two scalings) are exact p-bit
+    integers, so X = A'B' and C are exact."""
+    A = W.integers((190, 300), np.float64, 7)
+    B = W.integers((300, 170), np.float64, 8)
+    Cref, _ = oracle.matmul(A, B)
+    assert np.array_equal(oz2_matmul(A, B), Cref)
+    u, v = W.rank1_factors(300, 520, 5)
+    x, y = W.rank1_factors(520, 260, 6)
+    expect = (int(np.dot(v, x)) * np.outer(u, y)).astype(np.float64)
+    assert np.array_equal(oz2_matmul(np.outer(u, v).astype(np.float64), np.outer(x, y).astype(np.float64)), expect)
+    I = W.identity(256, 256, np.float64)
+    X = W.dyadic((256, 300), np.float64, 9)
+    assert np.array_equal(oz2_matmul(I, X), X)
+
+
+def test_zero_rows_columns_and_k0():
+    A = W.uniform((130, 90), np.float64, 3)
+    B = W.uniform((90, 70), np.float64, 4)
+    A[5] = 0.0
+    B[:, 7] = 0.0
+    C = oz2_matmul(A, B)
+    assert np.all(C[5] == 0.0) and np.all(C[:, 7] == 0.0)
+    check(C, A, B)
+
+
+def test_invariance_bitwise(monkeypatch):
+    """Scaling exponents come from whole rows of A / columns of B and the
+    CRT is exact, so Worker count, tile and pipelined staging change no bit."""
+    A = W.uniform((700, 390), np.float64, 11)
+    B = W.uniform((390, 333), np.float64, 12)
+    ref = oz2_matmul(A, B)
+    check(ref, A, B)
+    for workers, tile in ((2, 64), (4, 32), (8, 0)):
+        assert np.array_equal(oz2_matmul(A, B, tile=tile, workers=workers), ref)
+    monkeypatch.setenv("PDL_PIPELINE", "force")
+    assert np.array_equal(oz2_matmul(A, B, host=True), ref)
+
+
+def test_k_chunks_beyond_int32_window():
+    """K > 65536 is split into K chunks (each CRT-exact), summed in FP64."""
+    A = W.uniform((64, 70000), np.float64, 21)
+    B = W.uniform((70000, 48), np.float64, 22)
+    check(oz2_matmul(A, B), A, B)
+
+
+def test_wide_exponent_rows_columns():
+    A = W.signed((64, 256), np.float64, 31) * np.exp2(np.arange(64) - 32)[:, None]
+    B = W.signed((256, 48), np.float64, 32) * np.exp2(3 * np.arange(48) - 60)[None, :]
+    check(oz2_matmul(A, B), A, B)
+
+
+@pytest.mark.parametrize("moduli,tol", [(13, 1e-13), (14, 1e-14), (11, 1e-9)])
+def test_moduli_count_accuracy(moduli, tol):
+    """Fewer moduli force fewer scaling bits p (|X| <= K 2^(2p) < M/2)."""
+    A = W.uniform((256, 4096), np.float64, 41)
+    B = W.signed((4096, 256), np.float64, 42)
+    check(oz2_matmul(A, B, moduli=moduli), A, B, tol=tol)
+
+
+@pytest.mark.slow
+def test_c4_full_size_sampled():
+    c = W.CONFIGS["C4"]
+    A, B = W.config_inputs("C4", np.float64)
+    C = oz2_matmul(A, B, tile=c.tile)
+    check(C, A, B, rows=W.sampled_rows(c.M, (), c.tile, n_random=12))
+
+
+@pytest.mark.slow
+def test_c5_ragged_8_workers():
+    c = W.CONFIGS["C5"]
+    A, B = W.config_inputs("C5", np.float64)
+    C = oz2_matmul(A, B, tile=c.tile, workers=8)
+    rows = W.sampled_rows(c.M, (1248, 2496, 3744, 5008, 6256, 7504, 8752), c.tile, n_random=24)
+    check(C, A, B, rows=rows)
+
+
+def test_fp32_ozaki2_is_unsupported():
+    pdl.load(pdl.descriptor_xml(1, props={"SGEMM_VARIANT": "ozaki2"}))
+    A = torch.rand((64, 64), device="cuda")
+    C = torch.empty((64, 64), device="cuda")
+    pdl.task_matmul(A, A, C)
+    with pytest.raises(pdl.PDLError) as e:
+        pdl.run()
+    assert e.value.code == pdl.PDL_EUNSUPPORTED
