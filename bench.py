@@ -427,8 +427,9 @@ def main():
     if args.dtype == "f32":
         roofline["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
     if ozaki:
-        roofline["note"] = ("achieved counts int8 tensor ops (S(S+1)/2 slice products, 2 ops per MAC); "
-                            "useful FP64 FLOP = 2MNK")
+        prods = "one residue GEMM per modulus" if args.variant == "ozaki2" else "S(S+1)/2 slice products"
+        roofline["note"] = (f"achieved counts int8 tensor ops ({prods}, 2 ops per MAC); "
+                            f"useful {args.dtype.upper()} FLOP = 2MNK")
 
     # ---- e2e: host pinned operands through the public API ----
     e2e = None

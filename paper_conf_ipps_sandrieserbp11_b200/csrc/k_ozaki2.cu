@@ -221,66 +221,71 @@ __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
 // ------------------------------------------------------------------------
 struct Oz2Crt {
     int n, nch, p;
-    unsigned long long W[OZ2_MAX_MODULI][2];
-    unsigned long long Mw[2], Hw[2];
-    double Md;
+    unsigned int W[OZ2_MAX_MODULI][4];   // CRT weights as 32-bit limbs (W < M < 2^111)
+    unsigned int Ml[4];                  // M as 32-bit limbs
+    unsigned long long Mw[2], Hw[2];     // M and floor(M / 2) as 64-bit words
+    double invM;                         // 1 / M (rounded)
 };
 
-// 8 consecutive columns per thread: 8 bytes from each plane, 8 doubles out.
+// 4 consecutive columns per thread: 4 bytes from each plane, 4 doubles out.
+// S = sum_t u_t W_t is accumulated limb-wise (u_t < 2^8 times a 32-bit limb: one
+// IMAD.WIDE.U32 per limb, each limb sum < 14 * 2^40); q = floor(S / M) comes from a
+// double estimate (off by at most one), X = S - q M is formed limb-wise in signed
+// 64-bit words and carried into a 128-bit integer, then moved into [0, M) and to
+// the balanced representative in (-M/2, M/2].
+template <int NM>
 __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__restrict__ R, int64_t ldr,
                                                               int64_t plane, const int *__restrict__ ea,
                                                               const int *__restrict__ fb, const Oz2Crt crt,
                                                               double *__restrict__ C, int64_t ldc, int64_t rows,
                                                               int64_t cols) {
     const int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y;
-    const int64_t c8 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
-    if (row >= rows || c8 >= cols) return;
-    const u128 M = ((u128)crt.Mw[1] << 64) | crt.Mw[0];
-    const u128 H = ((u128)crt.Hw[1] << 64) | crt.Hw[0];
-    double acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    const int64_t c4 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4;
+    if (row >= rows || c4 >= cols) return;
+    const __int128 M = (__int128)(((u128)crt.Mw[1] << 64) | crt.Mw[0]);
+    const __int128 H = (__int128)(((u128)crt.Hw[1] << 64) | crt.Hw[0]);
+    double acc[4] = {0, 0, 0, 0};
     for (int c = 0; c < crt.nch; ++c) {
-        // S = sum_t u_t W_t in two 64-bit words per column (u_t < 2^8, W_t < M < 2^111:
-        // S < 14 * 2^119 < 2^128)
-        uint64_t slo[8], shi[8];
+        uint64_t a[4][4];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) slo[j] = shi[j] = 0;
-        for (int t = 0; t < crt.n; ++t) {
-            const uint8_t *pr = R + ((int64_t)c * crt.n + t) * plane + row * ldr + c8;
-            const uint64_t u8x8 = *reinterpret_cast<const uint64_t *>(pr);   // ldr, c8 multiples of 8
-            const uint64_t wl = crt.W[t][0], wh = crt.W[t][1];
+        for (int j = 0; j < 4; ++j)
 #pragma unroll
-            for (int j = 0; j < 8; ++j) {
-                const uint64_t u = (u8x8 >> (8 * j)) & 0xffu;
-                const uint64_t pl = u * wl;
-                const uint64_t ph = __umul64hi(u, wl) + u * wh;
-                slo[j] += pl;
-                shi[j] += ph + (slo[j] < pl ? 1u : 0u);
+            for (int l = 0; l < 4; ++l) a[j][l] = 0;
+        const uint8_t *pr = R + (int64_t)c * NM * plane + row * ldr + c4;
+        uint32_t u4[NM];
+#pragma unroll
+        for (int t = 0; t < NM; ++t)   // all planes' loads in flight together
+            u4[t] = __ldcs(reinterpret_cast<const unsigned int *>(pr + (int64_t)t * plane));   // ldr, c4 % 4 == 0
+#pragma unroll
+        for (int t = 0; t < NM; ++t) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const uint32_t u = __byte_perm(u4[t], 0u, 0x4440u + j);
+#pragma unroll
+                for (int l = 0; l < 4; ++l) a[j][l] += (uint64_t)u * crt.W[t][l];
             }
         }
-        u128 S[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) S[j] = ((u128)shi[j] << 64) | slo[j];
+        for (int j = 0; j < 4; ++j) {
+            const double Sd = fma((double)a[j][3], 79228162514264337593543950336.0,
+                                  fma((double)a[j][2], 18446744073709551616.0,
+                                      fma((double)a[j][1], 4294967296.0, (double)a[j][0])));
+            const uint64_t q = (uint64_t)(Sd * crt.invM);   // floor(S / M) or one off
+            __int128 X = 0;
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            // X = S mod M, then the balanced representative in (-M/2, M/2]
-            const double Sd = (double)(uint64_t)(S[j] >> 64) * 18446744073709551616.0 + (double)(uint64_t)S[j];
-            const uint64_t q = (uint64_t)floor(Sd / crt.Md);
-            __int128 X = (__int128)S[j] - (__int128)((u128)q * M);
-            if (X < 0) X += (__int128)M;
-            if (X < 0) X += (__int128)M;
-            if (X >= (__int128)M) X -= (__int128)M;
-            if (X >= (__int128)M) X -= (__int128)M;
-            if (X > (__int128)H) X -= (__int128)M;
-            const long long hi = (long long)(X >> 64);
-            const uint64_t lo = (uint64_t)X;
-            acc[j] += (double)hi * 18446744073709551616.0 + (double)lo;
+            for (int l = 3; l >= 0; --l)
+                X = X * (__int128)4294967296 + (__int128)((int64_t)a[j][l] - (int64_t)(q * crt.Ml[l]));
+            if (X < 0) X += M;
+            if (X >= M) X -= M;
+            if (X > H) X -= M;
+            acc[j] += (double)(long long)(X >> 64) * 18446744073709551616.0 + (double)(uint64_t)X;
         }
     }
     const int er = ea[row] - 2 * crt.p;
-    double *crow = C + row * ldc + c8;
+    double *crow = C + row * ldc + c4;
 #pragma unroll
-    for (int j = 0; j < 8; ++j)
-        if (c8 + j < cols) crow[j] = scale2(acc[j], er + fb[c8 + j]);
+    for (int j = 0; j < 4; ++j)
+        if (c4 + j < cols) crow[j] = scale2(acc[j], er + fb[c4 + j]);
 }
 
 // ------------------------------------------------------------------------
@@ -339,23 +344,29 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
                                       cudaStream_t s) {
     if (rows <= 0 || cols <= 0) return cudaSuccess;
-    if ((reinterpret_cast<uintptr_t>(R) & 7u) || (ldr & 7) || (plane & 7)) return cudaErrorInvalidValue;
+    if ((reinterpret_cast<uintptr_t>(R) & 3u) || (ldr & 3) || (plane & 3)) return cudaErrorInvalidValue;
     Oz2Crt crt;
     crt.n = P.n;
     crt.nch = P.nch;
     crt.p = P.p;
-    for (int t = 0; t < OZ2_MAX_MODULI; ++t) {
-        crt.W[t][0] = P.W[t][0];
-        crt.W[t][1] = P.W[t][1];
-    }
+    for (int t = 0; t < OZ2_MAX_MODULI; ++t)
+        for (int l = 0; l < 4; ++l) crt.W[t][l] = (unsigned int)(P.W[t][l >> 1] >> (32 * (l & 1)));
+    for (int l = 0; l < 4; ++l) crt.Ml[l] = (unsigned int)(P.Mw[l >> 1] >> (32 * (l & 1)));
     crt.Mw[0] = P.Mw[0];
     crt.Mw[1] = P.Mw[1];
     crt.Hw[0] = P.Hw[0];
     crt.Hw[1] = P.Hw[1];
-    crt.Md = P.Md;
+    crt.invM = 1.0 / P.Md;
     dim3 block(32, 8);
-    dim3 grid((unsigned)((cols + 255) / 256), (unsigned)((rows + 7) / 8));
-    oz2_reconstruct_kernel<<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, crt, C, ldc, rows, cols);
+    dim3 grid((unsigned)((cols + 127) / 128), (unsigned)((rows + 7) / 8));
+    switch (P.n) {
+#define OZ2_CASE(k) \
+    case k: oz2_reconstruct_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, crt, C, ldc, rows, cols); break;
+        OZ2_CASE(2) OZ2_CASE(3) OZ2_CASE(4) OZ2_CASE(5) OZ2_CASE(6) OZ2_CASE(7) OZ2_CASE(8) OZ2_CASE(9) OZ2_CASE(10)
+        OZ2_CASE(11) OZ2_CASE(12) OZ2_CASE(13) OZ2_CASE(14)
+#undef OZ2_CASE
+        default: return cudaErrorInvalidValue;
+    }
     return cudaGetLastError();
 }
 
