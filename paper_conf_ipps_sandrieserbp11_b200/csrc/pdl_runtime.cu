@@ -1392,6 +1392,30 @@ int pdl_query(const char *key, char *out, size_t len) {
     std::string k(key), res;
     if (k == "version") {
         res = kVersion;
+    } else if (k.rfind("ozaki2_plan/", 0) == 0) {
+        // "ozaki2_plan/<K>[/<bits>[/<moduli>]]": the Ozaki-II parameters the FP64
+        // variant ozaki2 uses for inner dimension K (host arithmetic, no device)
+        long long K = 0;
+        int bits = 43, nmod = 0;
+        if (sscanf(k.c_str() + 12, "%lld/%d/%d", &K, &bits, &nmod) < 1 || K < 0)
+            return set_err(PDL_EINVAL, "bad key '%s' (ozaki2_plan/<K>[/<bits>[/<moduli>]])", key);
+        const pdlk::Ozaki2Plan P = pdlk::ozaki2_plan(1, 1, K, nmod, std::max(8, std::min(52, bits)));
+        std::ostringstream o;
+        o << "{\"n\":" << P.n << ",\"p\":" << P.p << ",\"nch\":" << P.nch << ",\"Kc\":" << P.Kc << ",\"moduli\":[";
+        for (int t = 0; t < P.n; ++t) o << (t ? "," : "") << P.m[t];
+        auto dec = [](unsigned long long lo, unsigned long long hi) {   // 128-bit value as decimal text
+            unsigned __int128 v = ((unsigned __int128)hi << 64) | lo;
+            std::string d;
+            do {
+                d.insert(d.begin(), (char)('0' + (int)(v % 10)));
+                v /= 10;
+            } while (v);
+            return d;
+        };
+        o << "],\"W\":[";
+        for (int t = 0; t < P.n; ++t) o << (t ? "," : "") << "\"" << dec(P.W[t][0], P.W[t][1]) << "\"";
+        o << "],\"M\":\"" << dec(P.Mw[0], P.Mw[1]) << "\"}";
+        res = o.str();
     } else {
         int rc = check_loaded();
         if (rc) return rc;
