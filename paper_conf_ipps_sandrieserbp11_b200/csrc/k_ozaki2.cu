@@ -239,11 +239,14 @@ __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__r
                                                               const int *__restrict__ fb, const Oz2Crt crt,
                                                               double *__restrict__ C, int64_t ldc, int64_t rows,
                                                               int64_t cols) {
-    const int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y;
-    const int64_t c4 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4;
-    if (row >= rows || c4 >= cols) return;
     const __int128 M = (__int128)(((u128)crt.Mw[1] << 64) | crt.Mw[0]);
     const __int128 H = (__int128)(((u128)crt.Hw[1] << 64) | crt.Hw[0]);
+    // grid-stride over (row, 4-column group): a full grid visits each item once; the
+    // background launch (one 128-thread CTA per SM beside the GEMMs) strides
+    for (int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y; row < rows;
+         row += (int64_t)gridDim.y * blockDim.y)
+    for (int64_t c4 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4; c4 < cols;
+         c4 += (int64_t)gridDim.x * blockDim.x * 4) {
     double acc[4] = {0, 0, 0, 0};
     for (int c = 0; c < crt.nch; ++c) {
         uint64_t a[4][4];
@@ -286,6 +289,7 @@ __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__r
 #pragma unroll
     for (int j = 0; j < 4; ++j)
         if (c4 + j < cols) crow[j] = scale2(acc[j], er + fb[c4 + j]);
+    }
 }
 
 // ------------------------------------------------------------------------
@@ -314,12 +318,15 @@ static cudaError_t upload_moduli(const Ozaki2Plan &P) {
 }
 
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
-                                  int8_t *A8, int *ea, cudaStream_t s) {
+                                  int8_t *A8, int *ea, cudaStream_t s, bool background) {
     if (rows <= 0) return cudaSuccess;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
-    const int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
-    oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
+    // background: one 128-thread CTA per SM, small enough to sit beside a K6 GEMM CTA
+    const int cap = background ? 148 : 148 * 8;
+    const int blocks = (int)(rows < cap ? rows : cap);
+    oz2_split_rows_kernel<<<blocks, background ? 128 : 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8,
+                                                                  P.ld8, ea);
     return cudaGetLastError();
 }
 
@@ -342,7 +349,7 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
 
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                                      cudaStream_t s) {
+                                      cudaStream_t s, bool background) {
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 3u) || (ldr & 3) || (plane & 3)) return cudaErrorInvalidValue;
     Oz2Crt crt;
@@ -357,8 +364,12 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
     crt.Hw[0] = P.Hw[0];
     crt.Hw[1] = P.Hw[1];
     crt.invM = 1.0 / P.Md;
-    dim3 block(32, 8);
-    dim3 grid((unsigned)((cols + 127) / 128), (unsigned)((rows + 7) / 8));
+    dim3 block(32, background ? 4 : 8);
+    dim3 grid((unsigned)((cols + 127) / 128), (unsigned)((rows + block.y - 1) / block.y));
+    if (background) {   // 148 CTAs of 128 threads, grid-stride
+        grid.x = grid.x < 4u ? grid.x : 4u;
+        grid.y = (148u + grid.x - 1) / grid.x;
+    }
     switch (P.n) {
 #define OZ2_CASE(k) \
     case k: oz2_reconstruct_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, crt, C, ldc, rows, cols); break;
