@@ -241,8 +241,7 @@ __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__r
                                                               int64_t cols) {
     const __int128 M = (__int128)(((u128)crt.Mw[1] << 64) | crt.Mw[0]);
     const __int128 H = (__int128)(((u128)crt.Hw[1] << 64) | crt.Hw[0]);
-    // grid-stride over (row, 4-column group): a full grid visits each item once; the
-    // background launch (one 128-thread CTA per SM beside the GEMMs) strides
+    // grid-stride over (row, 4-column group); the launch covers every item once
     for (int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y; row < rows;
          row += (int64_t)gridDim.y * blockDim.y)
     for (int64_t c4 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4; c4 < cols;
@@ -318,15 +317,12 @@ static cudaError_t upload_moduli(const Ozaki2Plan &P) {
 }
 
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
-                                  int8_t *A8, int *ea, cudaStream_t s, bool background) {
+                                  int8_t *A8, int *ea, cudaStream_t s) {
     if (rows <= 0) return cudaSuccess;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
-    // background: one 128-thread CTA per SM, small enough to sit beside a K6 GEMM CTA
-    const int cap = background ? 148 : 148 * 8;
-    const int blocks = (int)(rows < cap ? rows : cap);
-    oz2_split_rows_kernel<<<blocks, background ? 128 : 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8,
-                                                                  P.ld8, ea);
+    const int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
+    oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
     return cudaGetLastError();
 }
 
@@ -349,7 +345,7 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
 
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                                      cudaStream_t s, bool background) {
+                                      cudaStream_t s) {
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 3u) || (ldr & 3) || (plane & 3)) return cudaErrorInvalidValue;
     Oz2Crt crt;
@@ -364,12 +360,8 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
     crt.Hw[0] = P.Hw[0];
     crt.Hw[1] = P.Hw[1];
     crt.invM = 1.0 / P.Md;
-    dim3 block(32, background ? 4 : 8);
-    dim3 grid((unsigned)((cols + 127) / 128), (unsigned)((rows + block.y - 1) / block.y));
-    if (background) {   // 148 CTAs of 128 threads, grid-stride
-        grid.x = grid.x < 4u ? grid.x : 4u;
-        grid.y = (148u + grid.x - 1) / grid.x;
-    }
+    dim3 block(32, 8);
+    dim3 grid((unsigned)((cols + 127) / 128), (unsigned)((rows + 7) / 8));
     switch (P.n) {
 #define OZ2_CASE(k) \
     case k: oz2_reconstruct_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, crt, C, ldc, rows, cols); break;

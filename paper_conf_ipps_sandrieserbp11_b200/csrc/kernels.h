@@ -89,10 +89,8 @@ struct Ozaki2Plan {
 };
 // nmod = 0: the fewest moduli that give p >= bits for this K chunk.
 Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits);
-// background = true: a grid of one 128-thread CTA per SM that co-resides with the K6
-// GEMM CTAs (run on a second stream while the GEMMs of another band execute)
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
-                                  int8_t *A8, int *ea, cudaStream_t s, bool background = false);
+                                  int8_t *A8, int *ea, cudaStream_t s);
 cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
                                   int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s);
 cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
@@ -100,7 +98,7 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
                                int *launches);
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                                      cudaStream_t s, bool background = false);
+                                      cudaStream_t s);
 
 // K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,

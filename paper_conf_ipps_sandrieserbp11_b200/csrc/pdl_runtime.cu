@@ -86,7 +86,6 @@ struct WorkerCtx {
     int sm_limit = 0;
     CUgreenCtx gctx = nullptr;
     cudaEvent_t ev_legacy = nullptr;   // orders the non-blocking green stream with the legacy stream
-    cudaStream_t prio[2] = {nullptr, nullptr};   // Ozaki-II banded schedule: high / low priority
     DevBuf buf[BUF_COUNT];
     cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr;   // around the dominant kernel of the last task
     int launches = 0;                               // kernels launched in the last run
@@ -469,8 +468,6 @@ void free_state() {
         for (auto ev : w.ev_pool) cudaEventDestroy(ev);
         for (auto st : w.aux)
             if (st) cudaStreamDestroy(st);
-        for (auto st : w.prio)
-            if (st) cudaStreamDestroy(st);
         if (w.gctx) green_api()->destroy(w.gctx);
     }
     if (g->dyn) {
@@ -756,90 +753,6 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     want.rn = ozaki ? OL.rn : ozaki2 ? P2.p : 0;
     const bool prep_b = K > 0 && (ozaki || ozaki2 || !f64);
     const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
-
-    // Ozaki-II on device-resident operands: row bands whose K6 GEMMs run on a
-    // high-priority stream while, on a low-priority stream, the K7 residues of the
-    // next band and the CRT pass of the previous band run as background grids (one
-    // 128-thread CTA per SM, small enough to sit beside a GEMM CTA), so the FP64 /
-    // ALU work hides under the tensor-core work.  Bitwise the one-band result.
-    int oz2_nb = 4;
-    if (const char *e = getenv("PDL_OZ2_BANDS")) oz2_nb = std::max(1, atoi(e));
-    oz2_nb = (int)std::min<int64_t>(oz2_nb, rows / 512);
-    if (ozaki2 && !piped && !a_st && !b_st && !w.gctx && oz2_nb >= 2 && flops >= 2e11) {
-        int pr_lo = 0, pr_hi = 0;
-        CUDA_TRY(cudaDeviceGetStreamPriorityRange(&pr_lo, &pr_hi));
-        if (!w.prio[0]) CUDA_TRY(cudaStreamCreateWithPriority(&w.prio[0], cudaStreamNonBlocking, pr_hi));
-        if (!w.prio[1]) CUDA_TRY(cudaStreamCreateWithPriority(&w.prio[1], cudaStreamNonBlocking, pr_lo));
-        cudaStream_t H = w.prio[0], L = w.prio[1];
-        size_t evn = 0;
-        auto rec = [&](cudaStream_t st) -> cudaEvent_t {
-            cudaEvent_t e = ev_get(w, evn);
-            if (e && cudaEventRecord(e, st) != cudaSuccess) return nullptr;
-            return e;
-        };
-        cudaEvent_t e0 = rec(w.stream);
-        if (!e0) return set_err(PDL_ECUDA, "event record failed");
-        CUDA_TRY(cudaStreamWaitEvent(H, e0, 0));
-        CUDA_TRY(cudaStreamWaitEvent(L, e0, 0));
-        std::vector<int64_t> bc(oz2_nb + 1);
-        for (int b = 0; b <= oz2_nb; ++b) bc[b] = std::min<int64_t>(rows, round_up((int64_t)b * rows / oz2_nb, 256));
-        bc[oz2_nb] = rows;
-        cudaError_t e = cudaSuccess;
-        if (!b_ready) {
-            e = pdlk::launch_ozaki2_split_b((const double *)Bd, ldb, K, cols, P2, b8, oz_fb, oz_bmax, H);
-            w.launches += 2;
-        }
-        if (e == cudaSuccess) {
-            e = pdlk::launch_ozaki2_split_a((const double *)Ad, lda, bc[1], K, P2, a8, oz_ea, H);
-            w.launches += 1;
-        }
-        if (e != cudaSuccess) return set_err(PDL_ECUDA, "K7 residue launch failed: %s", cudaGetErrorString(e));
-        cudaEvent_t ev_next = nullptr;
-        for (int b = 0; b < oz2_nb; ++b) {
-            const int64_t r0 = bc[b], nr = bc[b + 1] - bc[b];
-            if (nr <= 0) continue;
-            if (ev_next) CUDA_TRY(cudaStreamWaitEvent(H, ev_next, 0));
-            cudaEvent_t gs = rec(H);
-            if (!gs || kt_mark(w, true, H)) return set_err(PDL_ECUDA, "event record failed");
-            int nl = 0;
-            e = pdlk::launch_ozaki2_gemm(enc, a8 + r0 * P2.ld8, b8, P2, oz2_R + r0 * oz2_ldr, oz2_ldr, oz2_plane, nr,
-                                         cols, H, &nl);
-            if (e != cudaSuccess) return set_err(PDL_ECUDA, "K6 launch failed: %s", cudaGetErrorString(e));
-            w.launches += nl;
-            if (kt_mark(w, false, H)) return set_err(PDL_ECUDA, "event record failed");
-            cudaEvent_t gd = rec(H);
-            if (!gd) return set_err(PDL_ECUDA, "event record failed");
-            CUDA_TRY(cudaStreamWaitEvent(L, gs, 0));
-            ev_next = nullptr;
-            if (b + 1 < oz2_nb && bc[b + 2] > bc[b + 1]) {
-                e = pdlk::launch_ozaki2_split_a((const double *)(Ad + (size_t)(bc[b + 1] * lda) * es), lda,
-                                                bc[b + 2] - bc[b + 1], K, P2, a8 + bc[b + 1] * P2.ld8,
-                                                oz_ea + bc[b + 1], L, true);
-                if (e != cudaSuccess) return set_err(PDL_ECUDA, "K7 residue launch failed: %s", cudaGetErrorString(e));
-                w.launches += 1;
-                ev_next = rec(L);
-                if (!ev_next) return set_err(PDL_ECUDA, "event record failed");
-            }
-            CUDA_TRY(cudaStreamWaitEvent(L, gd, 0));
-            const bool last = b + 1 == oz2_nb;
-            e = pdlk::launch_ozaki2_reconstruct(oz2_R + r0 * oz2_ldr, oz2_ldr, oz2_plane, oz_ea + r0, oz_fb, P2,
-                                                (double *)(Cd + (size_t)(r0 * ldcd) * es), ldcd, nr, cols, L, !last);
-            if (e != cudaSuccess) return set_err(PDL_ECUDA, "K6 CRT launch failed: %s", cudaGetErrorString(e));
-            w.launches += 1;
-        }
-        cudaEvent_t eh = rec(H), el = rec(L);
-        if (!eh || !el) return set_err(PDL_ECUDA, "event record failed");
-        CUDA_TRY(cudaStreamWaitEvent(w.stream, eh, 0));
-        CUDA_TRY(cudaStreamWaitEvent(w.stream, el, 0));
-        w.timed = true;
-        w.bsig = want;
-        w.bsig.valid = !b_st;
-        if (c_st) {
-            CUDA_TRY(cudaMemcpy2DAsync(C, (size_t)(t.ldc * es), Cd, (size_t)(ldcd * es), (size_t)(cols * es),
-                                       (size_t)rows, cudaMemcpyDefault, w.stream));
-        }
-        return PDL_OK;
-    }
 
     std::vector<cudaEvent_t> ev_a(RB, nullptr), ev_b(CP, nullptr), ev_sa(RB, nullptr), ev_sb(CP, nullptr);
     cudaEvent_t ev_last_out = nullptr, ev_last_cmp1 = nullptr;
