@@ -173,7 +173,18 @@ constexpr int A_BYTES = BM * BK;        // 16 KiB
 constexpr int B_BYTES = BNH * BK;       // 16 KiB per N=256 sub-tile
 constexpr int EPI_WARPS = 16, FIRST_EPI_WARP = 2;
 constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
-constexpr int GROUP_M = 4;   // raster sweep (tools/sweep_group.sh): 4 best of {2,4,8,16,32}
+// Raster group (cluster-tile rows sweeping the columns together) from the K extent
+// of the launch: the group's A strips (256 rows x K' bytes each) should stay in L2
+// while the columns go by, so long diagonals take small groups.  Sweeps at C4
+// (profiles/r01_sweep_group*.txt): K' = 16384 -> 16 (Ozaki-II: DRAM 5.37 -> 3.52
+// GB per launch, 182.8 -> 189.7 TFLOP/s; 32, 64 thrash), FP32 Ozaki (K' <= 3K) 8
+// over 4, FP64 Ozaki-I (K' <= 6K) 4 ~ 8.  PDL_GROUP_M overrides.
+inline int group_for_k(int64_t kd) {
+    const int64_t strip = 256 * kd;
+    int g = 16;
+    while (g > 4 && (int64_t)g * strip > ((int64_t)96 << 20)) g >>= 1;
+    return raster_group_m(g);
+}
 template <int NSUB> struct Cfg {
     static constexpr int BN = BN1 * NSUB;
     static constexpr int STAGE_BYTES = A_BYTES + NSUB * B_BYTES;
@@ -533,11 +544,11 @@ static cudaError_t gemm_impl(EncodeTiledFn enc, const int8_t *A8, const int8_t *
             if (nsub == 2)
                 oz_gemm_2sm_kernel<2, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
                     ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
-                    tiles_n, raster_group_m(GROUP_M), vec_ok, 0, 0.f);
+                    tiles_n, group_for_k(kd), vec_ok, 0, 0.f);
             else
                 oz_gemm_2sm_kernel<1, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
                     ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
-                    tiles_n, raster_group_m(GROUP_M), vec_ok, 0, 0.f);
+                    tiles_n, group_for_k(kd), vec_ok, 0, 0.f);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             first = 0;
@@ -595,11 +606,11 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
             if (nsub == 2)
                 oz_gemm_2sm_kernel<2, uint8_t><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
                     ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, nullptr, nullptr, 0, 0, tiles_m, tiles_n,
-                    raster_group_m(GROUP_M), 1, P.m[t], inv);
+                    group_for_k(P.Kc), 1, P.m[t], inv);
             else
                 oz_gemm_2sm_kernel<1, uint8_t><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
                     ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, nullptr, nullptr, 0, 0, tiles_m, tiles_n,
-                    raster_group_m(GROUP_M), 1, P.m[t], inv);
+                    group_for_k(P.Kc), 1, P.m[t], inv);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             if (launches) ++*launches;
