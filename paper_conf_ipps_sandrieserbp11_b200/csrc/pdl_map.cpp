@@ -15,6 +15,7 @@
 #include <cmath>
 #include <cstdlib>
 #include <limits>
+#include <map>
 #include <sstream>
 
 #include "pdl_model.hpp"
@@ -24,6 +25,7 @@ namespace pdl {
 static int64_t cdiv(int64_t a, int64_t b) { return b ? (a + b - 1) / b : 0; }
 
 Rect Plan::rect(int w) const {
+    if (!wrect.empty()) return wrect[w];
     int r = w / Gc, c = w % Gc;
     return Rect{row[r], row[r + 1], col[c], col[c + 1]};
 }
@@ -200,6 +202,104 @@ Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec di
     return p;
 }
 
+// ---- hierarchical BLOCK (Hybrid PUs) ----
+namespace {
+struct TNode {
+    int pu = -1;            // model PU index (Master / Hybrid), or the Worker's
+    int worker = -1;        // group index for a leaf
+    std::vector<int> kids;  // node indices, document order
+    double weight = 0.0;    // total RELATIVE_SPEED of the subtree's group Workers
+};
+
+// Map C rows [r0, r1) (elements; task-row aligned) x all columns onto node n.
+void place(const std::vector<TNode> &T, int n, int64_t r0, int64_t r1, int64_t M, int64_t N, int64_t K, int64_t tile,
+           const std::vector<double> &speeds, int unit, Plan &P) {
+    const TNode &nd = T[n];
+    if (nd.worker >= 0) {
+        P.wrect[nd.worker] = Rect{r0, r1, 0, N};
+        P.wunit[nd.worker] = unit;
+        return;
+    }
+    if (nd.kids.size() == 1) {
+        place(T, nd.kids[0], r0, r1, M, N, K, tile, speeds, unit, P);
+        return;
+    }
+    bool leaves = true;
+    for (int k : nd.kids) leaves &= T[k].worker >= 0;
+    if (leaves) {   // a PU controlling only Workers: the flat BLOCK plan on its band
+        std::vector<double> sp;
+        for (int k : nd.kids) sp.push_back(speeds[T[k].worker]);
+        Plan sub = make_plan(r1 - r0, N, K, tile, (int)nd.kids.size(), DistSpec(), &sp);
+        for (size_t i = 0; i < nd.kids.size(); ++i) {
+            Rect R = sub.rect((int)i);
+            R.row0 += r0;
+            R.row1 += r0;
+            P.wrect[T[nd.kids[i]].worker] = R;
+            P.wunit[T[nd.kids[i]].worker] = unit;
+        }
+        return;
+    }
+    // row bands per child subtree, whole task rows, proportional to subtree speed
+    const int64_t edge = tile > 0 ? tile : 1;
+    const int64_t t0 = r0 / edge, units = (r1 - r0 + edge - 1) / edge;
+    double tot = 0.0;
+    for (int k : nd.kids) tot += T[k].weight;
+    double acc = 0.0;
+    int64_t prev = r0;
+    for (size_t i = 0; i < nd.kids.size(); ++i) {
+        acc += T[nd.kids[i]].weight;
+        const int64_t tb = i + 1 == nd.kids.size() ? t0 + units : t0 + (int64_t)std::llround(units * acc / tot);
+        const int64_t rb = std::min(r1, tb * edge);
+        place(T, nd.kids[i], prev, std::max(prev, rb), M, N, K, tile, speeds, unit < 0 ? (int)i : unit, P);
+        prev = std::max(prev, rb);
+    }
+}
+}  // namespace
+
+Plan make_plan_tree(int64_t M, int64_t N, int64_t K, int64_t tile, const Model &m, const std::vector<int> &gw,
+                    DistSpec dist, const std::vector<double> &speeds) {
+    const int G = (int)gw.size();
+    Plan flat = make_plan(M, N, K, tile, G, dist, &speeds);
+    if (dist.kind != Dist::Block || G < 2) return flat;
+    // tree of the controlling PUs of the group's Workers
+    std::vector<TNode> T(1);   // node 0: the virtual root above the Masters
+    std::map<int, int> node_of;   // model PU -> node
+    for (int w = 0; w < G; ++w) {
+        std::vector<int> chain;   // Worker, its controllers ..., top-level PU
+        for (int p = gw[w]; p >= 0; p = m.pus[p].parent) chain.push_back(p);
+        int parent = 0;
+        for (int i = (int)chain.size() - 1; i >= 0; --i) {
+            auto it = node_of.find(chain[i]);
+            int nd;
+            if (it == node_of.end()) {
+                nd = (int)T.size();
+                T.push_back(TNode());
+                T[nd].pu = chain[i];
+                if (i == 0) T[nd].worker = w;
+                node_of[chain[i]] = nd;
+                T[parent].kids.push_back(nd);
+            } else {
+                nd = it->second;
+            }
+            T[nd].weight += speeds[w];
+            parent = nd;
+        }
+        T[0].weight += speeds[w];
+    }
+    // flat when no PU below the Masters splits the group (all Workers are children of
+    // one controller, possibly through a chain of single-child Hybrids)
+    int n = 0;
+    while (T[n].worker < 0 && T[n].kids.size() == 1) n = T[n].kids[0];
+    bool leaves = T[n].worker < 0;
+    for (int k : T[n].kids) leaves &= T[k].worker >= 0;
+    if (leaves) return flat;
+    Plan P = flat;
+    P.wrect.assign(G, Rect());
+    P.wunit.assign(G, -1);
+    place(T, n, 0, M, M, N, K, tile, speeds, -1, P);
+    return P;
+}
+
 std::string Plan::to_json(const std::vector<int> &workers, const std::vector<std::string> &ids) const {
     std::ostringstream o;
     o << "{\"M\":" << M << ",\"N\":" << N << ",\"K\":" << K << ",\"tile\":" << tile << ",\"G\":" << G
@@ -207,11 +307,19 @@ std::string Plan::to_json(const std::vector<int> &workers, const std::vector<std
       << ",\"qb\":" << qb() << ",\"exchanged_elems\":" << (int64_t)exchanged_elems() << ",\"dist\":\""
       << (dist.kind == Dist::Block ? "BLOCK" : dist.kind == Dist::Cyclic ? "CYCLIC"
           : dist.kind == Dist::Dynamic ? "DYNAMIC" : "BLOCK-CYCLIC") << "\",\"dist_b\":"
-      << dist.b << ",\"workers\":[";
+      << dist.b << ",\"hierarchical\":" << (hierarchical() ? "true" : "false") << ",\"workers\":[";
     for (int w = 0; w < G; ++w) {
         Rect R = rect(w);
         int r = w / Gc, c = w % Gc;
         if (w) o << ",";
+        if (hierarchical()) {   // explicit rectangle inside its Hybrid subtree's band
+            const int64_t e = tile > 0 ? tile : 1;
+            o << "{\"w\":" << w << ",\"id\":\"" << (w < (int)ids.size() ? json_escape(ids[w]) : "")
+              << "\",\"unit\":" << wunit[w] << ",\"rows\":[" << R.row0 << "," << R.row1 << "],\"cols\":[" << R.col0
+              << "," << R.col1 << "],\"task_rows\":[" << R.row0 / e << "," << (R.row1 + e - 1) / e
+              << "],\"task_cols\":[" << R.col0 / e << "," << (R.col1 + e - 1) / e << "]}";
+            continue;
+        }
         if (dist.kind == Dist::Dynamic) {   // no static rectangle: tiles are claimed at run time
             o << "{\"w\":" << w << ",\"id\":\"" << (w < (int)ids.size() ? json_escape(ids[w]) : "")
               << "\",\"rows\":[0," << M << "],\"cols\":[0," << N << "],\"dynamic\":true}";

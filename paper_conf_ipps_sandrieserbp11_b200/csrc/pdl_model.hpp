@@ -121,6 +121,12 @@ struct Plan {
     int64_t Tm = 0, Tn = 0;                  // task grid
     std::vector<int64_t> trow, tcol;         // BLOCK: task-row / task-col boundaries per grid row / col
     std::vector<int64_t> row, col;           // BLOCK: element boundaries (Gr+1, Gc+1)
+    // Hierarchical BLOCK through Hybrid PUs: explicit per-Worker rectangles and the
+    // index of the Master's child subtree (level-1 unit) holding each Worker; empty
+    // for a flat plan
+    std::vector<Rect> wrect;
+    std::vector<int> wunit;
+    bool hierarchical() const { return !wrect.empty(); }
     Rect rect(int w) const;                  // BLOCK: the Worker's rectangle, w = r*Gc + c
     int64_t qa(int w) const;                 // rows per A chunk for Worker w
     int64_t qb() const;                      // K-rows per B chunk
@@ -143,6 +149,18 @@ struct Plan {
 // proportional to speed (cumulative rounding), so every Worker finishes together.
 Plan make_plan(int64_t M, int64_t N, int64_t K, int64_t tile, int G, DistSpec dist = DistSpec(),
                const std::vector<double> *speeds = nullptr);
+
+// Mapping through the PU hierarchy (Hybrid PUs "act as Master and
+// Worker ... inner nodes", L513-531): the group's Workers are arranged in the tree
+// of their controlling PUs below the Master.  Where a PU controls more than one
+// subtree holding group Workers, BLOCK splits its C block into row bands, one per
+// subtree in document order, sized by the subtree's total RELATIVE_SPEED in whole
+// task rows (cumulative rounding); a PU whose children are all Workers maps its
+// band with make_plan.  A flat tree (every Worker directly under the Master, or a
+// single chain) gives exactly make_plan.  gw = the group's Workers (PU indices,
+// document order); dist other than BLOCK ignores the hierarchy.
+Plan make_plan_tree(int64_t M, int64_t N, int64_t K, int64_t tile, const Model &m, const std::vector<int> &gw,
+                    DistSpec dist, const std::vector<double> &speeds);
 
 // RELATIVE_SPEED of the group's Workers (1 when absent or invalid).
 std::vector<double> worker_speeds(const Model &m, const std::vector<int> &workers);

@@ -1236,7 +1236,11 @@ int execute(bool sync) {
             return set_err(PDL_ENOWORKER, "group has %d Workers but %d ranks co-exist: one process per Worker", G,
                            g->nranks);
         const std::vector<double> speeds = worker_speeds(g->model, gw);
-        Plan plan = make_plan(t.M, t.N, t.K, t.tile, G, t.dist, &speeds);
+        // one process driving the Workers maps through the PU hierarchy (Hybrid
+        // subtrees, NEXT-4); the multi-rank panel exchange needs the flat grid
+        Plan plan = g->nranks == 1 && !(t.flags & PDL_TASK_PANELS)
+                        ? make_plan_tree(t.M, t.N, t.K, t.tile, g->model, gw, t.dist, speeds)
+                        : make_plan(t.M, t.N, t.K, t.tile, G, t.dist, &speeds);
         std::vector<std::string> ids;
         for (int x : gw) ids.push_back(g->model.pus[x].id);
         if (ti) pj << ",";
@@ -1378,8 +1382,18 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group, i
     const int G = (int)gw.size();
     if (worker < 0 || worker >= G) return set_err(PDL_EINVAL, "worker %d outside the group of %d", worker, G);
     const std::vector<double> speeds = worker_speeds(g->model, gw);
-    Plan p = make_plan(M, N, K, tile, G, DistSpec(), &speeds);
+    Plan p = g->nranks == 1 ? make_plan_tree(M, N, K, tile, g->model, gw, DistSpec(), speeds)
+                            : make_plan(M, N, K, tile, G, DistSpec(), &speeds);
     Rect R = p.rect(worker);
+    if (p.hierarchical()) {
+        // explicit rectangle (Hybrid subtrees): no Worker grid, no panel exchange
+        const int64_t e = p.tile > 0 ? p.tile : 1;
+        int64_t v[PDL_PLAN_LEN] = {G, G, 1, worker, 0, R.row0, R.row1, R.col0, R.col1, R.row1 - R.row0, K,
+                                   p.Tm, p.Tn, R.row0 / e, (R.row1 + e - 1) / e, R.col0 / e, (R.col1 + e - 1) / e,
+                                   p.tile};
+        for (int i = 0; i < PDL_PLAN_LEN; ++i) out[i] = v[i];
+        return PDL_OK;
+    }
     const int r = worker / p.Gc, c = worker % p.Gc;
     int64_t v[PDL_PLAN_LEN] = {G, p.Gr, p.Gc, r, c, R.row0, R.row1, R.col0, R.col1, p.qa(worker), p.qb(),
                                p.Tm, p.Tn, p.trow[r], p.trow[r + 1], p.tcol[c], p.tcol[c + 1], p.tile};
