@@ -147,7 +147,11 @@ int task_matmul_f32(const float *A, const float *B, float *C,
  *   process driving the Workers (pdl_load): with PDL_TASK_PANELS or
  *   pdl_load_rank they return PDL_EUNSUPPORTED.  Unknown names -> PDL_EINVAL.
  *   Workers whose PDL property RELATIVE_SPEED differs get a speed-weighted
- *   1-D BLOCK split (heterogeneous platforms, L1398-1402).
+ *   1-D BLOCK split (heterogeneous platforms, L1398-1402).  With one process
+ *   driving the Workers, BLOCK follows the PU hierarchy: a PU whose group
+ *   Workers lie in several subtrees (Hybrid PUs, L513-531) gives each subtree a
+ *   row band sized by its total RELATIVE_SPEED (pdl_plan then reports Gr = G,
+ *   Gc = 1 and the Worker's explicit rectangle).
  * flags: 0 or PDL_TASK_PANELS.
  */
 int task_matmul_ex(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb,
