@@ -448,11 +448,16 @@ OzakiLayout ozaki_layout(int64_t rows, int64_t cols, int64_t K, int S) {
     return L;
 }
 
+static int split_ctas() {
+    const char *e = getenv("PDL_SPLIT_CTAS");
+    return e && atoi(e) > 0 ? atoi(e) : 148 * 8;
+}
+
 template <typename T>
 static cudaError_t split_a_impl(const T *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L, int8_t *A8,
                                 int *ea, cudaStream_t s) {
     if (rows <= 0) return cudaSuccess;
-    int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
+    int blocks = (int)(rows < split_ctas() ? rows : split_ctas());
     oz_split_rows_kernel<T><<<blocks, 256, 0, s>>>(A, lda, rows, K, L.S, L.Kc, L.nch, A8, L.ld8, ea, L.rn);
     return cudaGetLastError();
 }

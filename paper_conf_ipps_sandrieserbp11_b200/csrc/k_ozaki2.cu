@@ -294,6 +294,15 @@ __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__r
 // ------------------------------------------------------------------------
 // host launchers
 // ------------------------------------------------------------------------
+// CTAs of the row-slicing kernels (tuning knob PDL_SPLIT_CTAS).  C4 sweep of
+// oz2_split_rows: 148 / 296 / 592 / 1184 CTAs -> 4.90 / 3.11 / 2.60 / 2.41 ms with
+// 2.4 / 2.4 / 3.3 / 3.5 GB DRAM read: fewer CTAs keep the second read of a row in
+// L2 but lose more latency hiding than they save bandwidth.
+static int split_ctas() {
+    const char *e = getenv("PDL_SPLIT_CTAS");
+    return e && atoi(e) > 0 ? atoi(e) : 148 * 8;
+}
+
 static cudaError_t upload_moduli(const Ozaki2Plan &P) {
     // identical for every plan (the moduli table is fixed); cheap synchronous copy
     static bool done = false;
@@ -321,7 +330,7 @@ cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, in
     if (rows <= 0) return cudaSuccess;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
-    const int blocks = (int)(rows < 148 * 8 ? rows : 148 * 8);
+    const int blocks = (int)(rows < split_ctas() ? rows : split_ctas());
     oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
     return cudaGetLastError();
 }
