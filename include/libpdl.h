@@ -71,6 +71,13 @@ extern "C" {
                                 (first) Worker: no mapping over the group.  The multi-rank
                                 runtime uses it to compute a Worker rectangle chunk by chunk
                                 while the exchange of the next chunk is in flight */
+#define PDL_TASK_GRAPH 8u    /* replay this task's launch sequence from a CUDA graph: the first
+                                run of a task signature (dtype, pointers, sizes, leading dims,
+                                tile, flags, stream) runs normally, the second is captured, later
+                                runs are one cudaGraphLaunch per Worker (launch-bound small
+                                tasks).  Env PDL_GRAPH=1 sets it for every task.  Ignored with
+                                PDL_TASK_REUSE_B and DYNAMIC; uncapturable work (pageable host
+                                memory) runs uncaptured */
 #define PDL_TASK_REUSE_B 4u  /* B (same pointer, ldb, K, N) is unchanged since the previous task
                                 of this Worker: reuse its prepared form (FP32 split / Ozaki
                                 slices) instead of recomputing it; ignored when no matching

@@ -22,6 +22,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <fstream>
+#include <map>
 #include <memory>
 #include <sstream>
 #include <string>
@@ -90,9 +91,26 @@ struct WorkerCtx {
     cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr;   // around the dominant kernel of the last task
     int launches = 0;                               // kernels launched in the last run
     bool timed = false;
-    // event pairs around every dominant-kernel launch since the last pdl_kernel_times()
-    std::vector<cudaEvent_t> kt_ev;
-    size_t kt_n = 0;
+    // event pairs around every dominant-kernel launch since the last pdl_kernel_times():
+    // kt_list holds the pairs in launch order; plain launches take events from kt_pool
+    // (kt_used of them in use), graph replays append the events their graph records
+    std::vector<cudaEvent_t> kt_pool;
+    size_t kt_used = 0;
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kt_list;
+    cudaEvent_t kt_open = nullptr;   // start event of the launch being bracketed
+    // CUDA graphs of repeated tasks (PDL_TASK_GRAPH / PDL_GRAPH=1): signature -> graph
+    struct GraphEntry {
+        cudaGraphExec_t exec = nullptr;
+        std::vector<cudaEvent_t> events;                              // owned; recorded by the graph
+        std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kt_pairs;
+        int launches = 0;
+        bool timed = false;
+    };
+    std::map<std::string, GraphEntry> graphs;
+    std::map<std::string, int> graph_seen;   // signatures run once (captured on the next run)
+    int buf_gen = 0;                         // bumped when a buffer is reallocated (graphs go stale)
+    bool capturing = false;
+    long long graph_replays = 0;
     // pipelined staging: copy-in, copy-out, second compute stream; reusable events
     cudaStream_t aux[3] = {nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> ev_pool;
@@ -112,20 +130,28 @@ struct WorkerCtx {
 
 constexpr size_t kMaxKernelTimes = 4096;
 
-// Record the start / end of a dominant-kernel launch on the worker's stream.
+// Record the start / end of a dominant-kernel launch on the worker's stream.  While a
+// graph is being captured the records are external event-record nodes of the graph
+// and the events move to its entry (they must not be reused by plain launches).
 int kt_mark(WorkerCtx &w, bool start, cudaStream_t st) {
+    auto record = [&](cudaEvent_t ev) {
+        return w.capturing ? cudaEventRecordWithFlags(ev, st, cudaEventRecordExternal) : cudaEventRecord(ev, st);
+    };
     cudaEvent_t &last = start ? w.ev_k0 : w.ev_k1;
-    cudaError_t e = cudaEventRecord(last, st);
-    if (e != cudaSuccess) return PDL_ECUDA;
-    if (w.kt_n >= kMaxKernelTimes) return PDL_OK;
-    size_t idx = 2 * w.kt_n + (start ? 0 : 1);
-    if (idx >= w.kt_ev.size()) {
+    if (record(last) != cudaSuccess) return PDL_ECUDA;
+    if (w.kt_list.size() >= kMaxKernelTimes) return PDL_OK;
+    if (w.kt_used >= w.kt_pool.size()) {
         cudaEvent_t ev;
         if (cudaEventCreate(&ev) != cudaSuccess) return PDL_ECUDA;
-        w.kt_ev.push_back(ev);
+        w.kt_pool.push_back(ev);
     }
-    if (cudaEventRecord(w.kt_ev[idx], st) != cudaSuccess) return PDL_ECUDA;
-    if (!start) w.kt_n++;
+    cudaEvent_t ev = w.kt_pool[w.kt_used++];
+    if (record(ev) != cudaSuccess) return PDL_ECUDA;
+    if (start) {
+        w.kt_open = ev;
+    } else {
+        w.kt_list.emplace_back(w.kt_open, ev);
+    }
     return PDL_OK;
 }
 
@@ -464,7 +490,11 @@ void free_state() {
         if (w.ev_k0) cudaEventDestroy(w.ev_k0);
         if (w.ev_k1) cudaEventDestroy(w.ev_k1);
         if (w.ev_legacy) cudaEventDestroy(w.ev_legacy);
-        for (auto ev : w.kt_ev) cudaEventDestroy(ev);
+        for (auto ev : w.kt_pool) cudaEventDestroy(ev);
+        for (auto &ge : w.graphs) {
+            if (ge.second.exec) cudaGraphExecDestroy(ge.second.exec);
+            for (auto ev : ge.second.events) cudaEventDestroy(ev);
+        }
         for (auto ev : w.ev_pool) cudaEventDestroy(ev);
         for (auto st : w.aux)
             if (st) cudaStreamDestroy(st);
@@ -494,6 +524,7 @@ int ensure_buf(WorkerCtx &w, int slot, size_t bytes, void **out) {
                            cudaGetErrorString(e));
         }
         b.bytes = bytes;
+        ++w.buf_gen;   // captured graphs hold the old pointer
         if (slot == BUF_BHI || slot == BUF_BLO || slot == BUF_OZB || slot == BUF_OZE) w.bsig.valid = false;
     }
     *out = b.ptr;
@@ -1115,6 +1146,98 @@ int run_dynamic(const Task &t, const std::vector<int> &gw) {
     return PDL_OK;
 }
 
+// ---- CUDA graphs of repeated tasks ----
+//
+// A Worker's launch sequence for one task (staging copies, split / slicing
+// pre-passes, tile kernels, CRT pass, copy-out, across its side streams) depends
+// only on the task's signature.  With PDL_TASK_GRAPH (or PDL_GRAPH=1) the first run
+// of a signature executes normally (sizing the Worker's buffers), the second is
+// captured from the Worker stream into a CUDA graph, and later runs replay it with
+// one cudaGraphLaunch -- for launch-bound small tasks.  Anything the capture cannot
+// hold (pageable host memory, a buffer reallocation) makes that signature run
+// uncaptured from then on.  Not used with PDL_TASK_REUSE_B (its launches depend on
+// state left by the previous task) or DYNAMIC.
+
+std::string graph_key(const WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows,
+                      int64_t cols) {
+    std::ostringstream k;
+    k << t.dtype << '|' << A << '|' << t.lda << '|' << B << '|' << t.ldb << '|' << C << '|' << t.ldc << '|' << t.M
+      << '|' << t.N << '|' << t.K << '|' << t.tile << '|' << t.flags << '|' << rows << '|' << cols << '|'
+      << (const void *)w.stream << '|' << w.buf_gen;
+    for (char **e = environ; e && *e; ++e)   // library knobs change the launch sequence
+        if (!strncmp(*e, "PDL_", 4)) k << '|' << *e;
+    return k.str();
+}
+
+int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
+    const bool want = (t.flags & PDL_TASK_GRAPH) || env_on("PDL_GRAPH");
+    if (!want || (t.flags & PDL_TASK_REUSE_B) || g->dry_run || rows <= 0 || cols <= 0)
+        return run_rect(w, t, A, B, C, rows, cols);
+    CUDA_TRY(cudaSetDevice(w.device));
+    const std::string key = graph_key(w, t, A, B, C, rows, cols);
+    auto replay = [&](WorkerCtx::GraphEntry &ge) -> int {
+        CUDA_TRY(cudaGraphLaunch(ge.exec, w.stream));
+        w.launches += ge.launches;
+        w.timed |= ge.timed;
+        for (auto &pr : ge.kt_pairs)
+            if (w.kt_list.size() < kMaxKernelTimes) w.kt_list.push_back(pr);
+        w.bsig.valid = false;
+        ++w.graph_replays;
+        return PDL_OK;
+    };
+    auto it = w.graphs.find(key);
+    if (it != w.graphs.end()) return replay(it->second);
+    int &seen = w.graph_seen[key];
+    if (seen <= 0) {   // first run (or not capturable): plain
+        const bool first = seen++ == 0;
+        const int rc = run_rect(w, t, A, B, C, rows, cols);
+        // the run may have sized the Worker's buffers: the next run has this key
+        if (first && !rc) {
+            int &s2 = w.graph_seen[graph_key(w, t, A, B, C, rows, cols)];
+            if (s2 == 0) s2 = 1;
+        }
+        return rc;
+    }
+    const size_t used0 = w.kt_used, list0 = w.kt_list.size();
+    const int launches0 = w.launches;
+    const int gen0 = w.buf_gen;
+    if (cudaStreamBeginCapture(w.stream, cudaStreamCaptureModeRelaxed) != cudaSuccess) {
+        cudaGetLastError();
+        seen = -1000000;
+        return run_rect(w, t, A, B, C, rows, cols);
+    }
+    w.capturing = true;
+    const int rc = run_rect(w, t, A, B, C, rows, cols);
+    w.capturing = false;
+    cudaGraph_t graph = nullptr;
+    cudaError_t e = cudaStreamEndCapture(w.stream, &graph);
+    cudaGraphExec_t exec = nullptr;
+    if (!rc && e == cudaSuccess && graph && w.buf_gen == gen0) e = cudaGraphInstantiate(&exec, graph, 0);
+    if (graph) cudaGraphDestroy(graph);
+    if (rc || e != cudaSuccess || !exec || w.buf_gen != gen0) {
+        // not capturable: drop what the capture recorded and run the task plainly
+        cudaGetLastError();
+        if (exec) cudaGraphExecDestroy(exec);
+        w.kt_used = used0;
+        w.kt_list.resize(list0);
+        w.launches = launches0;
+        seen = -1000000;
+        logf(1, "task not capturable into a CUDA graph (%s); running it uncaptured", rc ? g_err.c_str() : "capture");
+        return run_rect(w, t, A, B, C, rows, cols);
+    }
+    WorkerCtx::GraphEntry ge;
+    ge.exec = exec;
+    ge.launches = w.launches - launches0;
+    ge.timed = true;
+    ge.events.assign(w.kt_pool.begin() + used0, w.kt_pool.begin() + w.kt_used);   // now recorded by the graph
+    w.kt_pool.erase(w.kt_pool.begin() + used0, w.kt_pool.begin() + w.kt_used);
+    w.kt_used = used0;
+    ge.kt_pairs.assign(w.kt_list.begin() + list0, w.kt_list.end());
+    w.kt_list.resize(list0);
+    w.launches = launches0;
+    return replay(w.graphs.emplace(key, std::move(ge)).first->second);
+}
+
 int check_loaded() {
     if (!g || !g->loaded) return set_err(PDL_ESTATE, "no platform loaded (call pdl_load first)");
     return PDL_OK;
@@ -1162,7 +1285,7 @@ int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, v
     if (M < 0 || N < 0 || K < 0) return set_err(PDL_EINVAL, "negative size M=%lld N=%lld K=%lld", (long long)M,
                                                 (long long)N, (long long)K);
     if (tile < 0) return set_err(PDL_EINVAL, "negative tile %lld", (long long)tile);
-    if (flags & ~(PDL_TASK_PANELS | PDL_TASK_LOCAL | PDL_TASK_REUSE_B))
+    if (flags & ~(PDL_TASK_PANELS | PDL_TASK_LOCAL | PDL_TASK_REUSE_B | PDL_TASK_GRAPH))
         return set_err(PDL_EINVAL, "unknown flags 0x%x", flags);
     if ((flags & PDL_TASK_PANELS) && (flags & PDL_TASK_LOCAL))
         return set_err(PDL_EINVAL, "PDL_TASK_PANELS and PDL_TASK_LOCAL are exclusive");
@@ -1225,7 +1348,7 @@ int execute(bool sync) {
             pj << "{\"local\":true,\"M\":" << t.M << ",\"N\":" << t.N << ",\"K\":" << t.K << "}";
             if (g->dry_run) continue;
             if (g->workers.empty()) return set_err(PDL_ENOWORKER, "no Worker bound to this process");
-            rc = run_rect(g->workers[0], t, t.A, t.B, t.C, t.M, t.N);
+            rc = run_rect_g(g->workers[0], t, t.A, t.B, t.C, t.M, t.N);
             if (rc) return rc;
             continue;
         }
@@ -1267,7 +1390,7 @@ int execute(bool sync) {
                         const char *A = (const char *)t.A + (size_t)(rs.lo * t.lda) * es;
                         const char *B = (const char *)t.B + (size_t)cs.lo * es;
                         char *C = (char *)t.C + (size_t)(rs.lo * t.ldc + cs.lo) * es;
-                        rc = run_rect(w, t, A, B, C, rs.hi - rs.lo, cs.hi - cs.lo);
+                        rc = run_rect_g(w, t, A, B, C, rs.hi - rs.lo, cs.hi - cs.lo);
                         if (rc) return rc;
                     }
                 continue;
@@ -1290,7 +1413,7 @@ int execute(bool sync) {
             tt.lda = lda;
             tt.ldb = ldb;
             tt.ldc = ldc;
-            rc = run_rect(w, tt, A, B, C, rows, cols);
+            rc = run_rect_g(w, tt, A, B, C, rows, cols);
             if (rc) return rc;
         }
     }
@@ -1464,7 +1587,7 @@ int pdl_query(const char *key, char *out, size_t len) {
                 }
                 o << (first ? "" : ",") << "{\"id\":\"" << json_escape(m.pus[w.pu].id) << "\",\"device\":" << w.device
                   << ",\"kernel_ms\":" << ms << ",\"launches\":" << w.launches << ",\"sm_limit\":" << w.sm_limit
-                  << "}";
+                  << ",\"graphs\":" << w.graphs.size() << ",\"graph_replays\":" << w.graph_replays << "}";
                 first = false;
             }
             o << "]";
@@ -1529,12 +1652,13 @@ int pdl_kernel_times(int worker, float *ms, int n) {
     WorkerCtx &w = g->workers[worker];
     if (g->dry_run) return 0;
     CUDA_TRY(cudaSetDevice(w.device));
-    const int cnt = (int)w.kt_n;
+    const int cnt = (int)w.kt_list.size();
     for (int i = 0; i < cnt && i < n; ++i) {
-        CUDA_TRY(cudaEventSynchronize(w.kt_ev[2 * i + 1]));
-        CUDA_TRY(cudaEventElapsedTime(&ms[i], w.kt_ev[2 * i], w.kt_ev[2 * i + 1]));
+        CUDA_TRY(cudaEventSynchronize(w.kt_list[i].second));
+        CUDA_TRY(cudaEventElapsedTime(&ms[i], w.kt_list[i].first, w.kt_list[i].second));
     }
-    w.kt_n = 0;
+    w.kt_list.clear();
+    w.kt_used = 0;
     return cnt;
 }
 
