@@ -1158,6 +1158,8 @@ int run_dynamic(const Task &t, const std::vector<int> &gw) {
 // uncaptured from then on.  Not used with PDL_TASK_REUSE_B (its launches depend on
 // state left by the previous task) or DYNAMIC.
 
+constexpr size_t kMaxGraphs = 64;   // cached graphs per Worker
+
 std::string graph_key(const WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows,
                       int64_t cols) {
     std::ostringstream k;
@@ -1187,6 +1189,7 @@ int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *
     };
     auto it = w.graphs.find(key);
     if (it != w.graphs.end()) return replay(it->second);
+    if (w.graph_seen.size() >= 16 * kMaxGraphs) w.graph_seen.clear();
     int &seen = w.graph_seen[key];
     if (seen <= 0) {   // first run (or not capturable): plain
         const bool first = seen++ == 0;
@@ -1224,6 +1227,13 @@ int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *
         seen = -1000000;
         logf(1, "task not capturable into a CUDA graph (%s); running it uncaptured", rc ? g_err.c_str() : "capture");
         return run_rect(w, t, A, B, C, rows, cols);
+    }
+    if (w.graphs.size() >= kMaxGraphs) {   // bounded cache: start over
+        for (auto &kv : w.graphs) {
+            cudaGraphExecDestroy(kv.second.exec);
+            for (auto ev : kv.second.events) cudaEventDestroy(ev);
+        }
+        w.graphs.clear();
     }
     WorkerCtx::GraphEntry ge;
     ge.exec = exec;
