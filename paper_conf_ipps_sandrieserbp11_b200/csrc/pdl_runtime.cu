@@ -1231,7 +1231,8 @@ int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *
     if (w.graphs.size() >= kMaxGraphs) {   // bounded cache: start over
         for (auto &kv : w.graphs) {
             cudaGraphExecDestroy(kv.second.exec);
-            for (auto ev : kv.second.events) cudaEventDestroy(ev);
+            // the events may still be listed in kt_list: hand them back to the pool
+            w.kt_pool.insert(w.kt_pool.end(), kv.second.events.begin(), kv.second.events.end());
         }
         w.graphs.clear();
     }
