@@ -82,16 +82,31 @@ class Grid:
         self.Gr, self.Gc, self.rank = Gr, Gc, rank
         self.row_group = self.col_group = None
         self.row_ranks = [rank // Gc * Gc + c for c in range(Gc)]   # global ranks of my grid row
+        opts = _nccl_high_priority()
         for r in range(Gr):
             ranks = [r * Gc + c for c in range(Gc)]
-            g = dist.new_group(ranks) if Gc > 1 else None
+            g = dist.new_group(ranks, pg_options=opts) if Gc > 1 else None
             if rank in ranks:
                 self.row_group = g
         for c in range(Gc):
             ranks = [r * Gc + c for r in range(Gr)]
-            g = dist.new_group(ranks) if Gr > 1 else None
+            g = dist.new_group(ranks, pg_options=opts) if Gr > 1 else None
             if rank in ranks:
                 self.col_group = g
+
+
+def _nccl_high_priority():
+    """NCCL process-group options with high-priority streams, so the exchange
+    kernels get SMs ahead of queued tile-kernel CTAs when both are pending (the
+    A broadcasts must progress while the own-chunk kernel runs); None under gloo."""
+    if dist.get_backend() != "nccl":
+        return None
+    Options = getattr(dist, "ProcessGroupNCCL", None)
+    if Options is None or not hasattr(Options, "Options"):
+        return None
+    opts = Options.Options()
+    opts.is_high_priority_stream = True
+    return opts
 
 
 def chunk_from_full(A, B, wp: WorkerPlan):
