@@ -21,6 +21,11 @@ ORACLE    := oracle/liboracle.so
 
 all: $(LIB) $(ORACLE)
 
+examples: examples/dgemm_c_abi
+
+examples/dgemm_c_abi: examples/dgemm_c_abi.c include/libpdl.h $(LIB)
+	gcc -O2 -Wall -o $@ $< -L$(PKG) -lpdl -Wl,-rpath,'$$ORIGIN/../$(PKG)' -lm
+
 $(BUILD):
 	mkdir -p $(BUILD)
 
@@ -37,6 +42,6 @@ $(ORACLE): oracle/oracle.c
 	gcc -O3 -fopenmp -ffp-contract=off -fno-fast-math -shared -fPIC -o $@ $< -lm
 
 clean:
-	rm -rf $(BUILD) $(LIB) $(ORACLE)
+	rm -rf $(BUILD) $(LIB) $(ORACLE) examples/dgemm_c_abi
 
-.PHONY: all clean
+.PHONY: all clean examples
