@@ -181,3 +181,19 @@ def test_fp32_ozaki2_is_unsupported():
     with pytest.raises(pdl.PDLError) as e:
         pdl.run()
     assert e.value.code == pdl.PDL_EUNSUPPORTED
+
+
+def test_k0_and_tiny():
+    dA = torch.empty((40, 0), dtype=torch.float64, device="cuda")
+    dB = torch.empty((0, 30), dtype=torch.float64, device="cuda")
+    dC = torch.full((40, 30), float("nan"), dtype=torch.float64, device="cuda")
+    pdl.load(pdl.descriptor_xml(1, props={"DGEMM_VARIANT": "ozaki2"}))
+    pdl.task_matmul(dA, dB, dC, M=40, N=30, K=0)
+    pdl.run()
+    assert torch.count_nonzero(dC).item() == 0
+    pdl.unload()
+    A = W.signed((1, 1), np.float64, 3)
+    B = W.signed((1, 1), np.float64, 4)
+    check(oz2_matmul(A, B), A, B)           # 53-bit inputs, p-bit scaling: within the bar
+    A, B = np.array([[3.0]]), np.array([[-0.625]])
+    assert np.array_equal(oz2_matmul(A, B), A @ B)     # short mantissas: exact
