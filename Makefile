@@ -23,6 +23,13 @@ all: $(LIB) $(ORACLE)
 
 examples: examples/dgemm_c_abi
 
+# measurement tools (peaks, tensor-core behaviour, green-context splits)
+TOOLS := tools/microbench tools/tc_microbench tools/tc_probe tools/fp64_mix_probe tools/green_probe
+tools: $(TOOLS)
+
+tools/%: tools/%.cu
+	$(NVCC) $(ARCH) -O3 -lineinfo -std=c++17 -o $@ $< -lcuda
+
 examples/dgemm_c_abi: examples/dgemm_c_abi.c include/libpdl.h $(LIB)
 	gcc -O2 -Wall -o $@ $< -L$(PKG) -lpdl -Wl,-rpath,'$$ORIGIN/../$(PKG)' -lm
 
@@ -42,6 +49,6 @@ $(ORACLE): oracle/oracle.c
 	gcc -O3 -fopenmp -ffp-contract=off -fno-fast-math -shared -fPIC -o $@ $< -lm
 
 clean:
-	rm -rf $(BUILD) $(LIB) $(ORACLE) examples/dgemm_c_abi
+	rm -rf $(BUILD) $(LIB) $(ORACLE) examples/dgemm_c_abi $(TOOLS)
 
-.PHONY: all clean examples
+.PHONY: all clean examples tools
