@@ -21,6 +21,9 @@
 
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
+#include <cstring>
+#include <algorithm>
 
 #include "kernels.h"
 
@@ -32,6 +35,7 @@ static const int kModuli[OZ2_MAX_MODULI] = {256, 255, 253, 251, 247, 241, 239, 2
 
 __constant__ double c_oz2_m[OZ2_MAX_MODULI];
 __constant__ double c_oz2_inv[OZ2_MAX_MODULI];
+__constant__ int c_oz2_mi[OZ2_MAX_MODULI];
 
 // ------------------------------------------------------------------------
 // plan (host): moduli count, scaling bits, CRT constants
@@ -127,13 +131,30 @@ __device__ __forceinline__ int exp_of_max2(double mx) {   // mx < 2^e (0 -> 0)
     frexp(mx, &e);
     return e;
 }
-// v (an integer, |v| <= 2^52) mod m as a representative in [-128, 127]
+// v (an integer, |v| <= 2^52) mod m as a representative in [-128, 127].  Round-
+// to-integer by the 1.5 * 2^52 magic constant instead of rint / F2I: t = fma(v,
+// 1/m, magic) holds q = round(v/m) (one rounding of the exact product; |v/m| <
+// 2^45), q = t - magic and r = v - q m are exact (|q m| < 2^53), and r + magic
+// carries r in its low word -- four FP64-pipe operations, no conversion unit.
+// q may be one off when v/m sits within 2^-8 of a half-integer (1/m rounded);
+// the integer fix-ups fold r back into [-128, 127].
 __device__ __forceinline__ int res8(double v, int t) {
+    const double magic = 6755399441055744.0;   // 1.5 * 2^52
     const double m = c_oz2_m[t];
-    double r = fma(-rint(v * c_oz2_inv[t]), m, v);   // exact: |q m| < 2^53
-    if (r > 127.0) r -= m;
-    if (r < -128.0) r += m;
-    return (int)r;
+    const double q = fma(v, c_oz2_inv[t], magic) - magic;
+    const double r = fma(-q, m, v);
+    int ri = __double2loint(r + magic);
+    const int mi = c_oz2_mi[t];
+    ri -= ri > 127 ? mi : 0;
+    ri += ri < -128 ? mi : 0;
+    return ri;
+}
+
+// Low bytes of eight ints packed little-endian into 64 bits (PRMT, no shifts).
+__device__ __forceinline__ uint64_t pack8(const int (&r)[8]) {
+    const unsigned a = __byte_perm(__byte_perm(r[0], r[1], 0x0040), __byte_perm(r[2], r[3], 0x0040), 0x5410);
+    const unsigned b = __byte_perm(__byte_perm(r[4], r[5], 0x0040), __byte_perm(r[6], r[7], 0x0040), 0x5410);
+    return ((uint64_t)b << 32) | a;
 }
 
 // One CTA per row (grid-stride): A (rows x K) -> A8 rows [c][t][kk].
@@ -175,6 +196,50 @@ __global__ void oz2_split_rows_kernel(const double *__restrict__ A, int64_t lda,
     }
 }
 
+// Two-pass A residues (the default): a row-max pass, one warp per row with
+// coalesced loads, then an element-parallel residue pass over (row, 8-k group)
+// items -- every thread busy and 8 independent loads in flight, instead of one CTA
+// walking a row twice (oz2_split_rows_kernel, kept as PDL_OZ2_SPLIT=rows).
+__global__ void __launch_bounds__(256) oz2_rowmax_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
+                                                         int64_t K, int *__restrict__ ea) {
+    const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+    if (row >= M) return;
+    const int lane = threadIdx.x & 31;
+    const double *r = A + row * lda;
+    double mx = 0.0;
+    for (int64_t k = lane; k < K; k += 32) mx = fmax(mx, fabs(r[k]));
+    for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if (lane == 0) ea[row] = exp_of_max2(mx);
+}
+
+__global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
+                                                               int64_t K, int n, int p, int64_t Kc, int nch,
+                                                               int8_t *__restrict__ A8, int64_t ld8,
+                                                               const int *__restrict__ ea) {
+    const int64_t groups = (int64_t)nch * Kc / 8;   // Kc % 128 == 0
+    // 2-D grid-stride: rows along y, 8-k groups along x (no 64-bit divisions)
+    for (int64_t row = blockIdx.y; row < M; row += gridDim.y)
+    for (int64_t g8 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g8 < groups;
+         g8 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t k8 = g8 * 8;
+        const double *r = A + row * lda;
+        const int sh = p - ea[row];
+        double v[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? r[k8 + j] : 0.0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = rint(scale2(v[j], sh));
+        const int64_t c = nch == 1 ? 0 : k8 / Kc, kk = k8 - c * Kc;
+        int8_t *o = A8 + row * ld8 + (c * n) * Kc + kk;
+        for (int t = 0; t < n; ++t) {
+            int rr[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
+            *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+        }
+    }
+}
+
 __global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
                                   unsigned long long *__restrict__ bmax) {
     const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -209,10 +274,10 @@ __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
     const int64_t c = k8 / Kc, kk = k8 - c * Kc;
     int8_t *o = Bt8 + col * ld8 + (c * n) * Kc + kk;
     for (int t = 0; t < n; ++t) {
-        uint64_t pk = 0;
+        int rr[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) pk |= (uint64_t)(uint8_t)(int8_t)res8(v[j], t) << (8 * j);
-        *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pk;
+        for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
+        *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
     }
 }
 
@@ -315,8 +380,11 @@ static cudaError_t upload_moduli(const Ozaki2Plan &P) {
         m[t] = (double)kModuli[t];
         inv[t] = 1.0 / (double)kModuli[t];
     }
+    int mi[OZ2_MAX_MODULI];
+    for (int t = 0; t < OZ2_MAX_MODULI; ++t) mi[t] = kModuli[t];
     cudaError_t e = cudaMemcpyToSymbol(c_oz2_m, m, sizeof m);
     if (e == cudaSuccess) e = cudaMemcpyToSymbol(c_oz2_inv, inv, sizeof inv);
+    if (e == cudaSuccess) e = cudaMemcpyToSymbol(c_oz2_mi, mi, sizeof mi);
     if (e == cudaSuccess && dev < 64) {
         dev_done[dev] = 1;
         done = true;
@@ -326,12 +394,22 @@ static cudaError_t upload_moduli(const Ozaki2Plan &P) {
 }
 
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
-                                  int8_t *A8, int *ea, cudaStream_t s) {
+                                  int8_t *A8, int *ea, cudaStream_t s, int *launches) {
     if (rows <= 0) return cudaSuccess;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
-    const int blocks = (int)(rows < split_ctas() ? rows : split_ctas());
-    oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
+    const char *mode = getenv("PDL_OZ2_SPLIT");
+    if (mode && !strcmp(mode, "rows")) {
+        const int blocks = (int)(rows < split_ctas() ? rows : split_ctas());
+        oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
+        if (launches) *launches += 1;
+        return cudaGetLastError();
+    }
+    oz2_rowmax_kernel<<<(unsigned)((rows + 7) / 8), 256, 0, s>>>(A, lda, rows, K, ea);
+    const int64_t groups = (int64_t)P.nch * P.Kc / 8;
+    dim3 grid((unsigned)std::min<int64_t>((groups + 255) / 256, 64), (unsigned)std::min<int64_t>(rows, 65535));
+    oz2_residue_rows_kernel<<<grid, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
+    if (launches) *launches += 2;
     return cudaGetLastError();
 }
 

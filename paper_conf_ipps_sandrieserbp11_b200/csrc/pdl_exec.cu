@@ -322,8 +322,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (!a_prep[i]) {
                     a_prep[i] = 1;
                     e = pdlk::launch_ozaki2_split_a((const double *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K, P2,
-                                                    a8 + r0 * P2.ld8, oz_ea + r0, cs);
-                    w.launches += 1;
+                                                    a8 + r0 * P2.ld8, oz_ea + r0, cs, &w.launches);
                     if (piped) {
                         ev_sa[i] = ev_get(w, evn);
                         CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
