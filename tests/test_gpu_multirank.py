@@ -49,3 +49,7 @@ def test_distributed_ragged_8():
 
 def test_distributed_ozaki_4():
     _run(4, "f64", 777, 513, 1000, 128, "ozaki")
+
+
+def test_distributed_ozaki2_4():
+    _run(4, "f64", 777, 513, 1000, 128, "ozaki2")
