@@ -96,16 +96,21 @@ def tensor_peak(dtype):
     the conservative denominator.
     """
     pk, src = peaks()
+    sus = pk.get("bf16_tflops_sustained")
     if dtype == "i8":
+        alt = {"peak": round(pk["bf16_tflops"] * 2, 1), "source": f"{src} bf16 burst x nominal 4.5/2.25"}
+        if sus:
+            alt["peak_sustained"] = round(sus * 2, 1)
         return INT8_TCGEN05_PEAK_TOPS, ("INT8 tcgen05 issue rate measured (tools/tc_microbench; "
-                                        "profiles/r01_tc_microbench.json)"), \
-            {"peak": round(pk["bf16_tflops"] * 2, 1), "source": f"{src} bf16 burst x nominal 4.5/2.25"}
+                                        "profiles/r01_tc_microbench.json)"), alt
     if dtype == "f64":
         return FP64_DMMA_PEAK_TFLOPS, "FP64 DMMA.8x8x4 issue rate measured (tools/microbench; profiles/r01_microbench.json)", None
-    alt = pk["bf16_tflops"] * 1.1 / 2.25
+    alt = {"peak": round(pk["bf16_tflops"] * 1.1 / 2.25, 1),
+           "source": f"{src} bf16 burst {pk['bf16_tflops']} x nominal 1.1/2.25"}
+    if sus:
+        alt["peak_sustained"] = round(sus * 1.1 / 2.25, 1)
     return TF32_TCGEN05_PEAK_TFLOPS, ("TF32 tcgen05 issue rate measured (tools/tc_microbench; "
-                                      "profiles/r01_tc_microbench.json)"), \
-        {"peak": round(alt, 1), "source": f"{src} bf16 burst {pk['bf16_tflops']} x nominal 1.1/2.25"}
+                                      "profiles/r01_tc_microbench.json)"), alt
 
 
 class ClockSampler:
