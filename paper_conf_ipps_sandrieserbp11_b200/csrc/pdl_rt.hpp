@@ -19,6 +19,7 @@
 #include <string>
 #include <vector>
 
+#include <dlfcn.h>
 #include <unistd.h>
 
 #include "../../include/libpdl.h"

@@ -150,6 +150,66 @@ int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, v
 
 using namespace pdlrt;
 
+namespace pdlrt {
+
+// NVLink topology through NVML (dlopen'ed: the library must load where NVML is
+// absent), for pdl_describe's Worker properties and NVLink ICDescriptors
+// ("NVML NVLink topology").  links = active NVLink links of the
+// device, version = NVLink generation, via_switch = a link ends at an NVSwitch.
+struct NvLinkInfo {
+    int links = -1, version = 0;
+    bool via_switch = false;
+};
+
+std::vector<NvLinkInfo> nvlink_topology(int ndev) {
+    std::vector<NvLinkInfo> info(ndev);
+    void *h = dlopen("libnvidia-ml.so.1", RTLD_NOW | RTLD_LOCAL);
+    if (!h) return info;
+    typedef int (*init_t)();
+    typedef int (*byid_t)(const char *, void **);
+    typedef int (*state_t)(void *, unsigned, int *);
+    typedef int (*ver_t)(void *, unsigned, unsigned *);
+    typedef int (*rtype_t)(void *, unsigned, int *);
+    auto init = (init_t)dlsym(h, "nvmlInit_v2");
+    auto shutdown = (init_t)dlsym(h, "nvmlShutdown");
+    auto byid = (byid_t)dlsym(h, "nvmlDeviceGetHandleByPciBusId_v2");
+    auto state = (state_t)dlsym(h, "nvmlDeviceGetNvLinkState");
+    auto ver = (ver_t)dlsym(h, "nvmlDeviceGetNvLinkVersion");
+    auto rtype = (rtype_t)dlsym(h, "nvmlDeviceGetNvLinkRemoteDeviceType");
+    if (init && byid && state && init() == 0) {
+        for (int d = 0; d < ndev; ++d) {
+            char bus[32];
+            void *dev = nullptr;
+            if (cudaDeviceGetPCIBusId(bus, sizeof bus, d) != cudaSuccess || byid(bus, &dev) != 0) {
+                cudaGetLastError();
+                continue;
+            }
+            info[d].links = 0;
+            for (unsigned l = 0; l < 18; ++l) {   // NVML_NVLINK_MAX_LINKS
+                int active = 0;
+                if (state(dev, l, &active) != 0 || active != 1) continue;   // NVML_FEATURE_ENABLED
+                ++info[d].links;
+                unsigned v = 0;
+                if (ver && ver(dev, l, &v) == 0 && (int)v > info[d].version) info[d].version = (int)v;
+                int t = 0;
+                if (rtype && rtype(dev, l, &t) == 0 && t == 2) info[d].via_switch = true;   // ..._TYPE_SWITCH
+            }
+        }
+        if (shutdown) shutdown();
+    }
+    dlclose(h);
+    return info;
+}
+
+// NVML NVLink version enum -> generation ("5.0" on B200) and per-link GB/s per direction
+std::string nvlink_gen(int v) {
+    static const char *g[] = {"", "1.0", "2.0", "2.2", "3.0", "3.1", "4.0", "5.0"};
+    return v > 0 && v < 8 ? g[v] : std::to_string(v);
+}
+int nvlink_gbs(int v) { return v == 7 ? 50 : (v == 6 || v == 4 || v == 5) ? 25 : 0; }
+
+}  // namespace pdlrt
+
 // the C ABI is the only exported surface (built with -fvisibility=hidden)
 #pragma GCC visibility push(default)
 extern "C" {
@@ -411,6 +471,7 @@ int pdl_describe(char *out, size_t len) {
         }
         o << ">" << x << "</value></Property>\n";
     };
+    const std::vector<NvLinkInfo> nvl = nvlink_topology(ndev);
     std::ostringstream o;
     o << "<?xml version=\"1.0\"?>\n<!-- generated by pdl_describe (" << kVersion << ") -->\n";
     o << "<Master id=\"0\" quantity=\"1\">\n  <PUDescriptor>\n";
@@ -437,6 +498,10 @@ int pdl_describe(char *out, size_t len) {
         cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, d);
         prop(o, "CLOCK_RATE", std::to_string(clk), "kHz", false);
         prop(o, "PCI_BUS_ID", std::to_string(p.pciBusID), "", false);
+        if (nvl[d].links >= 0) {
+            prop(o, "NVLINK_LINKS", std::to_string(nvl[d].links), "", false);
+            if (nvl[d].version) prop(o, "NVLINK_VERSION", nvlink_gen(nvl[d].version), "", false);
+        }
         o << "    </PUDescriptor>\n    <MemoryRegion id=\"hbm\"><MRDescriptor>\n";
         prop(o, "SIZE", std::to_string((unsigned long long)p.totalGlobalMem), "B", false);
         o << "    </MRDescriptor></MemoryRegion>\n    <LogicGroupAttribute>gpus</LogicGroupAttribute>\n  </Worker>\n";
@@ -449,7 +514,21 @@ int pdl_describe(char *out, size_t len) {
                 cudaGetLastError();
                 can = 0;
             }
-            if (can) o << "  <Interconnect type=\"NVLink\" from=\"gpu" << a << "\" to=\"gpu" << b << "\" scheme=\"p2p\"/>\n";
+            if (!can) continue;
+            const bool sw = nvl[a].via_switch && nvl[b].via_switch;
+            o << "  <Interconnect type=\"NVLink\" from=\"gpu" << a << "\" to=\"gpu" << b << "\" scheme=\""
+              << (sw ? "switch" : "p2p") << "\"";
+            const int links = std::min(nvl[a].links, nvl[b].links);
+            if (links > 0) {
+                // NVLink 5 (B200): 50 GB/s per direction per link
+                o << ">\n    <ICDescriptor>\n";
+                prop(o, "LINKS", std::to_string(links), "", false);
+                const int per_link = nvlink_gbs(std::min(nvl[a].version, nvl[b].version));
+                if (per_link) prop(o, "BANDWIDTH", std::to_string(per_link * links), "GB/s", false);
+                o << "    </ICDescriptor>\n  </Interconnect>\n";
+            } else {
+                o << "/>\n";
+            }
         }
     o << "</Master>\n";
     const std::string res = o.str();
