@@ -362,7 +362,7 @@ def main():
             pdl.task_matmul(dA, dB, dC, tile=c.tile)
             pdl.run_async()
     else:
-        grid = runtime.Grid(wp.Gr, wp.Gc, rank)
+        grid = runtime.Grid(wp.Gr, wp.Gc, rank, via_host=runtime.exchange_path() == "host")
         Ach, Bch = runtime.chunk_from_full(torch.from_numpy(A), torch.from_numpy(B), wp)
         Ach, Bch = Ach.to(dev), Bch.to(dev)
         bufs = runtime.PanelBuffers(wp, tdt, dev)

@@ -217,7 +217,10 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group,
  *   each Worker claimed in the last DYNAMIC task -- read after pdl_sync),
  *   "worker/<i>/<PROPERTY>",
  *   "worker/<i>/device", "worker/<i>/id", "pu/<id>/<PROPERTY>",
- *   "interconnects" (JSON).
+ *   "interconnects" (JSON), "exchange_path[/<group>]" ("direct" when every
+ *   pair of the group's gpu Workers is joined by an Interconnect, else "host":
+ *   the transfer path the multi-rank exchange takes, L1336-1341),
+ *   "ozaki2_plan/<K>[/<bits>[/<moduli>]]" (JSON; no pdl_load needed).
  * Writes a NUL-terminated string (truncated to len-1) and returns the full
  * length, or a negative code (PDL_EINVAL for an unknown key).
  */

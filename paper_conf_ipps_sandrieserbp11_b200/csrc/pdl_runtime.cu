@@ -341,6 +341,19 @@ int pdl_query(const char *key, char *out, size_t len) {
         else if (k == "local_workers") res = std::to_string(g->workers.size());
         else if (k == "model") res = m.to_json();
         else if (k == "interconnects") res = m.ics_json();
+        else if (k == "exchange_path" || k.rfind("exchange_path/", 0) == 0) {
+            // the Worker<->Worker transfer path the descriptor allows for a group
+            // (L1336-1341: paths are derived from the explicit interconnects):
+            // "direct" when every pair of its gpu Workers is joined by an
+            // Interconnect (NVLink on a B200 box), else "host" (through the
+            // Master's memory region, over the Master<->Worker interconnects)
+            const std::string grp = k.size() > 14 ? k.substr(14) : std::string();
+            std::vector<int> gw = m.group_workers(grp.empty() ? nullptr : grp.c_str());
+            bool direct = true;
+            for (size_t i = 0; i < gw.size() && direct; ++i)
+                for (size_t j = i + 1; j < gw.size() && direct; ++j) direct = m.ic_between(gw[i], gw[j], "");
+            res = direct ? "direct" : "host";
+        }
         else if (k == "plan") res = g->plan_json;
         else if (k == "groups") {
             std::vector<std::string> gs;

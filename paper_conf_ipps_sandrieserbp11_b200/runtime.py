@@ -13,7 +13,9 @@ rectangle, which operand chunk each Worker holds) comes from libpdl's
   chunks inside each grid column over torch.distributed (NCCL over NVLink 5 /
   NVSwitch on the GPU box, gloo in the CPU tests).  This is the "derive
   data-transfer paths ... via the explicitly specified interconnect entity"
-  step (L1336-1341) for the Worker<->Worker NVLink interconnect;
+  step (L1336-1341) for the Worker<->Worker NVLink interconnect; a descriptor
+  that joins the Workers by no interconnect sends the exchange through the
+  Master's memory region instead (host-staged gloo groups, ``exchange_path``);
 * local task -- ``task_matmul_ex(..., PDL_TASK_PANELS)`` + ``pdl_run`` on the
   gathered panels (libpdl, sm_100a kernels).
 
@@ -74,23 +76,35 @@ def worker_plan(M, N, K, tile, rank, group=None) -> WorkerPlan:
                       p["col1"], p["qa"], p["qb"], M, N, K)
 
 
+def exchange_path(group=None) -> str:
+    """The Worker<->Worker path the loaded descriptor allows (libpdl query
+    "exchange_path"): "direct" when every pair of the group's Workers is joined
+    by an Interconnect (NVLink on a B200 box), else "host" -- the exchange then
+    stages through the Master's memory region ("derive data-transfer paths ...
+    via the explicitly specified interconnect entity")."""
+    return pdl.query("exchange_path" + (f"/{group}" if group else ""))
+
+
 class Grid:
     """Row / column process groups of the Gr x Gc Worker grid (created
-    collectively: every rank creates every group in the same order)."""
+    collectively: every rank creates every group in the same order).
+    via_host: exchange through host memory (gloo groups) because the
+    descriptor has no Worker<->Worker interconnect."""
 
-    def __init__(self, Gr, Gc, rank):
+    def __init__(self, Gr, Gc, rank, via_host=False):
         self.Gr, self.Gc, self.rank = Gr, Gc, rank
+        self.via_host = via_host
         self.row_group = self.col_group = None
         self.row_ranks = [rank // Gc * Gc + c for c in range(Gc)]   # global ranks of my grid row
-        opts = _nccl_high_priority()
+        kw = {"backend": "gloo"} if via_host else {"pg_options": _nccl_high_priority()}
         for r in range(Gr):
             ranks = [r * Gc + c for c in range(Gc)]
-            g = dist.new_group(ranks, pg_options=opts) if Gc > 1 else None
+            g = dist.new_group(ranks, **kw) if Gc > 1 else None
             if rank in ranks:
                 self.row_group = g
         for c in range(Gc):
             ranks = [r * Gc + c for r in range(Gr)]
-            g = dist.new_group(ranks, pg_options=opts) if Gr > 1 else None
+            g = dist.new_group(ranks, **kw) if Gr > 1 else None
             if rank in ranks:
                 self.col_group = g
 
@@ -245,13 +259,14 @@ def distributed_matmul(A_full, B_full, C_full, tile=0, group=None, overlap=True)
     """Public multi-Worker API: every rank passes the full (host or device)
     A, B and its own C; rank r writes its rectangle of C.  Host operands are
     copied chunk-wise to the Worker (PCIe), exchanged over NVLink (overlapped
-    with the tile kernels unless overlap=False), computed, and the C block
-    copied back (PCIe)."""
+    with the tile kernels unless overlap=False) -- or through host memory when
+    the descriptor joins the Workers by no interconnect -- computed, and the C
+    block copied back (PCIe)."""
     rank = dist.get_rank()
     M, K = A_full.shape
     N = B_full.shape[1]
     wp = worker_plan(M, N, K, tile, rank, group)
-    grid = Grid(wp.Gr, wp.Gc, rank)
+    grid = Grid(wp.Gr, wp.Gc, rank, via_host=exchange_path(group) == "host")
     dev = torch.device("cuda", torch.cuda.current_device())
     Ach, Bch = chunk_from_full(A_full, B_full, wp)
     Ach, Bch = Ach.to(dev, non_blocking=True), Bch.to(dev, non_blocking=True)
