@@ -561,6 +561,15 @@ int run_dynamic(const Task &t, const std::vector<int> &gw) {
         const int64_t Kp = round_up(K, pdlk::K2_BK);
         for (size_t i = 0; i < ws.size(); ++i) {
             WorkerCtx &w = *ws[i];
+            // the shared counter lives in the first Worker's memory region: a Worker on
+            // another device reaches it only over a Worker<->Worker interconnect of the
+            // descriptor (L1336-1341)
+            if (w.device != own.device && !g->model.ic_between(w.pu, own.pu, ""))
+                return set_err(PDL_EUNSUPPORTED,
+                               "DYNAMIC: the descriptor joins Workers %s and %s by no interconnect "
+                               "(the tile counter sits in %s's memory region)",
+                               g->model.pus[w.pu].id.c_str(), g->model.pus[own.pu].id.c_str(),
+                               g->model.pus[own.pu].id.c_str());
             if ((rc = enable_peer(w.device, g->dyn_dev)) || (rc = enable_peer(w.device, c_home))) return rc;
             CUDA_TRY(cudaSetDevice(w.device));
             if (&w != &own) CUDA_TRY(cudaStreamWaitEvent(w.stream, ev_reset, 0));
