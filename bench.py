@@ -154,7 +154,11 @@ class ClockSampler:
             if len(parts) < 9:
                 continue
             try:
-                rows.append((float(parts[1]), float(parts[2]), parts[5:9]))
+                try:
+                    pw = float(parts[3])
+                except ValueError:
+                    pw = float("nan")
+                rows.append((float(parts[1]), float(parts[2]), parts[5:9], pw))
             except ValueError:
                 continue
         os.unlink(self.path)
@@ -164,8 +168,12 @@ class ClockSampler:
         loaded = [r for r in rows if r[0] > 0.5 * maxmhz] or rows
         names = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
         reasons = sorted({names[i] for r in rows for i in range(4) if r[2][i].lower() == "active"})
-        return {"sm_mhz": float(np.median([r[0] for r in loaded])), "sm_max_mhz": maxmhz,
-                "reasons": reasons, "samples": len(rows)}
+        out = {"sm_mhz": float(np.median([r[0] for r in loaded])), "sm_max_mhz": maxmhz,
+               "reasons": reasons, "samples": len(rows)}
+        pw = [r[3] for r in loaded if r[3] == r[3]]
+        if pw:   # board power under load: the INT8 / TF32 paths sit at the 1000 W cap
+            out["power_w"] = round(float(np.median(pw)), 1)
+        return out
 
 
 def ncu_traffic(dtype, cfg):
