@@ -242,6 +242,15 @@ def variant_label(variant, dtype, S, K):
     return f"{dtype}-ozaki-i8x{S}", f"ozaki (K4/K5, {S} int8 slices)"
 
 
+def edge_waste(rows, cols, dtype, ozaki):
+    """Percent of the MMA work spent on padding of partial edge tiles (SURVEY
+    8(d)): K1 computes 128 x 128 CTA tiles, K2 / K4 / K6 256 x 256 (or 256 x 512)
+    CTA-pair tiles."""
+    e_m, e_n = (128, 128) if dtype == "f64" and not ozaki else (256, 256)
+    padded = -(-rows // e_m) * e_m * (-(-cols // e_n) * e_n)
+    return round(100.0 * (padded / max(1, rows * cols) - 1.0), 3)
+
+
 def host_inputs(cfg, np_dtype):
     return W.config_inputs(cfg, np_dtype)
 
@@ -434,6 +443,8 @@ def main():
                 "kernel": kname,
                 "kernel_ms": round(kavg, 3) if kavg else None,
                 "algorithmic_flops_per_launch": pipe_flops,
+                "algorithmic_dram_bytes_per_launch": int((wp.rows * K + K * wp.cols + wp.rows * wp.cols) * es),
+                "edge_waste_pct": edge_waste(wp.rows, wp.cols, args.dtype, ozaki),
                 "peak_source": peak_src}
     if peak_alt:
         roofline["peak_alt"] = peak_alt
