@@ -32,6 +32,8 @@
 
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
+#include <cstring>
 
 #include "kernels.h"
 #include "ptx.cuh"
@@ -171,8 +173,7 @@ constexpr int BM = 128, BN1 = 256, BNH = 128;
 constexpr int BK = 128, UMMA_K = 32;
 constexpr int A_BYTES = BM * BK;        // 16 KiB
 constexpr int B_BYTES = BNH * BK;       // 16 KiB per N=256 sub-tile
-constexpr int EPI_WARPS = 16, FIRST_EPI_WARP = 2;
-constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
+constexpr int FIRST_EPI_WARP = 2;
 // Raster group (cluster-tile rows sweeping the columns together) from the K extent
 // of the launch: the group's A strips (256 rows x K' bytes each) should stay in L2
 // while the columns go by, so long diagonals take small groups.  Sweeps at C4
@@ -185,11 +186,18 @@ inline int group_for_k(int64_t kd) {
     while (g > 4 && (int64_t)g * strip > ((int64_t)96 << 20)) g >>= 1;
     return raster_group_m(g);
 }
-template <int NSUB> struct Cfg {
+// OCC = CTAs per SM.  OCC = 1: one CTA (pair) owns the SM pair, 16 epilogue
+// warps, a 6-stage ring (4 for NSUB = 2).  OCC = 2 (NSUB = 1 only): two CTA pairs
+// share each SM pair, each with 256 TMEM columns, a 3-stage ring and 8 epilogue
+// warps, so one pair's epilogue (and prologue) overlaps the other's mainloop.
+template <int NSUB, int OCC = 1> struct Cfg {
+    static_assert(OCC == 1 || NSUB == 1, "two CTAs per SM need the 256-column tile");
     static constexpr int BN = BN1 * NSUB;
     static constexpr int STAGE_BYTES = A_BYTES + NSUB * B_BYTES;
-    static constexpr int STAGES = (6 * (A_BYTES + B_BYTES)) / STAGE_BYTES;   // 6 or 4
-    static constexpr int EPI_COLS = 64 * NSUB;
+    static constexpr int STAGES = OCC == 2 ? 3 : (6 * (A_BYTES + B_BYTES)) / STAGE_BYTES;   // 6, 4 or 3
+    static constexpr int EPI_WARPS = OCC == 2 ? 8 : 16;
+    static constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
+    static constexpr int EPI_COLS = 256 * NSUB / (EPI_WARPS / 4);
     static constexpr int TMEM_COLS = 256 * NSUB;
     static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
 };
@@ -221,15 +229,16 @@ __device__ __forceinline__ void umma_i8_2sm(uint32_t tmem_d, uint64_t adesc, uin
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
 }
 
-template <int NSUB, typename TC>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::THREADS, 1)
+template <int NSUB, typename TC, int OCC = 1>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, OCC>::THREADS, OCC)
     oz_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
                        TC *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
                        const int *__restrict__ fb, int scale_exp, int accumulate, int tiles_m, int tiles_n,
                        int group_m, int vec_ok, int modulus, float inv_mod) {
     using namespace koz;
-    constexpr int BN = Cfg<NSUB>::BN, STAGES = Cfg<NSUB>::STAGES, STAGE_BYTES = Cfg<NSUB>::STAGE_BYTES;
-    constexpr int EPI_COLS = Cfg<NSUB>::EPI_COLS, TMEM_COLS = Cfg<NSUB>::TMEM_COLS;
+    using CF = Cfg<NSUB, OCC>;
+    constexpr int BN = CF::BN, STAGES = CF::STAGES, STAGE_BYTES = CF::STAGE_BYTES;
+    constexpr int EPI_COLS = CF::EPI_COLS, TMEM_COLS = CF::TMEM_COLS;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
     const uint32_t bar_full = base + STAGES * STAGE_BYTES;
@@ -506,6 +515,71 @@ static bool map_i8(EncodeTiledFn enc, CUtensorMap *m, const int8_t *ptr, uint64_
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Kernel shape for one rectangle: 0 = 256 x 512 cluster tiles (NSUB 2), 1 = 256 x
+// 256 (NSUB 1), 2 = 256 x 256 with two CTA pairs per SM pair (OCC 2).  Exact INT32
+// sums: the shape does not change a bit of C.  Default: 256 x 512 when it still
+// gives >= 2 waves of CTA pairs (148 clusters), else 256 x 256 for parallelism.
+// PDL_OZ_SHAPE = 512 | 256 | 256x2 overrides (PDL_OZ_NSUB = 1 | 2 is the older knob).
+static int oz_shape(int64_t rows, int64_t cols) {
+    using namespace koz;
+    const int64_t clusters512 = ((rows + 2 * BM - 1) / (2 * BM)) * ((cols + 511) / 512);
+    int shape = (cols > 256 && clusters512 >= 148) ? 0 : 1;
+    if (const char *e = getenv("PDL_OZ_NSUB")) shape = atoi(e) == 1 ? 1 : 0;
+    if (const char *e = getenv("PDL_OZ_SHAPE")) {
+        if (!strcmp(e, "512")) shape = 0;
+        else if (!strcmp(e, "256")) shape = 1;
+        else if (!strcmp(e, "256x2")) shape = 2;
+    }
+    return shape;
+}
+
+template <typename TC>
+static cudaError_t oz_set_attrs() {
+    using namespace koz;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static bool attr_done[64] = {false};
+    if (dev < 64 && attr_done[dev]) return cudaSuccess;
+    cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1, TC, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         Cfg<1, 1>::SMEM_BYTES);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<2, TC, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 Cfg<2, 1>::SMEM_BYTES);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1, TC, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 Cfg<1, 2>::SMEM_BYTES);
+    if (e != cudaSuccess) return e;
+    if (dev < 64) attr_done[dev] = true;
+    return cudaSuccess;
+}
+
+template <int NSUB, int OCC, typename TC>
+static void oz_launch_one(const CUtensorMap &ta, const CUtensorMap &tb, TC *C, int64_t ldc, int64_t rows,
+                          int64_t cols, int64_t kd, const int *ea, const int *fb, int scale_exp, int accumulate,
+                          int vec_ok, int modulus, float inv_mod, cudaStream_t stream) {
+    using namespace koz;
+    using CF = Cfg<NSUB, OCC>;
+    const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + CF::BN - 1) / CF::BN);
+    oz_gemm_2sm_kernel<NSUB, TC, OCC><<<2 * tiles_m * tiles_n, CF::THREADS, CF::SMEM_BYTES, stream>>>(
+        ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, scale_exp, accumulate, tiles_m, tiles_n,
+        group_for_k(kd), vec_ok, modulus, inv_mod);
+}
+
+template <typename TC>
+static void oz_launch(int shape, const CUtensorMap &ta, const CUtensorMap &tb, TC *C, int64_t ldc, int64_t rows,
+                      int64_t cols, int64_t kd, const int *ea, const int *fb, int scale_exp, int accumulate,
+                      int vec_ok, int modulus, float inv_mod, cudaStream_t stream) {
+    if (shape == 0)
+        oz_launch_one<2, 1>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, inv_mod,
+                            stream);
+    else if (shape == 1)
+        oz_launch_one<1, 1>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, inv_mod,
+                            stream);
+    else
+        oz_launch_one<1, 2>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, inv_mod,
+                            stream);
+}
+
 // All diagonals and K chunks of one rectangle: S * nch int8 GEMM launches,
 // smallest diagonal first; the first launch overwrites C.
 template <typename TC>
@@ -514,27 +588,9 @@ static cudaError_t gemm_impl(EncodeTiledFn enc, const int8_t *A8, const int8_t *
                              int *launches) {
     using namespace koz;
     if (rows <= 0 || cols <= 0) return cudaSuccess;
-    int dev = 0;
-    cudaGetDevice(&dev);
-    static bool attr_done[64] = {false};
-    if (dev < 64 && !attr_done[dev]) {
-        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1, TC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             Cfg<1>::SMEM_BYTES);
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<2, TC>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     Cfg<2>::SMEM_BYTES);
-        if (e != cudaSuccess) return e;
-        attr_done[dev] = true;
-    }
-    // 256 x 512 cluster tiles unless the rectangle is narrow (PDL_OZ_NSUB=1|2 overrides).
-    // Exact INT32 sums: the tile shape does not change a bit of C.
-    // 256 x 512 only when it still gives >= 2 waves of CTA pairs (148 clusters);
-    // small rectangles keep 256 x 256 for parallelism
-    const int64_t clusters512 = ((rows + 2 * BM - 1) / (2 * BM)) * ((cols + 511) / 512);
-    int nsub = (cols > 256 && clusters512 >= 148) ? 2 : 1;
-    if (const char *e = getenv("PDL_OZ_NSUB")) nsub = atoi(e) == 1 ? 1 : 2;
-    const int BN = nsub == 2 ? Cfg<2>::BN : Cfg<1>::BN;
-    const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + BN - 1) / BN);
+    cudaError_t e0 = oz_set_attrs<TC>();
+    if (e0 != cudaSuccess) return e0;
+    const int shape = oz_shape(rows, cols);
     const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && ((ldc * sizeof(TC)) & 15) == 0) ? 1 : 0;
     int first = 1;
     for (int c = 0; c < L.nch; ++c) {
@@ -546,14 +602,8 @@ static cudaError_t gemm_impl(EncodeTiledFn enc, const int8_t *A8, const int8_t *
             if (!map_i8(enc, &ta, a, (uint64_t)kd, (uint64_t)rows, (uint64_t)L.ld8, BM) ||
                 !map_i8(enc, &tb, b, (uint64_t)kd, (uint64_t)cols, (uint64_t)L.ld8, BNH))
                 return cudaErrorInvalidValue;
-            if (nsub == 2)
-                oz_gemm_2sm_kernel<2, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
-                    ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
-                    tiles_n, group_for_k(kd), vec_ok, 0, 0.f);
-            else
-                oz_gemm_2sm_kernel<1, TC><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
-                    ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, -7 * (d + 2), first ? 0 : 1, tiles_m,
-                    tiles_n, group_for_k(kd), vec_ok, 0, 0.f);
+            oz_launch<TC>(shape, ta, tb, C, ldc, rows, cols, kd, ea, fb, -7 * (d + 2), first ? 0 : 1, vec_ok, 0, 0.f,
+                          stream);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             first = 0;
@@ -582,23 +632,9 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
     using namespace koz;
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 15u) || (ldr & 15) || (plane & 15)) return cudaErrorInvalidValue;
-    int dev = 0;
-    cudaGetDevice(&dev);
-    static bool attr_done[64] = {false};
-    if (dev < 64 && !attr_done[dev]) {
-        cudaError_t e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<1, uint8_t>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<1>::SMEM_BYTES);
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(oz_gemm_2sm_kernel<2, uint8_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     Cfg<2>::SMEM_BYTES);
-        if (e != cudaSuccess) return e;
-        attr_done[dev] = true;
-    }
-    const int64_t clusters512 = ((rows + 2 * BM - 1) / (2 * BM)) * ((cols + 511) / 512);
-    int nsub = (cols > 256 && clusters512 >= 148) ? 2 : 1;
-    if (const char *e = getenv("PDL_OZ_NSUB")) nsub = atoi(e) == 1 ? 1 : 2;
-    const int BN = nsub == 2 ? Cfg<2>::BN : Cfg<1>::BN;
-    const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + BN - 1) / BN);
+    cudaError_t e0 = oz_set_attrs<uint8_t>();
+    if (e0 != cudaSuccess) return e0;
+    const int shape = oz_shape(rows, cols);
     for (int c = 0; c < P.nch; ++c) {
         for (int t = 0; t < P.n; ++t) {
             const int64_t off = ((int64_t)c * P.n + t) * P.Kc;
@@ -607,15 +643,8 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
                 !map_i8(enc, &tb, Bt8 + off, (uint64_t)P.Kc, (uint64_t)cols, (uint64_t)P.ld8, BNH))
                 return cudaErrorInvalidValue;
             uint8_t *Rp = R + ((int64_t)c * P.n + t) * plane;
-            const float inv = 1.0f / (float)P.m[t];
-            if (nsub == 2)
-                oz_gemm_2sm_kernel<2, uint8_t><<<2 * tiles_m * tiles_n, THREADS, Cfg<2>::SMEM_BYTES, stream>>>(
-                    ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, nullptr, nullptr, 0, 0, tiles_m, tiles_n,
-                    group_for_k(P.Kc), 1, P.m[t], inv);
-            else
-                oz_gemm_2sm_kernel<1, uint8_t><<<2 * tiles_m * tiles_n, THREADS, Cfg<1>::SMEM_BYTES, stream>>>(
-                    ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, nullptr, nullptr, 0, 0, tiles_m, tiles_n,
-                    group_for_k(P.Kc), 1, P.m[t], inv);
+            oz_launch<uint8_t>(shape, ta, tb, Rp, ldr, rows, cols, P.Kc, nullptr, nullptr, 0, 0, 1, P.m[t],
+                               1.0f / (float)P.m[t], stream);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             if (launches) ++*launches;

@@ -150,6 +150,26 @@ __device__ __forceinline__ int res8(double v, int t) {
     return ri;
 }
 
+// Fast residue for p <= 50 (|v| < 2^51), one DFMA and one IMAD per modulus.
+// vm = v + 1.5 * 2^52 (exact), its low word = the low 32 bits of the integer v.
+// q = round(v / m) is EXACT here: for odd m, v / m = n + k / m lies at least
+// 1 / (2m) from a half-integer while v * rn(1/m) is within |v| / m * 2^-53 < 1 / (2m)
+// of v / m; for m = 256 the reciprocal is exact.  fma(v, 1/m, magic) = q + magic
+// carries q's low 32 bits in its low word, and r = v - q m (|r| <= m / 2 <= 128)
+// follows exactly from the low words in wrapping 32-bit arithmetic.  r = +-128
+// occurs only for m = 256, whose byte 0x80 is congruent to both.
+__device__ __forceinline__ int res8_fast(double v, int vlo, int t) {
+    const double qm = fma(v, c_oz2_inv[t], 6755399441055744.0);
+    return vlo - __double2loint(qm) * c_oz2_mi[t];
+}
+// rint(x 2^sh) + 1.5 * 2^52 in one DFMA (round-to-nearest-even on the integer grid
+// of [2^52, 2^53) is rint); off the normal exponent range through scale2.
+__device__ __forceinline__ double scaled_magic(double x, int sh) {
+    const double magic = 6755399441055744.0;
+    if (sh >= -1022 && sh <= 1023) return fma(x, pow2d(sh), magic);
+    return rint(scale2(x, sh)) + magic;
+}
+
 // Low bytes of eight ints packed little-endian into 64 bits (PRMT, no shifts).
 __device__ __forceinline__ uint64_t pack8(const int (&r)[8]) {
     const unsigned a = __byte_perm(__byte_perm(r[0], r[1], 0x0040), __byte_perm(r[2], r[3], 0x0040), 0x5410);
@@ -215,8 +235,9 @@ __global__ void __launch_bounds__(256) oz2_rowmax_kernel(const double *__restric
 __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
                                                                int64_t K, int n, int p, int64_t Kc, int nch,
                                                                int8_t *__restrict__ A8, int64_t ld8,
-                                                               const int *__restrict__ ea) {
+                                                               const int *__restrict__ ea, int vec) {
     const int64_t groups = (int64_t)nch * Kc / 8;   // Kc % 128 == 0
+    const bool fast = p <= 50;                      // |A'| < 2^51: res8_fast (uniform)
     // 2-D grid-stride: rows along y, 8-k groups along x (no 64-bit divisions)
     for (int64_t row = blockIdx.y; row < M; row += gridDim.y)
     for (int64_t g8 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g8 < groups;
@@ -225,17 +246,42 @@ __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__r
         const double *r = A + row * lda;
         const int sh = p - ea[row];
         double v[8];
+        if (vec && k8 + 8 <= K) {   // 16-byte aligned row and a full group: 4 x LDG.128
 #pragma unroll
-        for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? r[k8 + j] : 0.0;
+            for (int j = 0; j < 4; ++j) {
+                const double2 x = __ldcs(reinterpret_cast<const double2 *>(r + k8) + j);
+                v[2 * j] = x.x;
+                v[2 * j + 1] = x.y;
+            }
+        } else {
 #pragma unroll
-        for (int j = 0; j < 8; ++j) v[j] = rint(scale2(v[j], sh));
+            for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? r[k8 + j] : 0.0;
+        }
         const int64_t c = nch == 1 ? 0 : k8 / Kc, kk = k8 - c * Kc;
         int8_t *o = A8 + row * ld8 + (c * n) * Kc + kk;
-        for (int t = 0; t < n; ++t) {
-            int rr[8];
+        if (fast) {
+            int lo[8];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
-            *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+            for (int j = 0; j < 8; ++j) {
+                const double vm = scaled_magic(v[j], sh);
+                lo[j] = __double2loint(vm);
+                v[j] = vm - 6755399441055744.0;
+            }
+            for (int t = 0; t < n; ++t) {
+                int rr[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) rr[j] = res8_fast(v[j], lo[j], t);
+                *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[j] = rint(scale2(v[j], sh));
+            for (int t = 0; t < n; ++t) {
+                int rr[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
+                *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+            }
         }
     }
 }
@@ -250,16 +296,21 @@ __global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int
     atomicMax(bmax + n, (unsigned long long)__double_as_longlong(mx));
 }
 
-// B (K x N) -> Bt8 (N rows of [c][t][kk]) through a 64 k x 32 n shared tile.
+// B (K x N) -> Bt8 (N rows of [c][t][kk]) through a shared tile stored transposed
+// (32 n rows x 64 k, row pitch 66 doubles): coalesced loads along n, then each
+// thread reads its column's 8 consecutive k as four 16-byte shared loads (every
+// quarter-warp on distinct banks) and writes one 8-byte word per modulus.
 __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
     const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int n, int p, int64_t Kc, int nch,
     const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb) {
-    __shared__ double tl[64][33];
+    constexpr int PITCH = 66;
+    __shared__ __align__(16) double tl[32 * PITCH];
     const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
     const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+#pragma unroll
     for (int r = ty; r < 64; r += 8) {
         const int64_t k = k0 + r, nn = n0 + tx;
-        tl[r][tx] = (k < K && nn < N) ? B[k * ldb + nn] : 0.0;
+        tl[tx * PITCH + r] = (k < K && nn < N) ? __ldcs(B + k * ldb + nn) : 0.0;
     }
     __syncthreads();
     const int64_t Kpad = (int64_t)nch * Kc;
@@ -270,14 +321,36 @@ __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
     if (blockIdx.y == 0 && g == 0) fb[col] = f;
     double v[8];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) v[j] = rint(scale2(tl[8 * g + j][nl], p - f));
+    for (int j = 0; j < 4; ++j) {
+        const double2 x = *reinterpret_cast<const double2 *>(&tl[nl * PITCH + 8 * g + 2 * j]);
+        v[2 * j] = x.x;
+        v[2 * j + 1] = x.y;
+    }
     const int64_t c = k8 / Kc, kk = k8 - c * Kc;
     int8_t *o = Bt8 + col * ld8 + (c * n) * Kc + kk;
-    for (int t = 0; t < n; ++t) {
-        int rr[8];
+    if (p <= 50) {
+        int lo[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
-        *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+        for (int j = 0; j < 8; ++j) {
+            const double vm = scaled_magic(v[j], p - f);
+            lo[j] = __double2loint(vm);
+            v[j] = vm - 6755399441055744.0;
+        }
+        for (int t = 0; t < n; ++t) {
+            int rr[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) rr[j] = res8_fast(v[j], lo[j], t);
+            *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+        }
+    } else {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = rint(scale2(v[j], p - f));
+        for (int t = 0; t < n; ++t) {
+            int rr[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
+            *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+        }
     }
 }
 
@@ -408,7 +481,8 @@ cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, in
     oz2_rowmax_kernel<<<(unsigned)((rows + 7) / 8), 256, 0, s>>>(A, lda, rows, K, ea);
     const int64_t groups = (int64_t)P.nch * P.Kc / 8;
     dim3 grid((unsigned)std::min<int64_t>((groups + 255) / 256, 64), (unsigned)std::min<int64_t>(rows, 65535));
-    oz2_residue_rows_kernel<<<grid, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
+    const int vec = ((reinterpret_cast<uintptr_t>(A) & 15u) == 0 && (lda & 1) == 0) ? 1 : 0;
+    oz2_residue_rows_kernel<<<grid, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea, vec);
     if (launches) *launches += 2;
     return cudaGetLastError();
 }
