@@ -429,6 +429,94 @@ __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__r
     }
 }
 
+// FP64-pipe CRT (the default when the plan allows it, oz2_crt_fast_ok).  The
+// weights and M are split into three 39-bit pieces held as doubles, so
+//   S_i = sum_t u_t w_{t,i}        (u_t < 2^8, 14 terms: every partial sum < 2^51, exact)
+//   q   = rint(S / M)              (relative error ~ 2^-51 of S / M < 2^12; exact
+//                                   because |X| <= B = 2^(2p + lk) <= M / (2 r) with
+//                                   r >= 1 + 1/64, far from the half-integers)
+//   T_i = S_i - q M_i              (|T_i| < 2^51, exact in one FMA)
+//   X   = T_2 2^78 + T_1 2^39 + T_0, summed with two TwoSums: every intermediate is an
+//         integer, the two error terms add exactly, so X is rounded once.
+// Four FP64 operations per modulus and column (one DADD turns the byte into a double
+// through the 2^52 exponent trick, three DFMAs) instead of four IMAD.WIDE plus
+// 128-bit fix-ups: the integer pipes were the bottleneck of oz2_reconstruct_kernel.
+struct Oz2CrtF {
+    int p;
+    double w[OZ2_MAX_MODULI][3];   // W_t pieces (39 bits each)
+    double Mp[3];                  // M pieces
+    double invM39, invM;           // 2^39 / M, 1 / M
+};
+
+__device__ __forceinline__ void two_sum(double a, double b, double &s, double &e) {
+    s = a + b;
+    const double bb = s - a;
+    e = (a - (s - bb)) + (b - bb);
+}
+
+// 8 consecutive columns per thread: one 8-byte load per plane (all NM in flight),
+// then two groups of four columns through the FP64 pieces, each stored at once.
+// One K chunk (K <= 65536); longer K uses the integer pass.
+template <int NM>
+__global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__restrict__ R, int64_t ldr,
+                                                              int64_t plane, const int *__restrict__ ea,
+                                                              const int *__restrict__ fb, const Oz2CrtF crt,
+                                                              double *__restrict__ C, int64_t ldc, int64_t rows,
+                                                              int64_t cols, int vec) {
+    const double two52 = 4503599627370496.0, two39 = 549755813888.0, two78 = 302231454903657293676544.0;
+    for (int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y; row < rows;
+         row += (int64_t)gridDim.y * blockDim.y)
+    for (int64_t c16 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8; c16 < cols;
+         c16 += (int64_t)gridDim.x * blockDim.x * 8) {
+    const uint8_t *pr = R + row * ldr + c16;
+    uint2 u16[NM];
+#pragma unroll
+    for (int t = 0; t < NM; ++t)   // all planes' loads in flight together (ldr, plane % 16 == 0)
+        u16[t] = __ldcs(reinterpret_cast<const uint2 *>(pr + (int64_t)t * plane));
+    const int er = ea[row] - 2 * crt.p;
+    double *crow = C + row * ldc + c16;
+#pragma unroll
+    for (int g = 0; g < 2; ++g) {
+        double acc[4];
+        {
+            uint32_t w4[NM];
+#pragma unroll
+            for (int t = 0; t < NM; ++t) w4[t] = g == 0 ? u16[t].x : u16[t].y;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                double S0 = 0.0, S1 = 0.0, S2 = 0.0;
+#pragma unroll
+                for (int t = 0; t < NM; ++t) {
+                    const double ud = __hiloint2double(0x43300000, (int)__byte_perm(w4[t], 0u, 0x4440u + j)) - two52;
+                    S0 = fma(ud, crt.w[t][0], S0);
+                    S1 = fma(ud, crt.w[t][1], S1);
+                    S2 = fma(ud, crt.w[t][2], S2);
+                }
+                const double q = rint(fma(fma(S2, two39, S1), crt.invM39, S0 * crt.invM));
+                const double T0 = fma(-q, crt.Mp[0], S0);
+                const double T1 = fma(-q, crt.Mp[1], S1);
+                const double T2 = fma(-q, crt.Mp[2], S2);
+                double s1, e1, s2, e2;
+                two_sum(T2 * two78, T1 * two39, s1, e1);
+                two_sum(s1, T0, s2, e2);
+                acc[j] = s2 + (e1 + e2);
+            }
+        }
+        const int64_t c0 = c16 + 4 * g;
+        if (vec && c0 + 4 <= cols) {
+            __stcs(reinterpret_cast<double2 *>(crow + 4 * g),
+                   make_double2(scale2(acc[0], er + fb[c0]), scale2(acc[1], er + fb[c0 + 1])));
+            __stcs(reinterpret_cast<double2 *>(crow + 4 * g + 2),
+                   make_double2(scale2(acc[2], er + fb[c0 + 2]), scale2(acc[3], er + fb[c0 + 3])));
+        } else {
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                if (c0 + j < cols) crow[4 * g + j] = scale2(acc[j], er + fb[c0 + j]);
+        }
+    }
+    }
+}
+
 // ------------------------------------------------------------------------
 // host launchers
 // ------------------------------------------------------------------------
@@ -504,11 +592,50 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
     return cudaGetLastError();
 }
 
+// The FP64-pipe CRT needs one K chunk, M < 2^117 (three 39-bit pieces) and a clear gap between
+// the largest valid |X| (B = 2^(2p + ceil(log2 Kc))) and M / 2: M >= 2 B (1 + 1/64).
+// Holds for every plan of 2..14 moduli (M / 2^floor(log2 M) >= 1.029).
+bool oz2_crt_fast_ok(const Ozaki2Plan &P) {
+    const u128 M = ((u128)P.Mw[1] << 64) | P.Mw[0];
+    if (P.n < 2 || P.nch != 1 || (M >> 117) != 0) return false;
+    const int e = 2 * P.p + ilog2_ceil(P.Kc < 1 ? 1 : P.Kc);
+    if (e + 1 >= 127) return false;
+    const u128 twoB = (u128)1 << (e + 1);
+    return M >= twoB + (twoB >> 6);
+}
+
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
                                       cudaStream_t s) {
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 3u) || (ldr & 3) || (plane & 3)) return cudaErrorInvalidValue;
+    const char *crt_mode = getenv("PDL_OZ2_CRT");
+    if (oz2_crt_fast_ok(P) && !(crt_mode && !strcmp(crt_mode, "int"))) {
+        Oz2CrtF f;
+        f.p = P.p;
+        const u128 mask = ((u128)1 << 39) - 1;
+        for (int t = 0; t < OZ2_MAX_MODULI; ++t) {
+            const u128 W = ((u128)P.W[t][1] << 64) | P.W[t][0];
+            for (int i = 0; i < 3; ++i) f.w[t][i] = (double)(unsigned long long)((W >> (39 * i)) & mask);
+        }
+        const u128 M = ((u128)P.Mw[1] << 64) | P.Mw[0];
+        for (int i = 0; i < 3; ++i) f.Mp[i] = (double)(unsigned long long)((M >> (39 * i)) & mask);
+        f.invM39 = 549755813888.0 / P.Md;
+        f.invM = 1.0 / P.Md;
+        if ((reinterpret_cast<uintptr_t>(R) & 15u) || (ldr & 15) || (plane & 15)) return cudaErrorInvalidValue;
+        const int vec = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
+        dim3 block(32, 8);
+        dim3 grid((unsigned)((cols + 255) / 256), (unsigned)std::min<int64_t>((rows + 7) / 8, 65535));
+        switch (P.n) {
+#define OZ2_CASE(k) \
+    case k: oz2_crt_fp64_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec); break;
+            OZ2_CASE(2) OZ2_CASE(3) OZ2_CASE(4) OZ2_CASE(5) OZ2_CASE(6) OZ2_CASE(7) OZ2_CASE(8) OZ2_CASE(9)
+            OZ2_CASE(10) OZ2_CASE(11) OZ2_CASE(12) OZ2_CASE(13) OZ2_CASE(14)
+#undef OZ2_CASE
+            default: return cudaErrorInvalidValue;
+        }
+        return cudaGetLastError();
+    }
     Oz2Crt crt;
     crt.n = P.n;
     crt.nch = P.nch;

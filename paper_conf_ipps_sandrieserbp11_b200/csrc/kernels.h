@@ -96,6 +96,10 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
 cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
                                uint8_t *R, int64_t ldr, int64_t plane, int64_t rows, int64_t cols, cudaStream_t s,
                                int *launches);
+// The plan admits the FP64-pipe CRT pass (M < 2^117, M >= 2^(2p + lk + 1) (1 + 1/64));
+// otherwise launch_ozaki2_reconstruct uses the 128-bit integer pass.  PDL_OZ2_CRT=int
+// forces the integer pass.
+bool oz2_crt_fast_ok(const Ozaki2Plan &P);
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
                                       cudaStream_t s);

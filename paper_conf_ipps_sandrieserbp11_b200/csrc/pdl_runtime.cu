@@ -330,7 +330,8 @@ int pdl_query(const char *key, char *out, size_t len) {
         };
         o << "],\"W\":[";
         for (int t = 0; t < P.n; ++t) o << (t ? "," : "") << "\"" << dec(P.W[t][0], P.W[t][1]) << "\"";
-        o << "],\"M\":\"" << dec(P.Mw[0], P.Mw[1]) << "\"}";
+        o << "],\"M\":\"" << dec(P.Mw[0], P.Mw[1]) << "\",\"crt\":\"" << (pdlk::oz2_crt_fast_ok(P) ? "fp64" : "int")
+          << "\"}";
         res = o.str();
     } else {
         int rc = check_loaded();
