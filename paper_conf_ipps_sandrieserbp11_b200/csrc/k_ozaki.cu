@@ -213,11 +213,16 @@ __host__ __device__ constexpr uint32_t idesc_i8(int M, int N) {
 __device__ __forceinline__ double pow2_normal(int E) {   // E in [-1022, 1023]
     return __longlong_as_double((long long)(1023 + E) << 52);
 }
+// int32 -> double exactly on the FP64 pipe (the conversion unit runs at a quarter
+// of its rate): the bits 0x43380000:(x ^ 2^31) are 1.5 * 2^52 + 2^31 + x.
+__device__ __forceinline__ double i2d_exact(int32_t x) {
+    return __hiloint2double(0x43380000, x ^ (int)0x80000000) - 6755401588539392.0;
+}
 __device__ __forceinline__ double scale_pow2(int32_t x, int E) {
-    if (E >= -1022 && E <= 1023) return (double)x * pow2_normal(E);
+    if (E >= -1022 && E <= 1023) return i2d_exact(x) * pow2_normal(E);
     const int E1 = E < 0 ? -1022 : 1023;
     const int E2 = max(-1022, min(1023, E - E1));
-    return ((double)x * pow2_normal(E1)) * pow2_normal(E2);
+    return (i2d_exact(x) * pow2_normal(E1)) * pow2_normal(E2);
 }
 
 __device__ __forceinline__ void umma_i8_2sm(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
@@ -234,7 +239,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, OCC>:
     oz_gemm_2sm_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
                        TC *__restrict__ C, int64_t ldc, int M, int N, int Kd, const int *__restrict__ ea,
                        const int *__restrict__ fb, int scale_exp, int accumulate, int tiles_m, int tiles_n,
-                       int group_m, int vec_ok, int modulus, float inv_mod) {
+                       int group_m, int vec_ok, int modulus, unsigned mod_magic) {
     using namespace koz;
     using CF = Cfg<NSUB, OCC>;
     constexpr int BN = CF::BN, STAGES = CF::STAGES, STAGE_BYTES = CF::STAGE_BYTES;
@@ -324,9 +329,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, OCC>:
             // Ozaki-II (K6): the exact INT32 sum reduced mod m into a byte plane
             // (C = plane, ldc = its row pitch, 16-byte aligned).  Each thread owns
             // its TMEM lane = row and stores 16 consecutive residues per step.
+            // |x| <= Kc 2^14 <= 2^30, so xb = x + bias (bias = m ceil(2^30 / m)) lies in
+            // [0, 2^31 + m) and xb mod m = xb - m umulhi(xb, mag) >> 7 exactly, with
+            // mag = ceil(2^39 / m) < 2^32 (e = mag m - 2^39 < m and xb e < 2^39):
+            // four integer operations, no conversions.
             const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
             const int cbase = tn * BN + cg * EPI_COLS;
             uint8_t *prow = reinterpret_cast<uint8_t *>(C) + (int64_t)row * ldc + cbase;
+            const uint32_t mm = (uint32_t)modulus, bias = mm * ((1u << 30) / mm + 1u);
 #pragma unroll 1
             for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
                 uint32_t r[16];
@@ -335,18 +345,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, OCC>:
                 uint32_t pk[4];
 #pragma unroll
                 for (int w4 = 0; w4 < 4; ++w4) {
-                    uint32_t word = 0;
+                    uint32_t res[4];
 #pragma unroll
                     for (int b = 0; b < 4; ++b) {
-                        const int x = (int)r[4 * w4 + b];
-                        int res = x - __float2int_rn((float)x * inv_mod) * modulus;   // |q error| <= 1
-                        res += res < 0 ? modulus : 0;
-                        res += res < 0 ? modulus : 0;
-                        res -= res >= modulus ? modulus : 0;
-                        res -= res >= modulus ? modulus : 0;
-                        word |= (uint32_t)res << (8 * b);
+                        const uint32_t xb = r[4 * w4 + b] + bias;
+                        res[b] = xb - (__umulhi(xb, mod_magic) >> 7) * mm;
                     }
-                    pk[w4] = word;
+                    pk[w4] = __byte_perm(__byte_perm(res[0], res[1], 0x0040), __byte_perm(res[2], res[3], 0x0040), 0x5410);
                 }
                 if (cbase + c0 + 16 <= N) {
                     *reinterpret_cast<uint4 *>(prow + c0) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
@@ -556,27 +561,27 @@ static cudaError_t oz_set_attrs() {
 template <int NSUB, int OCC, typename TC>
 static void oz_launch_one(const CUtensorMap &ta, const CUtensorMap &tb, TC *C, int64_t ldc, int64_t rows,
                           int64_t cols, int64_t kd, const int *ea, const int *fb, int scale_exp, int accumulate,
-                          int vec_ok, int modulus, float inv_mod, cudaStream_t stream) {
+                          int vec_ok, int modulus, unsigned mod_magic, cudaStream_t stream) {
     using namespace koz;
     using CF = Cfg<NSUB, OCC>;
     const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + CF::BN - 1) / CF::BN);
     oz_gemm_2sm_kernel<NSUB, TC, OCC><<<2 * tiles_m * tiles_n, CF::THREADS, CF::SMEM_BYTES, stream>>>(
         ta, tb, C, ldc, (int)rows, (int)cols, (int)kd, ea, fb, scale_exp, accumulate, tiles_m, tiles_n,
-        group_for_k(kd), vec_ok, modulus, inv_mod);
+        group_for_k(kd), vec_ok, modulus, mod_magic);
 }
 
 template <typename TC>
 static void oz_launch(int shape, const CUtensorMap &ta, const CUtensorMap &tb, TC *C, int64_t ldc, int64_t rows,
                       int64_t cols, int64_t kd, const int *ea, const int *fb, int scale_exp, int accumulate,
-                      int vec_ok, int modulus, float inv_mod, cudaStream_t stream) {
+                      int vec_ok, int modulus, unsigned mod_magic, cudaStream_t stream) {
     if (shape == 0)
-        oz_launch_one<2, 1>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, inv_mod,
+        oz_launch_one<2, 1>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, mod_magic,
                             stream);
     else if (shape == 1)
-        oz_launch_one<1, 1>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, inv_mod,
+        oz_launch_one<1, 1>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, mod_magic,
                             stream);
     else
-        oz_launch_one<1, 2>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, inv_mod,
+        oz_launch_one<1, 2>(ta, tb, C, ldc, rows, cols, kd, ea, fb, scale_exp, accumulate, vec_ok, modulus, mod_magic,
                             stream);
 }
 
@@ -602,7 +607,7 @@ static cudaError_t gemm_impl(EncodeTiledFn enc, const int8_t *A8, const int8_t *
             if (!map_i8(enc, &ta, a, (uint64_t)kd, (uint64_t)rows, (uint64_t)L.ld8, BM) ||
                 !map_i8(enc, &tb, b, (uint64_t)kd, (uint64_t)cols, (uint64_t)L.ld8, BNH))
                 return cudaErrorInvalidValue;
-            oz_launch<TC>(shape, ta, tb, C, ldc, rows, cols, kd, ea, fb, -7 * (d + 2), first ? 0 : 1, vec_ok, 0, 0.f,
+            oz_launch<TC>(shape, ta, tb, C, ldc, rows, cols, kd, ea, fb, -7 * (d + 2), first ? 0 : 1, vec_ok, 0, 0u,
                           stream);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
@@ -643,8 +648,10 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
                 !map_i8(enc, &tb, Bt8 + off, (uint64_t)P.Kc, (uint64_t)cols, (uint64_t)P.ld8, BNH))
                 return cudaErrorInvalidValue;
             uint8_t *Rp = R + ((int64_t)c * P.n + t) * plane;
-            oz_launch<uint8_t>(shape, ta, tb, Rp, ldr, rows, cols, P.Kc, nullptr, nullptr, 0, 0, 1, P.m[t],
-                               1.0f / (float)P.m[t], stream);
+            // ceil(2^39 / m): the exact division-by-constant multiplier of the epilogue
+            const unsigned magic = (unsigned)((((unsigned long long)1 << 39) + (unsigned)P.m[t] - 1) / (unsigned)P.m[t]);
+            oz_launch<uint8_t>(shape, ta, tb, Rp, ldr, rows, cols, P.Kc, nullptr, nullptr, 0, 0, 1, P.m[t], magic,
+                               stream);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             if (launches) ++*launches;
