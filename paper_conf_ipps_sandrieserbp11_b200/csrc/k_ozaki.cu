@@ -34,6 +34,7 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <algorithm>
 
 #include "kernels.h"
 #include "ptx.cuh"
@@ -446,6 +447,180 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, OCC>:
     }
 }
 
+// K6, persistent: one CTA pair per TPC walks the residue GEMM's cluster tiles
+// (tile = cluster, cluster + clusters, ...).  Barriers and TMEM are set up once; the
+// producer runs ahead into the next tile while the epilogue drains the accumulator,
+// and the MMA warp starts the next tile as soon as both CTAs' epilogue warps have
+// read TMEM (bar_tempty on the leader, 2 x EPI_WARPS arrivals), so only the TMEM
+// read -- not the prologue, pipeline fill, residue arithmetic and stores -- sits
+// between two tiles' MMAs.  Epilogue as oz_gemm_2sm_kernel<NSUB, uint8_t>.
+template <int NSUB>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::THREADS, 1)
+    oz2_gemm_persistent_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
+                               uint8_t *__restrict__ R, int64_t ldr, int M, int N, int Kd, int tiles_m,
+                               int tiles_n, int group_m, int modulus, unsigned mod_magic, int hints) {
+    using namespace koz;
+    using CF = Cfg<NSUB, 1>;
+    constexpr int BN = CF::BN, STAGES = CF::STAGES, STAGE_BYTES = CF::STAGE_BYTES;
+    constexpr int EPI_COLS = CF::EPI_COLS, TMEM_COLS = CF::TMEM_COLS, EPI_WARPS = CF::EPI_WARPS;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
+    const uint32_t bar_full = base + STAGES * STAGE_BYTES;
+    const uint32_t bar_empty = bar_full + STAGES * 8;
+    const uint32_t bar_tfull = bar_empty + STAGES * 8;
+    const uint32_t bar_tempty = bar_tfull + 8;
+    const uint32_t tmem_slot = bar_tempty + 8;
+    uint8_t *const gbase = smem_raw + (base - smem_u32(smem_raw));
+    volatile uint32_t *tmem_slot_ptr = reinterpret_cast<volatile uint32_t *>(gbase + (tmem_slot - base));
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = cluster_ctarank();
+    const int ntiles = tiles_m * tiles_n, nclusters = (int)(gridDim.x >> 1), cl = (int)(blockIdx.x >> 1);
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(bar_full + 8 * s, 1);
+            mbar_init(bar_empty + 8 * s, 1);
+        }
+        mbar_init(bar_tfull, 1);
+        mbar_init(bar_tempty, 2 * EPI_WARPS);
+        fence_barrier_init();
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(tmem_slot),
+                     "n"(TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    cluster_sync_all();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem_base = *tmem_slot_ptr;
+    const int nk = Kd / BK;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            tma_prefetch_desc(&tA);
+            tma_prefetch_desc(&tB);
+            // hints & 1: A strips (reused across the raster group's column sweep) evict_last,
+            // B strips (read by one wave of the group) evict_first
+            const uint64_t pol_a = l2_policy_evict_last(), pol_b = l2_policy_evict_first();
+            uint32_t it = 0;
+            for (int tile = cl; tile < ntiles; tile += nclusters) {
+                int tm, tn;
+                raster_tile(tile, tiles_m, tiles_n, group_m, &tm, &tn);
+                const int m0 = tm * (2 * BM) + (int)rank * BM;
+                const int nb0 = tn * BN + (int)rank * BNH;
+                // hints & 4: odd rounds of tiles walk K backwards, so a round starts on the
+                // K blocks of the (shared) A strips the previous round touched last and
+                // still finds them in L2 (integer sums: the order does not change a bit)
+                const bool rev = (hints & 4) && (((tile / nclusters) & 1) != 0);
+                for (int kb = 0; kb < nk; ++kb, ++it) {
+                    const uint32_t s = it % STAGES, ph = (it / STAGES) & 1u;
+                    mbar_wait(bar_empty + 8 * s, ph ^ 1u);
+                    const uint32_t fb_leader = mapa_shared(bar_full + 8 * s, 0);
+                    if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * STAGE_BYTES);
+                    const uint32_t st = base + s * STAGE_BYTES;
+                    const int kx = (rev ? nk - 1 - kb : kb) * BK;
+                    if (hints & 1) {
+                        tma_load_2d_2sm_hint(st, &tA, fb_leader, kx, m0, pol_a);
+#pragma unroll
+                        for (int j = 0; j < NSUB; ++j)
+                            tma_load_2d_2sm_hint(st + A_BYTES + j * B_BYTES, &tB, fb_leader, kx, nb0 + j * BN1, pol_b);
+                    } else {
+                        tma_load_2d_2sm(st, &tA, fb_leader, kx, m0);
+#pragma unroll
+                        for (int j = 0; j < NSUB; ++j)
+                            tma_load_2d_2sm(st + A_BYTES + j * B_BYTES, &tB, fb_leader, kx, nb0 + j * BN1);
+                    }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (rank == 0 && lane == 0) {
+            constexpr uint32_t idesc = idesc_i8(2 * BM, BN1);
+            uint32_t it = 0, ti = 0;
+            for (int tile = cl; tile < ntiles; tile += nclusters, ++ti) {
+                mbar_wait(bar_tempty, (ti & 1u) ^ 1u);   // both CTAs' epilogues have read TMEM
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                for (int kb = 0; kb < nk; ++kb, ++it) {
+                    const uint32_t s = it % STAGES, ph = (it / STAGES) & 1u;
+                    mbar_wait(bar_full + 8 * s, ph);
+                    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                    const uint32_t st = base + s * STAGE_BYTES;
+#pragma unroll
+                    for (int kk = 0; kk < BK / UMMA_K; ++kk) {
+                        const uint32_t off = kk * UMMA_K;
+#pragma unroll
+                        for (int j = 0; j < NSUB; ++j)
+                            umma_i8_2sm(tmem_base + j * BN1, umma_desc_k_sw128(st + off),
+                                        umma_desc_k_sw128(st + A_BYTES + j * B_BYTES + off), idesc,
+                                        (kb | kk) ? 1u : 0u);
+                    }
+                    umma_commit_2sm(bar_empty + 8 * s);
+                }
+                umma_commit_2sm(bar_tfull);
+            }
+        }
+        __syncwarp();
+    } else {
+        const int e = warp - FIRST_EPI_WARP;
+        const int q = warp & 3;
+        const int cg = e >> 2;
+        const uint32_t tl = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(cg * EPI_COLS);
+        const uint32_t tempty_leader = mapa_shared(bar_tempty, 0);
+        const uint32_t mm = (uint32_t)modulus, bias = mm * ((1u << 30) / mm + 1u);
+        uint32_t ti = 0;
+        for (int tile = cl; tile < ntiles; tile += nclusters, ++ti) {
+            int tm, tn;
+            raster_tile(tile, tiles_m, tiles_n, group_m, &tm, &tn);
+            const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
+            const int cbase = tn * BN + cg * EPI_COLS;
+            uint8_t *prow = R + (int64_t)row * ldr + cbase;
+            mbar_wait(bar_tfull, ti & 1u);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll 1
+            for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
+                uint32_t r[16];
+                tmem_ld16(tl + c0, r);
+                if (c0 + 16 == EPI_COLS) {   // this warp's last TMEM read is complete
+                    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive_cluster(tempty_leader);
+                }
+                if (row >= M) continue;
+                uint32_t pk[4];
+#pragma unroll
+                for (int w4 = 0; w4 < 4; ++w4) {
+                    uint32_t res[4];
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) {
+                        const uint32_t xb = r[4 * w4 + b] + bias;
+                        res[b] = xb - (__umulhi(xb, mod_magic) >> 7) * mm;
+                    }
+                    pk[w4] = __byte_perm(__byte_perm(res[0], res[1], 0x0040), __byte_perm(res[2], res[3], 0x0040), 0x5410);
+                }
+                if (cbase + c0 + 16 <= N) {
+                    // hints & 2: streaming (evict-first) plane stores keep the operand strips in L2
+                    if (hints & 2)
+                        __stcs(reinterpret_cast<uint4 *>(prow + c0), make_uint4(pk[0], pk[1], pk[2], pk[3]));
+                    else
+                        *reinterpret_cast<uint4 *>(prow + c0) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                } else {
+#pragma unroll
+                    for (int jj = 0; jj < 16; ++jj)
+                        if (cbase + c0 + jj < N) prow[c0 + jj] = (uint8_t)(pk[jj >> 2] >> (8 * (jj & 3)));
+                }
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    cluster_sync_all();
+    if (warp == 1) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(TMEM_COLS));
+    }
+}
+
 // ------------------------------------------------------------------------
 // host side
 // ------------------------------------------------------------------------
@@ -558,6 +733,41 @@ static cudaError_t oz_set_attrs() {
     return cudaSuccess;
 }
 
+// Co-resident CTA pairs of the persistent K6 kernel (cudaOccupancyMaxActiveClusters,
+// cached per device); sets its shared-memory attribute on first use.
+static cudaError_t oz2_persistent_clusters(int *out) {
+    using namespace koz;
+    using CF = Cfg<2, 1>;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static int cached[64] = {0};
+    if (dev < 64 && cached[dev] > 0) {
+        *out = cached[dev];
+        return cudaSuccess;
+    }
+    cudaError_t e = cudaFuncSetAttribute(oz2_gemm_persistent_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         CF::SMEM_BYTES);
+    if (e != cudaSuccess) return e;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * 148, 1, 1);
+    cfg.blockDim = dim3(CF::THREADS, 1, 1);
+    cfg.dynamicSmemBytes = CF::SMEM_BYTES;
+    cudaLaunchAttribute attr;
+    attr.id = cudaLaunchAttributeClusterDimension;
+    attr.val.clusterDim.x = 2;
+    attr.val.clusterDim.y = 1;
+    attr.val.clusterDim.z = 1;
+    cfg.attrs = &attr;
+    cfg.numAttrs = 1;
+    int n = 0;
+    e = cudaOccupancyMaxActiveClusters(&n, oz2_gemm_persistent_kernel<2>, &cfg);
+    if (e != cudaSuccess) return e;
+    if (n < 1) return cudaErrorInvalidConfiguration;
+    if (dev < 64) cached[dev] = n;
+    *out = n;
+    return cudaSuccess;
+}
+
 template <int NSUB, int OCC, typename TC>
 static void oz_launch_one(const CUtensorMap &ta, const CUtensorMap &tb, TC *C, int64_t ldc, int64_t rows,
                           int64_t cols, int64_t kd, const int *ea, const int *fb, int scale_exp, int accumulate,
@@ -640,6 +850,16 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
     cudaError_t e0 = oz_set_attrs<uint8_t>();
     if (e0 != cudaSuccess) return e0;
     const int shape = oz_shape(rows, cols);
+    // persistent 256 x 512 tiles by default (PDL_OZ2_PERSIST=0: one cluster per tile)
+    const char *pe = getenv("PDL_OZ2_PERSIST");
+    const bool persist = shape == 0 && !(pe && !strcmp(pe, "0"));
+    int pclusters = 0;
+    const char *he = getenv("PDL_OZ2_HINTS");
+    const int hints = he ? atoi(he) : 0;
+    if (persist) {
+        e0 = oz2_persistent_clusters(&pclusters);
+        if (e0 != cudaSuccess) return e0;
+    }
     for (int c = 0; c < P.nch; ++c) {
         for (int t = 0; t < P.n; ++t) {
             const int64_t off = ((int64_t)c * P.n + t) * P.Kc;
@@ -650,8 +870,17 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
             uint8_t *Rp = R + ((int64_t)c * P.n + t) * plane;
             // ceil(2^39 / m): the exact division-by-constant multiplier of the epilogue
             const unsigned magic = (unsigned)((((unsigned long long)1 << 39) + (unsigned)P.m[t] - 1) / (unsigned)P.m[t]);
-            oz_launch<uint8_t>(shape, ta, tb, Rp, ldr, rows, cols, P.Kc, nullptr, nullptr, 0, 0, 1, P.m[t], magic,
-                               stream);
+            if (persist) {
+                using CF = Cfg<2, 1>;
+                const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + CF::BN - 1) / CF::BN);
+                const int ncl = std::min(tiles_m * tiles_n, pclusters);
+                oz2_gemm_persistent_kernel<2><<<2 * ncl, CF::THREADS, CF::SMEM_BYTES, stream>>>(
+                    ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, tiles_m, tiles_n, group_for_k(P.Kc), P.m[t],
+                    magic, hints);
+            } else {
+                oz_launch<uint8_t>(shape, ta, tb, Rp, ldr, rows, cols, P.Kc, nullptr, nullptr, 0, 0, 1, P.m[t], magic,
+                                   stream);
+            }
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             if (launches) ++*launches;
