@@ -136,6 +136,29 @@ def test_invariance_bitwise(monkeypatch):
     assert np.array_equal(oz2_matmul(A, B, host=True), ref)
 
 
+def test_gemm_shapes_and_crt_passes_bitwise(monkeypatch):
+    """The residue GEMMs are exact INT32 sums and the CRT is exact, so the K6
+    kernel shape (persistent 256 x 512 -- the default for this size, >= 148
+    cluster tiles --, one cluster per tile, 256 x 256, two CTA pairs per SM),
+    and the serpentine-K / cache-hint knobs change no bit; ragged edges in both
+    dimensions.  The 128-bit integer CRT pass rounds X twice (high and low words),
+    the FP64 pass once, so those agree to 2 ulps."""
+    A = W.uniform((5000, 1100), np.float64, 21) - 0.5
+    B = W.uniform((1100, 3999), np.float64, 22)
+    ref = oz2_matmul(A, B)
+    rows = [0, 1, 255, 256, 4095, 4999] + list(np.random.default_rng(3).integers(0, 5000, 24))
+    check(ref, A, B, rows=rows)
+    for env in ({"PDL_OZ2_PERSIST": "0"}, {"PDL_OZ_SHAPE": "256"}, {"PDL_OZ_SHAPE": "256x2"},
+                {"PDL_OZ2_HINTS": "7"}):
+        with monkeypatch.context() as mp:
+            for k, v in env.items():
+                mp.setenv(k, v)
+            assert np.array_equal(oz2_matmul(A, B), ref), env
+    monkeypatch.setenv("PDL_OZ2_CRT", "int")
+    Ci = oz2_matmul(A, B)
+    assert np.all(np.abs(Ci - ref) <= 2 * np.spacing(np.abs(ref)))
+
+
 def test_k_chunks_beyond_int32_window():
     """K > 65536 is split into K chunks (each CRT-exact), summed in FP64."""
     A = W.uniform((64, 70000), np.float64, 21)

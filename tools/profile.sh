@@ -23,9 +23,9 @@ for w in $WHAT; do
         ncu --set full --clock-control none --import-source on -k regex:oz_split -s 2 -c 2 -o $OUT/prof_ozsplit -f $P --variant ozaki > $OUT/prof_ozsplit.log 2>&1
         ncu $DR -k regex:oz_gemm -s 6 -c 6 --log-file $OUT/traffic_ozaki.csv $P --variant ozaki > $OUT/traffic_oz.log 2>&1 ;;
     oz2) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_oz2.csv $B --variant ozaki2 > $OUT/launches_oz2.log 2>&1
-        ncu --set full --clock-control none --import-source on -k regex:oz_gemm -s 14 -c 1 -o $OUT/prof_oz2 -f $P --variant ozaki2 > $OUT/prof_oz2.log 2>&1
-        ncu --set full --clock-control none --import-source on -k regex:oz2_ -s 4 -c 4 -o $OUT/prof_oz2aux -f $P --variant ozaki2 > $OUT/prof_oz2aux.log 2>&1
-        ncu $DR -k regex:oz_gemm -s 13 -c 13 --log-file $OUT/traffic_ozaki2.csv $P --variant ozaki2 > $OUT/traffic_oz2.log 2>&1 ;;
+        ncu --set full --clock-control none --import-source on -k 'regex:oz2?_gemm' -s 14 -c 1 -o $OUT/prof_oz2 -f $P --variant ozaki2 > $OUT/prof_oz2.log 2>&1
+        ncu --set full --clock-control none --import-source on -k 'regex:oz2_(rowmax|residue|colmax|split|crt|reconstruct)' -s 5 -c 5 -o $OUT/prof_oz2aux -f $P --variant ozaki2 > $OUT/prof_oz2aux.log 2>&1
+        ncu $DR -k 'regex:oz2?_gemm' -s 13 -c 13 --log-file $OUT/traffic_ozaki2.csv $P --variant ozaki2 > $OUT/traffic_oz2.log 2>&1 ;;
     oz32) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_oz32.csv $B --dtype f32 --variant ozaki > $OUT/launches_oz32.log 2>&1
         ncu $DR -k regex:oz_gemm -s 3 -c 3 --log-file $OUT/traffic_ozaki32.csv $P --dtype f32 --variant ozaki > $OUT/traffic_oz32.log 2>&1 ;;
   esac
