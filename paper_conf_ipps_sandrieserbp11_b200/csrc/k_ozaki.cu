@@ -57,14 +57,31 @@ __device__ __forceinline__ int exp_of_max(double mx, int rn) {
     return e;
 }
 
+// x 2^E (as ldexp): one DMUL by the bit-built power of two in the normal range
+__device__ __forceinline__ double ldexp_fast(double x, int E) {
+    if (E >= -1022 && E <= 1023) return x * __longlong_as_double((long long)(1023 + E) << 52);
+    return ldexp(x, E);
+}
+
 // One slicing step: v <- 128 v, q = round(v) (trunc or nearest), v <- v - q
 // (all exact in FP64).  trunc: |q| <= 127, remainders in (-1,1); nearest:
 // |q| <= 127 for the first slice, <= 64 after, remainders in [-1/2, 1/2].
-__device__ __forceinline__ double slice_q(double &v, int rn) {
+// Returns q as an int.  Nearest rounding runs on the FP64 pipe only: t =
+// fma(v, 128, 1.5 * 2^52) = magic + rint(128 v) (|128 v| < 2^51), q = t - magic,
+// v = fma(v, 128, -q) (exact), and q's low word is the int -- no FRND / F2I on the
+// quarter-rate conversion unit.
+__device__ __forceinline__ int slice_q(double &v, int rn) {
+    if (rn) {
+        const double magic = 6755399441055744.0;
+        const double t = fma(v, 128.0, magic);
+        const double q = t - magic;
+        v = fma(v, 128.0, -q);
+        return __double2loint(t);
+    }
     v *= 128.0;
-    const double q = rn ? rint(v) : trunc(v);
+    const double q = trunc(v);
     v -= q;
-    return q;
+    return (int)q;
 }
 
 // One CTA per row (grid-stride): A (M x K, lda) -> A8 rows [c][s][kk].
@@ -96,16 +113,13 @@ __global__ void oz_split_rows_kernel(const T *__restrict__ A, int64_t lda, int64
         for (int64_t k8 = (int64_t)threadIdx.x * 8; k8 < Kpad; k8 += (int64_t)blockDim.x * 8) {
             double v[8];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? ldexp((double)row[k8 + j], -e) : 0.0;
+            for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? ldexp_fast((double)row[k8 + j], -e) : 0.0;
             const int64_t c = k8 / Kc, kk = k8 - c * Kc;
             int8_t *o = out + (c * S) * Kc + kk;
             for (int s = 0; s < S; ++s) {
                 uint64_t pk = 0;
 #pragma unroll
-                for (int j = 0; j < 8; ++j) {
-                    const double q = slice_q(v[j], rn);
-                    pk |= (uint64_t)(uint8_t)(int8_t)(int)q << (8 * j);
-                }
+                for (int j = 0; j < 8; ++j) pk |= (uint64_t)(uint8_t)slice_q(v[j], rn) << (8 * j);
                 *reinterpret_cast<uint64_t *>(o + (int64_t)s * Kc) = pk;
             }
         }
@@ -125,20 +139,22 @@ __global__ void oz_colmax_kernel(const T *__restrict__ B, int64_t ldb, int64_t K
     atomicMax(bmax + n, (unsigned long long)__double_as_longlong(mx));
 }
 
-// B (K x N) -> Bt8 (N rows of [c][S-1-s][kk]) through a 32 x 32 smem transpose.
-// Tile of 64 k x 32 n: coalesced loads along n into shared memory, then each
-// thread slices 8 consecutive k of one column -> one 8-byte store per slice.
+// B (K x N) -> Bt8 (N rows of [c][S-1-s][kk]) through a shared tile stored
+// transposed (32 n rows x 64 k, pitch 66 doubles): coalesced loads along n, then
+// each thread slices 8 consecutive k of one column read as four 16-byte shared
+// loads (conflict-free per quarter-warp) -> one 8-byte store per slice.
 template <typename T>
 __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
     const T *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S, int64_t Kc, int nch,
     const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
     int rn) {
-    __shared__ double t[64][33];
+    constexpr int PITCH = 66;
+    __shared__ __align__(16) double t[32 * PITCH];
     const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
     const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;   // 32 x 8
     for (int r = ty; r < 64; r += 8) {
         const int64_t k = k0 + r, n = n0 + tx;
-        t[r][tx] = (k < K && n < N) ? (double)B[k * ldb + n] : 0.0;
+        t[tx * PITCH + r] = (k < K && n < N) ? (double)B[k * ldb + n] : 0.0;
     }
     __syncthreads();
     const int64_t Kpad = (int64_t)nch * Kc;
@@ -149,16 +165,17 @@ __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
     if (blockIdx.y == 0 && g == 0) fb[n] = f;
     double v[8];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) v[j] = ldexp(t[8 * g + j][nl], -f);
+    for (int j = 0; j < 4; ++j) {
+        const double2 x = *reinterpret_cast<const double2 *>(&t[nl * PITCH + 8 * g + 2 * j]);
+        v[2 * j] = ldexp_fast(x.x, -f);
+        v[2 * j + 1] = ldexp_fast(x.y, -f);
+    }
     const int64_t c = k8 / Kc, kk = k8 - c * Kc;
     int8_t *o = Bt8 + n * ld8 + (c * S) * Kc + kk;
     for (int s = 0; s < S; ++s) {
         uint64_t pk = 0;
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const double q = slice_q(v[j], rn);
-            pk |= (uint64_t)(uint8_t)(int8_t)(int)q << (8 * j);
-        }
+        for (int j = 0; j < 8; ++j) pk |= (uint64_t)(uint8_t)slice_q(v[j], rn) << (8 * j);
         *reinterpret_cast<uint64_t *>(o + (int64_t)(S - 1 - s) * Kc) = pk;
     }
 }
