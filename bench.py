@@ -255,24 +255,35 @@ def host_inputs(cfg, np_dtype):
     return W.config_inputs(cfg, np_dtype)
 
 
+def host_cores():
+    """Host cores this process may run on.  The oracle gets them explicitly:
+    torchrun sets OMP_NUM_THREADS=1 for N > 1, which would otherwise leave the
+    reference arm (rank 0 alone) on one core."""
+    try:
+        return max(1, len(os.sched_getaffinity(0)))
+    except AttributeError:
+        return max(1, os.cpu_count() or 1)
+
+
 def cpu_baseline(A, B, seconds):
     """Time the oracle (as it stands) on a bounded row sample of the workload."""
     import oracle
     M, K = A.shape
     N = B.shape[1]
+    nt = host_cores()
     rng = np.random.Generator(np.random.PCG64(99))
-    ncal = 2 * oracle.max_threads()          # one calibration row pair per thread
+    ncal = 2 * nt                            # one calibration row pair per thread
     t0 = time.perf_counter()
-    oracle.matmul(A, B, rows=rng.integers(0, M, size=ncal), with_mag=False)
+    oracle.matmul(A, B, rows=rng.integers(0, M, size=ncal), with_mag=False, nthreads=nt)
     t1 = time.perf_counter()
     per_row = max((t1 - t0) / ncal, 1e-6)
     nrows = int(max(2, min(M, seconds / per_row)))
     rows = rng.integers(0, M, size=nrows)
     t0 = time.perf_counter()
-    oracle.matmul(A, B, rows=rows, with_mag=False)
+    oracle.matmul(A, B, rows=rows, with_mag=False, nthreads=nt)
     dt = time.perf_counter() - t0
     gflops = 2.0 * nrows * N * K / dt / 1e9
-    return {"value": round(gflops, 3), "unit": "GFLOP/s", "cores": oracle.max_threads(), "kind": "oracle",
+    return {"value": round(gflops, 3), "unit": "GFLOP/s", "cores": nt, "kind": "oracle",
             "sample": f"{nrows} random rows x all {N} columns of the {M}x{N}x{K} product "
                       f"({2.0 * nrows * N * K:.3g} FLOP, {dt:.1f} s, double accumulation)"}
 
@@ -286,21 +297,22 @@ def run_reference(args):
     np_dtype = np.float64 if args.dtype == "f64" else np.float32
     A, B = host_inputs(args.config, np_dtype)
     import oracle
+    nt = host_cores()
     rng = np.random.Generator(np.random.PCG64(5))
     per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
-    ncal = 2 * oracle.max_threads()
+    ncal = 2 * nt
     t0 = time.perf_counter()
-    oracle.matmul(A, B, rows=rng.integers(0, c.M, size=ncal), with_mag=False)
+    oracle.matmul(A, B, rows=rng.integers(0, c.M, size=ncal), with_mag=False, nthreads=nt)
     per_row = max((time.perf_counter() - t0) / ncal, 1e-6)
     nrows = int(max(1, min(c.M, per_step / per_row)))
     flops = 2.0 * nrows * c.N * c.K
     for _ in range(args.warmup):
-        oracle.matmul(A, B, rows=rng.integers(0, c.M, size=nrows), with_mag=False)
+        oracle.matmul(A, B, rows=rng.integers(0, c.M, size=nrows), with_mag=False, nthreads=nt)
     times = []
     for _ in range(args.steps):
         rows = rng.integers(0, c.M, size=nrows)
         t0 = time.perf_counter()
-        oracle.matmul(A, B, rows=rows, with_mag=False)
+        oracle.matmul(A, B, rows=rows, with_mag=False, nthreads=nt)
         times.append(time.perf_counter() - t0)
     ms = 1e3 * sum(times) / len(times)
     value = flops / (ms / 1e3) / 1e9
@@ -310,7 +322,7 @@ def run_reference(args):
             "data": "synthetic", "impl": "reference",
             "config": {"workload": f"{args.config} {c.M}x{c.N}x{c.K} ({args.dtype}), oracle row sample",
                        "M": c.M, "N": c.N, "K": c.K, "tile": c.tile, "rows_per_step": nrows},
-            "cpu_baseline": {"value": round(value, 3), "unit": "GFLOP/s", "cores": oracle.max_threads(),
+            "cpu_baseline": {"value": round(value, 3), "unit": "GFLOP/s", "cores": nt,
                              "kind": "oracle",
                              "sample": f"{nrows} random rows x {c.N} columns per step (K={c.K})"},
             "e2e": {"value": round(value, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0,

@@ -98,3 +98,24 @@ def test_exchange_assembles_panels(world):
             assert Gr * Gc == world
             cover[r0:r1, c0:c1] += 1
         assert np.all(cover == 1)
+
+
+def test_reference_arm_uses_all_host_cores():
+    """bench.py --impl reference (the oracle on the host cores) under torchrun
+    with 2 ranks: rank 0 alone prints one line, on every core this process may
+    use, although torchrun sets OMP_NUM_THREADS=1 for N > 1."""
+    import json
+    import subprocess
+    import sys
+    env = dict(os.environ, OMP_NUM_THREADS="1")
+    out = subprocess.run(
+        [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+         "--master-addr", "127.0.0.1", "--master-port", "29587", os.path.join(ROOT, "bench.py"), "--gpus", "2",
+         "--impl", "reference", "--config", "C1", "--steps", "1", "--warmup", "1"],
+        capture_output=True, text=True, timeout=300, env=env, cwd=ROOT)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2
+    assert d["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
