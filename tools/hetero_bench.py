@@ -54,6 +54,9 @@ def main():
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--tile", type=int, default=256)
+    ap.add_argument("--mixed", type=float, default=0.0,
+                    help="also run per-Worker variants: ozaki2 on the first partition, dmma on the "
+                         "others, BLOCK weighted by this RELATIVE_SPEED of the first Worker (FP64)")
     args = ap.parse_args()
     dt = torch.float64 if args.dtype == "f64" else torch.float32
     n = args.n
@@ -79,6 +82,20 @@ def main():
         if "dynamic" in st:
             r["tiles"] = st["dynamic"]["tiles"]
         rows.append(r)
+    if args.mixed > 0 and args.dtype == "f64":
+        # the paper's premise: one task, a variant per PU pre-selected from the PDL
+        oz = pdl.descriptor_xml(1, props={"DGEMM_VARIANT": "ozaki2"})
+        t, st = timed(oz, A, B, C, None, args.reps, args.tile)
+        rows.append({"mapping": "whole device, 1 Worker, ozaki2", "ms": t, "tflops": flops / t / 1e9})
+        wp = [{"DGEMM_VARIANT": "ozaki2"}] + [{"DGEMM_VARIANT": "dmma"}] * (len(args.sm) - 1)
+        sp = [args.mixed] + [s / min(args.sm[1:]) for s in args.sm[1:]]
+        desc = pdl.partition_descriptor_xml(args.sm, speeds=sp, worker_props=wp)
+        t, st = timed(desc, A, B, C, None, args.reps, args.tile)
+        err = float(((C - ref).abs() / (A.abs() @ B.abs())).max())
+        rows.append({"mapping": f"per-Worker variants (ozaki2 | dmma), weighted {sp}", "ms": t,
+                     "tflops": flops / t / 1e9, "max_scaled_diff_vs_dmma": err,
+                     "worker_kernel_ms": [round(w["kernel_ms"], 2) for w in st["workers"]],
+                     "sm": [w["sm_limit"] for w in st["workers"]]})
     out = {"n": n, "dtype": args.dtype, "partitions": args.sm, "rows": rows}
     print(json.dumps(out))
     print(f"\n| mapping ({args.dtype} {n}^3, SMs {args.sm}) | ms | TFLOP/s | per-Worker kernel ms | tiles |")
