@@ -140,43 +140,52 @@ __global__ void oz_colmax_kernel(const T *__restrict__ B, int64_t ldb, int64_t K
 }
 
 // B (K x N) -> Bt8 (N rows of [c][S-1-s][kk]) through a shared tile stored
-// transposed (32 n rows x 64 k, pitch 66 doubles): coalesced loads along n, then
-// each thread slices 8 consecutive k of one column read as four 16-byte shared
-// loads (conflict-free per quarter-warp) -> one 8-byte store per slice.
+// transposed (32 n rows x KT k, pitch KT + 2 doubles): coalesced loads along n,
+// then each thread slices KG groups of 8 consecutive k of one column, read as
+// 16-byte shared loads (conflict-free per quarter-warp) -> one 8-byte store per
+// slice and group.  KT = 64 for FP64 inputs, 128 for FP32 (twice the work per CTA
+// for the half-size elements).
 template <typename T>
 __global__ void __launch_bounds__(256) oz_split_cols_t_kernel(
     const T *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int S, int64_t Kc, int nch,
     const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
     int rn) {
-    constexpr int PITCH = 66;
+    constexpr int KG = sizeof(T) == 4 ? 2 : 1, KT = 64 * KG, PITCH = KT + 2;
     __shared__ __align__(16) double t[32 * PITCH];
-    const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
+    const int64_t k0 = (int64_t)blockIdx.y * KT, n0 = (int64_t)blockIdx.x * 32;
     const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;   // 32 x 8
-    for (int r = ty; r < 64; r += 8) {
+#pragma unroll
+    for (int r = ty; r < KT; r += 8) {
         const int64_t k = k0 + r, n = n0 + tx;
         t[tx * PITCH + r] = (k < K && n < N) ? (double)B[k * ldb + n] : 0.0;
     }
     __syncthreads();
     const int64_t Kpad = (int64_t)nch * Kc;
     const int nl = threadIdx.x >> 3, g = threadIdx.x & 7;    // column, group of 8 k
-    const int64_t n = n0 + nl, k8 = k0 + 8 * g;
-    if (n >= N || k8 >= Kpad) return;
+    const int64_t n = n0 + nl;
+    if (n >= N) return;
     const int f = exp_of_max(__longlong_as_double((long long)bmax[n]), rn);
     if (blockIdx.y == 0 && g == 0) fb[n] = f;
-    double v[8];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const double2 x = *reinterpret_cast<const double2 *>(&t[nl * PITCH + 8 * g + 2 * j]);
-        v[2 * j] = ldexp_fast(x.x, -f);
-        v[2 * j + 1] = ldexp_fast(x.y, -f);
-    }
-    const int64_t c = k8 / Kc, kk = k8 - c * Kc;
-    int8_t *o = Bt8 + n * ld8 + (c * S) * Kc + kk;
-    for (int s = 0; s < S; ++s) {
-        uint64_t pk = 0;
+    for (int u = 0; u < KG; ++u) {
+        const int gl = g + 8 * u;                            // group within the tile
+        const int64_t k8 = k0 + 8 * gl;
+        if (k8 >= Kpad) break;
+        double v[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) pk |= (uint64_t)(uint8_t)slice_q(v[j], rn) << (8 * j);
-        *reinterpret_cast<uint64_t *>(o + (int64_t)(S - 1 - s) * Kc) = pk;
+        for (int j = 0; j < 4; ++j) {
+            const double2 x = *reinterpret_cast<const double2 *>(&t[nl * PITCH + 8 * gl + 2 * j]);
+            v[2 * j] = ldexp_fast(x.x, -f);
+            v[2 * j + 1] = ldexp_fast(x.y, -f);
+        }
+        const int64_t c = k8 / Kc, kk = k8 - c * Kc;
+        int8_t *o = Bt8 + n * ld8 + (c * S) * Kc + kk;
+        for (int s = 0; s < S; ++s) {
+            uint64_t pk = 0;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) pk |= (uint64_t)(uint8_t)slice_q(v[j], rn) << (8 * j);
+            *reinterpret_cast<uint64_t *>(o + (int64_t)(S - 1 - s) * Kc) = pk;
+        }
     }
 }
 
@@ -679,7 +688,8 @@ static cudaError_t split_b_impl(const T *B, int64_t ldb, int64_t K, int64_t cols
         oz_colmax_kernel<T><<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
     }
     const int64_t Kpad = (int64_t)L.nch * L.Kc;
-    dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 63) / 64));
+    const int64_t kt = sizeof(T) == 4 ? 128 : 64;   // k rows per CTA (oz_split_cols_t_kernel KT)
+    dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + kt - 1) / kt));
     oz_split_cols_t_kernel<T><<<g2, 256, 0, s>>>(B, ldb, K, cols, L.S, L.Kc, L.nch, bmax, Bt8, L.ld8, fb, L.rn);
     return cudaGetLastError();
 }
