@@ -146,11 +146,27 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             CP = (int)std::min<int64_t>(2, std::max<int64_t>(1, (cols + 127) / 128));
         }
     }
+    // tuning overrides of the cut counts (PDL_PIPE_RB / PDL_PIPE_CP)
+    if (RB * CP > 1 || force) {
+        if (const char *e = getenv("PDL_PIPE_RB")) RB = std::max(1, atoi(e));
+        if (const char *e = getenv("PDL_PIPE_CP")) CP = std::max(1, atoi(e));
+    }
     std::vector<int64_t> rb(RB + 1), cp(CP + 1);
     for (int i = 0; i <= RB; ++i) rb[i] = std::min<int64_t>(rows, round_up((int64_t)i * rows / RB, 128));
     for (int j = 0; j <= CP; ++j) cp[j] = std::min<int64_t>(cols, round_up((int64_t)j * cols / CP, 128));
     rb[RB] = rows;
     cp[CP] = cols;
+    // PDL_PIPE_FIRST=f: the first row band is 1/f of the others (the first kernel waits
+    // for less staging; the rest of the rows spread over the remaining bands)
+    if (RB > 1) {
+        if (const char *e = getenv("PDL_PIPE_FIRST")) {
+            const int f = std::max(1, atoi(e));
+            const int64_t first = std::max<int64_t>(128, round_up(rows / RB / f, 128));
+            rb[1] = std::min<int64_t>(rows, first);
+            for (int i = 2; i < RB; ++i)
+                rb[i] = std::min<int64_t>(rows, round_up(first + (int64_t)(i - 1) * (rows - first) / (RB - 1), 128));
+        }
+    }
     const bool piped = RB * CP > 1;
     int rc;
     if (piped && (rc = ensure_aux(w))) return rc;
