@@ -172,6 +172,23 @@ def test_wide_exponent_rows_columns():
     check(oz2_matmul(A, B), A, B)
 
 
+def test_scaling_bits_above_50_residue_fallback():
+    """14 moduli at K <= 128 give p = 51 > 50: |A'| may reach 2^51, beyond the
+    one-DFMA residue path's exactness bound, so K7 takes the four-op residue path
+    with fix-ups (k_ozaki2.cu res8); both sides of the bound stay within the bar."""
+    import json
+    pdl.load(pdl.descriptor_xml(1))
+    try:
+        assert json.loads(pdl.query("ozaki2_plan/100/43/14"))["p"] == 51
+        assert json.loads(pdl.query("ozaki2_plan/300/43/14"))["p"] == 50
+    finally:
+        pdl.unload()
+    for K in (100, 300):
+        A = W.signed((96, K), np.float64, 51) * np.exp2(np.arange(96) % 7 - 3)[:, None]
+        B = W.uniform((K, 80), np.float64, 52)
+        check(oz2_matmul(A, B, moduli=14), A, B, tol=1e-15)
+
+
 @pytest.mark.parametrize("moduli,tol", [(13, 1e-13), (14, 1e-14), (11, 1e-9)])
 def test_moduli_count_accuracy(moduli, tol):
     """Fewer moduli force fewer scaling bits p (|X| <= K 2^(2p) < M/2)."""
