@@ -101,6 +101,16 @@ extern "C" {
  *   share a device, and get disjoint partitions (the device is split into groups
  *   of gcd(n_i) SMs; PDL_EINVAL when the device cannot supply enough groups or
  *   the sum exceeds its SMs).  This emulates heterogeneous Workers on one GPU.
+ * Task variants (one task interface, several implementations pre-selected per
+ *   Worker from its properties): DGEMM_VARIANT = dmma
+ *   (default: K1, IEEE FP64 on DMMA) | ozaki (K4/K5, OZAKI_SLICES, default 6,
+ *   OZAKI_ROUNDING nearest | trunc) | ozaki2 (K6/K7, OZAKI2_MODULI, default
+ *   the fewest giving OZAKI2_BITS = 43 scaling bits); SGEMM_VARIANT = 3xtf32
+ *   (default: K3 + K2) | ozaki (OZAKI_SLICES_F32, default 3).  The Ozaki
+ *   variants assume finite inputs and meet the 1e-12 / 1e-5 bars for rows and
+ *   columns of moderate dynamic range (R19, R20).  RELATIVE_SPEED
+ *   weights the BLOCK mapping.  Env PDL_<PROPERTY> overrides a property for
+ *   every Worker.
  * This process is the single Master driving every Worker of the descriptor.
  * Env: PDL_DRY_RUN=1 skips device binding (plans only; no device work);
  *   PDL_ALLOW_OVERSUBSCRIBE=1 lets several Workers share a device.
@@ -220,7 +230,9 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group,
  *   "interconnects" (JSON), "exchange_path[/<group>]" ("direct" when every
  *   pair of the group's gpu Workers is joined by an Interconnect, else "host":
  *   the transfer path the multi-rank exchange takes, L1336-1341),
- *   "ozaki2_plan/<K>[/<bits>[/<moduli>]]" (JSON; no pdl_load needed).
+ *   "ozaki2_plan/<K>[/<bits>[/<moduli>]]" (JSON; no pdl_load needed: moduli,
+ *   scaling bits p, K chunks, CRT weights W_t and M as decimal strings, and
+ *   "crt": "fp64" when the FP64-pipe reconstruction applies, else "int").
  * Writes a NUL-terminated string (truncated to len-1) and returns the full
  * length, or a negative code (PDL_EINVAL for an unknown key).
  */
