@@ -35,16 +35,28 @@
 namespace pdlk {
 
 namespace k1 {
-constexpr int BM = 128, BN = 128, BK = 16, STAGES = 4;
-constexpr int A_BYTES = BM * BK * 8;   // 16 KiB
-constexpr int B_BYTES = BK * BN * 8;   // 16 KiB, as BN/16 sub-boxes of 16 x 16 doubles
-constexpr int B_SUB_BYTES = BK * 16 * 8;
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int NCONS = 8;               // DMMA warps; thread 0 also issues the TMA loads
-constexpr int THREADS = NCONS * 32;    // 256: keeps the 255-register budget per thread
+// Two CTA shapes with the same warp tile (64 x 32) and the same per-element
+// summation order, so they give bitwise the same C (pin P7): 128 x 128 (eight
+// DMMA warps, one CTA per SM) and, for grids too small to fill the 148 SMs,
+// 64 x 128 (four warps, two CTAs per SM).
+template <int BM_>
+struct Shape {
+    static constexpr int BM = BM_, BN = 128, BK = 16, STAGES = 4;
+    static constexpr int A_BYTES = BM * BK * 8;   // 16 KiB (BM 128) / 8 KiB (BM 64)
+    static constexpr int B_BYTES = BK * BN * 8;   // 16 KiB, as BN/16 sub-boxes of 16 x 16 doubles
+    static constexpr int B_SUB_BYTES = BK * 16 * 8;
+    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+    static constexpr int NCONS = BM / 16;          // DMMA warps (2 or 1 warp rows x 4); thread 0 also issues TMA
+    static constexpr int THREADS = NCONS * 32;     // keeps the 255-register budget per thread
+    static constexpr int MIN_CTAS = 128 / BM;      // CTAs per SM
+    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 2 * STAGES * 8 + 1024;
+};
 constexpr int GROUP_M = 8;             // tile rows per raster group (ncu sweep: 8 -> least DRAM traffic)
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 2 * STAGES * 8 + 1024;
 }  // namespace k1
+
+// Rate of a 64-row CTA relative to the 128-row CTA's per-SM rate: alone on an
+// SM (four DMMA warps) and two per SM (measured, tools/k1_shape_sweep.py).
+constexpr double K1_E1 = 0.69, K1_E2 = 0.93;
 
 // 128B-swizzled byte offset of (row, 8-byte column j in [0,16)) inside a
 // buffer of 128-byte rows whose base is 1024-byte aligned.
@@ -62,11 +74,14 @@ __device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b)
                  : "d"(a), "d"(b));
 }
 
-__global__ void __launch_bounds__(k1::THREADS, 1)
+template <int BM_>
+__global__ void __launch_bounds__(k1::Shape<BM_>::THREADS, k1::Shape<BM_>::MIN_CTAS)
     dgemm_k1_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     double *__restrict__ C, int64_t ldc, int M, int N, int K, int tiles_m, int tiles_n,
                     int group_m, int vec_ok, int *dyn_next, int *dyn_mine) {
-    using namespace k1;
+    using S = k1::Shape<BM_>;
+    constexpr int BM = S::BM, BN = S::BN, BK = S::BK, STAGES = S::STAGES, NCONS = S::NCONS;
+    constexpr int A_BYTES = S::A_BYTES, B_SUB_BYTES = S::B_SUB_BYTES, STAGE_BYTES = S::STAGE_BYTES;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
     const uint32_t bar_full = base + STAGES * STAGE_BYTES;
@@ -128,7 +143,7 @@ __global__ void __launch_bounds__(k1::THREADS, 1)
     // (columns 2j and 2j+1).  The k order per 16-wide block is
     // {0,4,10,14},{1,5,11,15},{2,6,8,12},{3,7,9,13}; with the 128B swizzle every
     // quarter-warp of every ld.shared.v2.f64 hits 8 distinct bank groups.
-    const int wm = warp >> 2, wn = warp & 3;   // 2 x 4 warps, warp tile 64 x 32
+    const int wm = warp >> 2, wn = warp & 3;   // (BM / 64) x 4 warps, warp tile 64 x 32
     const uint32_t g4 = (uint32_t)lane >> 2;   // groupID (MMA row / B column pair)
     const uint32_t p = (uint32_t)lane & 3u;    // thread in group (MMA k index)
     const uint32_t cA = (0x7520u >> (4u * p)) & 0xFu;
@@ -240,38 +255,75 @@ static bool make_map_2d(EncodeTiledFn enc, CUtensorMap *m, CUtensorMapDataType d
     return r == CUDA_SUCCESS;
 }
 
-int k1_smem_bytes() { return k1::SMEM_BYTES; }
+int k1_smem_bytes() { return k1::Shape<128>::SMEM_BYTES; }
+
+// CTA rows for a grid of M x N, from a wave model with W = the time of one
+// 128 x 128 tile on an SM: 128-row grid ceil(t128 / sms) W; 64-row grid
+// W / (2 K1_E1) when every CTA has an SM to itself, else ceil(t64 / 2 sms)
+// waves of two co-resident CTAs at K1_E2 of the 128-row rate.  Constants from
+// tools/k1_shape_sweep.py on the B200 (profiles/r01_k1_shape_sweep.jsonl).
+// DYNAMIC keeps 128 x 128 tiles: every Worker claims from one tile grid.
+static int k1_pick_bm(int64_t M, int64_t N, int sms, bool dynamic) {
+    const char *f = getenv("PDL_K1_BM");   // measurement knob: force 64 or 128
+    if (f && (atoi(f) == 64 || atoi(f) == 128)) return atoi(f);
+    if (dynamic || sms <= 0) return 128;
+    const int64_t tn = (N + 127) / 128;
+    const int64_t t128 = (M + 127) / 128 * tn, t64 = (M + 63) / 64 * tn;
+    const double w128 = (double)((t128 + sms - 1) / sms);
+    const double w64 =
+        t64 <= sms ? 0.5 / K1_E1 : (double)((t64 + 2 * sms - 1) / (2 * sms)) / K1_E2;
+    return w64 < w128 ? 64 : 128;
+}
+
+template <int BM_>
+static cudaError_t launch_k1_shape(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
+                                   double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, int dev,
+                                   cudaStream_t stream, int *dyn_next, int *dyn_mine) {
+    using S = k1::Shape<BM_>;
+    CUtensorMap ta, tb;
+    if (!make_map_2d(enc, &ta, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 8, A, (uint64_t)K, (uint64_t)M, (uint64_t)lda, S::BK,
+                     S::BM, CU_TENSOR_MAP_SWIZZLE_128B))
+        return cudaErrorInvalidValue;
+    if (!make_map_2d(enc, &tb, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 8, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, 16,
+                     S::BK, CU_TENSOR_MAP_SWIZZLE_128B))
+        return cudaErrorInvalidValue;
+    static bool attr_done[64] = {false};
+    if (dev < 64 && !attr_done[dev]) {
+        cudaError_t e =
+            cudaFuncSetAttribute(dgemm_k1_kernel<BM_>, cudaFuncAttributeMaxDynamicSharedMemorySize, S::SMEM_BYTES);
+        if (e != cudaSuccess) return e;
+        attr_done[dev] = true;
+    }
+    const int tiles_m = (int)((M + S::BM - 1) / S::BM), tiles_n = (int)((N + S::BN - 1) / S::BN);
+    const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
+    const char *gm = getenv("PDL_GROUP_M_K1");   // raster tuning knob
+    const int group_m = gm && atoi(gm) > 0 ? atoi(gm) : k1::GROUP_M * (128 / BM_);
+    dgemm_k1_kernel<BM_><<<tiles_m * tiles_n, S::THREADS, S::SMEM_BYTES, stream>>>(
+        ta, tb, C, ldc, (int)M, (int)N, (int)K, tiles_m, tiles_n, group_m, vec_ok, dyn_next, dyn_mine);
+    return cudaGetLastError();
+}
 
 // Host launcher.  A: rows x K (lda), B: K x cols (ldb), both device-resident,
 // 16 B aligned base, lda*8 and ldb*8 multiples of 16 (checked by the runtime).
 cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
                             double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream,
                             int *dyn_next, int *dyn_mine) {
-    using namespace k1;
     if (M <= 0 || N <= 0) return cudaSuccess;
-    CUtensorMap ta, tb;
-    if (!make_map_2d(enc, &ta, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 8, A, (uint64_t)K, (uint64_t)M, (uint64_t)lda, BK, BM,
-                     CU_TENSOR_MAP_SWIZZLE_128B))
-        return cudaErrorInvalidValue;
-    if (!make_map_2d(enc, &tb, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 8, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, 16, BK,
-                     CU_TENSOR_MAP_SWIZZLE_128B))
-        return cudaErrorInvalidValue;
-    int dev = 0;
+    int dev = 0, sms = 0;
     cudaGetDevice(&dev);
-    static bool attr_done[64] = {false};
-    if (dev < 64 && !attr_done[dev]) {
-        cudaError_t e = cudaFuncSetAttribute(dgemm_k1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
-        if (e != cudaSuccess) return e;
-        attr_done[dev] = true;
-    }
-    const int tiles_m = (int)((M + BM - 1) / BM), tiles_n = (int)((N + BN - 1) / BN);
-    const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
-    const char *gm = getenv("PDL_GROUP_M_K1");   // raster tuning knob
-    const int group_m = gm && atoi(gm) > 0 ? atoi(gm) : GROUP_M;
-    dgemm_k1_kernel<<<tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(ta, tb, C, ldc, (int)M, (int)N, (int)K,
-                                                                        tiles_m, tiles_n, group_m, vec_ok, dyn_next,
-                                                                        dyn_mine);
-    return cudaGetLastError();
+    static int sm_count[64] = {0};
+    if (dev < 64 && !sm_count[dev]) cudaDeviceGetAttribute(&sm_count[dev], cudaDevAttrMultiProcessorCount, dev);
+    if (dev < 64) sms = sm_count[dev];
+    if (k1_pick_bm(M, N, sms, dyn_next != nullptr) == 64)
+        return launch_k1_shape<64>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine);
+    return launch_k1_shape<128>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine);
+}
+
+int k1_cta_rows(int64_t M, int64_t N, int dynamic) {
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return k1_pick_bm(M, N, sms, dynamic != 0);
 }
 
 }  // namespace pdlk

@@ -117,6 +117,20 @@ bool worker_sgemm_ozaki2(const WorkerCtx &w) {
     return lower(trim(v)) == "ozaki2";
 }
 
+// K2 shape for an nr x nc launch: the 1-SM 128 x 128 kernel when the CTA-pair
+// grid of 256 x 256 tiles leaves TPCs idle, from a wave model with W = one pair
+// tile's time: pairs ceil(p / (sms/2)) W, 1-SM ceil(t1 / sms) W / (2 e), e = the
+// 1-SM kernel's per-SM rate relative to the pair's (0.8 measured at 4096^3 --
+// 8192^3, tools/k1_shape_sweep.py f32; profiles/r01_k2_shape_sweep.jsonl).  Both
+// give bitwise the same C (same K chunks and MMA order).
+static bool k2_pick_1sm(int64_t nr, int64_t nc, int sms) {
+    if (sms < 2) return false;
+    const int64_t p = ((nr + 255) / 256) * ((nc + 255) / 256), t1 = ((nr + 127) / 128) * ((nc + 127) / 128);
+    const double w2 = (double)((p + sms / 2 - 1) / (sms / 2));
+    const double w1 = (double)((t1 + sms - 1) / sms) / (2 * 0.8);
+    return w1 < w2;
+}
+
 int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
     if (rows <= 0 || cols <= 0) return PDL_OK;
     CUDA_TRY(cudaSetDevice(w.device));
@@ -226,8 +240,9 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     }
     pdlk::EncodeTiledFn enc = nullptr;
     if (K > 0 && (rc = get_encoder(&enc))) return rc;
-    const char *k2v = getenv("PDL_K2");
-    const bool k2_1sm = k2v && !strcmp(k2v, "1sm");
+    const char *k2v = getenv("PDL_K2");   // measurement knob: force "1sm" or "2sm"
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, w.device);
 
     pdlk::OzakiLayout OL;
     int8_t *a8 = nullptr, *b8 = nullptr;
@@ -445,7 +460,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 }
                 if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
                 if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
-                if (k2_1sm)
+                if (k2v ? !strcmp(k2v, "1sm") : k2_pick_1sm(nr, nc, sms))
                     e = pdlk::launch_gemm_3xtf32(enc, ahi + r0 * Kp, alo + r0 * Kp, bhi + c0 * Kp, blo + c0 * Kp, Kp,
                                                  (float *)Cs, ldcd, nr, nc, cs);
                 else
