@@ -228,7 +228,8 @@ def ozaki2_moduli(K, bits=43):
 def ozaki2_ops(rows, cols, K):
     n, p, nch, kc = ozaki2_moduli(K)
     ops = 2.0 * rows * cols * kc * nch * n
-    return ops, f"K6 oz_gemm_2sm_kernel<uint8> x {n * nch} residue GEMMs (tcgen05 kind::i8, p = {p}) + CRT pass"
+    return ops, (f"K6 oz2_gemm_persistent_kernel: {n * nch} residue GEMMs in {nch} persistent launch(es) "
+                 f"(tcgen05 kind::i8, p = {p}) + CRT pass")
 
 
 def variant_ops(variant, rows, cols, K, S):

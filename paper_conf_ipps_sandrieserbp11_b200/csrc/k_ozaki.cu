@@ -473,18 +473,29 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, OCC>:
     }
 }
 
-// K6, persistent: one CTA pair per TPC walks the residue GEMM's cluster tiles
-// (tile = cluster, cluster + clusters, ...).  Barriers and TMEM are set up once; the
-// producer runs ahead into the next tile while the epilogue drains the accumulator,
-// and the MMA warp starts the next tile as soon as both CTAs' epilogue warps have
-// read TMEM (bar_tempty on the leader, 2 x EPI_WARPS arrivals), so only the TMEM
-// read -- not the prologue, pipeline fill, residue arithmetic and stores -- sits
-// between two tiles' MMAs.  Epilogue as oz_gemm_2sm_kernel<NSUB, uint8_t>.
+// K6, persistent: one CTA pair per TPC walks the work items (modulus t, cluster
+// tile) of all nmod residue GEMMs of a K chunk, modulus-major (item = cluster,
+// cluster + clusters, ...), so the last partial round of tiles is paid once per
+// K chunk instead of once per modulus.  The operands of modulus t are the K
+// columns [t Kd, (t+1) Kd) of the tensor maps (the residues of a row are
+// contiguous per modulus), its residues go to plane t of R.  Barriers and TMEM
+// are set up once; the producer runs ahead into the next item while the
+// epilogue drains the accumulator, and the MMA warp starts the next item as soon
+// as both CTAs' epilogue warps have read TMEM (bar_tempty on the leader, 2 x
+// EPI_WARPS arrivals), so only the TMEM read -- not the prologue, pipeline fill,
+// residue arithmetic and stores -- sits between two items' MMAs.  Epilogue as
+// oz_gemm_2sm_kernel<NSUB, uint8_t>.
+struct Oz2Moduli {
+    int m[OZ2_MAX_MODULI];
+    unsigned magic[OZ2_MAX_MODULI];   // ceil(2^39 / m): exact division-by-constant multiplier
+};
+
 template <int NSUB>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::THREADS, 1)
     oz2_gemm_persistent_kernel(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB,
-                               uint8_t *__restrict__ R, int64_t ldr, int M, int N, int Kd, int tiles_m,
-                               int tiles_n, int group_m, int modulus, unsigned mod_magic, int hints) {
+                               uint8_t *__restrict__ R, int64_t ldr, int64_t plane, int M, int N, int Kd,
+                               int tiles_m, int tiles_n, int group_m, int nmod, const __grid_constant__ Oz2Moduli mods,
+                               int hints) {
     using namespace koz;
     using CF = Cfg<NSUB, 1>;
     constexpr int BN = CF::BN, STAGES = CF::STAGES, STAGE_BYTES = CF::STAGE_BYTES;
@@ -502,6 +513,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t rank = cluster_ctarank();
     const int ntiles = tiles_m * tiles_n, nclusters = (int)(gridDim.x >> 1), cl = (int)(blockIdx.x >> 1);
+    const int nitems = nmod * ntiles;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
@@ -531,7 +543,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
             // B strips (read by one wave of the group) evict_first
             const uint64_t pol_a = l2_policy_evict_last(), pol_b = l2_policy_evict_first();
             uint32_t it = 0;
-            for (int tile = cl; tile < ntiles; tile += nclusters) {
+            for (int item = cl; item < nitems; item += nclusters) {
+                const int t = item / ntiles, tile = item - t * ntiles;
                 int tm, tn;
                 raster_tile(tile, tiles_m, tiles_n, group_m, &tm, &tn);
                 const int m0 = tm * (2 * BM) + (int)rank * BM;
@@ -539,14 +552,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
                 // hints & 4: odd rounds of tiles walk K backwards, so a round starts on the
                 // K blocks of the (shared) A strips the previous round touched last and
                 // still finds them in L2 (integer sums: the order does not change a bit)
-                const bool rev = (hints & 4) && (((tile / nclusters) & 1) != 0);
+                const bool rev = (hints & 4) && (((item / nclusters) & 1) != 0);
                 for (int kb = 0; kb < nk; ++kb, ++it) {
                     const uint32_t s = it % STAGES, ph = (it / STAGES) & 1u;
                     mbar_wait(bar_empty + 8 * s, ph ^ 1u);
                     const uint32_t fb_leader = mapa_shared(bar_full + 8 * s, 0);
                     if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * STAGE_BYTES);
                     const uint32_t st = base + s * STAGE_BYTES;
-                    const int kx = (rev ? nk - 1 - kb : kb) * BK;
+                    const int kx = t * Kd + (rev ? nk - 1 - kb : kb) * BK;
                     if (hints & 1) {
                         tma_load_2d_2sm_hint(st, &tA, fb_leader, kx, m0, pol_a);
 #pragma unroll
@@ -565,7 +578,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
         if (rank == 0 && lane == 0) {
             constexpr uint32_t idesc = idesc_i8(2 * BM, BN1);
             uint32_t it = 0, ti = 0;
-            for (int tile = cl; tile < ntiles; tile += nclusters, ++ti) {
+            for (int item = cl; item < nitems; item += nclusters, ++ti) {
                 mbar_wait(bar_tempty, (ti & 1u) ^ 1u);   // both CTAs' epilogues have read TMEM
                 asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
                 for (int kb = 0; kb < nk; ++kb, ++it) {
@@ -594,14 +607,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
         const int cg = e >> 2;
         const uint32_t tl = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(cg * EPI_COLS);
         const uint32_t tempty_leader = mapa_shared(bar_tempty, 0);
-        const uint32_t mm = (uint32_t)modulus, bias = mm * ((1u << 30) / mm + 1u);
         uint32_t ti = 0;
-        for (int tile = cl; tile < ntiles; tile += nclusters, ++ti) {
+        for (int item = cl; item < nitems; item += nclusters, ++ti) {
+            const int t = item / ntiles, tile = item - t * ntiles;
+            const uint32_t mm = (uint32_t)mods.m[t], bias = mm * ((1u << 30) / mm + 1u);
+            const unsigned mod_magic = mods.magic[t];
             int tm, tn;
             raster_tile(tile, tiles_m, tiles_n, group_m, &tm, &tn);
             const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
             const int cbase = tn * BN + cg * EPI_COLS;
-            uint8_t *prow = R + (int64_t)row * ldr + cbase;
+            uint8_t *prow = R + (int64_t)t * plane + (int64_t)row * ldr + cbase;
             mbar_wait(bar_tfull, ti & 1u);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #pragma unroll 1
@@ -876,7 +891,14 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
     if ((reinterpret_cast<uintptr_t>(R) & 15u) || (ldr & 15) || (plane & 15)) return cudaErrorInvalidValue;
     cudaError_t e0 = oz_set_attrs<uint8_t>();
     if (e0 != cudaSuccess) return e0;
-    const int shape = oz_shape(rows, cols);
+    // persistent 256 x 512 tiles by default, small grids included: the moduli of a
+    // launch fill the rounds (PDL_OZ2_PERSIST=0: one cluster per tile, shape by
+    // oz_shape); 256 x 256 for N <= 256
+    int shape = cols > 256 ? 0 : 1;
+    {
+        const char *pe0 = getenv("PDL_OZ2_PERSIST");
+        if ((pe0 && !strcmp(pe0, "0")) || getenv("PDL_OZ_SHAPE") || getenv("PDL_OZ_NSUB")) shape = oz_shape(rows, cols);
+    }
     // persistent 256 x 512 tiles by default (PDL_OZ2_PERSIST=0: one cluster per tile)
     const char *pe = getenv("PDL_OZ2_PERSIST");
     const bool persist = shape == 0 && !(pe && !strcmp(pe, "0"));
@@ -887,7 +909,62 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
         e0 = oz2_persistent_clusters(&pclusters);
         if (e0 != cudaSuccess) return e0;
     }
-    for (int c = 0; c < P.nch; ++c) {
+    // Moduli per persistent launch.  A launch walks the tiles of a group of moduli
+    // (modulus-major), so a small rectangle (a multi-GPU chunk: < 1 round of
+    // tiles per modulus) pays the idle tail of a last round once per launch
+    // instead of once per modulus.  Long launches lose L2 locality: at C4 (28
+    // rounds per modulus) one launch for all 13 moduli read 2x the DRAM bytes (L2
+    // hit 73 -> 62 %: the clusters drift apart over 360 rounds and the live
+    // strips spread) and the power-capped clock fell 10 %.  So: the fewest
+    // launches nl with at most kOz2MaxRounds rounds each that minimise the idle
+    // rounds sum_l (ceil(r_l) - r_l), moduli spread evenly.  PDL_OZ2_MERGE = g
+    // forces groups of about g moduli (1: one launch per modulus).
+    constexpr double kOz2MaxRounds = 24.0;
+    using CF2 = Cfg<2, 1>;
+    const int tiles_m2 = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n2 = (int)((cols + CF2::BN - 1) / CF2::BN);
+    int nl = P.n;
+    if (persist) {
+        const double rmod = (double)tiles_m2 * tiles_n2 / std::max(1, pclusters);   // rounds per modulus
+        double best = 1e30;
+        for (int L = std::max(1, (int)std::ceil(rmod * P.n / kOz2MaxRounds - 1e-9)); L <= P.n; ++L) {
+            double idle = 0.0;
+            for (int l = 0; l < L; ++l) {
+                const double r = rmod * ((l + 1) * P.n / L - l * P.n / L);
+                idle += std::ceil(r - 1e-9) - r;
+            }
+            if (idle < best - 1e-6) {
+                best = idle;
+                nl = L;
+            }
+        }
+        if (const char *me = getenv("PDL_OZ2_MERGE")) nl = (P.n + std::max(1, atoi(me)) - 1) / std::max(1, atoi(me));
+        nl = std::max(1, std::min(P.n, nl));
+    }
+    const bool merge = persist && nl < P.n;
+    for (int c = 0; c < P.nch && merge; ++c) {
+        for (int l = 0; l < nl; ++l) {
+            const int t0 = l * P.n / nl, t1 = (l + 1) * P.n / nl, gl = t1 - t0;
+            const int64_t off = ((int64_t)c * P.n + t0) * P.Kc;
+            CUtensorMap ta, tb;
+            if (!map_i8(enc, &ta, A8 + off, (uint64_t)(gl * P.Kc), (uint64_t)rows, (uint64_t)P.ld8, BM) ||
+                !map_i8(enc, &tb, Bt8 + off, (uint64_t)(gl * P.Kc), (uint64_t)cols, (uint64_t)P.ld8, BNH))
+                return cudaErrorInvalidValue;
+            Oz2Moduli mods = {};
+            for (int t = 0; t < gl; ++t) {
+                const unsigned m = (unsigned)P.m[t0 + t];
+                mods.m[t] = (int)m;
+                mods.magic[t] = (unsigned)((((unsigned long long)1 << 39) + m - 1) / m);
+            }
+            const int ncl = std::min(gl * tiles_m2 * tiles_n2, pclusters);
+            oz2_gemm_persistent_kernel<2><<<2 * ncl, CF2::THREADS, CF2::SMEM_BYTES, stream>>>(
+                ta, tb, R + ((int64_t)c * P.n + t0) * plane, ldr, plane, (int)rows, (int)cols, (int)P.Kc, tiles_m2,
+                tiles_n2, group_for_k(P.Kc), gl, mods, hints);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return e;
+            if (launches) ++*launches;
+        }
+    }
+    for (int c = 0; c < P.nch && !merge; ++c) {
         for (int t = 0; t < P.n; ++t) {
             const int64_t off = ((int64_t)c * P.n + t) * P.Kc;
             CUtensorMap ta, tb;
@@ -901,9 +978,12 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
                 using CF = Cfg<2, 1>;
                 const int tiles_m = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((cols + CF::BN - 1) / CF::BN);
                 const int ncl = std::min(tiles_m * tiles_n, pclusters);
+                Oz2Moduli one = {};
+                one.m[0] = P.m[t];
+                one.magic[0] = magic;
                 oz2_gemm_persistent_kernel<2><<<2 * ncl, CF::THREADS, CF::SMEM_BYTES, stream>>>(
-                    ta, tb, Rp, ldr, (int)rows, (int)cols, (int)P.Kc, tiles_m, tiles_n, group_for_k(P.Kc), P.m[t],
-                    magic, hints);
+                    ta, tb, Rp, ldr, plane, (int)rows, (int)cols, (int)P.Kc, tiles_m, tiles_n, group_for_k(P.Kc), 1,
+                    one, hints);
             } else {
                 oz_launch<uint8_t>(shape, ta, tb, Rp, ldr, rows, cols, P.Kc, nullptr, nullptr, 0, 0, 1, P.m[t], magic,
                                    stream);

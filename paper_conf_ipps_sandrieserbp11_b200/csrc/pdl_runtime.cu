@@ -355,6 +355,19 @@ int pdl_query(const char *key, char *out, size_t len) {
                 for (size_t j = i + 1; j < gw.size() && direct; ++j) direct = m.ic_between(gw[i], gw[j], "");
             res = direct ? "direct" : "host";
         }
+        else if (k == "concurrent_tasks/f64" || k == "concurrent_tasks/f32") {
+            // whether two tasks on device-resident operands may run at once on
+            // different streams of a local Worker: only task variants that use no
+            // Worker scratch buffers (FP64 DMMA, K1) qualify; the FP32 split and
+            // the Ozaki slices / residues live in per-Worker buffers
+            bool yes = k == "concurrent_tasks/f64" && !g->workers.empty();
+            for (auto &w : g->workers) {
+                int s = 0, rn = 0, nm = 0, bits = 0;
+                if (!yes) break;
+                yes = !worker_ozaki(w, true, &s, &rn) && !worker_ozaki2(w, &nm, &bits);
+            }
+            res = yes ? "yes" : "no";
+        }
         else if (k == "plan") res = g->plan_json;
         else if (k == "groups") {
             std::vector<std::string> gs;

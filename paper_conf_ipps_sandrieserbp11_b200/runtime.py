@@ -192,7 +192,7 @@ def chunk_rows(wp: WorkerPlan, j):
     return lo, min(lo + wp.qa, wp.rows)
 
 
-def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers, compute):
+def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers, compute, concurrent=None):
     """Exchange with the A transfer overlapped by compute.
 
     The B column-panel is all-gathered first (every C row needs it).  The A
@@ -202,7 +202,8 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
     the chunks after it, each group as one launch once its broadcasts have
     landed (the stream waits on the NCCL work, the host does not), so the
     other (Gc-1)/Gc of the A traffic hides behind the own-chunk kernel.
-    Results are bitwise identical to the non-overlapped path (R14)."""
+    Results are bitwise identical to the non-overlapped path (R14).
+    concurrent: see compute_groups (None = ask libpdl)."""
     if wp.Gr > 1:
         _all_gather(bufs.B, Bch, grid.col_group)
     else:
@@ -214,24 +215,91 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
     if wp.Gc > 1:
         for j in range(wp.Gc):   # same order on every rank of the row
             works[j] = _broadcast(bufs.A[j * qa:(j + 1) * qa], grid.row_ranks[j], grid.row_group)
-    # Compute in at most three launches so each stays wave-efficient: the own
-    # chunk at once, then the chunks before it (broadcast first, so they land
-    # first), then the chunks after it.
-    groups = [[c], list(range(0, c)), list(range(c + 1, wp.Gc))]
-    first = True
-    for grp in groups:
-        if not grp:
-            continue
-        for j in grp:
-            if j != c and j in works:
-                works[j].wait()
-        lo, hi = chunk_rows(wp, grp[0])[0], chunk_rows(wp, grp[-1])[1]
-        if hi > lo and wp.cols > 0:
-            compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first)
-            first = False
+    compute_groups(wp, bufs, Bp, compute, works, concurrent)
     for w in works.values():
         w.wait()
     return bufs.A[: wp.rows], Bp
+
+
+_side_streams = {}
+
+
+def _side_stream(i):
+    dev = torch.cuda.current_device()
+    if (dev, i) not in _side_streams:
+        _side_streams[(dev, i)] = torch.cuda.Stream(device=dev)
+    return _side_streams[(dev, i)]
+
+
+def tasks_may_overlap(*panels) -> bool:
+    """Whether two tasks on these device panels may run on different streams of
+    the Worker at once, i.e. neither touches a Worker scratch buffer: libpdl
+    answers "yes" for task variants without one (FP64 DMMA, K1), and K1 stages
+    nothing when every operand is on the Worker's device, 16-byte aligned, with
+    16-byte row pitches."""
+    dt = panels[0].dtype
+    key = "concurrent_tasks/" + ("f64" if dt == torch.float64 else "f32")
+    if not all(t.is_cuda for t in panels):
+        return False
+    dev = torch.cuda.current_device()
+    for t in panels:
+        es = t.element_size()
+        if not t.is_cuda or t.device.index != dev or t.data_ptr() % 16 or (t.stride(0) * es) % 16:
+            return False
+    return pdl.query(key) == "yes"
+
+
+def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concurrent=None):
+    """The chunk computations of exchange_overlapped, in at most three launches
+    so each stays wave-efficient: the own chunk at once, then the chunks before
+    it (broadcast first, so they land first), then the chunks after it.
+    works: chunk -> broadcast handle (absent = already resident).
+
+    concurrent (default: tasks_may_overlap(A panel, B panel)): the
+    later groups go on side streams that wait only for their own broadcasts, so
+    their CTAs fill the SMs the previous launch leaves idle in its last wave
+    (three serial launches each round up to whole waves); the Worker stream
+    joins them before returning.  C regions are disjoint, so C is bitwise the
+    serial result."""
+    c = wp.c
+    if concurrent is None:
+        concurrent = tasks_may_overlap(bufs.A, Bp)
+    main = torch.cuda.current_stream() if concurrent else None
+    groups = [[c], list(range(0, c)), list(range(c + 1, wp.Gc))]
+    first = True
+    joins = []
+    if concurrent:
+        ready = torch.cuda.Event()
+        ready.record(main)   # everything the chunks need (B panel, own chunk) is enqueued
+    for grp in groups:
+        if not grp:
+            continue
+        lo, hi = chunk_rows(wp, grp[0])[0], chunk_rows(wp, grp[-1])[1]
+        if hi <= lo or wp.cols <= 0:
+            continue
+        if first or not concurrent:
+            for j in grp:
+                if j != c and j in works:
+                    works[j].wait()
+            compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first)
+        else:
+            side = _side_stream(len(joins))
+            side.wait_event(ready)
+            with torch.cuda.stream(side):
+                for j in grp:
+                    if j in works:
+                        works[j].wait()
+                pdl.set_stream(side)
+                try:
+                    compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first)
+                finally:
+                    pdl.set_stream(main)
+                done = torch.cuda.Event()
+                done.record(side)
+            joins.append(done)
+        first = False
+    for ev in joins:
+        main.wait_event(ev)
 
 
 def chunk_task(Cblock, wp: WorkerPlan, tile=0):

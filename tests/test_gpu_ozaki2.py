@@ -62,10 +62,11 @@ def check(C, A, B, rows=None, tol=1e-12):
     return float(err.max())
 
 
-def test_variant_selected_and_launch_count():
+def test_variant_selected_and_launch_count(monkeypatch):
     """13 moduli at the default 43 scaling bits for K <= 16384: A residues
     (row max, residues) + B residues (column max, residues) + 13 residue GEMMs
-    + the CRT pass."""
+    (one launch each with PDL_OZ2_MERGE=1) + the CRT pass."""
+    monkeypatch.setenv("PDL_OZ2_MERGE", "1")
     pdl.load(pdl.descriptor_xml(1, props={"DGEMM_VARIANT": "ozaki2"}))
     assert pdl.query("worker/0/DGEMM_VARIANT") == "ozaki2"
     A = W.uniform((300, 200), np.float64, 1)
@@ -140,6 +141,8 @@ def test_gemm_shapes_and_crt_passes_bitwise(monkeypatch):
     """The residue GEMMs are exact INT32 sums and the CRT is exact, so the K6
     kernel shape (persistent 256 x 512 -- the default for this size, >= 148
     cluster tiles --, one cluster per tile, 256 x 256, two CTA pairs per SM),
+    the moduli per persistent launch (default 4 here: 2.2 rounds of tiles per
+    modulus; 1, 5 and all 13 forced),
     and the serpentine-K / cache-hint knobs change no bit; ragged edges in both
     dimensions.  The 128-bit integer CRT pass rounds X twice (high and low words),
     the FP64 pass once, so those agree to 2 ulps."""
@@ -149,7 +152,8 @@ def test_gemm_shapes_and_crt_passes_bitwise(monkeypatch):
     rows = [0, 1, 255, 256, 4095, 4999] + list(np.random.default_rng(3).integers(0, 5000, 24))
     check(ref, A, B, rows=rows)
     for env in ({"PDL_OZ2_PERSIST": "0"}, {"PDL_OZ_SHAPE": "256"}, {"PDL_OZ_SHAPE": "256x2"},
-                {"PDL_OZ2_HINTS": "7"}):
+                {"PDL_OZ2_HINTS": "7"}, {"PDL_OZ2_MERGE": "1"}, {"PDL_OZ2_MERGE": "5"},
+                {"PDL_OZ2_MERGE": "13"}):
         with monkeypatch.context() as mp:
             for k, v in env.items():
                 mp.setenv(k, v)

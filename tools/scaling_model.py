@@ -1,8 +1,11 @@
 """Strong-scaling model of the multi-Worker path (NVLink scaling is not
 measurable with one GPU per gpurun call; this predicts it from measured parts).
 
-Per Worker (plan from libpdl, dry run): compute time = its FLOPs / the measured
-single-B200 rate of the task variant (profiles/r01_bench_table.jsonl, C4);
+Per Worker (plan from libpdl, dry run): compute time = the measured time of the
+Worker's own chunk launches on one B200 where tools/worker_emulate.py has it
+(profiles/r01_worker_emulate_*.jsonl: the worst Worker position, launch grouping
+and wave quantisation included), else its FLOPs / the measured single-B200 rate
+of the task variant (profiles/r01_bench_table.jsonl, C4);
 exchange = B column-panel all-gather (exposed) + A-chunk broadcasts overlapped
 with the chunk kernels (exposed only if a chunk transfer outlasts the previous
 chunk's compute).  NVLink: 770 GB/s per direction per GPU (the measured peer
@@ -33,14 +36,29 @@ def rates():
     return r
 
 
-def model(M, N, K, tile, G, rate, es):
+def emulated():
+    """(dtype, variant, G) -> measured worst-Worker compute seconds."""
+    out = {}
+    for fn in sorted(os.listdir(os.path.join(ROOT, "profiles"))):
+        if fn.startswith("r01_worker_emulate_") and fn.endswith(".jsonl"):
+            with open(os.path.join(ROOT, "profiles", fn)) as f:
+                for line in f:
+                    d = json.loads(line)
+                    if "G" in d:
+                        var = {"default": "dmma" if d["dtype"] == "f64" else "3xtf32"}.get(
+                            d.get("variant", "default"), d.get("variant"))
+                        out[(d["dtype"], var, d["G"])] = d["max_concurrent_ms"] / 1e3
+    return out
+
+
+def model(M, N, K, tile, G, rate, es, t_meas=None):
     pdl.unload()
     pdl.load(pdl.descriptor_path(G))
     worst = 0.0
     for w in range(G):
         p = pdl.plan(M, N, K, tile, worker=w)
         rows, cols = p["row1"] - p["row0"], p["col1"] - p["col0"]
-        t_comp = 2.0 * rows * cols * K / rate
+        t_comp = t_meas if t_meas is not None else 2.0 * rows * cols * K / rate
         b_bytes = K * cols * es * (1 - 1 / p["Gr"])            # received B chunks
         a_chunk = p["qa"] * K * es                              # one A chunk
         t_b = b_bytes / NVLINK
@@ -54,12 +72,14 @@ def model(M, N, K, tile, G, rate, es):
 
 def main():
     r = rates()
+    em = emulated()
     M = N = K = 16384
     rows = ["| variant | G=1 ms | G=2 | G=4 | G=8 | predicted S_8 |", "|---|---|---|---|---|---|"]
     for (dt, var), rate in sorted(r.items()):
         es = 8 if dt == "f64" else 4
-        ts = [model(M, N, K, 1024, G, rate, es) for G in (1, 2, 4, 8)]
-        rows.append(f"| {dt} {var} | {ts[0] * 1e3:.1f} | {ts[1] * 1e3:.1f} | {ts[2] * 1e3:.1f} | "
+        ts = [model(M, N, K, 1024, G, rate, es, em.get((dt, var, G))) for G in (1, 2, 4, 8)]
+        src = "measured" if all((dt, var, G) in em for G in (1, 2, 4, 8)) else "rate"
+        rows.append(f"| {dt} {var} ({src}) | {ts[0] * 1e3:.1f} | {ts[1] * 1e3:.1f} | {ts[2] * 1e3:.1f} | "
                     f"{ts[3] * 1e3:.1f} | {ts[0] / ts[3]:.2f} |")
     print("\n".join(rows))
 

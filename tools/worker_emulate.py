@@ -1,0 +1,117 @@
+"""Per-Worker compute time of the multi-GPU C4 step, measured on one B200.
+
+For G = 1, 2, 4, 8 Workers, every distinct Worker position c in its grid row
+(the launch grouping of runtime.compute_groups depends on c) runs exactly the
+chunk launches of runtime.exchange_overlapped on its own panels -- the
+rectangle, chunk sizes and launch groups of libpdl's plan for that Worker --
+with the panels already resident (the NVLink exchange is modelled separately
+in tools/scaling_model.py).  Serial launches on the Worker stream and
+runtime.compute_groups' own choice (side streams where libpdl reports the task
+variant scratch-free, else serial) are both timed with CUDA events (median of
+`--reps`), and C is compared bitwise.
+
+    python tools/worker_emulate.py [--dtype f64] [--config C4] [--reps 3]
+"""
+import argparse
+import json
+import os
+import sys
+
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import workloads as W  # noqa: E402
+from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime  # noqa: E402
+
+
+def plans(M, N, K, tile, G):
+    os.environ["PDL_ALLOW_OVERSUBSCRIBE"] = "1"
+    os.environ["PDL_DRY_RUN"] = "1"
+    pdl.load(pdl.descriptor_path(G))
+    try:
+        return [runtime.worker_plan(M, N, K, tile, r) for r in range(G)]
+    finally:
+        pdl.unload()
+        os.environ.pop("PDL_DRY_RUN", None)
+
+
+def time_worker(wp, dt, tile, concurrent, reps):
+    dev = torch.device("cuda", torch.cuda.current_device())
+    g = torch.Generator(device="cuda").manual_seed(11)
+    bufs = runtime.PanelBuffers(wp, dt, dev)
+    bufs.A.uniform_(generator=g)
+    bufs.B.uniform_(generator=g)
+    Bp = bufs.B[: wp.K]
+    C = torch.full((wp.rows, wp.cols), float("nan"), dtype=dt, device=dev)
+    compute = runtime.chunk_task(C, wp, tile=tile)
+    main = torch.cuda.current_stream()
+    pdl.set_stream(main)
+    for _ in range(2):
+        runtime.compute_groups(wp, bufs, Bp, compute, {}, concurrent)
+    pdl.sync()
+    torch.cuda.synchronize()
+    ms = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(main)
+        runtime.compute_groups(wp, bufs, Bp, compute, {}, concurrent)
+        e1.record(main)
+        pdl.sync()
+        torch.cuda.synchronize()
+        ms.append(e0.elapsed_time(e1))
+    ms.sort()
+    return ms[len(ms) // 2], C
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--dtype", choices=("f64", "f32"), default="f64")
+    ap.add_argument("--config", default="C4")
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--gs", default="1,2,4,8")
+    ap.add_argument("--variant", default=None, help="task variant (PDL_DGEMM_VARIANT / PDL_SGEMM_VARIANT)")
+    args = ap.parse_args()
+    if args.variant:
+        os.environ["PDL_DGEMM_VARIANT" if args.dtype == "f64" else "PDL_SGEMM_VARIANT"] = args.variant
+    c = W.CONFIGS[args.config]
+    dt = torch.float64 if args.dtype == "f64" else torch.float32
+    out = []
+    for G in [int(x) for x in args.gs.split(",")]:
+        wps = plans(c.M, c.N, c.K, c.tile, G)
+        pdl.load(pdl.descriptor_path(1))
+        try:
+            seen = set()
+            rows = []
+            for wp in wps:
+                key = (wp.c, wp.rows, wp.cols)
+                if key in seen:
+                    continue
+                seen.add(key)
+                t_ser, C_ser = time_worker(wp, dt, c.tile, False, args.reps)
+                C_ser = C_ser.clone()
+                t_con, C_con = time_worker(wp, dt, c.tile, None, args.reps)   # libpdl decides
+                flops = 2.0 * wp.rows * wp.cols * wp.K
+                rows.append({"c": wp.c, "rect": [wp.rows, wp.cols], "qa": wp.qa, "serial_ms": round(t_ser, 3),
+                             "concurrent_ms": round(t_con, 3), "bitwise": bool(torch.equal(C_ser, C_con)),
+                             "concurrent_tflops": round(flops / t_con / 1e9, 1)})
+                del C_ser, C_con
+                torch.cuda.empty_cache()
+        finally:
+            pdl.unload()
+        r = {"config": args.config, "dtype": args.dtype, "variant": args.variant or "default", "G": G, "grid": [wps[0].Gr, wps[0].Gc],
+             "max_serial_ms": max(x["serial_ms"] for x in rows),
+             "max_concurrent_ms": max(x["concurrent_ms"] for x in rows), "workers": rows}
+        print(json.dumps(r), flush=True)
+        out.append(r)
+    t1 = out[0]["max_concurrent_ms"] if out[0]["G"] == 1 else None
+    if t1:
+        for r in out:
+            r["compute_speedup_serial"] = round(t1 / r["max_serial_ms"], 2)
+            r["compute_speedup_concurrent"] = round(t1 / r["max_concurrent_ms"], 2)
+        print(json.dumps({"speedups": {r["G"]: [r["compute_speedup_serial"], r["compute_speedup_concurrent"]]
+                                       for r in out}}))
+
+
+if __name__ == "__main__":
+    main()
