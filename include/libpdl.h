@@ -82,6 +82,16 @@ extern "C" {
                                 of this Worker: reuse its prepared form (FP32 split / Ozaki
                                 slices) instead of recomputing it; ignored when no matching
                                 prepared B exists */
+#define PDL_TASK_SLOT(s) (((unsigned)(s) & 3u) << 4)
+                             /* scratch slot s in 0..2 of the Worker: a task's own buffers (A
+                                split / slices / residues and exponents, residue planes,
+                                staging) exist once per slot, so tasks of different slots with
+                                device-resident, 16-byte aligned operands may run at once on
+                                different streams (pdl_set_stream between them); the prepared
+                                B (PDL_TASK_REUSE_B) is shared and a reusing task on another
+                                stream waits for its preparation.  Slot 3 -> PDL_EINVAL.
+                                pdl_query("concurrent_tasks/f64"|"concurrent_tasks/f32") says
+                                whether the loaded Workers support it ("yes") */
 
 /*
  * pdl_load -- parse a PDL descriptor and build the machine model.

@@ -117,6 +117,27 @@ bool worker_sgemm_ozaki2(const WorkerCtx &w) {
     return lower(trim(v)) == "ozaki2";
 }
 
+// Ozaki exponent arrays of a task: the B side [bmax: cols u64][fb: cols int] in the
+// shared BUF_OZE of slot 0 (it does not move with `rows`, so a prepared B survives
+// row-chunk tasks, REUSE_B), the A side ea (rows int) after it for slot 0, in the
+// slot's own BUF_OZE otherwise.
+static int oz_exponents(WorkerCtx &w, int slot, int64_t rows, int64_t cols, unsigned long long **bmax, int **fb,
+                        int **ea) {
+    void *p = nullptr, *q = nullptr;
+    const size_t bside = (size_t)round_up(cols, 2) * 4 + (size_t)cols * 8;
+    int rc = ensure_buf(w, BUF_OZE, bside + (slot == 0 ? (size_t)round_up(rows, 2) * 4 : 0), &p);
+    if (rc) return rc;
+    *bmax = (unsigned long long *)p;
+    *fb = (int *)(*bmax + cols);
+    if (slot == 0) {
+        *ea = *fb + round_up(cols, 2);
+        return PDL_OK;
+    }
+    if ((rc = ensure_buf(w, slot_buf(BUF_OZE, slot), (size_t)round_up(rows, 2) * 4, &q))) return rc;
+    *ea = (int *)q;
+    return PDL_OK;
+}
+
 // K2 shape for an nr x nc launch: the 1-SM 128 x 128 kernel when the CTA-pair
 // grid of 256 x 256 tiles leaves TPCs idle, from a wave model with W = one pair
 // tile's time: pairs ceil(p / (sms/2)) W, 1-SM ceil(t1 / sms) W / (2 e), e = the
@@ -134,6 +155,8 @@ static bool k2_pick_1sm(int64_t nr, int64_t nc, int sms) {
 int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
     if (rows <= 0 || cols <= 0) return PDL_OK;
     CUDA_TRY(cudaSetDevice(w.device));
+    const int slot = (int)((t.flags >> 4) & 3u) % kTaskSlots;   // PDL_TASK_SLOT
+    auto ensure = [&](int buf, size_t bytes, void **out) { return ensure_buf(w, slot_buf(buf, slot), bytes, out); };
     const int es = t.dtype == PDL_F64 ? 8 : 4;
     const bool f64 = t.dtype == PDL_F64;
     const int64_t K = t.K;
@@ -202,7 +225,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     void *p;
     if (a_st) {
         lda = round_up(std::max<int64_t>(K, 1), pe);
-        if ((rc = ensure_buf(w, BUF_A, (size_t)(lda * rows * es), &p))) return rc;
+        if ((rc = ensure(BUF_A, (size_t)(lda * rows * es), &p))) return rc;
         Ad = (const char *)p;
     }
     if (b_st) {
@@ -212,7 +235,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     }
     if (c_st) {
         ldcd = round_up(cols, pe);
-        if ((rc = ensure_buf(w, BUF_C, (size_t)(ldcd * rows * es), &p))) return rc;
+        if ((rc = ensure(BUF_C, (size_t)(ldcd * rows * es), &p))) return rc;
         Cd = (char *)p;
     }
     // Task variant of this Worker, pre-selected from its PDL properties (task
@@ -229,9 +252,9 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     const int64_t Kp = round_up(std::max<int64_t>(K, 1), pdlk::K2_BK);
     float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
     if (!f64 && K > 0 && !ozaki) {
-        if ((rc = ensure_buf(w, BUF_AHI, (size_t)(rows * Kp * 4), &p))) return rc;
+        if ((rc = ensure(BUF_AHI, (size_t)(rows * Kp * 4), &p))) return rc;
         ahi = (float *)p;
-        if ((rc = ensure_buf(w, BUF_ALO, (size_t)(rows * Kp * 4), &p))) return rc;
+        if ((rc = ensure(BUF_ALO, (size_t)(rows * Kp * 4), &p))) return rc;
         alo = (float *)p;
         if ((rc = ensure_buf(w, BUF_BHI, (size_t)(cols * Kp * 4), &p))) return rc;
         bhi = (float *)p;
@@ -251,17 +274,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     if (ozaki) {
         OL = pdlk::ozaki_layout(rows, cols, K, oz_slices);
         OL.rn = oz_rn;
-        if ((rc = ensure_buf(w, BUF_OZA, OL.a8_bytes, &p))) return rc;
+        if ((rc = ensure(BUF_OZA, OL.a8_bytes, &p))) return rc;
         a8 = (int8_t *)p;
         if ((rc = ensure_buf(w, BUF_OZB, OL.b8_bytes, &p))) return rc;
         b8 = (int8_t *)p;
-        const size_t eb = (size_t)round_up(rows, 2) * 4 + (size_t)round_up(cols, 2) * 4 + (size_t)cols * 8;
-        if ((rc = ensure_buf(w, BUF_OZE, eb, &p))) return rc;
-        // [bmax: cols u64][fb: cols int][ea: rows int] -- the B-side part does not
-        // move with `rows`, so a prepared B survives row-chunk tasks (REUSE_B)
-        oz_bmax = (unsigned long long *)p;
-        oz_fb = (int *)(oz_bmax + cols);
-        oz_ea = oz_fb + round_up(cols, 2);
+        if ((rc = oz_exponents(w, slot, rows, cols, &oz_bmax, &oz_fb, &oz_ea))) return rc;
     }
 
     pdlk::Ozaki2Plan P2;
@@ -269,18 +286,14 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     int64_t oz2_ldr = 0, oz2_plane = 0;
     if (ozaki2) {
         P2 = pdlk::ozaki2_plan(rows, cols, K, oz2_nmod, oz2_bits);
-        if ((rc = ensure_buf(w, BUF_OZA, P2.a8_bytes, &p))) return rc;
+        if ((rc = ensure(BUF_OZA, P2.a8_bytes, &p))) return rc;
         a8 = (int8_t *)p;
         if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
         b8 = (int8_t *)p;
-        const size_t eb = (size_t)round_up(rows, 2) * 4 + (size_t)round_up(cols, 2) * 4 + (size_t)cols * 8;
-        if ((rc = ensure_buf(w, BUF_OZE, eb, &p))) return rc;
-        oz_bmax = (unsigned long long *)p;
-        oz_fb = (int *)(oz_bmax + cols);
-        oz_ea = oz_fb + round_up(cols, 2);
+        if ((rc = oz_exponents(w, slot, rows, cols, &oz_bmax, &oz_fb, &oz_ea))) return rc;
         oz2_ldr = round_up(cols, 16);
         oz2_plane = oz2_ldr * rows;
-        if ((rc = ensure_buf(w, BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
+        if ((rc = ensure(BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
         oz2_R = (uint8_t *)p;
     }
 
@@ -297,6 +310,14 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     want.rn = ozaki ? OL.rn : ozaki2 ? P2.p : 0;
     const bool prep_b = K > 0 && (ozaki || ozaki2 || !f64);
     const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
+    // a B prepared on another stream (a task of another slot): wait for it
+    if (b_ready && w.ev_bprep) CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_bprep, 0));
+    auto mark_bprep = [&](cudaStream_t st) -> int {
+        if (piped) return PDL_OK;
+        if (!w.ev_bprep && cudaEventCreateWithFlags(&w.ev_bprep, cudaEventDisableTiming) != cudaSuccess)
+            return PDL_ECUDA;
+        return cudaEventRecord(w.ev_bprep, st) == cudaSuccess ? PDL_OK : PDL_ECUDA;
+    };
 
     std::vector<cudaEvent_t> ev_a(RB, nullptr), ev_b(CP, nullptr), ev_sa(RB, nullptr), ev_sb(CP, nullptr);
     cudaEvent_t ev_last_out = nullptr, ev_last_cmp1 = nullptr;
@@ -366,6 +387,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                     e = pdlk::launch_ozaki2_split_b((const double *)(Bd + (size_t)c0 * es), ldb, K, nc, P2,
                                                     b8 + c0 * P2.ld8, oz_fb + c0, oz_bmax + c0, cs);
                     w.launches += 2;
+                    if (e == cudaSuccess && mark_bprep(cs)) return set_err(PDL_ECUDA, "event record failed");
                     if (piped) {
                         ev_sb[j] = ev_get(w, evn);
                         CUDA_TRY(cudaEventRecord(ev_sb[j], cs));
@@ -409,6 +431,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                             : pdlk::launch_ozaki_split_b((const float *)Bp, ldb, K, nc, OL, b8 + c0 * OL.ld8,
                                                          oz_fb + c0, oz_bmax + c0, cs);
                     w.launches += 2;
+                    if (e == cudaSuccess && mark_bprep(cs)) return set_err(PDL_ECUDA, "event record failed");
                     if (piped) {
                         ev_sb[j] = ev_get(w, evn);
                         CUDA_TRY(cudaEventRecord(ev_sb[j], cs));
@@ -451,6 +474,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                     e = pdlk::launch_split_cols_t((const float *)(Bd + (size_t)c0 * es), ldb, K, nc, bhi + c0 * Kp,
                                                   blo + c0 * Kp, Kp, cs);
                     w.launches += 1;
+                    if (e == cudaSuccess && mark_bprep(cs)) return set_err(PDL_ECUDA, "event record failed");
                     if (piped) {
                         ev_sb[j] = ev_get(w, evn);
                         CUDA_TRY(cudaEventRecord(ev_sb[j], cs));

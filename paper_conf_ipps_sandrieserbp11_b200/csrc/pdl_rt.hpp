@@ -43,6 +43,14 @@ struct DevBuf {
 };
 
 enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_OZA, BUF_OZB, BUF_OZE, BUF_OZR, BUF_COUNT };
+// Scratch slots (PDL_TASK_SLOT): the per-task buffers (A staging, C staging, A
+// split / slices / residues, A exponents, residue planes) exist once per slot, so
+// tasks of different slots may run at once on different streams of the Worker;
+// the B-side buffers (the prepared B of PDL_TASK_REUSE_B) are shared.
+constexpr int kTaskSlots = 3;
+inline int slot_buf(int buf, int slot) {
+    return (buf == BUF_B || buf == BUF_BHI || buf == BUF_BLO || buf == BUF_OZB) ? buf : buf + slot * BUF_COUNT;
+}
 
 struct WorkerCtx {
     int pu = -1;         // PU instance index in the model
@@ -55,7 +63,8 @@ struct WorkerCtx {
     int sm_limit = 0;
     CUgreenCtx gctx = nullptr;
     cudaEvent_t ev_legacy = nullptr;   // orders the non-blocking green stream with the legacy stream
-    DevBuf buf[BUF_COUNT];
+    DevBuf buf[BUF_COUNT * kTaskSlots];
+    cudaEvent_t ev_bprep = nullptr;   // after the last B preparation (REUSE_B tasks on other streams wait)
     cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr;   // around the dominant kernel of the last task
     int launches = 0;                               // kernels launched in the last run
     bool timed = false;

@@ -113,8 +113,9 @@ int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, v
     if (M < 0 || N < 0 || K < 0) return set_err(PDL_EINVAL, "negative size M=%lld N=%lld K=%lld", (long long)M,
                                                 (long long)N, (long long)K);
     if (tile < 0) return set_err(PDL_EINVAL, "negative tile %lld", (long long)tile);
-    if (flags & ~(PDL_TASK_PANELS | PDL_TASK_LOCAL | PDL_TASK_REUSE_B | PDL_TASK_GRAPH))
+    if (flags & ~(PDL_TASK_PANELS | PDL_TASK_LOCAL | PDL_TASK_REUSE_B | PDL_TASK_GRAPH | PDL_TASK_SLOT(3)))
         return set_err(PDL_EINVAL, "unknown flags 0x%x", flags);
+    if (((flags >> 4) & 3u) >= 3u) return set_err(PDL_EINVAL, "scratch slot %u out of range (0..2)", (flags >> 4) & 3u);
     if ((flags & PDL_TASK_PANELS) && (flags & PDL_TASK_LOCAL))
         return set_err(PDL_EINVAL, "PDL_TASK_PANELS and PDL_TASK_LOCAL are exclusive");
     DistSpec ds;
@@ -356,17 +357,12 @@ int pdl_query(const char *key, char *out, size_t len) {
             res = direct ? "direct" : "host";
         }
         else if (k == "concurrent_tasks/f64" || k == "concurrent_tasks/f32") {
-            // whether two tasks on device-resident operands may run at once on
-            // different streams of a local Worker: only task variants that use no
-            // Worker scratch buffers (FP64 DMMA, K1) qualify; the FP32 split and
-            // the Ozaki slices / residues live in per-Worker buffers
-            bool yes = k == "concurrent_tasks/f64" && !g->workers.empty();
-            for (auto &w : g->workers) {
-                int s = 0, rn = 0, nm = 0, bits = 0;
-                if (!yes) break;
-                yes = !worker_ozaki(w, true, &s, &rn) && !worker_ozaki2(w, &nm, &bits);
-            }
-            res = yes ? "yes" : "no";
+            // whether two tasks on device-resident, 16-byte aligned operands may
+            // run at once on different streams of a local Worker when they use
+            // different scratch slots (PDL_TASK_SLOT): every task variant keeps its
+            // per-task buffers per slot, and a REUSE_B task waits for the B
+            // preparation on the other stream
+            res = g->workers.empty() ? "no" : "yes";
         }
         else if (k == "plan") res = g->plan_json;
         else if (k == "groups") {

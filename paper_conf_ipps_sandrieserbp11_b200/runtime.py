@@ -232,11 +232,11 @@ def _side_stream(i):
 
 
 def tasks_may_overlap(*panels) -> bool:
-    """Whether two tasks on these device panels may run on different streams of
-    the Worker at once, i.e. neither touches a Worker scratch buffer: libpdl
-    answers "yes" for task variants without one (FP64 DMMA, K1), and K1 stages
-    nothing when every operand is on the Worker's device, 16-byte aligned, with
-    16-byte row pitches."""
+    """Whether tasks on these device panels may run on different streams of the
+    Worker at once: libpdl keeps every task variant's own buffers per scratch
+    slot (PDL_TASK_SLOT; query "concurrent_tasks/<dtype>"), and stages nothing
+    when every operand is on the Worker's device, 16-byte aligned, with 16-byte
+    row pitches."""
     dt = panels[0].dtype
     key = "concurrent_tasks/" + ("f64" if dt == torch.float64 else "f32")
     if not all(t.is_cuda for t in panels):
@@ -256,7 +256,8 @@ def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concu
     works: chunk -> broadcast handle (absent = already resident).
 
     concurrent (default: tasks_may_overlap(A panel, B panel)): the
-    later groups go on side streams that wait only for their own broadcasts, so
+    later groups go on side streams, each with its own scratch slot, that wait
+    only for their own broadcasts (and the B panel libpdl prepared), so
     their CTAs fill the SMs the previous launch leaves idle in its last wave
     (three serial launches each round up to whole waves); the Worker stream
     joins them before returning.  C regions are disjoint, so C is bitwise the
@@ -291,7 +292,7 @@ def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concu
                         works[j].wait()
                 pdl.set_stream(side)
                 try:
-                    compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first)
+                    compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first, slot=len(joins) + 1)
                 finally:
                     pdl.set_stream(main)
                 done = torch.cuda.Event()
@@ -304,11 +305,14 @@ def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concu
 
 def chunk_task(Cblock, wp: WorkerPlan, tile=0):
     """compute() for exchange_overlapped: one PDL_TASK_LOCAL task per A chunk
-    on this process's Worker; the prepared B panel is reused after the first."""
-    def compute(j, lo, hi, Arows, Bp, first):
+    on this process's Worker; the prepared B panel is reused after the first;
+    `slot` is the task's scratch slot (compute_groups gives each concurrent
+    launch group its own)."""
+    def compute(j, lo, hi, Arows, Bp, first, slot=0):
         Cv = Cblock[lo:hi]
         pdl.task_matmul(Arows, Bp, Cv, M=hi - lo, N=wp.cols, K=wp.K, tile=tile,
-                        lda=Arows.stride(0), ldb=Bp.stride(0), ldc=Cv.stride(0), local=True, reuse_b=not first)
+                        lda=Arows.stride(0), ldb=Bp.stride(0), ldc=Cv.stride(0), local=True, reuse_b=not first,
+                        slot=slot)
         pdl.run_async()
     return compute
 

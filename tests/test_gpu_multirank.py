@@ -55,12 +55,14 @@ def test_distributed_ozaki2_4():
     _run(4, "f64", 777, 513, 1000, 128, "ozaki2")
 
 
-@pytest.mark.parametrize("G", [4, 8])
-def test_concurrent_chunk_groups_bitwise(G):
-    """runtime.compute_groups with the later chunk groups on side streams (the
-    FP64 DMMA path, libpdl "concurrent_tasks/f64" = yes) gives bitwise the
-    serial launches' C for every Worker position of a G-Worker plan, and
-    sampled rows match the oracle; the FP32 task reports no overlap."""
+@pytest.mark.parametrize("G,dt,variant", [(4, "f64", None), (8, "f64", None), (8, "f32", None),
+                                          (8, "f64", "ozaki"), (8, "f64", "ozaki2"), (4, "f32", "ozaki")])
+def test_concurrent_chunk_groups_bitwise(G, dt, variant, monkeypatch):
+    """runtime.compute_groups with the later chunk groups on side streams, each
+    task in its own libpdl scratch slot (PDL_TASK_SLOT) and reusing the B panel
+    prepared on the Worker stream, gives bitwise the serial launches' C for
+    every Worker position of a G-Worker plan and every task variant, and sampled
+    rows match the oracle."""
     torch = pytest.importorskip("torch")
     import numpy as np
 
@@ -68,41 +70,44 @@ def test_concurrent_chunk_groups_bitwise(G):
     import oracle
     from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime
 
+    if variant:
+        monkeypatch.setenv("PDL_DGEMM_VARIANT" if dt == "f64" else "PDL_SGEMM_VARIANT", variant)
     M, N, K, tile = 1500, 1100, 260, 128
-    os.environ["PDL_ALLOW_OVERSUBSCRIBE"] = "1"
-    os.environ["PDL_DRY_RUN"] = "1"
+    monkeypatch.setenv("PDL_ALLOW_OVERSUBSCRIBE", "1")
+    monkeypatch.setenv("PDL_DRY_RUN", "1")
     pdl.load(pdl.descriptor_path(G))
     try:
         wps = [runtime.worker_plan(M, N, K, tile, r) for r in range(G)]
     finally:
         pdl.unload()
-        os.environ.pop("PDL_DRY_RUN", None)
+        monkeypatch.delenv("PDL_DRY_RUN")
+    npdt, tdt = (np.float64, torch.float64) if dt == "f64" else (np.float32, torch.float32)
     rng = np.random.default_rng(5)
-    A = rng.uniform(-1, 1, (M, K))
-    B = rng.uniform(-1, 1, (K, N))
+    A = rng.uniform(-1, 1, (M, K)).astype(npdt)
+    B = rng.uniform(-1, 1, (K, N)).astype(npdt)
     dev = torch.device("cuda", 0)
+    tol = 1e-12 if dt == "f64" else 1e-5
     pdl.load(pdl.descriptor_path(1))
     try:
-        f32 = torch.zeros((8, 8), dtype=torch.float32, device=dev)
-        assert not runtime.tasks_may_overlap(f32, f32)
+        assert pdl.query("concurrent_tasks/" + dt) == "yes"
         for wp in wps:
-            bufs = runtime.PanelBuffers(wp, torch.float64, dev)
+            bufs = runtime.PanelBuffers(wp, tdt, dev)
             bufs.A.zero_()
             bufs.A[: wp.rows].copy_(torch.from_numpy(A[wp.row0: wp.row1]))
             bufs.B[: wp.K].copy_(torch.from_numpy(B[:, wp.col0: wp.col1]))
             Bp = bufs.B[: wp.K]
             assert runtime.tasks_may_overlap(bufs.A, Bp)
             out = []
-            for conc in (False, True):
-                C = torch.full((wp.rows, wp.cols), float("nan"), dtype=torch.float64, device=dev)
+            for conc in (False, True, True):
+                C = torch.full((wp.rows, wp.cols), float("nan"), dtype=tdt, device=dev)
                 pdl.set_stream(torch.cuda.current_stream())
                 runtime.compute_groups(wp, bufs, Bp, runtime.chunk_task(C, wp, tile), {}, conc)
                 pdl.sync()
                 torch.cuda.synchronize()
                 out.append(C.cpu().numpy())
-            assert np.array_equal(out[0], out[1]), (wp.r, wp.c)
+            assert np.array_equal(out[0], out[1]) and np.array_equal(out[0], out[2]), (wp.r, wp.c)
             rows = np.arange(0, wp.rows, 97)
             Cref, D = oracle.matmul(A[wp.row0: wp.row1][rows], B[:, wp.col0: wp.col1])
-            assert (oracle.scaled_error(out[1][rows], Cref, D) <= 1e-12).all()
+            assert (oracle.scaled_error(out[1][rows], Cref, D) <= tol).all()
     finally:
         pdl.unload()
