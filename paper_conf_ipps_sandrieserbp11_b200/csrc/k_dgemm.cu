@@ -255,8 +255,6 @@ static bool make_map_2d(EncodeTiledFn enc, CUtensorMap *m, CUtensorMapDataType d
     return r == CUDA_SUCCESS;
 }
 
-int k1_smem_bytes() { return k1::Shape<128>::SMEM_BYTES; }
-
 // CTA rows for a grid of M x N, from a wave model with W = the time of one
 // 128 x 128 tile on an SM: 128-row grid ceil(t128 / sms) W; 64-row grid
 // W / (2 K1_E1) when every CTA has an SM to itself, else ceil(t64 / 2 sms)
@@ -319,11 +317,5 @@ cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, con
     return launch_k1_shape<128>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine);
 }
 
-int k1_cta_rows(int64_t M, int64_t N, int dynamic) {
-    int dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    return k1_pick_bm(M, N, sms, dynamic != 0);
-}
 
 }  // namespace pdlk

@@ -21,10 +21,6 @@ cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, con
                             int *dyn_next = nullptr, int *dyn_mine = nullptr);
 // dyn_next / dyn_mine (K1, K2): DYNAMIC distribution -- CTAs claim raster tiles
 // from the shared counter *dyn_next and count their claims in *dyn_mine.
-int k1_smem_bytes();
-// CTA rows K1 launches for an M x N grid on the current device (64 or 128;
-// both give bitwise the same C).
-int k1_cta_rows(int64_t M, int64_t N, int dynamic);
 
 // K3 -- TF32 hi/lo split pre-pass.  Kp = K rounded up to K2's BK (32).
 //  split_rows:   A (M x K, lda, fp32)  -> Ahi, Alo  (M x Kp, K-major, zero padded)
