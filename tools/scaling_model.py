@@ -44,7 +44,7 @@ def emulated():
             with open(os.path.join(ROOT, "profiles", fn)) as f:
                 for line in f:
                     d = json.loads(line)
-                    if "G" in d:
+                    if "G" in d and d.get("config") == "C4":
                         var = {"default": "dmma" if d["dtype"] == "f64" else "3xtf32"}.get(
                             d.get("variant", "default"), d.get("variant"))
                         out[(d["dtype"], var, d["G"])] = d["max_concurrent_ms"] / 1e3
