@@ -881,6 +881,39 @@ cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t 
     return gemm_impl(enc, A8, Bt8, ea, fb, L, C, ldc, rows, cols, stream, launches);
 }
 
+// Moduli per persistent K6 launch (host arithmetic).  A launch walks the tiles of
+// a group of moduli (modulus-major), so a small rectangle (a multi-GPU chunk: < 1
+// round of tiles per modulus) pays the idle tail of a last round once per launch
+// instead of once per modulus.  Long launches lose L2 locality: at C4 (28 rounds
+// per modulus) one launch for all 13 moduli read 2x the DRAM bytes (L2 hit 73 ->
+// 62 %: the clusters drift apart over 360 rounds and the live strips spread) and
+// the power-capped clock fell 10 %.  So: the fewest launches nl with at most
+// kOz2MaxRounds rounds each (a single modulus may exceed it) that minimise the
+// idle rounds sum_l (ceil(r_l) - r_l),
+// moduli spread evenly (launch l: moduli [l n / nl, (l+1) n / nl)).
+int oz2_launches_per_chunk(int n, int64_t rows, int64_t cols, int clusters) {
+    constexpr double kOz2MaxRounds = 24.0;
+    if (n <= 1 || rows <= 0 || cols <= 0 || clusters <= 0) return std::max(1, n);
+    const int64_t tiles = ((rows + 2 * koz::BM - 1) / (2 * koz::BM)) * ((cols + 511) / 512);
+    const double rmod = (double)tiles / clusters;   // rounds per modulus
+    int nl = n;
+    double best = 1e30;
+    for (int L = 1; L <= n; ++L) {
+        const int gmax = (n + L - 1) / L;   // the largest group of an even spread
+        if (gmax > 1 && gmax * rmod > kOz2MaxRounds + 1e-9) continue;
+        double idle = 0.0;
+        for (int l = 0; l < L; ++l) {
+            const double r = rmod * ((l + 1) * n / L - l * n / L);
+            idle += std::ceil(r - 1e-9) - r;
+        }
+        if (idle < best - 1e-6) {
+            best = idle;
+            nl = L;
+        }
+    }
+    return nl;
+}
+
 // Ozaki-II (K6): one INT8 GEMM per modulus and K chunk, each writing its byte
 // plane of residues (k_ozaki2.cu builds the operands and rebuilds C).
 cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
@@ -909,37 +942,14 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
         e0 = oz2_persistent_clusters(&pclusters);
         if (e0 != cudaSuccess) return e0;
     }
-    // Moduli per persistent launch.  A launch walks the tiles of a group of moduli
-    // (modulus-major), so a small rectangle (a multi-GPU chunk: < 1 round of
-    // tiles per modulus) pays the idle tail of a last round once per launch
-    // instead of once per modulus.  Long launches lose L2 locality: at C4 (28
-    // rounds per modulus) one launch for all 13 moduli read 2x the DRAM bytes (L2
-    // hit 73 -> 62 %: the clusters drift apart over 360 rounds and the live
-    // strips spread) and the power-capped clock fell 10 %.  So: the fewest
-    // launches nl with at most kOz2MaxRounds rounds each that minimise the idle
-    // rounds sum_l (ceil(r_l) - r_l), moduli spread evenly.  PDL_OZ2_MERGE = g
-    // forces groups of about g moduli (1: one launch per modulus).
-    constexpr double kOz2MaxRounds = 24.0;
-    using CF2 = Cfg<2, 1>;
-    const int tiles_m2 = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n2 = (int)((cols + CF2::BN - 1) / CF2::BN);
     int nl = P.n;
     if (persist) {
-        const double rmod = (double)tiles_m2 * tiles_n2 / std::max(1, pclusters);   // rounds per modulus
-        double best = 1e30;
-        for (int L = std::max(1, (int)std::ceil(rmod * P.n / kOz2MaxRounds - 1e-9)); L <= P.n; ++L) {
-            double idle = 0.0;
-            for (int l = 0; l < L; ++l) {
-                const double r = rmod * ((l + 1) * P.n / L - l * P.n / L);
-                idle += std::ceil(r - 1e-9) - r;
-            }
-            if (idle < best - 1e-6) {
-                best = idle;
-                nl = L;
-            }
-        }
+        nl = oz2_launches_per_chunk(P.n, rows, cols, pclusters);
         if (const char *me = getenv("PDL_OZ2_MERGE")) nl = (P.n + std::max(1, atoi(me)) - 1) / std::max(1, atoi(me));
         nl = std::max(1, std::min(P.n, nl));
     }
+    using CF2 = Cfg<2, 1>;
+    const int tiles_m2 = (int)((rows + 2 * BM - 1) / (2 * BM)), tiles_n2 = (int)((cols + CF2::BN - 1) / CF2::BN);
     const bool merge = persist && nl < P.n;
     for (int c = 0; c < P.nch && merge; ++c) {
         for (int l = 0; l < nl; ++l) {

@@ -88,6 +88,9 @@ struct Ozaki2Plan {
 };
 // nmod = 0: the fewest moduli that give p >= bits for this K chunk.
 Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits);
+// Persistent K6 launches per K chunk for n moduli on a rows x cols rectangle with
+// `clusters` co-resident CTA pairs (k_ozaki.cu).
+int oz2_launches_per_chunk(int n, int64_t rows, int64_t cols, int clusters);
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
                                   int8_t *A8, int *ea, cudaStream_t s, int *launches = nullptr);
 cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,

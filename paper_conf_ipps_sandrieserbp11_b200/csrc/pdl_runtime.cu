@@ -334,6 +334,20 @@ int pdl_query(const char *key, char *out, size_t len) {
         o << "],\"M\":\"" << dec(P.Mw[0], P.Mw[1]) << "\",\"crt\":\"" << (pdlk::oz2_crt_fast_ok(P) ? "fp64" : "int")
           << "\"}";
         res = o.str();
+    } else if (k.rfind("ozaki2_launches/", 0) == 0) {
+        // "ozaki2_launches/<rows>/<cols>/<moduli>/<clusters>": persistent K6 launches
+        // per K chunk and the moduli of each (host arithmetic, no device)
+        long long rows = 0, cols = 0;
+        int n = 0, cl = 0;
+        if (sscanf(k.c_str() + 16, "%lld/%lld/%d/%d", &rows, &cols, &n, &cl) != 4 || rows < 0 || cols < 0 || n < 1 ||
+            n > pdlk::OZ2_MAX_MODULI || cl < 1)
+            return set_err(PDL_EINVAL, "bad key '%s' (ozaki2_launches/<rows>/<cols>/<moduli>/<clusters>)", key);
+        const int nl = pdlk::oz2_launches_per_chunk(n, rows, cols, cl);
+        std::ostringstream o;
+        o << "[";
+        for (int l = 0; l < nl; ++l) o << (l ? "," : "") << (l + 1) * n / nl - l * n / nl;
+        o << "]";
+        res = o.str();
     } else {
         int rc = check_loaded();
         if (rc) return rc;

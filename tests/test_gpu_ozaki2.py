@@ -141,8 +141,8 @@ def test_gemm_shapes_and_crt_passes_bitwise(monkeypatch):
     """The residue GEMMs are exact INT32 sums and the CRT is exact, so the K6
     kernel shape (persistent 256 x 512 -- the default for this size, >= 148
     cluster tiles --, one cluster per tile, 256 x 256, two CTA pairs per SM),
-    the moduli per persistent launch (default 4 here: 2.2 rounds of tiles per
-    modulus; 1, 5 and all 13 forced),
+    the moduli per persistent launch (default 6 + 7 here: 2.2 rounds of tiles
+    per modulus; 1, 5 and all 13 forced),
     and the serpentine-K / cache-hint knobs change no bit; ragged edges in both
     dimensions.  The 128-bit integer CRT pass rounds X twice (high and low words),
     the FP64 pass once, so those agree to 2 ulps."""
