@@ -242,7 +242,11 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group,
  *   the transfer path the multi-rank exchange takes, L1336-1341),
  *   "ozaki2_plan/<K>[/<bits>[/<moduli>]]" (JSON; no pdl_load needed: moduli,
  *   scaling bits p, K chunks, CRT weights W_t and M as decimal strings, and
- *   "crt": "fp64" when the FP64-pipe reconstruction applies, else "int").
+ *   "crt": "fp64" when the FP64-pipe reconstruction applies, else "int"),
+ *   "ozaki2_launches/<rows>/<cols>/<moduli>/<clusters>" (JSON list, no pdl_load
+ *   needed: moduli per persistent residue-GEMM launch of one K chunk),
+ *   "concurrent_tasks/f64" | "concurrent_tasks/f32" ("yes" when tasks of
+ *   different PDL_TASK_SLOTs may overlap on different streams).
  * Writes a NUL-terminated string (truncated to len-1) and returns the full
  * length, or a negative code (PDL_EINVAL for an unknown key).
  */
