@@ -37,7 +37,7 @@ __device__ __forceinline__ float tf32_rna(float x) {
 }
 
 __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int64_t M, int64_t K,
-                                  float *__restrict__ hi, float *__restrict__ lo, int64_t Kp) {
+                                  float *__restrict__ hi, float *__restrict__ lo, int64_t Kp, int vec) {
     // one thread per 4 consecutive k of one row (Kp % 4 == 0)
     const int64_t q = Kp >> 2;
     const int64_t total = M * q;
@@ -45,8 +45,13 @@ __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int6
         const int64_t i = t / q, k0 = (t - i * q) << 2;
         const float *src = A + i * lda;
         float v[4], h[4], l[4];
+        if (vec && k0 + 3 < K) {   // 16-byte aligned rows: one LDG.128
+            const float4 x = __ldcs(reinterpret_cast<const float4 *>(src + k0));
+            v[0] = x.x, v[1] = x.y, v[2] = x.z, v[3] = x.w;
+        } else {
 #pragma unroll
-        for (int u = 0; u < 4; ++u) v[u] = (k0 + u < K) ? __ldg(src + k0 + u) : 0.0f;
+            for (int u = 0; u < 4; ++u) v[u] = (k0 + u < K) ? __ldg(src + k0 + u) : 0.0f;
+        }
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
             h[u] = tf32_rna(v[u]);
@@ -57,23 +62,46 @@ __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int6
     }
 }
 
-// B (K x N) -> B^T split (N x Kp); 32 x 32 tiles through shared memory.
-__global__ void split_cols_t_kernel(const float *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
-                                    float *__restrict__ hi, float *__restrict__ lo, int64_t Kp) {
-    __shared__ float t[32][33];
-    const int64_t k0 = (int64_t)blockIdx.y * 32, n0 = (int64_t)blockIdx.x * 32;
-    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
-        const int64_t k = k0 + r, n = n0 + threadIdx.x;
-        t[r][threadIdx.x] = (k < K && n < N) ? __ldg(B + k * ldb + n) : 0.0f;
+// B (K x N) -> B^T split (N x Kp); 64 x 64 tiles through shared memory, 16-byte
+// loads along n and 16-byte stores along k (4 of each per thread).  The 32 x 32
+// scalar version moved 4 KB per CTA with 4-byte accesses and ran at 48 % of HBM
+// (profiles/r01_ncu_prof_k3.json).
+__global__ void __launch_bounds__(256) split_cols_t_kernel(const float *__restrict__ B, int64_t ldb, int64_t K,
+                                                           int64_t N, float *__restrict__ hi, float *__restrict__ lo,
+                                                           int64_t Kp, int vec) {
+    __shared__ float t[64][65];
+    const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 64;
+    const int cq = threadIdx.x & 15, r0 = threadIdx.x >> 4;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int r = r0 + 16 * i;
+        const int64_t k = k0 + r, n = n0 + 4 * cq;
+        float v[4];
+        if (vec && k < K && n + 3 < N) {
+            const float4 x = __ldcs(reinterpret_cast<const float4 *>(B + k * ldb + n));
+            v[0] = x.x, v[1] = x.y, v[2] = x.z, v[3] = x.w;
+        } else {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) v[j] = (k < K && n + j < N) ? __ldg(B + k * ldb + n + j) : 0.0f;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) t[r][4 * cq + j] = v[j];
     }
     __syncthreads();
-    for (int r = threadIdx.y; r < 32; r += blockDim.y) {
-        const int64_t n = n0 + r, k = k0 + threadIdx.x;
-        if (n < N && k < Kp) {
-            const float v = t[threadIdx.x][r];
-            const float h = tf32_rna(v);
-            hi[n * Kp + k] = h;
-            lo[n * Kp + k] = tf32_rna(v - h);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int nr = r0 + 16 * i;
+        const int64_t n = n0 + nr, k = k0 + 4 * cq;
+        if (n < N && k < Kp) {   // Kp % 32 == 0: a group of 4 k is all inside or all outside
+            float h[4], l[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const float v = t[4 * cq + j][nr];
+                h[j] = tf32_rna(v);
+                l[j] = tf32_rna(v - h[j]);
+            }
+            *reinterpret_cast<float4 *>(hi + n * Kp + k) = make_float4(h[0], h[1], h[2], h[3]);
+            *reinterpret_cast<float4 *>(lo + n * Kp + k) = make_float4(l[0], l[1], l[2], l[3]);
         }
     }
 }
@@ -84,15 +112,17 @@ cudaError_t launch_split_rows(const float *A, int64_t lda, int64_t M, int64_t K,
     const int64_t total = M * (Kp >> 2);
     int blocks = (int)((total + 255) / 256);
     if (blocks > 148 * 16) blocks = 148 * 16;
-    split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, M, K, hi, lo, Kp);
+    const int vec = ((reinterpret_cast<uintptr_t>(A) & 15u) == 0 && (lda & 3) == 0) ? 1 : 0;
+    split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, M, K, hi, lo, Kp, vec);
     return cudaGetLastError();
 }
 
 cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t N, float *hi, float *lo, int64_t Kp,
                                 cudaStream_t s) {
     if (N <= 0 || Kp <= 0) return cudaSuccess;
-    dim3 grid((unsigned)((N + 31) / 32), (unsigned)((Kp + 31) / 32));
-    split_cols_t_kernel<<<grid, dim3(32, 8), 0, s>>>(B, ldb, K, N, hi, lo, Kp);
+    dim3 grid((unsigned)((N + 63) / 64), (unsigned)((Kp + 63) / 64));
+    const int vec = ((reinterpret_cast<uintptr_t>(B) & 15u) == 0 && (ldb & 3) == 0) ? 1 : 0;
+    split_cols_t_kernel<<<grid, 256, 0, s>>>(B, ldb, K, N, hi, lo, Kp, vec);
     return cudaGetLastError();
 }
 
