@@ -192,7 +192,35 @@ def chunk_rows(wp: WorkerPlan, j):
     return lo, min(lo + wp.qa, wp.rows)
 
 
-def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers, compute, concurrent=None):
+# NVLink 5 peer bandwidth per direction (the measured peer-copy figure quoted in
+# /opt/skills/guides/B200_PROFILING.md) and the A exchange below which one launch
+# over the whole Worker rectangle beats the chunked overlap: tools/worker_emulate.py
+# (profiles/r01_worker_emulate_single_*.jsonl) measured the chunk launches 0.41-0.46
+# ms slower than one launch for C3 at G = 4 / 8 (host issue of three short tasks
+# outlasts their kernels) against 0.13 / 0.07 ms of A transfer, and 0.03 ms slower
+# for C0 / C5 at G = 8 and C0 at G = 2 against 0.12-0.35 ms.
+NVLINK_BPS = 770e9
+SINGLE_LAUNCH_BELOW_S = 2e-4
+
+
+def a_exchange_seconds(wp: WorkerPlan, elem_bytes: int) -> float:
+    """Time the other Gc - 1 A chunks take over NVLink (what a single launch
+    over the whole rectangle leaves exposed)."""
+    return (wp.Gc - 1) * wp.qa * wp.K * elem_bytes / NVLINK_BPS
+
+
+def overlap_pays(wp: WorkerPlan, elem_bytes: int) -> bool:
+    """Chunked overlap (True) or one launch after the A exchange (False);
+    env PDL_OVERLAP_A = 1 / 0 forces either."""
+    import os
+    f = os.environ.get("PDL_OVERLAP_A")
+    if f in ("0", "1"):
+        return f == "1"
+    return a_exchange_seconds(wp, elem_bytes) >= SINGLE_LAUNCH_BELOW_S
+
+
+def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers, compute, concurrent=None,
+                        overlap_a=None):
     """Exchange with the A transfer overlapped by compute.
 
     The B column-panel is all-gathered first (every C row needs it).  The A
@@ -203,7 +231,9 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
     landed (the stream waits on the NCCL work, the host does not), so the
     other (Gc-1)/Gc of the A traffic hides behind the own-chunk kernel.
     Results are bitwise identical to the non-overlapped path (R14).
-    concurrent: see compute_groups (None = ask libpdl)."""
+    concurrent: see compute_groups (None = ask libpdl).  overlap_a: False =
+    wait for every A chunk, then one compute over the whole rectangle (None =
+    overlap_pays for device panels; host panels always chunk)."""
     if wp.Gr > 1:
         _all_gather(bufs.B, Bch, grid.col_group)
     else:
@@ -215,7 +245,15 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
     if wp.Gc > 1:
         for j in range(wp.Gc):   # same order on every rank of the row
             works[j] = _broadcast(bufs.A[j * qa:(j + 1) * qa], grid.row_ranks[j], grid.row_group)
-    compute_groups(wp, bufs, Bp, compute, works, concurrent)
+    if overlap_a is None:
+        overlap_a = wp.Gc == 1 or not bufs.A.is_cuda or overlap_pays(wp, bufs.A.element_size())
+    if overlap_a:
+        compute_groups(wp, bufs, Bp, compute, works, concurrent)
+    else:
+        for w in works.values():
+            w.wait()
+        if wp.rows > 0 and wp.cols > 0:
+            compute(wp.c, 0, wp.rows, bufs.A[: wp.rows], Bp, True)
     for w in works.values():
         w.wait()
     return bufs.A[: wp.rows], Bp

@@ -24,13 +24,13 @@ def _port():
     return p
 
 
-def _run(world, *args):
+def _run(world, *args, env_extra=None):
     torch = pytest.importorskip("torch")
     backend = "nccl" if torch.cuda.device_count() >= world else "gloo"
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
            "--master-addr=127.0.0.1", f"--master-port={_port()}", os.path.join(ROOT, "tests", "dist_check.py"),
            *[str(a) for a in args[:5]], backend, *[str(a) for a in args[5:]]]
-    env = dict(os.environ, PDL_ALLOW_OVERSUBSCRIBE="1")
+    env = dict(os.environ, PDL_ALLOW_OVERSUBSCRIBE="1", **(env_extra or {}))
     env.pop("PDL_DRY_RUN", None)
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
@@ -43,8 +43,11 @@ def test_distributed_matmul(world, dt):
     _run(world, dt, 1000, 700, 300, 128)
 
 
-def test_distributed_ragged_8():
-    _run(8, "f64", 1000, 700, 300, 64)
+@pytest.mark.parametrize("overlap", ["0", "1"])
+def test_distributed_ragged_8(overlap):
+    """Both A-exchange policies: one launch after the whole exchange (the default
+    at this size) and the chunked overlap (PDL_OVERLAP_A=1)."""
+    _run(8, "f64", 1000, 700, 300, 64, env_extra={"PDL_OVERLAP_A": overlap})
 
 
 def test_distributed_ozaki_4():

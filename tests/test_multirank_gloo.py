@@ -64,6 +64,11 @@ def _worker(rank, world, port, shapes, q):
                 ok_a = ok_a and seen[0][3] and not any(s[3] for s in seen[1:])
                 ok_a = ok_a and (hi_c == lo_c or seen[0][0] == wp.c)
             ok_a = ok_a and sum(s[2] - s[1] for s in seen) == (wp.rows if wp.cols else 0)
+            # single launch after the whole A exchange (overlap_a=False): one call, all rows
+            bufs3 = runtime.PanelBuffers(wp, A.dtype, A.device)
+            seen.clear()
+            runtime.exchange_overlapped(Ach, Bch, wp, grid, bufs3, compute, overlap_a=False)
+            ok_a = ok_a and (seen == ([(wp.c, 0, wp.rows, True)] if wp.rows and wp.cols else []))
             out.append((M, N, K, tile, wp.row0, wp.row1, wp.col0, wp.col1, wp.Gr, wp.Gc, ok_a, ok_b))
         pdl.unload()
         q.put((rank, out, None))

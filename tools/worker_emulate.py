@@ -64,6 +64,39 @@ def time_worker(wp, dt, tile, concurrent, reps):
     return ms[len(ms) // 2], C
 
 
+def time_single(wp, dt, tile, reps):
+    """The Worker's whole rectangle as one task (the non-overlapped exchange:
+    every A chunk landed first)."""
+    dev = torch.device("cuda", torch.cuda.current_device())
+    bufs = runtime.PanelBuffers(wp, dt, dev)
+    bufs.A.uniform_()
+    bufs.B.uniform_()
+    C = torch.empty((wp.rows, wp.cols), dtype=dt, device=dev)
+    Ap, Bp = bufs.A[: wp.rows], bufs.B[: wp.K]
+    main_s = torch.cuda.current_stream()
+    pdl.set_stream(main_s)
+
+    def once():
+        pdl.task_matmul(Ap, Bp, C, M=wp.rows, N=wp.cols, K=wp.K, tile=tile, lda=Ap.stride(0), ldb=Bp.stride(0),
+                        ldc=C.stride(0), local=True)
+        pdl.run_async()
+    for _ in range(2):
+        once()
+    pdl.sync()
+    torch.cuda.synchronize()
+    ms = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(main_s)
+        once()
+        e1.record(main_s)
+        pdl.sync()
+        torch.cuda.synchronize()
+        ms.append(e0.elapsed_time(e1))
+    ms.sort()
+    return ms[len(ms) // 2]
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--dtype", choices=("f64", "f32"), default="f64")
@@ -91,9 +124,11 @@ def main():
                 t_ser, C_ser = time_worker(wp, dt, c.tile, False, args.reps)
                 C_ser = C_ser.clone()
                 t_con, C_con = time_worker(wp, dt, c.tile, None, args.reps)   # libpdl decides
+                t_one = time_single(wp, dt, c.tile, args.reps)
                 flops = 2.0 * wp.rows * wp.cols * wp.K
                 rows.append({"c": wp.c, "rect": [wp.rows, wp.cols], "qa": wp.qa, "serial_ms": round(t_ser, 3),
-                             "concurrent_ms": round(t_con, 3), "bitwise": bool(torch.equal(C_ser, C_con)),
+                             "concurrent_ms": round(t_con, 3), "single_launch_ms": round(t_one, 3),
+                             "bitwise": bool(torch.equal(C_ser, C_con)),
                              "concurrent_tflops": round(flops / t_con / 1e9, 1)})
                 del C_ser, C_con
                 torch.cuda.empty_cache()
@@ -101,7 +136,8 @@ def main():
             pdl.unload()
         r = {"config": args.config, "dtype": args.dtype, "variant": args.variant or "default", "G": G, "grid": [wps[0].Gr, wps[0].Gc],
              "max_serial_ms": max(x["serial_ms"] for x in rows),
-             "max_concurrent_ms": max(x["concurrent_ms"] for x in rows), "workers": rows}
+             "max_concurrent_ms": max(x["concurrent_ms"] for x in rows),
+             "max_single_launch_ms": max(x["single_launch_ms"] for x in rows), "workers": rows}
         print(json.dumps(r), flush=True)
         out.append(r)
     t1 = out[0]["max_concurrent_ms"] if out[0]["G"] == 1 else None
