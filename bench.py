@@ -60,7 +60,7 @@ def parse():
     p.add_argument("--dtype", choices=("f64", "f32"), default="f64")
     p.add_argument("--config", default="C4")
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    p.add_argument("--e2e-steps", type=int, default=3)
+    p.add_argument("--e2e-steps", type=int, default=None, help="default: --steps")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="oracle sample budget")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
@@ -72,8 +72,10 @@ def parse():
     p.add_argument("--slices", type=int, default=None,
                    help="Ozaki slices (default 6 for FP64, 3 for FP32; round-to-nearest)")
     p.add_argument("--no-alt", action="store_true", help="skip timing the other task variants")
-    p.add_argument("--dist-backend", choices=("nccl", "gloo"), default="nccl",
-                   help="gloo only to validate the N>1 flow with ranks sharing one GPU")
+    p.add_argument("--dist-backend", choices=("auto", "nccl", "gloo"), default="auto",
+                   help="auto: NCCL when every rank has its own GPU, else gloo (ranks share GPUs: "
+                        "validates the N>1 flow only)")
+    p.add_argument("--no-f32", action="store_true", help="skip the FP32 3xTF32 leg of the FP64 N=1 line")
     return p.parse_args()
 
 
@@ -225,10 +227,18 @@ def ozaki2_moduli(K, bits=43):
     return n, p, nch, kc
 
 
+# co-resident CTA pairs of the persistent K6 kernel on a B200 (148 SMs, one
+# 2-CTA cluster per SM pair; grid (148, 1, 1) in profiles/r01_launches_oz2.csv)
+OZ2_CLUSTERS = 74
+
+
 def ozaki2_ops(rows, cols, K):
     n, p, nch, kc = ozaki2_moduli(K)
     ops = 2.0 * rows * cols * kc * nch * n
-    return ops, (f"K6 oz2_gemm_persistent_kernel: {n * nch} residue GEMMs in {nch} persistent launch(es) "
+    from paper_conf_ipps_sandrieserbp11_b200 import pdl
+    per_chunk = json.loads(pdl.query(f"ozaki2_launches/{rows}/{cols}/{n}/{OZ2_CLUSTERS}"))
+    return ops, (f"K6 oz2_gemm_persistent_kernel: {n * nch} residue GEMMs ({n} moduli x {nch} K chunk(s)) in "
+                 f"{len(per_chunk) * nch} persistent launch(es) of {per_chunk} moduli "
                  f"(tcgen05 kind::i8, p = {p}) + CRT pass")
 
 
@@ -331,34 +341,115 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def spawn_ranks(args):
+    """`python bench.py --gpus N` with N > 1 and no torchrun environment: start
+    N ranks under torch.distributed.run (one process per GPU, rendezvous on
+    127.0.0.1) with the same arguments; rank 0 prints the JSON line."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd, cwd=ROOT)
+
+
+def setup_dist(args, torch, dist):
+    """Rank / device / process group of this process.  --dist-backend auto:
+    NCCL when every rank has its own GPU, else gloo with the ranks sharing
+    devices (validates the N > 1 flow; its timings are not a scaling number)."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    ndev = torch.cuda.device_count()
+    backend = args.dist_backend
+    if backend == "auto":
+        backend = "nccl" if ndev >= world else "gloo"
+    shared = ndev < world
+    if shared and backend == "nccl":
+        raise SystemExit(f"{world} NCCL ranks need {world} GPUs ({ndev} visible): use --dist-backend gloo")
+    local = local % ndev   # gloo validation: several ranks may share one GPU
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
+    return world, rank, local, dev, backend, shared
+
+
+def device_timed(torch, dist, step, steps, stream, world, dev, local, sync):
+    """K steps bracketed by barrier + synchronize on both sides, CUDA events on
+    the launching stream, nvidia-smi clocks sampled during the region; returns
+    (max-over-ranks ms, clocks)."""
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(steps):
+            step()
+        e1.record(stream)
+        sync()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    ms = e0.elapsed_time(e1)
+    if world > 1:
+        t = torch.tensor([ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    return ms, clk.summary()
+
+
+def k_roofline(ktimes, steps, pipe_flops, peak_dtype, kname, traffic_key, cfg, alg_bytes, rows, cols, dtype, ozaki):
+    """roofline object of the dominant kernel: algorithmic work per step over
+    its device time per step (CUDA events around every launch, summed over the
+    Worker's chunk launches at N > 1)."""
+    kavg = float(np.sum(ktimes)) / steps if ktimes else None
+    peak_tf, peak_src, peak_alt = tensor_peak(peak_dtype)
+    achieved = pipe_flops / (kavg / 1e3) / 1e12 if kavg else None
+    r = {"bound": "tensor", "achieved": round(achieved, 2) if achieved else None,
+         "peak": round(peak_tf, 1), "unit": "TFLOP/s",
+         "frac": round(achieved / peak_tf, 4) if achieved else None,
+         "traffic": ncu_traffic(traffic_key, cfg),
+         "traffic_source": "ncu --set full capture of this kernel (profiles/ncu_traffic.json), per launch",
+         "kernel": kname, "kernel_ms": round(kavg, 3) if kavg else None,
+         "algorithmic_flops_per_launch": pipe_flops,
+         "algorithmic_dram_bytes_per_launch": int(alg_bytes),
+         "edge_waste_pct": edge_waste(rows, cols, dtype, ozaki),
+         "peak_source": peak_src}
+    if peak_alt:
+        r["peak_alt"] = peak_alt
+    return r
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
         return
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args))
     import torch
     import torch.distributed as dist
 
     from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world != args.gpus:
-        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}: launch N>1 with torchrun")
-    if args.dist_backend == "gloo":
-        local = local % torch.cuda.device_count()   # several ranks may share one GPU
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
-    if world > 1:
-        if args.dist_backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
-        else:   # validation of the N>1 flow with several ranks on one GPU (timings meaningless)
-            dist.init_process_group("gloo")
+    world, rank, local, dev, backend, shared = setup_dist(args, torch, dist)
     os.environ.pop("PDL_DRY_RUN", None)
+    if shared:
+        os.environ["PDL_ALLOW_OVERSUBSCRIBE"] = "1"
 
     c = W.CONFIGS[args.config]
     M, N, K = c.M, c.N, c.K
+    e2e_steps = args.e2e_steps or args.steps
     np_dtype = np.float64 if args.dtype == "f64" else np.float32
     tdt = torch.float64 if args.dtype == "f64" else torch.float32
     es = 8 if args.dtype == "f64" else 4
@@ -381,6 +472,10 @@ def main():
     wp = runtime.worker_plan(M, N, K, c.tile, rank)
     flops_total = 2.0 * M * N * K
     flops_worker = 2.0 * wp.rows * wp.cols * K
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
 
     # ---- device-resident operands ----
     if world == 1:
@@ -405,62 +500,29 @@ def main():
             # Worker's own chunk (and each landed chunk) computes
             runtime.exchange_overlapped(Ach, Bch, wp, grid, bufs, compute)
 
-    def barrier():
-        if world > 1:
-            dist.barrier()
-
     for _ in range(args.warmup):
         step()
     pdl.sync()
     torch.cuda.synchronize()
     pdl.kernel_times()   # clear
     launches0 = pdl.query_json("stats")["total_launches"]
-
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
-        barrier()
-        torch.cuda.synchronize()
-        e0.record(stream)
-        for _ in range(args.steps):
-            step()
-        e1.record(stream)
-        torch.cuda.synchronize()
-        barrier()
-    ms_total = e0.elapsed_time(e1)
+    ms_total, clocks = device_timed(torch, dist, step, args.steps, stream, world, dev, local, pdl.sync)
     ktimes = pdl.kernel_times()
     timed_launches = pdl.query_json("stats")["total_launches"] - launches0
-    clocks = clk.summary()
-    if world > 1:
-        t = torch.tensor([ms_total], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_total = float(t.item())
     ms_step = ms_total / args.steps
     value = flops_total * args.steps / (ms_total / 1e3) / 1e9   # GFLOP/s, whole job
 
     # ---- roofline of the dominant kernel (K1, or K2 for FP32) ----
-    # dominant-kernel device time per step (N > 1: summed over the Worker's chunk tasks)
-    kavg = float(np.sum(ktimes)) / args.steps if ktimes else None
-    peak_tf, peak_src, peak_alt = tensor_peak("i8" if ozaki else args.dtype)
+    peak_dtype = "i8" if ozaki else args.dtype
     if ozaki:
         pipe_flops, kname = variant_ops(args.variant, wp.rows, wp.cols, K, args.slices)
     else:
         pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
         kname = "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_2sm_kernel (tcgen05)"
-    achieved_tf = pipe_flops / (kavg / 1e3) / 1e12 if kavg else None
-    roofline = {"bound": "tensor", "achieved": round(achieved_tf, 2) if achieved_tf else None,
-                "peak": round(peak_tf, 1), "unit": "TFLOP/s",
-                "frac": round(achieved_tf / peak_tf, 4) if achieved_tf else None,
-                "traffic": ncu_traffic((args.variant if args.dtype == "f64" else "ozaki32") if ozaki else args.dtype,
-                                       args.config),
-                "kernel": kname,
-                "kernel_ms": round(kavg, 3) if kavg else None,
-                "algorithmic_flops_per_launch": pipe_flops,
-                "algorithmic_dram_bytes_per_launch": int((wp.rows * K + K * wp.cols + wp.rows * wp.cols) * es),
-                "edge_waste_pct": edge_waste(wp.rows, wp.cols, args.dtype, ozaki),
-                "peak_source": peak_src}
-    if peak_alt:
-        roofline["peak_alt"] = peak_alt
+    traffic_key = (args.variant if args.dtype == "f64" else "ozaki32") if ozaki else args.dtype
+    roofline = k_roofline(ktimes, args.steps, pipe_flops, peak_dtype, kname, traffic_key, args.config,
+                          (wp.rows * K + K * wp.cols + wp.rows * wp.cols) * es, wp.rows, wp.cols, args.dtype, ozaki)
+    peak_tf = roofline["peak"]
     if args.dtype == "f32":
         roofline["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
     if ozaki:
@@ -468,7 +530,7 @@ def main():
         roofline["note"] = (f"achieved counts int8 tensor ops ({prods}, 2 ops per MAC); "
                             f"useful {args.dtype.upper()} FLOP = 2MNK")
 
-    # ---- e2e: host pinned operands through the public API ----
+    # ---- e2e: host pinned operands through the public API, --steps steps ----
     e2e = None
     if not args.no_e2e:
         if world == 1:
@@ -497,28 +559,20 @@ def main():
                 hCb.copy_(dC, non_blocking=True)
             h2d = ((a1 - a0) * K + (b1 - b0) * wp.cols) * es
             d2h = wp.rows * wp.cols * es
-        estep()
-        pdl.sync()
-        torch.cuda.synchronize()
-        barrier()
-        t0 = torch.cuda.Event(enable_timing=True)
-        t1 = torch.cuda.Event(enable_timing=True)
-        t0.record(stream)
-        for _ in range(args.e2e_steps):
+
+        def estep_synced():
             estep()
             pdl.sync()
             torch.cuda.synchronize()   # the step's result is on the host
-        t1.record(stream)
-        torch.cuda.synchronize()
+        estep_synced()
         barrier()
-        ems = t0.elapsed_time(t1)
-        if world > 1:
-            t = torch.tensor([ems], device=dev, dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ems = float(t.item())
-        e2e = {"value": round(flops_total * args.e2e_steps / (ems / 1e3) / 1e9, 1), "unit": "GFLOP/s",
+        ems, _ = device_timed(torch, dist, estep_synced, e2e_steps, stream, world, dev, local, pdl.sync)
+        e2e = {"value": round(flops_total * e2e_steps / (ems / 1e3) / 1e9, 1), "unit": "GFLOP/s",
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
-               "ms_per_step": round(ems / args.e2e_steps, 3)}
+               "ms_per_step": round(ems / e2e_steps, 3), "steps": e2e_steps,
+               "api": ("pdl.task_matmul + pdl.run on pinned host A, B, C (C ABI task_matmul_ex/pdl_run)"
+                       if world == 1 else
+                       "per rank: pinned host chunks -> runtime.exchange_overlapped -> pinned host C block")}
         if world == 1:
             del hA, hB, hC
         pdl.kernel_times()
@@ -550,15 +604,7 @@ def main():
         pdl.sync()
         torch.cuda.synchronize()
         pdl.kernel_times()
-        t0 = torch.cuda.Event(enable_timing=True)
-        t1 = torch.cuda.Event(enable_timing=True)
-        with ClockSampler(local) as clk2:
-            t0.record(stream)
-            for _ in range(args.steps):
-                step()
-            t1.record(stream)
-            torch.cuda.synchronize()
-        ams = t0.elapsed_time(t1)
+        ams, aclk = device_timed(torch, dist, step, args.steps, stream, world, dev, local, pdl.sync)
         akt = pdl.kernel_times()
         aops, akname = variant_ops(av, M, N, K, args.slices)
         apeak, apsrc, _ = tensor_peak("i8")
@@ -577,21 +623,28 @@ def main():
                                   "kernel": akname,
                                   "kernel_ms": round(float(np.mean(akt)), 3) if akt else None,
                                   "peak_source": apsrc},
-                     "clocks": clk2.summary()})
+                     "clocks": aclk})
 
+    # ---- FP32 (north star (2)): the tcgen05/TMEM 3xTF32 path K3+K2 on the same config ----
+    f32 = None
+    if world == 1 and args.dtype == "f64" and not args.no_f32:
+        f32 = fp32_leg(args, torch, dist, pdl, stream, dev, local, c)
+
+    # ---- the oracle on the host cores, after the GPU timings (rank 0, every N) ----
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline:
         cpu = cpu_baseline(A, B, args.cpu_seconds)
+    barrier()
 
     if rank == 0:
+        workload = (f"{args.config} {M}x{N}x{K} blocked matmul, task tile {c.tile}, PDL b200_x{world}")
         line = {
             "metric": METRIC, "value": round(value, 1), "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": variant_label(args.variant, args.dtype, args.slices, K)[0] if ozaki else args.dtype,
             "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} ({args.dtype})",
-            "config": {"workload": f"{args.config} {M}x{N}x{K} blocked matmul, task tile {c.tile}, "
-                                   f"PDL b200_x{world}",
+            "config": {"workload": workload,
                        "M": M, "N": N, "K": K, "tile": c.tile, "parallelism": f"block2d {wp.Gr}x{wp.Gc}",
                        "task_variant": (variant_label(args.variant, args.dtype, args.slices, K)[1] if ozaki else
                                         ("dmma (K1)" if args.dtype == "f64" else "3xtf32 (K3+K2)")),
@@ -601,14 +654,71 @@ def main():
             "gpu_launches": int(timed_launches),
             "clocks": clocks,
         }
+        if world > 1:
+            line["config"]["dist_backend"] = backend
+            if shared:
+                line["config"]["note"] = (f"{world} ranks share {torch.cuda.device_count()} GPU(s) over gloo: "
+                                          "validates the N>1 flow, not a scaling measurement")
         if cublas is not None:
             line["cublas_gflops_same_operands"] = cublas
         if alts:
             line["alt_variants"] = alts
+        if f32 is not None:
+            line["f32_3xtf32"] = f32
         print(json.dumps(line), flush=True)
     pdl.unload()
     if world > 1:
         dist.destroy_process_group()
+
+
+def fp32_leg(args, torch, dist, pdl, stream, dev, local, c):
+    """FP32 inputs through the default SGEMM variant (K3 TF32 split + K2 3xTF32
+    tcgen05 CTA-pair kernel), device-resident and end to end, on the same
+    config: the tcgen05/TMEM kernel of north star (2) with a driver-run number."""
+    M, N, K = c.M, c.N, c.K
+    A, B = host_inputs(args.config, np.float32)
+    pdl.unload()
+    pdl.load(pdl.descriptor_xml(1))
+    pdl.set_stream(stream)
+    dA = torch.from_numpy(A).to(dev)
+    dB = torch.from_numpy(B).to(dev)
+    dC = torch.empty((M, N), dtype=torch.float32, device=dev)
+
+    def step():
+        pdl.task_matmul(dA, dB, dC, tile=c.tile)
+        pdl.run_async()
+    for _ in range(max(2, args.warmup)):
+        step()
+    pdl.sync()
+    torch.cuda.synchronize()
+    pdl.kernel_times()
+    ms, clk = device_timed(torch, dist, step, args.steps, stream, 1, dev, local, pdl.sync)
+    kt = pdl.kernel_times()
+    flops = 2.0 * M * N * K
+    roof = k_roofline(kt, args.steps, 3 * flops, "f32", "K2 gemm_3xtf32_2sm_kernel (tcgen05 cta_group::2 kind::tf32)",
+                      "f32", args.config, (M * K + K * N + M * N) * 4, M, N, "f32", False)
+    roof["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
+    out = {"value": round(flops * args.steps / (ms / 1e3) / 1e9, 1), "unit": "GFLOP/s", "dtype": "f32",
+           "ms_per_step": round(ms / args.steps, 3), "task_variant": "3xtf32 (K3+K2)",
+           "parity": "max rel err <= 1e-5 vs oracle (tests/test_gpu_parity.py)",
+           "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} (f32)",
+           "roofline": roof, "clocks": clk}
+    if not args.no_e2e:
+        hA = torch.from_numpy(A).pin_memory()
+        hB = torch.from_numpy(B).pin_memory()
+        hC = torch.empty((M, N), dtype=torch.float32).pin_memory()
+
+        def estep():
+            pdl.task_matmul(hA, hB, hC, tile=c.tile)
+            pdl.run()
+            torch.cuda.synchronize()
+        estep()
+        ems, _ = device_timed(torch, dist, estep, args.steps, stream, 1, dev, local, pdl.sync)
+        out["e2e"] = {"value": round(flops * args.steps / (ems / 1e3) / 1e9, 1), "unit": "GFLOP/s",
+                      "h2d_bytes_per_step": (M * K + K * N) * 4, "d2h_bytes_per_step": M * N * 4,
+                      "ms_per_step": round(ems / args.steps, 3)}
+    del dA, dB, dC
+    return out
 
 
 if __name__ == "__main__":

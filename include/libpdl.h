@@ -205,7 +205,9 @@ int pdl_sync(void);
  * library's own stream, which is a blocking stream, i.e. ordered with the
  * legacy default stream; pass cudaStreamLegacy = (void*)1 for the legacy
  * default stream itself).  Lets a caller order the library with its own
- * stream and time it with its own events.
+ * stream and time it with its own events.  A Worker on an SM partition
+ * (SM_LIMIT, a green context) keeps its partition's stream: each run then
+ * waits for the prior work of `stream` and `stream` waits for the run.
  */
 int pdl_set_stream(int worker, void *stream);
 

@@ -301,17 +301,26 @@ static cudaError_t launch_k1_shape(EncodeTiledFn enc, const double *A, int64_t l
     return cudaGetLastError();
 }
 
+static int g_worker_sms = 0;
+void set_worker_sms(int sms) { g_worker_sms = sms > 0 ? sms : 0; }
+int worker_sms() {
+    if (g_worker_sms > 0) return g_worker_sms;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    static int sm_count[64] = {0};
+    if (dev < 64 && !sm_count[dev]) cudaDeviceGetAttribute(&sm_count[dev], cudaDevAttrMultiProcessorCount, dev);
+    return dev < 64 ? sm_count[dev] : 148;
+}
+
 // Host launcher.  A: rows x K (lda), B: K x cols (ldb), both device-resident,
 // 16 B aligned base, lda*8 and ldb*8 multiples of 16 (checked by the runtime).
 cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
                             double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream,
                             int *dyn_next, int *dyn_mine) {
     if (M <= 0 || N <= 0) return cudaSuccess;
-    int dev = 0, sms = 0;
+    int dev = 0;
     cudaGetDevice(&dev);
-    static int sm_count[64] = {0};
-    if (dev < 64 && !sm_count[dev]) cudaDeviceGetAttribute(&sm_count[dev], cudaDevAttrMultiProcessorCount, dev);
-    if (dev < 64) sms = sm_count[dev];
+    const int sms = worker_sms();
     if (k1_pick_bm(M, N, sms, dyn_next != nullptr) == 64)
         return launch_k1_shape<64>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine);
     return launch_k1_shape<128>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine);

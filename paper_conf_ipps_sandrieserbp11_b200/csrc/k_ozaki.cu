@@ -745,7 +745,7 @@ static bool map_i8(EncodeTiledFn enc, CUtensorMap *m, const int8_t *ptr, uint64_
 static int oz_shape(int64_t rows, int64_t cols) {
     using namespace koz;
     const int64_t clusters512 = ((rows + 2 * BM - 1) / (2 * BM)) * ((cols + 511) / 512);
-    int shape = (cols > 256 && clusters512 >= 148) ? 0 : 1;
+    int shape = (cols > 256 && clusters512 >= worker_sms()) ? 0 : 1;
     if (const char *e = getenv("PDL_OZ_NSUB")) shape = atoi(e) == 1 ? 1 : 0;
     if (const char *e = getenv("PDL_OZ_SHAPE")) {
         if (!strcmp(e, "512")) shape = 0;
@@ -807,6 +807,15 @@ static cudaError_t oz2_persistent_clusters(int *out) {
     if (n < 1) return cudaErrorInvalidConfiguration;
     if (dev < 64) cached[dev] = n;
     *out = n;
+    return cudaSuccess;
+}
+
+// Co-resident CTA pairs for the launching Worker: an SM-partition Worker holds one
+// pair per two of its SMs at most.
+static cudaError_t oz2_worker_clusters(int *out) {
+    cudaError_t e = oz2_persistent_clusters(out);
+    if (e != cudaSuccess) return e;
+    *out = std::max(1, std::min(*out, worker_sms() / 2));
     return cudaSuccess;
 }
 
@@ -939,7 +948,7 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
     const char *he = getenv("PDL_OZ2_HINTS");
     const int hints = he ? atoi(he) : 0;
     if (persist) {
-        e0 = oz2_persistent_clusters(&pclusters);
+        e0 = oz2_worker_clusters(&pclusters);
         if (e0 != cudaSuccess) return e0;
     }
     int nl = P.n;

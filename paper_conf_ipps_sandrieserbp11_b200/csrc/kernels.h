@@ -14,6 +14,13 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t
                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
+// SM count of the Worker whose kernels launch next: its green-context partition
+// (PDL property SM_LIMIT) or 0 for the whole device.  The runtime sets it before
+// a Worker's launches (one Master thread drives the library); the shape pickers
+// and persistent grids size their wave models by worker_sms().
+void set_worker_sms(int sms);
+int worker_sms();   // the partition's SMs if set, else the current device's
+
 // K1 -- FP64 DMMA tile kernel.  Requirements (checked by the caller):
 // A, B device pointers, 16 B aligned, lda*8 % 16 == 0, ldb*8 % 16 == 0.
 cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,

@@ -205,6 +205,42 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         }
     }
     const bool piped = RB * CP > 1;
+    // Task variant of this Worker, pre-selected from its PDL properties (task
+    // repository + static pre-selection, L1307-1326): FP64 K1 (DMMA) or K4
+    // (Ozaki), FP32 K3+K2 (3xTF32) or K4 (Ozaki).
+    int oz_slices = 0;
+    int oz_rn = 0;
+    int oz2_nmod = 0, oz2_bits = 0;
+    if (!f64 && K > 0 && worker_sgemm_ozaki2(w))
+        return set_err(PDL_EUNSUPPORTED, "SGEMM_VARIANT ozaki2: Ozaki scheme II is an FP64 variant (use ozaki)");
+    const bool ozaki2 = K > 0 && f64 && worker_ozaki2(w, &oz2_nmod, &oz2_bits);
+    const bool ozaki = K > 0 && !ozaki2 && worker_ozaki(w, f64, &oz_slices, &oz_rn);
+    pdlk::OzakiLayout OL;
+    if (ozaki) {
+        OL = pdlk::ozaki_layout(rows, cols, K, oz_slices);
+        OL.rn = oz_rn;
+    }
+    pdlk::Ozaki2Plan P2;
+    if (ozaki2) P2 = pdlk::ozaki2_plan(rows, cols, K, oz2_nmod, oz2_bits);
+    // B prepared by a previous task of this Worker (PDL_TASK_REUSE_B)?
+    WorkerCtx::BSig want;
+    want.valid = true;
+    want.B = B;
+    want.ldb = t.ldb;
+    want.K = K;
+    want.cols = cols;
+    want.dtype = t.dtype;
+    want.oz = ozaki ? 1 : ozaki2 ? 2 : 0;
+    want.S = ozaki ? OL.S : ozaki2 ? P2.n : 0;
+    want.rn = ozaki ? OL.rn : ozaki2 ? P2.p : 0;
+    const bool prep_b = K > 0 && (ozaki || ozaki2 || !f64);
+    const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
+    // A task that re-prepares B while another task of this Worker may still read
+    // the shared B-side buffers on another stream (a side-stream chunk task, slot
+    // != 0, after the main task was replayed from a graph or ran on other
+    // operands) waits for the last B-using task first.
+    const bool b_writes = prep_b && !b_ready;
+    if (b_writes && slot != 0 && w.ev_blast) CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_blast, 0));
     int rc;
     if (piped && (rc = ensure_aux(w))) return rc;
     cudaStream_t s_in = piped ? w.aux[0] : w.stream, s_out = piped ? w.aux[1] : w.stream;
@@ -238,16 +274,6 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         if ((rc = ensure(BUF_C, (size_t)(ldcd * rows * es), &p))) return rc;
         Cd = (char *)p;
     }
-    // Task variant of this Worker, pre-selected from its PDL properties (task
-    // repository + static pre-selection, L1307-1326): FP64 K1 (DMMA) or K4
-    // (Ozaki), FP32 K3+K2 (3xTF32) or K4 (Ozaki).
-    int oz_slices = 0;
-    int oz_rn = 0;
-    int oz2_nmod = 0, oz2_bits = 0;
-    if (!f64 && K > 0 && worker_sgemm_ozaki2(w))
-        return set_err(PDL_EUNSUPPORTED, "SGEMM_VARIANT ozaki2: Ozaki scheme II is an FP64 variant (use ozaki)");
-    const bool ozaki2 = K > 0 && f64 && worker_ozaki2(w, &oz2_nmod, &oz2_bits);
-    const bool ozaki = K > 0 && !ozaki2 && worker_ozaki(w, f64, &oz_slices, &oz_rn);
     // FP32 split buffers (K-major hi/lo of A rows and of B^T rows)
     const int64_t Kp = round_up(std::max<int64_t>(K, 1), pdlk::K2_BK);
     float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
@@ -264,16 +290,14 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     pdlk::EncodeTiledFn enc = nullptr;
     if (K > 0 && (rc = get_encoder(&enc))) return rc;
     const char *k2v = getenv("PDL_K2");   // measurement knob: force "1sm" or "2sm"
-    int sms = 0;
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, w.device);
+    // wave models of the shape pickers see this Worker's SMs (its partition)
+    pdlk::set_worker_sms(w.sm_limit);
+    const int sms = pdlk::worker_sms();
 
-    pdlk::OzakiLayout OL;
     int8_t *a8 = nullptr, *b8 = nullptr;
     int *oz_ea = nullptr, *oz_fb = nullptr;
     unsigned long long *oz_bmax = nullptr;
     if (ozaki) {
-        OL = pdlk::ozaki_layout(rows, cols, K, oz_slices);
-        OL.rn = oz_rn;
         if ((rc = ensure(BUF_OZA, OL.a8_bytes, &p))) return rc;
         a8 = (int8_t *)p;
         if ((rc = ensure_buf(w, BUF_OZB, OL.b8_bytes, &p))) return rc;
@@ -281,11 +305,9 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         if ((rc = oz_exponents(w, slot, rows, cols, &oz_bmax, &oz_fb, &oz_ea))) return rc;
     }
 
-    pdlk::Ozaki2Plan P2;
     uint8_t *oz2_R = nullptr;
     int64_t oz2_ldr = 0, oz2_plane = 0;
     if (ozaki2) {
-        P2 = pdlk::ozaki2_plan(rows, cols, K, oz2_nmod, oz2_bits);
         if ((rc = ensure(BUF_OZA, P2.a8_bytes, &p))) return rc;
         a8 = (int8_t *)p;
         if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
@@ -297,19 +319,6 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         oz2_R = (uint8_t *)p;
     }
 
-    // B prepared by a previous task of this Worker (PDL_TASK_REUSE_B)?
-    WorkerCtx::BSig want;
-    want.valid = true;
-    want.B = B;
-    want.ldb = t.ldb;
-    want.K = K;
-    want.cols = cols;
-    want.dtype = t.dtype;
-    want.oz = ozaki ? 1 : ozaki2 ? 2 : 0;
-    want.S = ozaki ? OL.S : ozaki2 ? P2.n : 0;
-    want.rn = ozaki ? OL.rn : ozaki2 ? P2.p : 0;
-    const bool prep_b = K > 0 && (ozaki || ozaki2 || !f64);
-    const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
     // a B prepared on another stream (a task of another slot): wait for it
     if (b_ready && w.ev_bprep) CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_bprep, 0));
     auto mark_bprep = [&](cudaStream_t st) -> int {
@@ -517,6 +526,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         // the B-side buffers now hold this task's prepared B (whole panel only when unpiped)
         w.bsig = want;
         w.bsig.valid = !piped && !b_st;
+        ++w.bsig_gen;
     }
     if (piped) {
         // join: the Worker stream completes after every side stream's work
@@ -527,6 +537,12 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         cudaEvent_t ein = ev_get(w, evn);
         CUDA_TRY(cudaEventRecord(ein, s_in));
         CUDA_TRY(cudaStreamWaitEvent(w.stream, ein, 0));
+    }
+    // end of this task's use of the B-side buffers (a graph replay records it
+    // after the launch instead: an event recorded inside a capture is a graph node)
+    if (prep_b && !w.capturing) {
+        if (!w.ev_blast) CUDA_TRY(cudaEventCreateWithFlags(&w.ev_blast, cudaEventDisableTiming));
+        CUDA_TRY(cudaEventRecord(w.ev_blast, w.stream));
     }
     return PDL_OK;
 }
@@ -616,6 +632,7 @@ int run_dynamic(const Task &t, const std::vector<int> &gw) {
         const int64_t Kp = round_up(K, pdlk::K2_BK);
         for (size_t i = 0; i < ws.size(); ++i) {
             WorkerCtx &w = *ws[i];
+            pdlk::set_worker_sms(w.sm_limit);
             // the shared counter lives in the first Worker's memory region: a Worker on
             // another device reaches it only over a Worker<->Worker interconnect of the
             // descriptor (L1336-1341)
@@ -728,7 +745,16 @@ int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *
         w.timed |= ge.timed;
         for (auto &pr : ge.kt_pairs)
             if (w.kt_list.size() < kMaxKernelTimes) w.kt_list.push_back(pr);
-        w.bsig.valid = false;
+        // the replay leaves the captured task's prepared B in the B-side buffers:
+        // REUSE_B tasks may use it once the replay is done (ev_bprep), and a task
+        // re-preparing B on another stream waits for it (ev_blast)
+        w.bsig = ge.bsig;
+        if (ge.bsig.valid || ge.uses_b) {
+            for (cudaEvent_t *ev : {&w.ev_bprep, &w.ev_blast}) {
+                if (!*ev) CUDA_TRY(cudaEventCreateWithFlags(ev, cudaEventDisableTiming));
+                CUDA_TRY(cudaEventRecord(*ev, w.stream));
+            }
+        }
         ++w.graph_replays;
         return PDL_OK;
     };
@@ -749,6 +775,7 @@ int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *
     const size_t used0 = w.kt_used, list0 = w.kt_list.size();
     const int launches0 = w.launches;
     const int gen0 = w.buf_gen;
+    const long long bsig_gen0 = w.bsig_gen;
     if (cudaStreamBeginCapture(w.stream, cudaStreamCaptureModeRelaxed) != cudaSuccess) {
         cudaGetLastError();
         seen = -1000000;
@@ -789,6 +816,8 @@ int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *
     w.kt_pool.erase(w.kt_pool.begin() + used0, w.kt_pool.begin() + w.kt_used);
     w.kt_used = used0;
     ge.kt_pairs.assign(w.kt_list.begin() + list0, w.kt_list.end());
+    ge.bsig = w.bsig;
+    ge.uses_b = w.bsig.dtype >= 0 && w.bsig_gen != bsig_gen0;
     w.kt_list.resize(list0);
     w.launches = launches0;
     return replay(w.graphs.emplace(key, std::move(ge)).first->second);
@@ -806,14 +835,15 @@ int execute(bool sync) {
         w.timed = false;
     }
     // Green-context streams are non-blocking: give them the ordering of the
-    // blocking Worker streams (after the legacy default stream's prior work,
-    // and the legacy stream after them -- see the end of this function).
+    // blocking Worker streams (after the prior work of the legacy default stream,
+    // or of the caller's stream given to pdl_set_stream, and that stream after
+    // them -- see the end of this function).
     if (!g->dry_run)
         for (auto &w : g->workers)
             if (w.gctx && w.own_stream) {
                 CUDA_TRY(cudaSetDevice(w.device));
                 if (!w.ev_legacy) CUDA_TRY(cudaEventCreateWithFlags(&w.ev_legacy, cudaEventDisableTiming));
-                CUDA_TRY(cudaEventRecord(w.ev_legacy, cudaStreamLegacy));
+                CUDA_TRY(cudaEventRecord(w.ev_legacy, w.join_stream ? w.join_stream : cudaStreamLegacy));
                 CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_legacy, 0));
             }
     for (size_t ti = 0; ti < q.size(); ++ti) {
@@ -901,7 +931,7 @@ int execute(bool sync) {
             if (w.gctx && w.own_stream) {
                 CUDA_TRY(cudaSetDevice(w.device));
                 CUDA_TRY(cudaEventRecord(w.ev_legacy, w.stream));
-                CUDA_TRY(cudaStreamWaitEvent(cudaStreamLegacy, w.ev_legacy, 0));
+                CUDA_TRY(cudaStreamWaitEvent(w.join_stream ? w.join_stream : cudaStreamLegacy, w.ev_legacy, 0));
             }
     if (sync) return pdl_sync();
     return PDL_OK;

@@ -65,6 +65,11 @@ struct WorkerCtx {
     cudaEvent_t ev_legacy = nullptr;   // orders the non-blocking green stream with the legacy stream
     DevBuf buf[BUF_COUNT * kTaskSlots];
     cudaEvent_t ev_bprep = nullptr;   // after the last B preparation (REUSE_B tasks on other streams wait)
+    cudaEvent_t ev_blast = nullptr;   // after the last task that used the shared B-side buffers (a task
+                                      // re-preparing B on another stream waits for it)
+    // the caller's stream (pdl_set_stream) of a green-context Worker: the Worker
+    // keeps its partition's stream and joins this one around every run
+    cudaStream_t join_stream = nullptr;   // nullptr = cudaStreamLegacy
     cudaEvent_t ev_k0 = nullptr, ev_k1 = nullptr;   // around the dominant kernel of the last task
     int launches = 0;                               // kernels launched in the last run
     bool timed = false;
@@ -75,22 +80,6 @@ struct WorkerCtx {
     size_t kt_used = 0;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kt_list;
     cudaEvent_t kt_open = nullptr;   // start event of the launch being bracketed
-    // CUDA graphs of repeated tasks (PDL_TASK_GRAPH / PDL_GRAPH=1): signature -> graph
-    struct GraphEntry {
-        cudaGraphExec_t exec = nullptr;
-        std::vector<cudaEvent_t> events;                              // owned; recorded by the graph
-        std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kt_pairs;
-        int launches = 0;
-        bool timed = false;
-    };
-    std::map<std::string, GraphEntry> graphs;
-    std::map<std::string, int> graph_seen;   // signatures run once (captured on the next run)
-    int buf_gen = 0;                         // bumped when a buffer is reallocated (graphs go stale)
-    bool capturing = false;
-    long long graph_replays = 0;
-    // pipelined staging: copy-in, copy-out, second compute stream; reusable events
-    cudaStream_t aux[3] = {nullptr, nullptr, nullptr};
-    std::vector<cudaEvent_t> ev_pool;
     // identity of the B operand whose prepared form (FP32 split / Ozaki slices)
     // sits in the B-side buffers (PDL_TASK_REUSE_B)
     struct BSig {
@@ -102,7 +91,27 @@ struct WorkerCtx {
             return valid && o.valid && B == o.B && ldb == o.ldb && K == o.K && cols == o.cols && dtype == o.dtype &&
                    oz == o.oz && S == o.S && rn == o.rn;
         }
-    } bsig;
+    };
+    BSig bsig;
+    long long bsig_gen = 0;   // bumped whenever a task writes the B-side buffers
+    // CUDA graphs of repeated tasks (PDL_TASK_GRAPH / PDL_GRAPH=1): signature -> graph
+    struct GraphEntry {
+        cudaGraphExec_t exec = nullptr;
+        std::vector<cudaEvent_t> events;                              // owned; recorded by the graph
+        std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kt_pairs;
+        int launches = 0;
+        bool timed = false;
+        BSig bsig;            // the prepared B the captured task leaves in the B-side buffers
+        bool uses_b = false;  // the captured task writes the B-side buffers
+    };
+    std::map<std::string, GraphEntry> graphs;
+    std::map<std::string, int> graph_seen;   // signatures run once (captured on the next run)
+    int buf_gen = 0;                         // bumped when a buffer is reallocated (graphs go stale)
+    bool capturing = false;
+    long long graph_replays = 0;
+    // pipelined staging: copy-in, copy-out, second compute stream; reusable events
+    cudaStream_t aux[3] = {nullptr, nullptr, nullptr};
+    std::vector<cudaEvent_t> ev_pool;
 };
 
 constexpr size_t kMaxKernelTimes = 4096;

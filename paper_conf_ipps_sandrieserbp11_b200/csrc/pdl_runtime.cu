@@ -260,6 +260,12 @@ int pdl_set_stream(int worker, void *stream) {
     WorkerCtx &w = g->workers[worker];
     if (g->dry_run) return PDL_OK;
     CUDA_TRY(cudaSetDevice(w.device));
+    if (w.gctx) {
+        // an SM-partition Worker keeps its green-context stream (replacing it would
+        // drop the partition); runs join the caller's stream on both sides instead
+        w.join_stream = (cudaStream_t)stream;
+        return PDL_OK;
+    }
     if (stream) {
         if (w.own_stream && w.stream) {
             cudaStreamSynchronize(w.stream);
@@ -375,8 +381,13 @@ int pdl_query(const char *key, char *out, size_t len) {
             // run at once on different streams of a local Worker when they use
             // different scratch slots (PDL_TASK_SLOT): every task variant keeps its
             // per-task buffers per slot, and a REUSE_B task waits for the B
-            // preparation on the other stream
-            res = g->workers.empty() ? "no" : "yes";
+            // preparation on the other stream (a task re-preparing B there -- e.g.
+            // after a graph replay of the first task -- waits for the last B-using
+            // task).  SM-partition Workers keep their one green-context stream, so
+            // their tasks serialise: "no"
+            bool any_green = false;
+            for (auto &w : g->workers) any_green |= w.gctx != nullptr;
+            res = g->workers.empty() || any_green ? "no" : "yes";
         }
         else if (k == "plan") res = g->plan_json;
         else if (k == "groups") {

@@ -373,8 +373,13 @@ def distributed_matmul(A_full, B_full, C_full, tile=0, group=None, overlap=True)
     the descriptor joins the Workers by no interconnect -- computed, and the C
     block copied back (PCIe)."""
     rank = dist.get_rank()
+    if not (A_full.dtype == B_full.dtype == C_full.dtype):
+        raise TypeError(f"A, B, C must have one dtype (got {A_full.dtype}, {B_full.dtype}, {C_full.dtype})")
     M, K = A_full.shape
     N = B_full.shape[1]
+    if B_full.shape[0] != K or tuple(C_full.shape) != (M, N):
+        raise ValueError(f"shapes do not chain: A {tuple(A_full.shape)} @ B {tuple(B_full.shape)} -> "
+                         f"C {tuple(C_full.shape)}")
     wp = worker_plan(M, N, K, tile, rank, group)
     grid = Grid(wp.Gr, wp.Gc, rank, via_host=exchange_path(group) == "host")
     dev = torch.device("cuda", torch.cuda.current_device())
