@@ -11,7 +11,7 @@ NVFLAGS   := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisi
 CXXFLAGS  := -O2 -std=c++17 -fPIC -fvisibility=hidden -Wall -Wextra -Wno-unused-parameter
 
 HOST_SRC  := $(CSRC)/pdl_xml.cpp $(CSRC)/pdl_model.cpp $(CSRC)/pdl_map.cpp
-CU_SRC    := $(CSRC)/pdl_runtime.cu $(CSRC)/pdl_devices.cu $(CSRC)/pdl_exec.cu $(CSRC)/k_dgemm.cu $(CSRC)/k_tf32.cu $(CSRC)/k_tf32_2sm.cu $(CSRC)/k_ozaki.cu $(CSRC)/k_ozaki2.cu
+CU_SRC    := $(CSRC)/pdl_runtime.cu $(CSRC)/pdl_devices.cu $(CSRC)/pdl_exec.cu $(CSRC)/pdl_xchg.cu $(CSRC)/k_dgemm.cu $(CSRC)/k_tf32.cu $(CSRC)/k_tf32_2sm.cu $(CSRC)/k_ozaki.cu $(CSRC)/k_ozaki2.cu
 HOST_OBJ  := $(patsubst $(CSRC)/%.cpp,$(BUILD)/%.o,$(HOST_SRC))
 CU_OBJ    := $(patsubst $(CSRC)/%.cu,$(BUILD)/%.o,$(CU_SRC))
 HDRS      := $(wildcard $(CSRC)/*.h $(CSRC)/*.hpp $(CSRC)/*.cuh) include/libpdl.h

@@ -44,6 +44,15 @@ int main(int argc, char **argv) {
     printf("gpu Workers in the descriptor: %s\n", buf);
     check(task_matmul(A, B, C, n, n, n, 256), "task_matmul");
     check(pdl_run(), "pdl_run");
+    /* bytes moved along the descriptor's interconnects: with several Workers joined
+       by NVLink, host operands cross PCIe once and the panels move Worker<->Worker */
+    char stats[8192];
+    check(pdl_query("stats", stats, sizeof stats), "pdl_query(stats)");
+    const char *tr = strstr(stats, "\"transfers\"");
+    if (tr) {
+        const char *end = strchr(tr, '}');
+        printf("%.*s}\n", end ? (int)(end - tr) : (int)strlen(tr), tr);
+    }
     int64_t plan[PDL_PLAN_LEN];
     check(pdl_plan(n, n, n, 256, NULL, 0, plan, PDL_PLAN_LEN), "pdl_plan");
     printf("Worker 0 of %lld: rows [%lld, %lld) cols [%lld, %lld), %lld x %lld tile tasks in all\n",

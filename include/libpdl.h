@@ -55,7 +55,10 @@ extern "C" {
 #define PDL_ENOWORKER    -3  /* no gpu Worker in the execution group, or more Workers than devices */
 #define PDL_ENOMEM       -4  /* device or host allocation failed */
 #define PDL_ECUDA        -5  /* a CUDA runtime/driver call failed */
-#define PDL_ENCCL        -6  /* reserved: collective failure (the exchange runs in the Python runtime) */
+#define PDL_ENCCL        -6  /* Worker<->Worker exchange failed: a peer copy of pdl_run's exchange
+                                failed or had not completed within PDL_SYNC_TIMEOUT_MS (pdl_sync);
+                                the multi-rank Python runtime maps NCCL / gloo collective
+                                failures and timeouts to the same code */
 #define PDL_ESTATE       -7  /* call out of order (task before load, load twice, ...) */
 #define PDL_EUNSUPPORTED -8  /* valid request this build does not implement */
 
@@ -189,6 +192,18 @@ int task_matmul_ex(int dtype, const void *A, int64_t lda, const void *B, int64_t
  * pdl_run -- map and execute all queued tasks in program order (access-mode
  * dependencies reduce to queue order for one task type), then synchronise,
  * harvest errors and clear the queue.  Blocks until C is written.
+ * Transfer paths follow the descriptor's interconnects (SS IV-C step 3,
+ * L1336-1341): with A and B in the Master's memory region (host), a BLOCK
+ * task over G > 1 Workers that an Interconnect joins pairwise (the shipped
+ * descriptors' NVLink) moves each operand byte over the Master->Worker
+ * interconnect once -- Worker (r, c) receives chunk c of its A row-panel and
+ * chunk r of its B column-panel -- and the Workers pull the rest of their
+ * panels from each other (peer copies, overlapped with the tile kernels: own
+ * A chunk first).  Otherwise each Worker stages its whole panels from the
+ * Master's memory region.  Bytes per path: pdl_query("stats")["transfers"].
+ * Env PDL_EXCHANGE=0 disables the Worker<->Worker path; PDL_SYNC_TIMEOUT_MS
+ * bounds the wait (then PDL_ENCCL if an exchange copy is unfinished, else
+ * PDL_ECUDA; the work stays in flight: unload the platform).
  */
 int pdl_run(void);
 
@@ -235,7 +250,10 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group,
  * pdl_query -- the "simple query API" over the loaded PDL (L935-937).
  * Keys: "version", "masters", "workers", "groups", "model" (JSON),
  *   "plan" (JSON of the last run's mappings), "stats" (JSON: launches,
- *   kernel time and SM partition per Worker of the last run; "dynamic": tiles
+ *   kernel time and SM partition per Worker of the last run; "transfers":
+ *   bytes moved Master->Worker, Worker->Master and Worker<->Worker in the
+ *   last run, the tasks that ran the Worker<->Worker exchange, and the
+ *   descriptor's interconnect types of those paths; "dynamic": tiles
  *   each Worker claimed in the last DYNAMIC task -- read after pdl_sync),
  *   "worker/<i>/<PROPERTY>",
  *   "worker/<i>/device", "worker/<i>/id", "pu/<id>/<PROPERTY>",

@@ -275,6 +275,10 @@ void free_state() {
         for (auto ev : w.ev_pool) cudaEventDestroy(ev);
         for (auto st : w.aux)
             if (st) cudaStreamDestroy(st);
+        if (w.xs) cudaStreamDestroy(w.xs);
+        for (auto ev : w.xev_pool) cudaEventDestroy(ev);
+        for (cudaEvent_t ev : {w.ev_xdone, w.ev_bprep, w.ev_blast})
+            if (ev) cudaEventDestroy(ev);
         if (w.gctx) green_api()->destroy(w.gctx);
     }
     if (g->dyn) {

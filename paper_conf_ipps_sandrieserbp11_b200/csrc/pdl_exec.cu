@@ -222,7 +222,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     }
     pdlk::Ozaki2Plan P2;
     if (ozaki2) P2 = pdlk::ozaki2_plan(rows, cols, K, oz2_nmod, oz2_bits);
-    // B prepared by a previous task of this Worker (PDL_TASK_REUSE_B)?
+    // the prepared-B signature of this task (PDL_TASK_REUSE_B)
     WorkerCtx::BSig want;
     want.valid = true;
     want.B = B;
@@ -234,13 +234,12 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     want.S = ozaki ? OL.S : ozaki2 ? P2.n : 0;
     want.rn = ozaki ? OL.rn : ozaki2 ? P2.p : 0;
     const bool prep_b = K > 0 && (ozaki || ozaki2 || !f64);
-    const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
     // A task that re-prepares B while another task of this Worker may still read
     // the shared B-side buffers on another stream (a side-stream chunk task, slot
     // != 0, after the main task was replayed from a graph or ran on other
-    // operands) waits for the last B-using task first.
-    const bool b_writes = prep_b && !b_ready;
-    if (b_writes && slot != 0 && w.ev_blast) CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_blast, 0));
+    // operands) waits for the last B-using task first (piped tasks here, before
+    // their side streams fork; unpiped ones below, once b_ready is known).
+    if (piped && prep_b && slot != 0 && w.ev_blast) CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_blast, 0));
     int rc;
     if (piped && (rc = ensure_aux(w))) return rc;
     cudaStream_t s_in = piped ? w.aux[0] : w.stream, s_out = piped ? w.aux[1] : w.stream;
@@ -319,6 +318,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         oz2_R = (uint8_t *)p;
     }
 
+    // B prepared by a previous task of this Worker (PDL_TASK_REUSE_B)?  Decided after
+    // the buffers above are sized: a reallocated B-side buffer invalidates it.
+    const bool b_ready = prep_b && (t.flags & PDL_TASK_REUSE_B) && !piped && !b_st && w.bsig == want;
+    if (!piped && prep_b && !b_ready && slot != 0 && w.ev_blast)
+        CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_blast, 0));
     // a B prepared on another stream (a task of another slot): wait for it
     if (b_ready && w.ev_bprep) CUDA_TRY(cudaStreamWaitEvent(w.stream, w.ev_bprep, 0));
     auto mark_bprep = [&](cudaStream_t st) -> int {
@@ -352,6 +356,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                                               (const char *)A + (size_t)(r0 * t.lda) * es, (size_t)(t.lda * es),
                                               (size_t)(K * es), (size_t)nr, cudaMemcpyDefault, s_in);
             if (e != cudaSuccess) return set_err(PDL_ECUDA, "A staging copy failed: %s", cudaGetErrorString(e));
+            g->xfer.count(locate(A), w.device, nr * K * es);
             if (piped) {
                 ev_a[i] = ev_get(w, evn);
                 CUDA_TRY(cudaEventRecord(ev_a[i], s_in));
@@ -364,6 +369,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                                                   (const char *)B + (size_t)c0 * es, (size_t)(t.ldb * es),
                                                   (size_t)(nc * es), (size_t)K, cudaMemcpyDefault, s_in);
                 if (e != cudaSuccess) return set_err(PDL_ECUDA, "B staging copy failed: %s", cudaGetErrorString(e));
+                g->xfer.count(locate(B), w.device, nc * K * es);
                 if (piped) {
                     ev_b[j] = ev_get(w, evn);
                     CUDA_TRY(cudaEventRecord(ev_b[j], s_in));
@@ -517,6 +523,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 e = cudaMemcpy2DAsync((char *)C + (size_t)(r0 * t.ldc + c0) * es, (size_t)(t.ldc * es), Cs,
                                       (size_t)(ldcd * es), (size_t)(nc * es), (size_t)nr, cudaMemcpyDefault, s_out);
                 if (e != cudaSuccess) return set_err(PDL_ECUDA, "result gather copy failed: %s", cudaGetErrorString(e));
+                g->xfer.count(w.device, locate(C), nr * nc * es);
             }
             ++launch_idx;
         }
@@ -833,7 +840,9 @@ int execute(bool sync) {
     for (auto &w : g->workers) {
         w.launches = 0;
         w.timed = false;
+        w.xpending = false;
     }
+    g->xfer = XferStats();
     // Green-context streams are non-blocking: give them the ordering of the
     // blocking Worker streams (after the prior work of the legacy default stream,
     // or of the caller's stream given to pdl_set_stream, and that stream after
@@ -877,6 +886,13 @@ int execute(bool sync) {
         if (g->dry_run) continue;
         if (t.dist.kind == Dist::Dynamic) {
             rc = run_dynamic(t, gw);
+            if (rc) return rc;
+            continue;
+        }
+        if (exchange_applies(t, plan, gw)) {
+            // operands in the Master's memory region cross PCIe once, then move
+            // Worker <-> Worker over the descriptor's interconnect (pdl_xchg.cu)
+            rc = run_exchange(t, plan, gw);
             if (rc) return rc;
             continue;
         }

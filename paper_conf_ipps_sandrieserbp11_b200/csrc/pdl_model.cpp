@@ -129,6 +129,13 @@ bool Model::ic_between(int a, int b, const std::string &type_ci) const {
     return false;
 }
 
+std::string Model::ic_type_between(int a, int b) const {
+    const std::string &ta = pus[a].tid, &tb = pus[b].tid;
+    for (auto &ic : ics)
+        if ((ic.from == ta && ic.to == tb) || (ic.from == tb && ic.to == ta)) return ic.type;
+    return "";
+}
+
 namespace {
 
 bool is_pu(const XmlNode &n) {

@@ -74,6 +74,8 @@ struct Model {
     std::vector<int> group_workers(const char *group) const;  // gpu Workers, document order
     std::vector<int> all_gpu_workers() const;
     bool ic_between(int a, int b, const std::string &type_ci) const;
+    // type of the first Interconnect joining PU instances a and b ("" if none)
+    std::string ic_type_between(int a, int b) const;
     std::string to_json() const;
     std::string ics_json() const;
 };

@@ -42,7 +42,9 @@ struct DevBuf {
     size_t bytes = 0;
 };
 
-enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_OZA, BUF_OZB, BUF_OZE, BUF_OZR, BUF_COUNT };
+enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_OZA, BUF_OZB, BUF_OZE, BUF_OZR,
+               BUF_XA, BUF_XB,   // A row-panel / B column-panel gathered by the Worker<->Worker exchange
+               BUF_COUNT };
 // Scratch slots (PDL_TASK_SLOT): the per-task buffers (A staging, C staging, A
 // split / slices / residues, A exponents, residue planes) exist once per slot, so
 // tasks of different slots may run at once on different streams of the Worker;
@@ -112,6 +114,12 @@ struct WorkerCtx {
     // pipelined staging: copy-in, copy-out, second compute stream; reusable events
     cudaStream_t aux[3] = {nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> ev_pool;
+    // Worker<->Worker exchange (pdl_xchg.cu): its copy stream, events, and the
+    // event after the last exchange copy of the last run (sync timeouts)
+    cudaStream_t xs = nullptr;
+    std::vector<cudaEvent_t> xev_pool;
+    cudaEvent_t ev_xdone = nullptr;
+    bool xpending = false;
 };
 
 constexpr size_t kMaxKernelTimes = 4096;
@@ -131,8 +139,22 @@ struct Task {
     DistSpec dist;
 };
 
+// Bytes moved along the descriptor's interconnects in the last run (pdl_query
+// "stats"): Master MR <-> Worker MR (host staging, gather) and Worker MR <->
+// Worker MR (the exchange, and device operands read by another device's Worker).
+struct XferStats {
+    long long m2w = 0, w2m = 0, w2w = 0;
+    int exchange_tasks = 0;   // tasks that ran the Worker<->Worker exchange
+    void count(int src_dev, int dst_dev, long long bytes) {
+        if (src_dev < 0 && dst_dev >= 0) m2w += bytes;
+        else if (src_dev >= 0 && dst_dev < 0) w2m += bytes;
+        else if (src_dev >= 0 && dst_dev >= 0) w2w += bytes;
+    }
+};
+
 struct State {
     bool loaded = false;
+    XferStats xfer;
     bool dry_run = false;
     bool oversub = false;
     int rank = 0, nranks = 1;
@@ -200,5 +222,9 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
 int run_dynamic(const Task &t, const std::vector<int> &gw);
 int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols);
 int execute(bool sync);
+int enable_peer(int from, int to);
+// pdl_xchg.cu
+bool exchange_applies(const Task &t, const Plan &plan, const std::vector<int> &gw);
+int run_exchange(const Task &t, const Plan &plan, const std::vector<int> &gw);
 
 }  // namespace pdlrt

@@ -14,6 +14,8 @@
 // one-process-per-GPU mode runs in the Python runtime over torch.distributed.
 #include "pdl_rt.hpp"
 
+#include <chrono>
+
 namespace pdlrt {
 
 
@@ -242,11 +244,40 @@ int pdl_sync(void) {
     if (rc) return rc;
     if (g->dry_run) return PDL_OK;
     int launches = 0;
+    // PDL_SYNC_TIMEOUT_MS = t > 0: give up after t ms instead of blocking (a hung
+    // Worker<->Worker transfer or kernel); the device work stays in flight and the
+    // platform must be unloaded.  An unfinished exchange -> PDL_ENCCL.
+    const char *te = getenv("PDL_SYNC_TIMEOUT_MS");
+    const double tmo = te ? atof(te) : 0.0;
+    const auto t0 = std::chrono::steady_clock::now();
     for (auto &w : g->workers) {
         CUDA_TRY(cudaSetDevice(w.device));
-        cudaError_t e = cudaStreamSynchronize(w.stream);
-        if (e != cudaSuccess) return set_err(PDL_ECUDA, "device work failed on device %d: %s", w.device,
-                                             cudaGetErrorString(e));
+        cudaError_t e;
+        if (tmo > 0) {
+            while ((e = cudaStreamQuery(w.stream)) == cudaErrorNotReady) {
+                const double ms =
+                    std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+                if (ms > tmo) {
+                    if (w.xpending && w.ev_xdone && cudaEventQuery(w.ev_xdone) == cudaErrorNotReady)
+                        return set_err(PDL_ENCCL,
+                                       "Worker<->Worker exchange into Worker %s (device %d) did not complete "
+                                       "within %.0f ms",
+                                       g->model.pus[w.pu].id.c_str(), w.device, tmo);
+                    cudaGetLastError();
+                    return set_err(PDL_ECUDA, "device work of Worker %s (device %d) did not complete within %.0f ms",
+                                   g->model.pus[w.pu].id.c_str(), w.device, tmo);
+                }
+                usleep(50);
+            }
+        } else {
+            e = cudaStreamSynchronize(w.stream);
+        }
+        if (e != cudaSuccess) {
+            const bool xfail = w.xpending && w.ev_xdone && cudaEventQuery(w.ev_xdone) != cudaSuccess;
+            return set_err(xfail ? PDL_ENCCL : PDL_ECUDA, "device work failed on device %d%s: %s", w.device,
+                           xfail ? " (Worker<->Worker exchange)" : "", cudaGetErrorString(e));
+        }
+        w.xpending = false;
         launches += w.launches;
     }
     g->last_launches = launches;
@@ -418,6 +449,16 @@ int pdl_query(const char *key, char *out, size_t len) {
                 first = false;
             }
             o << "]";
+            // bytes moved along the interconnects in the last run, by path (the
+            // descriptor's IC types: Master<->Worker, Worker<->Worker)
+            std::string mw_ic, ww_ic;
+            const std::vector<int> gws = m.all_gpu_workers();
+            if (!gws.empty() && !m.masters.empty()) mw_ic = m.ic_type_between(m.masters[0], gws[0]);
+            if (gws.size() > 1) ww_ic = m.ic_type_between(gws[0], gws[1]);
+            o << ",\"transfers\":{\"master_to_worker\":" << g->xfer.m2w << ",\"worker_to_master\":" << g->xfer.w2m
+              << ",\"worker_to_worker\":" << g->xfer.w2w << ",\"exchange_tasks\":" << g->xfer.exchange_tasks
+              << ",\"master_worker_ic\":\"" << json_escape(mw_ic) << "\",\"worker_worker_ic\":\""
+              << json_escape(ww_ic) << "\"}";
             // tiles each Worker claimed in the last DYNAMIC task (valid after pdl_sync)
             if (g->dyn_n > 0 && g->dyn && !g->dry_run) {
                 std::vector<int> claims(g->dyn_n + 1, 0);

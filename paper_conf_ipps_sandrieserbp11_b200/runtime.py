@@ -141,6 +141,11 @@ class PanelBuffers:
     def __init__(self, wp: WorkerPlan, dtype, device):
         self.A = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dtype, device=device)
         self.B = torch.empty((wp.Gr * wp.qb, wp.cols), dtype=dtype, device=device)
+        if _test_delay_cycles():
+            # fault injection (tests): panels start as NaN, so a compute that does
+            # not wait for its chunk's landing produces NaN rows of C
+            self.A.fill_(float("nan"))
+            self.B.fill_(float("nan"))
 
 
 def exchange(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers):
@@ -157,33 +162,142 @@ def exchange(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers):
     return bufs.A[: wp.rows], bufs.B[: wp.K]
 
 
+# ---- collectives ------------------------------------------------------------
+#
+# NCCL (the B200 box): asynchronous work on NCCL's streams; Work.wait() makes the
+# CURRENT stream wait for it, the host does not block.  gloo (CPU tests; several
+# ranks sharing one GPU): gloo moves host tensors only, so device tensors are
+# staged through pinned host memory, and _HostStaged gives the same stream
+# semantics -- the landing copy runs on a comm stream and wait() makes the current
+# stream wait for it -- so the ordering logic of compute_groups faces work that
+# has not finished.  Fault injection for the tests: PDL_TEST_EXCHANGE_DELAY_US
+# delays every landing on the comm stream (a spin kernel) and poisons the panel
+# buffers with NaN; PDL_TEST_DROP_WAITS=1 drops the A-chunk waits (the test that
+# the ordering matters must then see corrupt C).
+# Failures of the collectives surface as pdl.PDLError(PDL_ENCCL); a hang is
+# bounded by the process group's timeout (init_process_group(timeout=...)) and,
+# for the broadcast handles, PDL_EXCHANGE_TIMEOUT_S.
+
+
+def _test_delay_cycles():
+    import os
+    us = float(os.environ.get("PDL_TEST_EXCHANGE_DELAY_US", "0") or 0)
+    return int(us * 2000)   # ~2 GHz SM clock
+
+
+_comm_streams = {}
+
+
+def _comm_stream():
+    dev = torch.cuda.current_device()
+    if dev not in _comm_streams:
+        _comm_streams[dev] = torch.cuda.Stream(device=dev)
+    return _comm_streams[dev]
+
+
+def _exchange_error(what, e):
+    return pdl.PDLError(pdl.PDL_ENCCL, f"{what} failed over {dist.get_backend()}: {e}")
+
+
+class _HostStaged:
+    """A gloo collective on pinned host memory whose result lands in a device
+    tensor on the comm stream, with NCCL's wait() semantics (see above)."""
+
+    def __init__(self, work, tmp, dst, drop_wait=False):
+        self.work, self.tmp, self.dst = work, tmp, dst
+        self.drop_wait = drop_wait
+        self.issued = torch.cuda.Event()
+        self.issued.record()   # the landing copy must not overtake earlier users of dst
+        self.landed = None
+
+    def _land(self):
+        if self.landed is None:
+            try:
+                self.work.wait()   # the host copy is complete
+            except RuntimeError as e:
+                raise _exchange_error("host-staged collective", e) from e
+            cs = _comm_stream()
+            cs.wait_event(self.issued)
+            with torch.cuda.stream(cs):
+                cyc = _test_delay_cycles()
+                if cyc:
+                    torch.cuda._sleep(cyc)
+                self.dst.copy_(self.tmp, non_blocking=True)
+                self.landed = torch.cuda.Event()
+                self.landed.record(cs)
+
+    def wait(self):
+        self._land()
+        if not self.drop_wait:
+            torch.cuda.current_stream().wait_event(self.landed)
+
+
+class _Async:
+    """Async work handle (NCCL: wait() = the current stream waits, no host block;
+    gloo on host tensors: the host waits);
+    errors (including the NCCL watchdog's async-error abort) -> PDL_ENCCL."""
+
+    def __init__(self, work, what, drop_wait=False):
+        self.work, self.what, self.drop_wait = work, what, drop_wait
+
+    def wait(self):
+        if self.drop_wait:
+            return
+        import os
+        from datetime import timedelta
+        try:
+            t = os.environ.get("PDL_EXCHANGE_TIMEOUT_S")
+            if t:
+                self.work.wait(timeout=timedelta(seconds=float(t)))
+            else:
+                self.work.wait()
+        except RuntimeError as e:
+            raise _exchange_error(self.what, e) from e
+
+
+def _staged(t, group):
+    return t.is_cuda and dist.get_backend(group) == "gloo"
+
+
 def _all_gather(out, chunk, group):
-    """NCCL all-gather into a contiguous buffer.  Under the gloo backend
-    (CPU tests; several ranks sharing one GPU in the 1-GPU validation run)
-    device tensors are staged through host memory, since gloo gathers host
-    tensors only."""
-    if out.is_cuda and dist.get_backend(group) == "gloo":
-        tmp = torch.empty(out.shape, dtype=out.dtype)
-        dist.all_gather_into_tensor(tmp, chunk.contiguous().cpu(), group=group)
-        out.copy_(tmp)
-    else:
-        dist.all_gather_into_tensor(out, chunk.contiguous(), group=group)
+    """All-gather into a contiguous buffer (the current stream waits for it)."""
+    try:
+        if _staged(out, group):
+            tmp = torch.empty(out.shape, dtype=out.dtype, pin_memory=True)
+            w = dist.all_gather_into_tensor(tmp, chunk.contiguous().cpu(), group=group, async_op=True)
+            _HostStaged(w, tmp, out).wait()
+        else:
+            dist.all_gather_into_tensor(out, chunk.contiguous(), group=group)
+    except RuntimeError as e:
+        if isinstance(e, pdl.PDLError):
+            raise
+        raise _exchange_error("all-gather", e) from e
+
+
+def _broadcast(t, src, group):
+    """Asynchronous broadcast of one A chunk inside the grid row; returns a
+    handle whose wait() orders the current stream after the chunk's landing."""
+    import os
+    drop = os.environ.get("PDL_TEST_DROP_WAITS") == "1"
+    try:
+        if _staged(t, group):
+            mine = dist.get_rank() == src
+            tmp = t.cpu().pin_memory() if mine else torch.empty(t.shape, dtype=t.dtype, pin_memory=True)
+            w = dist.broadcast(tmp, src=src, group=group, async_op=True)
+            if mine:   # the source's chunk is already in place
+                w.wait()
+                return _Done()
+            return _HostStaged(w, tmp, t, drop_wait=drop)
+        return _Async(dist.broadcast(t, src=src, group=group, async_op=True), f"broadcast from rank {src}", drop)
+    except RuntimeError as e:
+        if isinstance(e, pdl.PDLError):
+            raise
+        raise _exchange_error("broadcast", e) from e
 
 
 class _Done:
     def wait(self):
         pass
-
-
-def _broadcast(t, src, group):
-    """Asynchronous broadcast of one A chunk inside the grid row (NCCL);
-    host-staged and synchronous under gloo (see _all_gather)."""
-    if t.is_cuda and dist.get_backend(group) == "gloo":
-        tmp = t.cpu() if dist.get_rank() == src else torch.empty(t.shape, dtype=t.dtype)
-        dist.broadcast(tmp, src=src, group=group)
-        t.copy_(tmp)
-        return _Done()
-    return dist.broadcast(t, src=src, group=group, async_op=True)
 
 
 def chunk_rows(wp: WorkerPlan, j):

@@ -114,3 +114,33 @@ def test_concurrent_chunk_groups_bitwise(G, dt, variant, monkeypatch):
             assert (oracle.scaled_error(out[1][rows], Cref, D) <= tol).all()
     finally:
         pdl.unload()
+
+
+def _run_rc(world, *args, env_extra=None):
+    torch = pytest.importorskip("torch")
+    backend = "nccl" if torch.cuda.device_count() >= world else "gloo"
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
+           "--master-addr=127.0.0.1", f"--master-port={_port()}", os.path.join(ROOT, "tests", "dist_check.py"),
+           *[str(a) for a in args[:5]], backend, *[str(a) for a in args[5:]]]
+    env = dict(os.environ, PDL_ALLOW_OVERSUBSCRIBE="1", **(env_extra or {}))
+    env.pop("PDL_DRY_RUN", None)
+    return subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
+
+
+@pytest.mark.parametrize("world,dt", [(4, "f64"), (8, "f64"), (8, "f32")])
+def test_late_chunks_are_waited_for(world, dt):
+    """Every A chunk and B chunk lands 3 ms late on the comm stream (a spin kernel
+    before the landing copy) into NaN-poisoned panel buffers, while the host runs
+    ahead (the collectives have NCCL's stream semantics): C is still correct, so
+    every compute launch of compute_groups waits for its own chunks."""
+    _run(world, dt, 1000, 700, 300, 64,
+         env_extra={"PDL_TEST_EXCHANGE_DELAY_US": "3000", "PDL_OVERLAP_A": "1"})
+
+
+def test_a_missing_wait_corrupts_c():
+    """Negative control for the test above: with the A-chunk waits dropped
+    (PDL_TEST_DROP_WAITS=1) the same run computes on chunks that have not landed
+    and the oracle check fails -- the ordering test can see a missing wait."""
+    r = _run_rc(4, "f64", 1000, 700, 300, 64,
+                env_extra={"PDL_TEST_EXCHANGE_DELAY_US": "3000", "PDL_OVERLAP_A": "1", "PDL_TEST_DROP_WAITS": "1"})
+    assert r.returncode != 0 or "ok=False" in r.stdout, r.stdout[-2000:]

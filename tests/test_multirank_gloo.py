@@ -124,3 +124,46 @@ def test_reference_arm_uses_all_host_cores():
     d = json.loads(lines[0])
     assert d["impl"] == "reference" and d["n_gpus"] == 2
     assert d["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
+
+
+def _stalled_peer(rank, world, port, q):
+    """Rank 0 waits for a broadcast rank 1 never sends (rank 1 is stuck in host
+    work): the handle's wait times out after PDL_EXCHANGE_TIMEOUT_S and the
+    runtime reports it as PDL_ENCCL, the library's exchange-failure code."""
+    import sys
+    import time
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), PDL_EXCHANGE_TIMEOUT_S="2")
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime
+    res = None
+    try:
+        if rank == 0:
+            t = torch.zeros(16)
+            try:
+                runtime._broadcast(t, 1, None).wait()
+                res = "no error"
+            except pdl.PDLError as e:
+                res = e.code
+        else:
+            time.sleep(8)
+            res = "peer"
+    except Exception as e:  # pragma: no cover
+        res = repr(e)
+    q.put((rank, res))
+
+
+def test_exchange_timeout_maps_to_pdl_enccl():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_stalled_peer, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in range(2))
+    for p in procs:
+        p.join(timeout=30)
+        if p.is_alive():
+            p.kill()
+    from paper_conf_ipps_sandrieserbp11_b200 import pdl
+    assert res[0] == pdl.PDL_ENCCL, res
