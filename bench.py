@@ -65,12 +65,10 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cublas", action="store_true")
-    p.add_argument("--variant", choices=("default", "ozaki", "ozaki2"), default="default",
-                   help="task variant pinned in the PDL descriptor: default (FP64 K1 DMMA / FP32 K3+K2 3xTF32), "
-                        "ozaki (K4/K5 INT8 slices; DGEMM_VARIANT / SGEMM_VARIANT) or ozaki2 (FP64 only: "
-                        "K6/K7 Ozaki scheme II, INT8 residue GEMMs + CRT)")
-    p.add_argument("--slices", type=int, default=None,
-                   help="Ozaki slices (default 6 for FP64, 3 for FP32; round-to-nearest)")
+    p.add_argument("--variant", choices=("default", "ozaki2"), default="default",
+                   help="task variant pinned in the PDL descriptor: default (FP64 K1 DMMA / FP32 K3+K2 3xTF32) "
+                        "or ozaki2 (FP64 only: K6/K7 Ozaki scheme II, INT8 residue GEMMs + CRT, with its "
+                        "certificate and K1 recompute, DESIGN.md R21)")
     p.add_argument("--no-alt", action="store_true", help="skip timing the other task variants")
     p.add_argument("--dist-backend", choices=("auto", "nccl", "gloo"), default="auto",
                    help="auto: NCCL when every rank has its own GPU, else gloo (ranks share GPUs: "
@@ -189,24 +187,11 @@ def ncu_traffic(dtype, cfg):
         return None
 
 
-def variant_descriptor(pdl, world, dtype, variant, S):
-    """PDL descriptor XML with the task variant pinned as Worker properties."""
+def variant_descriptor(pdl, world, dtype, variant):
+    """PDL descriptor XML with the task variant pinned as a Worker property."""
     if variant == "default":
         return pdl.descriptor_xml(world)
-    if variant == "ozaki2":
-        return pdl.descriptor_xml(world, props={"DGEMM_VARIANT": "ozaki2"})
-    if dtype == "f64":
-        return pdl.descriptor_xml(world, "ozaki", S)
-    return pdl.descriptor_xml(world, props={"SGEMM_VARIANT": "ozaki", "OZAKI_SLICES_F32": S})
-
-
-def ozaki_ops(rows, cols, K, S):
-    """INT8 tensor ops of the Ozaki variant: S slice diagonals, diagonal d is a
-    GEMM with K' = (d+1) Kc per K chunk (k_ozaki.cu)."""
-    nch = max(1, -(-K // 16384))
-    kc = -(-(-(-K // nch)) // 128) * 128
-    ops = 2.0 * rows * cols * kc * nch * S * (S + 1) / 2
-    return ops, f"K4 oz_gemm_2sm_kernel x {S * nch} slice-diagonal launches (tcgen05 kind::i8)"
+    return pdl.descriptor_xml(world, props={"DGEMM_VARIANT": "ozaki2"})
 
 
 OZ2_MODULI = (256, 255, 253, 251, 247, 241, 239, 233, 229, 227, 223, 217, 211, 199)
@@ -234,23 +219,22 @@ OZ2_CLUSTERS = 74
 
 def ozaki2_ops(rows, cols, K):
     n, p, nch, kc = ozaki2_moduli(K)
-    ops = 2.0 * rows * cols * kc * nch * n
+    # the n residue GEMMs and the certificate GEMM (one K chunk: K <= 65536)
+    ops = 2.0 * rows * cols * kc * nch * (n + 1)
     from paper_conf_ipps_sandrieserbp11_b200 import pdl
-    per_chunk = json.loads(pdl.query(f"ozaki2_launches/{rows}/{cols}/{n}/{OZ2_CLUSTERS}"))
-    return ops, (f"K6 oz2_gemm_persistent_kernel: {n * nch} residue GEMMs ({n} moduli x {nch} K chunk(s)) in "
-                 f"{len(per_chunk) * nch} persistent launch(es) of {per_chunk} moduli "
-                 f"(tcgen05 kind::i8, p = {p}) + CRT pass")
+    per_chunk = json.loads(pdl.query(f"ozaki2_launches/{rows}/{cols}/{n + 1}/{OZ2_CLUSTERS}"))
+    return ops, (f"K6 oz2_gemm_persistent_kernel: {n} residue GEMMs + 1 certificate GEMM in "
+                 f"{len(per_chunk) * nch} persistent launch(es) of {per_chunk} items "
+                 f"(tcgen05 kind::i8, p = {p}) + CRT pass + K1 recompute of uncertified elements")
 
 
-def variant_ops(variant, rows, cols, K, S):
-    return ozaki2_ops(rows, cols, K) if variant == "ozaki2" else ozaki_ops(rows, cols, K, S)
+def variant_ops(variant, rows, cols, K):
+    return ozaki2_ops(rows, cols, K)
 
 
-def variant_label(variant, dtype, S, K):
-    if variant == "ozaki2":
-        n = ozaki2_moduli(K)[0]
-        return f"{dtype}-ozaki2-i8x{n}", f"ozaki2 (K6/K7, {n} moduli, CRT)"
-    return f"{dtype}-ozaki-i8x{S}", f"ozaki (K4/K5, {S} int8 slices)"
+def variant_label(variant, dtype, K):
+    n = ozaki2_moduli(K)[0]
+    return f"{dtype}-ozaki2-i8x{n}", f"ozaki2 (K6/K7, {n} moduli + certificate GEMM, CRT, K1 recompute)"
 
 
 def edge_waste(rows, cols, dtype, ozaki):
@@ -457,11 +441,9 @@ def main():
 
     if args.variant == "ozaki2" and args.dtype != "f64":
         sys.exit("--variant ozaki2 is an FP64 task variant")
-    ozaki = args.variant in ("ozaki", "ozaki2")
-    S = args.slices or (6 if args.dtype == "f64" else 3)
-    args.slices = S
+    ozaki = args.variant == "ozaki2"
     # the task variant is pre-selected through the Worker's PDL properties (L1316-1326)
-    desc = variant_descriptor(pdl, world, args.dtype, args.variant, S)
+    desc = variant_descriptor(pdl, world, args.dtype, args.variant)
     if world == 1:
         pdl.load(desc)
     else:
@@ -515,20 +497,19 @@ def main():
     # ---- roofline of the dominant kernel (K1, or K2 for FP32) ----
     peak_dtype = "i8" if ozaki else args.dtype
     if ozaki:
-        pipe_flops, kname = variant_ops(args.variant, wp.rows, wp.cols, K, args.slices)
+        pipe_flops, kname = variant_ops(args.variant, wp.rows, wp.cols, K)
     else:
         pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
         kname = "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_2sm_kernel (tcgen05)"
-    traffic_key = (args.variant if args.dtype == "f64" else "ozaki32") if ozaki else args.dtype
+    traffic_key = args.variant if ozaki else args.dtype
     roofline = k_roofline(ktimes, args.steps, pipe_flops, peak_dtype, kname, traffic_key, args.config,
                           (wp.rows * K + K * wp.cols + wp.rows * wp.cols) * es, wp.rows, wp.cols, args.dtype, ozaki)
     peak_tf = roofline["peak"]
     if args.dtype == "f32":
         roofline["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
     if ozaki:
-        prods = "one residue GEMM per modulus" if args.variant == "ozaki2" else "S(S+1)/2 slice products"
-        roofline["note"] = (f"achieved counts int8 tensor ops ({prods}, 2 ops per MAC); "
-                            f"useful {args.dtype.upper()} FLOP = 2MNK")
+        roofline["note"] = ("achieved counts int8 tensor ops (one residue GEMM per modulus + the certificate "
+                            "GEMM, 2 ops per MAC); useful FP64 FLOP = 2MNK")
 
     # ---- e2e: host pinned operands through the public API, --steps steps ----
     e2e = None
@@ -594,10 +575,10 @@ def main():
 
     # ---- the other task variants on the same resident operands (PDL-selected) ----
     alts = []
-    others = [v for v in (("ozaki", "ozaki2") if args.dtype == "f64" else ("ozaki",)) if v != args.variant]
+    others = ["ozaki2"] if args.dtype == "f64" and args.variant != "ozaki2" else []
     for av in (others if world == 1 and not args.no_alt else []):
         pdl.unload()
-        pdl.load(variant_descriptor(pdl, 1, args.dtype, av, args.slices))
+        pdl.load(variant_descriptor(pdl, 1, args.dtype, av))
         pdl.set_stream(stream)
         for _ in range(2):
             step()
@@ -606,20 +587,23 @@ def main():
         pdl.kernel_times()
         ams, aclk = device_timed(torch, dist, step, args.steps, stream, world, dev, local, pdl.sync)
         akt = pdl.kernel_times()
-        aops, akname = variant_ops(av, M, N, K, args.slices)
+        guard = pdl.query_json("stats").get("ozaki_guard", [])
+        aops, akname = variant_ops(av, M, N, K)
         apeak, apsrc, _ = tensor_peak("i8")
         aach = aops / (float(np.mean(akt)) / 1e3) / 1e12 if akt else None
-        tol = "1e-12" if args.dtype == "f64" else "1e-5"
-        adt, alabel = variant_label(av, args.dtype, args.slices, K)
-        alts.append({"variant": f"{alabel}: {args.dtype.upper()} matmul on INT8 tcgen05",
+        adt, alabel = variant_label(av, args.dtype, K)
+        alts.append({"variant": f"{alabel}: FP64 matmul on INT8 tcgen05",
                      "dtype": adt,
                      "value": round(flops_total * args.steps / (ams / 1e3) / 1e9, 1), "unit": "GFLOP/s",
                      "ms_per_step": round(ams / args.steps, 3),
-                     "parity": f"max scaled err <= {tol} vs oracle (tests/test_gpu_{av}.py)",
+                     "parity": "certified |C - AB| <= 5e-13 |A||B| per element (DESIGN.md R21; "
+                               "tests/test_gpu_ozaki2.py, tests/test_ozaki2_certificate.py)",
+                     "certificate": {"tiles_checked": sum(w["tiles_checked"] for w in guard),
+                                     "elements_recomputed_by_k1": sum(w["elements_recomputed"] for w in guard)},
                      "roofline": {"bound": "tensor", "achieved": round(aach, 1) if aach else None,
                                   "peak": apeak, "unit": "TFLOP/s",
                                   "frac": round(aach / apeak, 4) if aach else None,
-                                  "traffic": ncu_traffic(av if args.dtype == "f64" else "ozaki32", args.config),
+                                  "traffic": ncu_traffic(av, args.config),
                                   "kernel": akname,
                                   "kernel_ms": round(float(np.mean(akt)), 3) if akt else None,
                                   "peak_source": apsrc},
@@ -642,11 +626,11 @@ def main():
             "metric": METRIC, "value": round(value, 1), "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-            "dtype": variant_label(args.variant, args.dtype, args.slices, K)[0] if ozaki else args.dtype,
+            "dtype": variant_label(args.variant, args.dtype, K)[0] if ozaki else args.dtype,
             "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} ({args.dtype})",
             "config": {"workload": workload,
                        "M": M, "N": N, "K": K, "tile": c.tile, "parallelism": f"block2d {wp.Gr}x{wp.Gc}",
-                       "task_variant": (variant_label(args.variant, args.dtype, args.slices, K)[1] if ozaki else
+                       "task_variant": (variant_label(args.variant, args.dtype, K)[1] if ozaki else
                                         ("dmma (K1)" if args.dtype == "f64" else "3xtf32 (K3+K2)")),
                        "l2": "inputs larger than L2 (operands >> 126 MB), no flush needed"},
             "pct_of_tensor_peak": round(100 * (pipe_flops / flops_worker) * value / world / (peak_tf * 1e3), 2),

@@ -116,14 +116,18 @@ extern "C" {
  *   the sum exceeds its SMs).  This emulates heterogeneous Workers on one GPU.
  * Task variants (one task interface, several implementations pre-selected per
  *   Worker from its properties): DGEMM_VARIANT = dmma
- *   (default: K1, IEEE FP64 on DMMA) | ozaki (K4/K5, OZAKI_SLICES, default 6,
- *   OZAKI_ROUNDING nearest | trunc) | ozaki2 (K6/K7, OZAKI2_MODULI, default
- *   the fewest giving OZAKI2_BITS = 43 scaling bits); SGEMM_VARIANT = 3xtf32
- *   (default: K3 + K2) | ozaki (OZAKI_SLICES_F32, default 3).  The Ozaki
- *   variants assume finite inputs and meet the 1e-12 / 1e-5 bars for rows and
- *   columns of moderate dynamic range (R19, R20).  RELATIVE_SPEED
- *   weights the BLOCK mapping.  Env PDL_<PROPERTY> overrides a property for
- *   every Worker.
+ *   (default: K1, IEEE FP64 on DMMA) | ozaki2 (K6/K7: Ozaki scheme II on the
+ *   INT8 tensor cores, OZAKI2_MODULI, default the fewest giving OZAKI2_BITS =
+ *   43 scaling bits, finite inputs only).  ozaki2 carries a certificate
+ *   (OZAKI2_GUARD = on | off, default on; OZAKI2_GUARD_TOL = tau, default
+ *   5e-13): one more INT8 GEMM bounds every element's error against a lower
+ *   bound of |A||B|, and K1 recomputes each element whose bound exceeds
+ *   tau |A||B| -- so |C - AB| <= tau |A||B| holds element by element for any
+ *   finite input (R20, R21); tasks with K > 65536 run K1.
+ *   SGEMM_VARIANT = 3xtf32 (default: K3 + K2).  The round-1 variant "ozaki"
+ *   (Ozaki scheme I) is retired: PDL_EUNSUPPORTED at pdl_run.
+ *   RELATIVE_SPEED weights the BLOCK mapping.  Env PDL_<PROPERTY> overrides a
+ *   property for every Worker.
  * This process is the single Master driving every Worker of the descriptor.
  * Env: PDL_DRY_RUN=1 skips device binding (plans only; no device work);
  *   PDL_ALLOW_OVERSUBSCRIBE=1 lets several Workers share a device.
@@ -263,8 +267,11 @@ int pdl_plan(int64_t M, int64_t N, int64_t K, int64_t tile, const char *group,
  *   "ozaki2_plan/<K>[/<bits>[/<moduli>]]" (JSON; no pdl_load needed: moduli,
  *   scaling bits p, K chunks, CRT weights W_t and M as decimal strings, and
  *   "crt": "fp64" when the FP64-pipe reconstruction applies, else "int"),
- *   "ozaki2_launches/<rows>/<cols>/<moduli>/<clusters>" (JSON list, no pdl_load
- *   needed: moduli per persistent residue-GEMM launch of one K chunk),
+ *   "ozaki2_launches/<rows>/<cols>/<items>/<clusters>" (JSON list, no pdl_load
+ *   needed: GEMM items -- moduli, plus 1 for the certificate -- per persistent
+ *   launch of one K chunk), "ozaki_guard" inside "stats" (JSON: per Worker the
+ *   128 x 128 tiles the Ozaki-II certificate checked in the last run and the
+ *   tiles / elements K1 recomputed),
  *   "concurrent_tasks/f64" | "concurrent_tasks/f32" ("yes" when tasks of
  *   different PDL_TASK_SLOTs may overlap on different streams).
  * Writes a NUL-terminated string (truncated to len-1) and returns the full

@@ -78,7 +78,8 @@ template <int BM_>
 __global__ void __launch_bounds__(k1::Shape<BM_>::THREADS, k1::Shape<BM_>::MIN_CTAS)
     dgemm_k1_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     double *__restrict__ C, int64_t ldc, int M, int N, int K, int tiles_m, int tiles_n,
-                    int group_m, int vec_ok, int *dyn_next, int *dyn_mine) {
+                    int group_m, int vec_ok, int *dyn_next, int *dyn_mine, const uint32_t *tile_mask,
+                    int64_t ld_mask, const uint32_t *elem_mask, int64_t ld_emask) {
     using S = k1::Shape<BM_>;
     constexpr int BM = S::BM, BN = S::BN, BK = S::BK, STAGES = S::STAGES, NCONS = S::NCONS;
     constexpr int A_BYTES = S::A_BYTES, B_SUB_BYTES = S::B_SUB_BYTES, STAGE_BYTES = S::STAGE_BYTES;
@@ -103,6 +104,8 @@ __global__ void __launch_bounds__(k1::Shape<BM_>::THREADS, k1::Shape<BM_>::MIN_C
     const int gsz = min(tiles_m - first_m, group_m);
     const int tm = first_m + (bid % per_group) % gsz;
     const int tn = (bid % per_group) / gsz;
+    // recompute set of the Ozaki-II certificate: other tiles exit untouched
+    if (tile_mask && !tile_mask[(int64_t)((tm * BM) >> 7) * ld_mask + ((tn * BN) >> 7)]) return;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
@@ -230,7 +233,13 @@ __global__ void __launch_bounds__(k1::Shape<BM_>::THREADS, k1::Shape<BM_>::MIN_C
             const int col = tn * BN + 32 * wn + 16 * q + 4 * (int)p;
             const double v0 = acc[mi][2 * q][0], v1 = acc[mi][2 * q + 1][0];
             const double v2 = acc[mi][2 * q][1], v3 = acc[mi][2 * q + 1][1];
-            if (vec_ok && col + 3 < N) {
+            if (elem_mask) {   // recompute set: only the flagged elements (4 bits of one word)
+                const uint32_t bits = col < N ? elem_mask[(int64_t)row * ld_emask + (col >> 5)] >> (col & 31) : 0u;
+                if ((bits & 1u) && col < N) crow[col] = v0;
+                if ((bits & 2u) && col + 1 < N) crow[col + 1] = v1;
+                if ((bits & 4u) && col + 2 < N) crow[col + 2] = v2;
+                if ((bits & 8u) && col + 3 < N) crow[col + 3] = v3;
+            } else if (vec_ok && col + 3 < N) {
                 *reinterpret_cast<double2 *>(crow + col) = make_double2(v0, v1);
                 *reinterpret_cast<double2 *>(crow + col + 2) = make_double2(v2, v3);
             } else {
@@ -276,7 +285,8 @@ static int k1_pick_bm(int64_t M, int64_t N, int sms, bool dynamic) {
 template <int BM_>
 static cudaError_t launch_k1_shape(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
                                    double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, int dev,
-                                   cudaStream_t stream, int *dyn_next, int *dyn_mine) {
+                                   cudaStream_t stream, int *dyn_next, int *dyn_mine, const uint32_t *tile_mask,
+                                   int64_t ld_mask, const uint32_t *elem_mask, int64_t ld_emask) {
     using S = k1::Shape<BM_>;
     CUtensorMap ta, tb;
     if (!make_map_2d(enc, &ta, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 8, A, (uint64_t)K, (uint64_t)M, (uint64_t)lda, S::BK,
@@ -297,7 +307,8 @@ static cudaError_t launch_k1_shape(EncodeTiledFn enc, const double *A, int64_t l
     const char *gm = getenv("PDL_GROUP_M_K1");   // raster tuning knob
     const int group_m = gm && atoi(gm) > 0 ? atoi(gm) : k1::GROUP_M * (128 / BM_);
     dgemm_k1_kernel<BM_><<<tiles_m * tiles_n, S::THREADS, S::SMEM_BYTES, stream>>>(
-        ta, tb, C, ldc, (int)M, (int)N, (int)K, tiles_m, tiles_n, group_m, vec_ok, dyn_next, dyn_mine);
+        ta, tb, C, ldc, (int)M, (int)N, (int)K, tiles_m, tiles_n, group_m, vec_ok, dyn_next, dyn_mine, tile_mask,
+        ld_mask, elem_mask, ld_emask);
     return cudaGetLastError();
 }
 
@@ -316,14 +327,17 @@ int worker_sms() {
 // 16 B aligned base, lda*8 and ldb*8 multiples of 16 (checked by the runtime).
 cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
                             double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream,
-                            int *dyn_next, int *dyn_mine) {
+                            int *dyn_next, int *dyn_mine, const uint32_t *tile_mask, int64_t ld_mask,
+                            const uint32_t *elem_mask, int64_t ld_emask) {
     if (M <= 0 || N <= 0) return cudaSuccess;
     int dev = 0;
     cudaGetDevice(&dev);
     const int sms = worker_sms();
     if (k1_pick_bm(M, N, sms, dyn_next != nullptr) == 64)
-        return launch_k1_shape<64>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine);
-    return launch_k1_shape<128>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine);
+        return launch_k1_shape<64>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine, tile_mask,
+                                   ld_mask, elem_mask, ld_emask);
+    return launch_k1_shape<128>(enc, A, lda, B, ldb, C, ldc, M, N, K, dev, stream, dyn_next, dyn_mine, tile_mask,
+                                ld_mask, elem_mask, ld_emask);
 }
 
 

@@ -71,7 +71,12 @@ static int bits_for(u128 M, int64_t Kc) {
     return p;
 }
 
-Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits) {
+bool oz2_guard_ok(const Ozaki2Plan &P, int64_t K) {
+    return P.nch == 1 && 16129 * P.Kc < ((int64_t)1 << 31) && P.p >= 7 &&
+           P.p + 2 + ilog2_ceil(K < 1 ? 1 : K) <= 62;
+}
+
+Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits, bool guard) {
     Ozaki2Plan P;
     P.nch = (int)((K + OZ2_KC_MAX - 1) / OZ2_KC_MAX);
     if (P.nch < 1) P.nch = 1;
@@ -107,7 +112,9 @@ Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits
     P.Hw[0] = (unsigned long long)H;
     P.Hw[1] = (unsigned long long)(H >> 64);
     P.Md = (double)P.Mw[1] * 18446744073709551616.0 + (double)P.Mw[0];
-    P.ld8 = (int64_t)P.nch * n * P.Kc;
+    P.check = guard && oz2_guard_ok(P, K) ? 1 : 0;
+    P.np = n + P.check;
+    P.ld8 = (int64_t)P.nch * P.np * P.Kc;
     P.a8_bytes = (size_t)rows * P.ld8;
     P.b8_bytes = (size_t)cols * P.ld8;
     return P;
@@ -170,6 +177,21 @@ __device__ __forceinline__ double scaled_magic(double x, int sh) {
     return rint(scale2(x, sh)) + magic;
 }
 
+// Certificate operand of one scaled integer v = rint(x 2^(p-e)) (|v| <= 2^p):
+// max(0, |v| - 1) 2^(7-p) rounded down, in [0, 127] and at most |x| 2^(7-e)
+// (|v| - 1 < |x| 2^(p-e)); and the row / column sum term 2|v| + 1 for x != 0
+// (|x| 2^(p-e) <= |v| + 1/2).  DESIGN.md R21.
+__device__ __forceinline__ int cert8(double v, int p) {
+    return (int)floor(fmax(fabs(v) - 1.0, 0.0) * pow2d(7 - p));
+}
+__device__ __forceinline__ unsigned long long cert_sum(double v, bool nz) {
+    return nz ? (unsigned long long)(2.0 * fabs(v) + 1.0) : 0ull;   // < 2^53: exact
+}
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x, int width) {
+    for (int o = 1; o < width; o <<= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+    return x;
+}
+
 // Low bytes of eight ints packed little-endian into 64 bits (PRMT, no shifts).
 __device__ __forceinline__ uint64_t pack8(const int (&r)[8]) {
     const unsigned a = __byte_perm(__byte_perm(r[0], r[1], 0x0040), __byte_perm(r[2], r[3], 0x0040), 0x5410);
@@ -204,7 +226,7 @@ __global__ void oz2_split_rows_kernel(const double *__restrict__ A, int64_t lda,
 #pragma unroll
             for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? rint(scale2(row[k8 + j], p - e)) : 0.0;
             const int64_t c = k8 / Kc, kk = k8 - c * Kc;
-            int8_t *o = out + (c * n) * Kc + kk;
+            int8_t *o = out + (c * n) * Kc + kk;   // (no certificate plane: np == n here)
             for (int t = 0; t < n; ++t) {
                 uint64_t pk = 0;
 #pragma unroll
@@ -233,13 +255,16 @@ __global__ void __launch_bounds__(256) oz2_rowmax_kernel(const double *__restric
 }
 
 __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
-                                                               int64_t K, int n, int p, int64_t Kc, int nch,
+                                                               int64_t K, int n, int np, int p, int64_t Kc, int nch,
                                                                int8_t *__restrict__ A8, int64_t ld8,
-                                                               const int *__restrict__ ea, int vec) {
+                                                               const int *__restrict__ ea, int vec,
+                                                               unsigned long long *__restrict__ sa) {
     const int64_t groups = (int64_t)nch * Kc / 8;   // Kc % 128 == 0
     const bool fast = p <= 50;                      // |A'| < 2^51: res8_fast (uniform)
+    const bool check = np > n;                      // certificate plane n (one K chunk)
     // 2-D grid-stride: rows along y, 8-k groups along x (no 64-bit divisions)
-    for (int64_t row = blockIdx.y; row < M; row += gridDim.y)
+    for (int64_t row = blockIdx.y; row < M; row += gridDim.y) {
+    unsigned long long rsum = 0;
     for (int64_t g8 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g8 < groups;
          g8 += (int64_t)gridDim.x * blockDim.x) {
         const int64_t k8 = g8 * 8;
@@ -258,7 +283,10 @@ __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__r
             for (int j = 0; j < 8; ++j) v[j] = (k8 + j < K) ? r[k8 + j] : 0.0;
         }
         const int64_t c = nch == 1 ? 0 : k8 / Kc, kk = k8 - c * Kc;
-        int8_t *o = A8 + row * ld8 + (c * n) * Kc + kk;
+        int8_t *o = A8 + row * ld8 + (c * np) * Kc + kk;
+        bool nz[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) nz[j] = v[j] != 0.0;
         if (fast) {
             int lo[8];
 #pragma unroll
@@ -283,6 +311,20 @@ __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__r
                 *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
             }
         }
+        if (check) {
+            int cc[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                cc[j] = cert8(v[j], p);
+                rsum += cert_sum(v[j], nz[j]);
+            }
+            *reinterpret_cast<uint64_t *>(o + (int64_t)n * Kc) = pack8(cc);
+        }
+    }
+    if (check) {   // the warp's 32 lanes share the row (blockDim.x = 256 along k)
+        rsum = warp_sum_u64(rsum, 32);
+        if ((threadIdx.x & 31) == 0 && rsum) atomicAdd(sa + row, rsum);
+    }
     }
 }
 
@@ -301,8 +343,9 @@ __global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int
 // thread reads its column's 8 consecutive k as four 16-byte shared loads (every
 // quarter-warp on distinct banks) and writes one 8-byte word per modulus.
 __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
-    const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int n, int p, int64_t Kc, int nch,
-    const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb) {
+    const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int n, int np, int p, int64_t Kc, int nch,
+    const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
+    unsigned long long *__restrict__ sb) {
     constexpr int PITCH = 66;
     __shared__ __align__(16) double tl[32 * PITCH];
     const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
@@ -316,7 +359,9 @@ __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
     const int64_t Kpad = (int64_t)nch * Kc;
     const int nl = threadIdx.x >> 3, g = threadIdx.x & 7;
     const int64_t col = n0 + nl, k8 = k0 + 8 * g;
-    if (col >= N || k8 >= Kpad) return;
+    const bool check = np > n;
+    unsigned long long csum = 0;
+    if (col < N && k8 < Kpad) {   // (predicated, not returned: the certificate sum reduces over g)
     const int f = exp_of_max2(__longlong_as_double((long long)bmax[col]));
     if (blockIdx.y == 0 && g == 0) fb[col] = f;
     double v[8];
@@ -326,8 +371,11 @@ __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
         v[2 * j] = x.x;
         v[2 * j + 1] = x.y;
     }
+    bool nz[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) nz[j] = v[j] != 0.0;
     const int64_t c = k8 / Kc, kk = k8 - c * Kc;
-    int8_t *o = Bt8 + col * ld8 + (c * n) * Kc + kk;
+    int8_t *o = Bt8 + col * ld8 + (c * np) * Kc + kk;
     if (p <= 50) {
         int lo[8];
 #pragma unroll
@@ -351,6 +399,20 @@ __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
             for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
             *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
         }
+    }
+    if (check) {
+        int cc[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            cc[j] = cert8(v[j], p);
+            csum += cert_sum(v[j], nz[j]);
+        }
+        *reinterpret_cast<uint64_t *>(o + (int64_t)n * Kc) = pack8(cc);
+    }
+    }
+    if (check) {   // the 8 lanes of a column are consecutive: reduce, one atomic per column and CTA
+        csum = warp_sum_u64(csum, 8);
+        if (g == 0 && csum) atomicAdd(sb + col, csum);
     }
 }
 
@@ -555,12 +617,16 @@ static cudaError_t upload_moduli(const Ozaki2Plan &P) {
 }
 
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
-                                  int8_t *A8, int *ea, cudaStream_t s, int *launches) {
+                                  int8_t *A8, int *ea, cudaStream_t s, int *launches, unsigned long long *sa) {
     if (rows <= 0) return cudaSuccess;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
+    if (P.check) {
+        if (!sa) return cudaErrorInvalidValue;
+        if ((e = cudaMemsetAsync(sa, 0, (size_t)rows * sizeof(unsigned long long), s)) != cudaSuccess) return e;
+    }
     const char *mode = getenv("PDL_OZ2_SPLIT");
-    if (mode && !strcmp(mode, "rows")) {
+    if (mode && !strcmp(mode, "rows") && !P.check) {
         const int blocks = (int)(rows < split_ctas() ? rows : split_ctas());
         oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
         if (launches) *launches += 1;
@@ -570,16 +636,22 @@ cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, in
     const int64_t groups = (int64_t)P.nch * P.Kc / 8;
     dim3 grid((unsigned)std::min<int64_t>((groups + 255) / 256, 64), (unsigned)std::min<int64_t>(rows, 65535));
     const int vec = ((reinterpret_cast<uintptr_t>(A) & 15u) == 0 && (lda & 1) == 0) ? 1 : 0;
-    oz2_residue_rows_kernel<<<grid, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea, vec);
+    oz2_residue_rows_kernel<<<grid, 256, 0, s>>>(A, lda, rows, K, P.n, P.np, P.p, P.Kc, P.nch, A8, P.ld8, ea, vec,
+                                                 sa);
     if (launches) *launches += 2;
     return cudaGetLastError();
 }
 
 cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
-                                  int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s) {
+                                  int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s,
+                                  unsigned long long *sb) {
     if (cols <= 0) return cudaSuccess;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
+    if (P.check) {
+        if (!sb) return cudaErrorInvalidValue;
+        if ((e = cudaMemsetAsync(sb, 0, (size_t)cols * sizeof(unsigned long long), s)) != cudaSuccess) return e;
+    }
     e = cudaMemsetAsync(bmax, 0, (size_t)cols * sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
     if (K > 0) {
@@ -588,7 +660,8 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
     }
     const int64_t Kpad = (int64_t)P.nch * P.Kc;
     dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 63) / 64));
-    oz2_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, P.n, P.p, P.Kc, P.nch, bmax, Bt8, P.ld8, fb);
+    oz2_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, P.n, P.np, P.p, P.Kc, P.nch, bmax, Bt8, P.ld8, fb,
+                                               sb);
     return cudaGetLastError();
 }
 

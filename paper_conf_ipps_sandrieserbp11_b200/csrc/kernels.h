@@ -25,9 +25,15 @@ int worker_sms();   // the partition's SMs if set, else the current device's
 // A, B device pointers, 16 B aligned, lda*8 % 16 == 0, ldb*8 % 16 == 0.
 cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, const double *B, int64_t ldb,
                             double *C, int64_t ldc, int64_t M, int64_t N, int64_t K, cudaStream_t stream,
-                            int *dyn_next = nullptr, int *dyn_mine = nullptr);
+                            int *dyn_next = nullptr, int *dyn_mine = nullptr, const uint32_t *tile_mask = nullptr,
+                            int64_t ld_mask = 0, const uint32_t *elem_mask = nullptr, int64_t ld_emask = 0);
 // dyn_next / dyn_mine (K1, K2): DYNAMIC distribution -- CTAs claim raster tiles
 // from the shared counter *dyn_next and count their claims in *dyn_mine.
+// tile_mask (K1): compute only the 128 x 128 tiles t with tile_mask[(row / 128) *
+// ld_mask + col / 128] != 0; the other CTAs exit before touching memory.
+// elem_mask: of those, store only the elements whose bit (col % 32) of
+// elem_mask[row * ld_emask + col / 32] is set (the Ozaki-II certificate's recompute
+// set).  A stored element is bitwise the plain K1 result.
 
 // K3 -- TF32 hi/lo split pre-pass.  Kp = K rounded up to K2's BK (32).
 //  split_rows:   A (M x K, lda, fp32)  -> Ahi, Alo  (M x Kp, K-major, zero padded)
@@ -43,35 +49,6 @@ cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t 
 cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
                                cudaStream_t stream);
-// K4/K5 -- FP64 DGEMM variant on INT8 tensor cores (Ozaki scheme, k_ozaki.cu).
-// Slices: A8 = rows x ld8 int8, row layout [chunk][slice][Kc]; Bt8 = cols x ld8
-// int8, row layout [chunk][S-1-slice][Kc]; ea/fb = per-row / per-column
-// power-of-two exponents; bmax = cols x u64 scratch.
-constexpr int64_t OZ_KC_MAX = 16384;   // (d+1)*Kc*127^2 < 2^31 for S <= 8
-struct OzakiLayout {
-    int S = 7, nch = 1;
-    int rn = 0;          // slice rounding: 0 = truncation, 1 = round-to-nearest
-    int64_t Kc = 0, ld8 = 0;
-    size_t a8_bytes = 0, b8_bytes = 0;
-};
-OzakiLayout ozaki_layout(int64_t rows, int64_t cols, int64_t K, int S);
-cudaError_t launch_ozaki_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
-                                 int8_t *A8, int *ea, cudaStream_t s);
-cudaError_t launch_ozaki_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
-                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s);
-cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
-                              const OzakiLayout &L, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                              cudaStream_t stream, int *launches);
-// FP32 task variant on the same machinery: FP32 inputs promoted exactly, each
-// diagonal added in double and rounded once into the FP32 C.
-cudaError_t launch_ozaki_split_a(const float *A, int64_t lda, int64_t rows, int64_t K, const OzakiLayout &L,
-                                 int8_t *A8, int *ea, cudaStream_t s);
-cudaError_t launch_ozaki_split_b(const float *B, int64_t ldb, int64_t K, int64_t cols, const OzakiLayout &L,
-                                 int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s);
-cudaError_t launch_ozaki_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const int *ea, const int *fb,
-                              const OzakiLayout &L, float *C, int64_t ldc, int64_t rows, int64_t cols,
-                              cudaStream_t stream, int *launches);
-
 // K6/K7 -- FP64 DGEMM variant "ozaki2" (Ozaki scheme II: integer scaling and the
 // Chinese remainder theorem over INT8 GEMMs, k_ozaki2.cu).  A' = rint(A 2^(p-e_i))
 // row-wise, B' = rint(B 2^(p-f_j)) column-wise (|A'|, |B'| <= 2^p); for each of n
@@ -86,6 +63,8 @@ struct Ozaki2Plan {
     int n = 0;                            // moduli in use
     int p = 0;                            // integer scaling bits
     int nch = 1;
+    int check = 0;                        // 1: plane n of the operands is the certificate operand
+    int np = 0;                           // operand planes per K chunk: n + check
     int64_t Kc = 0, ld8 = 0;
     size_t a8_bytes = 0, b8_bytes = 0;
     int m[OZ2_MAX_MODULI] = {};
@@ -93,18 +72,46 @@ struct Ozaki2Plan {
     unsigned long long Mw[2] = {}, Hw[2] = {};      // M and floor(M / 2)
     double Md = 0.0;
 };
-// nmod = 0: the fewest moduli that give p >= bits for this K chunk.
-Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits);
+// nmod = 0: the fewest moduli that give p >= bits for this K chunk.  guard: add the
+// certificate plane when the plan admits it (oz2_guard_ok).
+Ozaki2Plan ozaki2_plan(int64_t rows, int64_t cols, int64_t K, int nmod, int bits, bool guard = false);
+// The componentwise certificate (R21) needs one K chunk, an exact INT32
+// certificate sum (127^2 Kc < 2^31) and the u64 row / column sums ((2^(p+1)+1) K < 2^63).
+bool oz2_guard_ok(const Ozaki2Plan &P, int64_t K);
+// Certificate of one Ozaki-II launch (R21).  With A' = rint(A 2^(p-e_i))
+// and B' = rint(B 2^(p-f_j)) the componentwise error of C_ij is at most
+//   2^(e_i+f_j-2p-2) (sa_i + sb_j + min(sa_i, sb_j))  + rounding of X to double,
+// sa_i = sum_k (2|A'_ik| + 1)[A_ik != 0] (sb_j likewise), and D_ij = sum_k |A_ik||B_kj|
+// is at least 2^(e_i+f_j-14) X^c_ij, X^c = a^c b^c with a^c_ik = max(0, |A'_ik| - 1) >>
+// (p - 7) in [0, 127] (b^c likewise): the certificate plane, one more INT8 GEMM.  A
+// 128 x 128 tile holding an element whose bound exceeds tau D_ij is flagged and
+// recomputed by K1 (IEEE FP64); K1 stores only the flagged elements, so every
+// element's value depends on its own certificate alone (bitwise invariance, R14).
+struct Oz2Guard {
+    unsigned long long *sa = nullptr;     // rows of the launch's rectangle
+    unsigned long long *sb = nullptr;     // its columns
+    uint32_t *flags = nullptr;            // tile (row / 128, col / 128) at flags[(row / 128) * ldf + col / 128]
+    int64_t ldf = 0;
+    uint32_t *emask = nullptr;            // element (row, col): bit col % 32 of emask[row * ldw + col / 32]
+    int64_t ldw = 0;
+    unsigned *fallback = nullptr;         // [0] += flagged tiles, [1] += flagged elements (stats)
+    double tau = 5e-13;
+};
 // Persistent K6 launches per K chunk for n moduli on a rows x cols rectangle with
 // `clusters` co-resident CTA pairs (k_ozaki.cu).
 int oz2_launches_per_chunk(int n, int64_t rows, int64_t cols, int clusters);
+// sa / sb (P.check): the certificate's row / column sums, zeroed and accumulated here.
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
-                                  int8_t *A8, int *ea, cudaStream_t s, int *launches = nullptr);
+                                  int8_t *A8, int *ea, cudaStream_t s, int *launches = nullptr,
+                                  unsigned long long *sa = nullptr);
 cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
-                                  int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s);
+                                  int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s,
+                                  unsigned long long *sb = nullptr);
+// guard (P.check): the certificate GEMM runs as one more item of the persistent
+// launches and flags tiles into guard->flags (zeroed by the caller).
 cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
                                uint8_t *R, int64_t ldr, int64_t plane, int64_t rows, int64_t cols, cudaStream_t s,
-                               int *launches);
+                               int *launches, const Oz2Guard *guard = nullptr);
 // The plan admits the FP64-pipe CRT pass (M < 2^117, M >= 2^(2p + lk + 1) (1 + 1/64));
 // otherwise launch_ozaki2_reconstruct uses the 128-bit integer pass.  PDL_OZ2_CRT=int
 // forces the integer pass.

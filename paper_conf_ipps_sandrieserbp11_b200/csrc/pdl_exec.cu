@@ -63,32 +63,17 @@ int ensure_aux(WorkerCtx &w) {
     return PDL_OK;
 }
 
-// Task variant of a Worker (task repository + static pre-selection, L1307-1326):
-//   FP64: PDL property DGEMM_VARIANT ("dmma" default | "ozaki"), OZAKI_SLICES (default 6)
-//   FP32: PDL property SGEMM_VARIANT ("3xtf32" default | "ozaki"), OZAKI_SLICES_F32 (default 3)
-// OZAKI_ROUNDING ("nearest" default | "trunc") for both; env PDL_<NAME> overrides
-// the descriptor (tests, bench).
+// The retired task variant "ozaki" (Ozaki scheme I, round 1's K4/K5): true when the
+// Worker's PDL property DGEMM_VARIANT (FP64) / SGEMM_VARIANT (FP32), or env
+// PDL_<NAME>, names it -- run_rect then reports PDL_EUNSUPPORTED.
 bool worker_ozaki(const WorkerCtx &w, bool f64, int *slices, int *rn) {
     const char *vname = f64 ? "DGEMM_VARIANT" : "SGEMM_VARIANT";
-    const char *sname = f64 ? "OZAKI_SLICES" : "OZAKI_SLICES_F32";
     std::string v;
     if (const char *e = getenv((std::string("PDL_") + vname).c_str())) v = e;
     else if (const Property *p = g->model.prop(w.pu, vname)) v = p->value;
-    if (lower(trim(v)) != "ozaki") return false;
-    // Defaults from the measured accuracy sweeps (profiles/r01_ozaki_accuracy*.txt):
-    // FP64 -- round-to-nearest slices, S = 6 -> max scaled error 3.7e-14 at K = 16384
-    // (truncation needs S = 7 for 3.0e-14; truncation S = 6 gives 1.6e-12);
-    // FP32 -- S = 3 (8+7+7 bits) -> max 3.3e-7 (K = 256) .. 4.3e-8 (K = 16384), 1e-5 bar.
-    int s = f64 ? 6 : 3;
-    if (const char *e = getenv((std::string("PDL_") + sname).c_str())) s = atoi(e);
-    else if (const Property *p = g->model.prop(w.pu, sname)) s = atoi(p->value.c_str());
-    *slices = std::max(2, std::min(8, s));
-    // OZAKI_ROUNDING: "nearest" (default) | "trunc"
-    std::string r;
-    if (const char *e = getenv("PDL_OZAKI_ROUNDING")) r = e;
-    else if (const Property *p = g->model.prop(w.pu, "OZAKI_ROUNDING")) r = p->value;
-    *rn = lower(trim(r)) == "trunc" ? 0 : 1;
-    return true;
+    *slices = 0;
+    *rn = 1;
+    return lower(trim(v)) == "ozaki";
 }
 
 // FP64 variant "ozaki2" (Ozaki scheme II, K6/K7): DGEMM_VARIANT = "ozaki2";
@@ -117,25 +102,44 @@ bool worker_sgemm_ozaki2(const WorkerCtx &w) {
     return lower(trim(v)) == "ozaki2";
 }
 
-// Ozaki exponent arrays of a task: the B side [bmax: cols u64][fb: cols int] in the
-// shared BUF_OZE of slot 0 (it does not move with `rows`, so a prepared B survives
-// row-chunk tasks, REUSE_B), the A side ea (rows int) after it for slot 0, in the
-// slot's own BUF_OZE otherwise.
+// Ozaki-II per-row / per-column arrays of a task: the B side [bmax: cols u64][sb:
+// cols u64][fb: cols int] in the shared BUF_OZE of slot 0 (it does not move with
+// `rows`, so a prepared B survives row-chunk tasks, REUSE_B), the A side [ea: rows
+// int][sa: rows u64] after it for slot 0, in the slot's own BUF_OZE otherwise.
+// sa / sb: the certificate's row / column sums (R21).
 static int oz_exponents(WorkerCtx &w, int slot, int64_t rows, int64_t cols, unsigned long long **bmax, int **fb,
-                        int **ea) {
+                        int **ea, unsigned long long **sb, unsigned long long **sa) {
     void *p = nullptr, *q = nullptr;
-    const size_t bside = (size_t)round_up(cols, 2) * 4 + (size_t)cols * 8;
-    int rc = ensure_buf(w, BUF_OZE, bside + (slot == 0 ? (size_t)round_up(rows, 2) * 4 : 0), &p);
+    const size_t bside = (size_t)cols * 16 + (size_t)round_up(cols, 2) * 4;
+    const size_t aside = (size_t)round_up(rows, 2) * 4 + (size_t)rows * 8;
+    int rc = ensure_buf(w, BUF_OZE, bside + (slot == 0 ? aside : 0), &p);
     if (rc) return rc;
     *bmax = (unsigned long long *)p;
-    *fb = (int *)(*bmax + cols);
+    *sb = *bmax + cols;
+    *fb = (int *)(*sb + cols);
     if (slot == 0) {
         *ea = *fb + round_up(cols, 2);
-        return PDL_OK;
+    } else {
+        if ((rc = ensure_buf(w, slot_buf(BUF_OZE, slot), aside, &q))) return rc;
+        *ea = (int *)q;
     }
-    if ((rc = ensure_buf(w, slot_buf(BUF_OZE, slot), (size_t)round_up(rows, 2) * 4, &q))) return rc;
-    *ea = (int *)q;
+    *sa = (unsigned long long *)(*ea + round_up(rows, 2));
     return PDL_OK;
+}
+
+// Certificate of the Ozaki-II variant (R21): PDL property OZAKI2_GUARD =
+// "on" (default) | "off", OZAKI2_GUARD_TOL = tau (default 5e-13: the certified
+// componentwise bound |C - AB| <= tau |A||B|, half the 1e-12 bar); env PDL_<NAME>.
+static bool worker_oz2_guard(const WorkerCtx &w, double *tau) {
+    std::string v;
+    if (const char *e = getenv("PDL_OZAKI2_GUARD")) v = e;
+    else if (const Property *p = g->model.prop(w.pu, "OZAKI2_GUARD")) v = p->value;
+    *tau = 5e-13;
+    if (const char *e = getenv("PDL_OZAKI2_GUARD_TOL")) *tau = atof(e);
+    else if (const Property *p = g->model.prop(w.pu, "OZAKI2_GUARD_TOL")) *tau = atof(p->value.c_str());
+    if (!(*tau > 0.0)) *tau = 5e-13;
+    v = lower(trim(v));
+    return !(v == "off" || v == "0" || v == "false");
 }
 
 // K2 shape for an nr x nc launch: the 1-SM 128 x 128 kernel when the CTA-pair
@@ -206,22 +210,29 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     }
     const bool piped = RB * CP > 1;
     // Task variant of this Worker, pre-selected from its PDL properties (task
-    // repository + static pre-selection, L1307-1326): FP64 K1 (DMMA) or K4
-    // (Ozaki), FP32 K3+K2 (3xTF32) or K4 (Ozaki).
-    int oz_slices = 0;
-    int oz_rn = 0;
+    // repository + static pre-selection, L1307-1326): FP64 K1 (DMMA) or K6/K7
+    // (Ozaki scheme II with its certificate), FP32 K3+K2 (3xTF32).
     int oz2_nmod = 0, oz2_bits = 0;
-    if (!f64 && K > 0 && worker_sgemm_ozaki2(w))
-        return set_err(PDL_EUNSUPPORTED, "SGEMM_VARIANT ozaki2: Ozaki scheme II is an FP64 variant (use ozaki)");
-    const bool ozaki2 = K > 0 && f64 && worker_ozaki2(w, &oz2_nmod, &oz2_bits);
-    const bool ozaki = K > 0 && !ozaki2 && worker_ozaki(w, f64, &oz_slices, &oz_rn);
-    pdlk::OzakiLayout OL;
-    if (ozaki) {
-        OL = pdlk::ozaki_layout(rows, cols, K, oz_slices);
-        OL.rn = oz_rn;
+    if (K > 0 && (f64 ? false : worker_sgemm_ozaki2(w)))
+        return set_err(PDL_EUNSUPPORTED, "SGEMM_VARIANT ozaki2: Ozaki scheme II is an FP64 variant");
+    {
+        int sl = 0, rn = 0;
+        if (K > 0 && worker_ozaki(w, f64, &sl, &rn))
+            return set_err(PDL_EUNSUPPORTED,
+                           "%s_VARIANT ozaki (Ozaki scheme I) is retired: its dropped slice products bound the "
+                           "error only by %s of K max|a| max|b|, which cannot certify the componentwise bar; use %s",
+                           f64 ? "DGEMM" : "SGEMM", f64 ? "~2^-42" : "~2^-21",
+                           f64 ? "DGEMM_VARIANT=ozaki2 (certified, DESIGN.md R21) or dmma" : "the default 3xtf32");
     }
+    bool ozaki2 = K > 0 && f64 && worker_ozaki2(w, &oz2_nmod, &oz2_bits);
+    double oz2_tau = 0.0;
+    const bool oz2_guard = ozaki2 && worker_oz2_guard(w, &oz2_tau);
     pdlk::Ozaki2Plan P2;
-    if (ozaki2) P2 = pdlk::ozaki2_plan(rows, cols, K, oz2_nmod, oz2_bits);
+    if (ozaki2) {
+        P2 = pdlk::ozaki2_plan(rows, cols, K, oz2_nmod, oz2_bits, oz2_guard);
+        // the certificate needs one K chunk (K <= 65536): longer tasks run K1 (IEEE FP64)
+        if (oz2_guard && !P2.check) ozaki2 = false;
+    }
     // the prepared-B signature of this task (PDL_TASK_REUSE_B)
     WorkerCtx::BSig want;
     want.valid = true;
@@ -230,10 +241,10 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     want.K = K;
     want.cols = cols;
     want.dtype = t.dtype;
-    want.oz = ozaki ? 1 : ozaki2 ? 2 : 0;
-    want.S = ozaki ? OL.S : ozaki2 ? P2.n : 0;
-    want.rn = ozaki ? OL.rn : ozaki2 ? P2.p : 0;
-    const bool prep_b = K > 0 && (ozaki || ozaki2 || !f64);
+    want.oz = ozaki2 ? 2 + P2.check : 0;
+    want.S = ozaki2 ? P2.n : 0;
+    want.rn = ozaki2 ? P2.p : 0;
+    const bool prep_b = K > 0 && (ozaki2 || !f64);
     // A task that re-prepares B while another task of this Worker may still read
     // the shared B-side buffers on another stream (a side-stream chunk task, slot
     // != 0, after the main task was replayed from a graph or ran on other
@@ -276,7 +287,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     // FP32 split buffers (K-major hi/lo of A rows and of B^T rows)
     const int64_t Kp = round_up(std::max<int64_t>(K, 1), pdlk::K2_BK);
     float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
-    if (!f64 && K > 0 && !ozaki) {
+    if (!f64 && K > 0) {
         if ((rc = ensure(BUF_AHI, (size_t)(rows * Kp * 4), &p))) return rc;
         ahi = (float *)p;
         if ((rc = ensure(BUF_ALO, (size_t)(rows * Kp * 4), &p))) return rc;
@@ -295,27 +306,39 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
 
     int8_t *a8 = nullptr, *b8 = nullptr;
     int *oz_ea = nullptr, *oz_fb = nullptr;
-    unsigned long long *oz_bmax = nullptr;
-    if (ozaki) {
-        if ((rc = ensure(BUF_OZA, OL.a8_bytes, &p))) return rc;
-        a8 = (int8_t *)p;
-        if ((rc = ensure_buf(w, BUF_OZB, OL.b8_bytes, &p))) return rc;
-        b8 = (int8_t *)p;
-        if ((rc = oz_exponents(w, slot, rows, cols, &oz_bmax, &oz_fb, &oz_ea))) return rc;
-    }
-
+    unsigned long long *oz_bmax = nullptr, *oz_sa = nullptr, *oz_sb = nullptr;
     uint8_t *oz2_R = nullptr;
     int64_t oz2_ldr = 0, oz2_plane = 0;
+    pdlk::Oz2Guard G2;
     if (ozaki2) {
         if ((rc = ensure(BUF_OZA, P2.a8_bytes, &p))) return rc;
         a8 = (int8_t *)p;
         if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
         b8 = (int8_t *)p;
-        if ((rc = oz_exponents(w, slot, rows, cols, &oz_bmax, &oz_fb, &oz_ea))) return rc;
+        if ((rc = oz_exponents(w, slot, rows, cols, &oz_bmax, &oz_fb, &oz_ea, &oz_sb, &oz_sa))) return rc;
         oz2_ldr = round_up(cols, 16);
         oz2_plane = oz2_ldr * rows;
         if ((rc = ensure(BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
         oz2_R = (uint8_t *)p;
+        if (P2.check) {
+            // recompute flags of the rectangle's 128 x 128 tiles, and the Worker's
+            // count of flagged tiles in this run (pdl_query "stats")
+            G2.ldf = (cols + 127) / 128;
+            if ((rc = ensure(BUF_OZF, (size_t)(((rows + 127) / 128) * G2.ldf * 4), &p))) return rc;
+            G2.flags = (uint32_t *)p;
+            G2.ldw = (cols + 31) / 32;
+            if ((rc = ensure(BUF_OZM, (size_t)(rows * G2.ldw * 4), &p))) return rc;
+            G2.emask = (uint32_t *)p;
+            if ((rc = ensure_buf(w, BUF_OZG, 16, &p))) return rc;
+            G2.fallback = (unsigned *)p;
+            if (w.guard_epoch != g->run_epoch) {
+                CUDA_TRY(cudaMemsetAsync(G2.fallback, 0, 16, w.stream));
+                w.guard_epoch = g->run_epoch;
+                w.guard_tiles = 0;
+            }
+            w.guard_tiles += ((rows + 127) / 128) * G2.ldf;
+            G2.tau = oz2_tau;
+        }
     }
 
     // B prepared by a previous task of this Worker (PDL_TASK_REUSE_B)?  Decided after
@@ -389,7 +412,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (!a_prep[i]) {
                     a_prep[i] = 1;
                     e = pdlk::launch_ozaki2_split_a((const double *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K, P2,
-                                                    a8 + r0 * P2.ld8, oz_ea + r0, cs, &w.launches);
+                                                    a8 + r0 * P2.ld8, oz_ea + r0, cs, &w.launches, oz_sa + r0);
                     if (piped) {
                         ev_sa[i] = ev_get(w, evn);
                         CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
@@ -400,7 +423,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (e == cudaSuccess && !b_prep[j] && !b_ready) {
                     b_prep[j] = 1;
                     e = pdlk::launch_ozaki2_split_b((const double *)(Bd + (size_t)c0 * es), ldb, K, nc, P2,
-                                                    b8 + c0 * P2.ld8, oz_fb + c0, oz_bmax + c0, cs);
+                                                    b8 + c0 * P2.ld8, oz_fb + c0, oz_bmax + c0, cs, oz_sb + c0);
                     w.launches += 2;
                     if (e == cudaSuccess && mark_bprep(cs)) return set_err(PDL_ECUDA, "event record failed");
                     if (piped) {
@@ -414,55 +437,34 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
                 int nl = 0;
                 uint8_t *Rs = oz2_R + r0 * oz2_ldr + c0;
-                e = pdlk::launch_ozaki2_gemm(enc, a8 + r0 * P2.ld8, b8 + c0 * P2.ld8, P2, Rs, oz2_ldr, oz2_plane, nr,
-                                             nc, cs, &nl);
+                // the certificate of this band / panel (r0, c0: multiples of 128)
+                pdlk::Oz2Guard gs = G2;
+                if (P2.check) {
+                    gs.sa = oz_sa + r0;
+                    gs.sb = oz_sb + c0;
+                    gs.flags = G2.flags + (r0 / 128) * G2.ldf + c0 / 128;
+                    gs.emask = G2.emask + r0 * G2.ldw + c0 / 32;
+                    e = cudaMemset2DAsync(gs.flags, (size_t)(G2.ldf * 4), 0, (size_t)((nc + 127) / 128) * 4,
+                                          (size_t)((nr + 127) / 128), cs);
+                    if (e == cudaSuccess)
+                        e = cudaMemset2DAsync(gs.emask, (size_t)(G2.ldw * 4), 0, (size_t)((nc + 31) / 32) * 4,
+                                              (size_t)nr, cs);
+                }
+                if (e == cudaSuccess)
+                    e = pdlk::launch_ozaki2_gemm(enc, a8 + r0 * P2.ld8, b8 + c0 * P2.ld8, P2, Rs, oz2_ldr, oz2_plane,
+                                                 nr, nc, cs, &nl, P2.check ? &gs : nullptr);
                 if (e == cudaSuccess)
                     e = pdlk::launch_ozaki2_reconstruct(Rs, oz2_ldr, oz2_plane, oz_ea + r0, oz_fb + c0, P2,
                                                         (double *)Cs, ldcd, nr, nc, cs);
+                // flagged tiles: recomputed by K1 over the same operands (IEEE FP64)
+                if (e == cudaSuccess && P2.check) {
+                    e = pdlk::launch_dgemm_k1(enc, (const double *)(Ad + (size_t)(r0 * lda) * es), lda,
+                                              (const double *)(Bd + (size_t)c0 * es), ldb, (double *)Cs, ldcd, nr, nc,
+                                              K, cs, nullptr, nullptr, gs.flags, G2.ldf, gs.emask, G2.ldw);
+                    ++nl;
+                }
                 if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
                 w.launches += nl + 1;
-            } else if (ozaki) {
-                // K5 slicing of this band / panel once, shared by both compute streams
-                if (!a_prep[i]) {
-                    a_prep[i] = 1;
-                    const char *Ab = Ad + (size_t)(r0 * lda) * es;
-                    e = f64 ? pdlk::launch_ozaki_split_a((const double *)Ab, lda, nr, K, OL, a8 + r0 * OL.ld8,
-                                                         oz_ea + r0, cs)
-                            : pdlk::launch_ozaki_split_a((const float *)Ab, lda, nr, K, OL, a8 + r0 * OL.ld8,
-                                                         oz_ea + r0, cs);
-                    w.launches += 1;
-                    if (piped) {
-                        ev_sa[i] = ev_get(w, evn);
-                        CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
-                    }
-                } else if (ev_sa[i]) {
-                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sa[i], 0));
-                }
-                if (e == cudaSuccess && !b_prep[j] && !b_ready) {
-                    b_prep[j] = 1;
-                    const char *Bp = Bd + (size_t)c0 * es;
-                    e = f64 ? pdlk::launch_ozaki_split_b((const double *)Bp, ldb, K, nc, OL, b8 + c0 * OL.ld8,
-                                                         oz_fb + c0, oz_bmax + c0, cs)
-                            : pdlk::launch_ozaki_split_b((const float *)Bp, ldb, K, nc, OL, b8 + c0 * OL.ld8,
-                                                         oz_fb + c0, oz_bmax + c0, cs);
-                    w.launches += 2;
-                    if (e == cudaSuccess && mark_bprep(cs)) return set_err(PDL_ECUDA, "event record failed");
-                    if (piped) {
-                        ev_sb[j] = ev_get(w, evn);
-                        CUDA_TRY(cudaEventRecord(ev_sb[j], cs));
-                    }
-                } else if (ev_sb[j]) {
-                    CUDA_TRY(cudaStreamWaitEvent(cs, ev_sb[j], 0));
-                }
-                if (e != cudaSuccess) return set_err(PDL_ECUDA, "K5 slicing launch failed: %s", cudaGetErrorString(e));
-                if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
-                int nl = 0;
-                e = f64 ? pdlk::launch_ozaki_gemm(enc, a8 + r0 * OL.ld8, b8 + c0 * OL.ld8, oz_ea + r0, oz_fb + c0,
-                                                  OL, (double *)Cs, ldcd, nr, nc, cs, &nl)
-                        : pdlk::launch_ozaki_gemm(enc, a8 + r0 * OL.ld8, b8 + c0 * OL.ld8, oz_ea + r0, oz_fb + c0,
-                                                  OL, (float *)Cs, ldcd, nr, nc, cs, &nl);
-                if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
-                w.launches += nl;
             } else if (f64) {
                 if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
                 e = pdlk::launch_dgemm_k1(enc, (const double *)(Ad + (size_t)(r0 * lda) * es), lda,
@@ -596,8 +598,8 @@ int run_dynamic(const Task &t, const std::vector<int> &gw) {
         int n2, b2;
         if (K > 0 && (worker_ozaki(*w, f64, &sl, &rn) || (f64 && worker_ozaki2(*w, &n2, &b2))))
             return set_err(PDL_EUNSUPPORTED,
-                           "DYNAMIC needs a single-launch task variant (dmma / 3xtf32); Worker %s runs Ozaki "
-                           "(S diagonal launches updating C)",
+                           "DYNAMIC needs a single-launch task variant (dmma / 3xtf32); Worker %s runs an Ozaki "
+                           "variant (residue GEMMs, CRT pass and certificate recompute)",
                            g->model.pus[w->pu].id.c_str());
     }
     WorkerCtx &own = *ws[0];
@@ -843,6 +845,7 @@ int execute(bool sync) {
         w.xpending = false;
     }
     g->xfer = XferStats();
+    ++g->run_epoch;
     // Green-context streams are non-blocking: give them the ordering of the
     // blocking Worker streams (after the prior work of the legacy default stream,
     // or of the caller's stream given to pdl_set_stream, and that stream after

@@ -44,6 +44,7 @@ struct DevBuf {
 
 enum BufSlot { BUF_A = 0, BUF_B, BUF_C, BUF_AHI, BUF_ALO, BUF_BHI, BUF_BLO, BUF_OZA, BUF_OZB, BUF_OZE, BUF_OZR,
                BUF_XA, BUF_XB,   // A row-panel / B column-panel gathered by the Worker<->Worker exchange
+               BUF_OZF, BUF_OZM, BUF_OZG,   // Ozaki-II certificate: tile flags, element mask (per slot), counters
                BUF_COUNT };
 // Scratch slots (PDL_TASK_SLOT): the per-task buffers (A staging, C staging, A
 // split / slices / residues, A exponents, residue planes) exist once per slot, so
@@ -120,6 +121,9 @@ struct WorkerCtx {
     std::vector<cudaEvent_t> xev_pool;
     cudaEvent_t ev_xdone = nullptr;
     bool xpending = false;
+    // Ozaki-II certificate of the current run: tiles checked (host) and the device
+    // counter of tiles recomputed by K1 (BUF_OZG), reset at the first use in a run
+    long long guard_epoch = -1, guard_tiles = 0;
 };
 
 constexpr size_t kMaxKernelTimes = 4096;
@@ -155,6 +159,7 @@ struct XferStats {
 struct State {
     bool loaded = false;
     XferStats xfer;
+    long long run_epoch = 0;   // pdl_run / pdl_run_async calls since pdl_load
     bool dry_run = false;
     bool oversub = false;
     int rank = 0, nranks = 1;

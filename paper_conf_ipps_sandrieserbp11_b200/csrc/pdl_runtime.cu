@@ -459,6 +459,26 @@ int pdl_query(const char *key, char *out, size_t len) {
               << ",\"worker_to_worker\":" << g->xfer.w2w << ",\"exchange_tasks\":" << g->xfer.exchange_tasks
               << ",\"master_worker_ic\":\"" << json_escape(mw_ic) << "\",\"worker_worker_ic\":\""
               << json_escape(ww_ic) << "\"}";
+            // Ozaki-II certificate of the last run (valid after pdl_sync): 128 x 128 tiles
+            // checked per Worker and those recomputed by K1 (R21)
+            bool any_guard = false;
+            for (auto &w : g->workers) any_guard |= w.guard_epoch == g->run_epoch;
+            if (any_guard && !g->dry_run) {
+                o << ",\"ozaki_guard\":[";
+                bool f1 = true;
+                for (auto &w : g->workers) {
+                    if (w.guard_epoch != g->run_epoch) continue;
+                    unsigned cnt[2] = {0, 0};
+                    cudaSetDevice(w.device);
+                    if (cudaMemcpy(cnt, w.buf[BUF_OZG].ptr, sizeof cnt, cudaMemcpyDeviceToHost) != cudaSuccess)
+                        cudaGetLastError();
+                    o << (f1 ? "" : ",") << "{\"id\":\"" << json_escape(m.pus[w.pu].id)
+                      << "\",\"tiles_checked\":" << w.guard_tiles << ",\"tiles_recomputed\":" << cnt[0]
+                      << ",\"elements_recomputed\":" << cnt[1] << "}";
+                    f1 = false;
+                }
+                o << "]";
+            }
             // tiles each Worker claimed in the last DYNAMIC task (valid after pdl_sync)
             if (g->dyn_n > 0 && g->dyn && !g->dry_run) {
                 std::vector<int> claims(g->dyn_n + 1, 0);

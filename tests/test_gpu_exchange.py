@@ -72,8 +72,7 @@ CASES = [
     (8, np.float64, 1000, 700, 300, 64, None),
     (8, np.float32, 1000, 700, 300, 64, None),
     (8, np.float64, 777, 513, 1000, 128, "ozaki2"),
-    (4, np.float64, 777, 513, 1000, 128, "ozaki"),
-    (8, np.float32, 1500, 1100, 260, 128, "ozaki"),
+    (4, np.float64, 1500, 1100, 260, 128, "ozaki2"),
 ]
 
 

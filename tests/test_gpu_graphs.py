@@ -54,8 +54,7 @@ def runs(desc, A, B, n, graph, tile=0, host=False, pinned=False):
         pdl.unload()
 
 
-@pytest.mark.parametrize("dt,variant", [(np.float64, None), (np.float32, None), (np.float64, "ozaki"),
-                                        (np.float64, "ozaki2"), (np.float32, "ozaki")])
+@pytest.mark.parametrize("dt,variant", [(np.float64, None), (np.float32, None), (np.float64, "ozaki2")])
 def test_graph_replay_bitwise(dt, variant):
     A = W.uniform((1000, 700), dt, 1)
     B = W.uniform((700, 900), dt, 2)
@@ -76,8 +75,11 @@ def test_graph_replay_bitwise(dt, variant):
 
 def test_graph_multiworker_pinned_pipelined(monkeypatch):
     """4 Workers, pinned host operands through the pipelined staging path
-    (copy-in / copy-out / second compute stream, all joined by events)."""
+    (copy-in / copy-out / second compute stream, all joined by events).  The
+    Worker<->Worker exchange (which runs uncaptured, its chunk tasks on device
+    panels) is off, so each Worker stages its panels through this path."""
     monkeypatch.setenv("PDL_PIPELINE", "force")
+    monkeypatch.setenv("PDL_EXCHANGE", "0")
     A = W.signed((777, 513), np.float64, 3)
     B = W.signed((513, 640), np.float64, 4)
     ref, _, _, _ = runs(pdl.descriptor_xml(4), A, B, 1, graph=False, tile=64, host=True, pinned=True)

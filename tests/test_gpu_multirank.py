@@ -50,16 +50,12 @@ def test_distributed_ragged_8(overlap):
     _run(8, "f64", 1000, 700, 300, 64, env_extra={"PDL_OVERLAP_A": overlap})
 
 
-def test_distributed_ozaki_4():
-    _run(4, "f64", 777, 513, 1000, 128, "ozaki")
-
-
 def test_distributed_ozaki2_4():
     _run(4, "f64", 777, 513, 1000, 128, "ozaki2")
 
 
 @pytest.mark.parametrize("G,dt,variant", [(4, "f64", None), (8, "f64", None), (8, "f32", None),
-                                          (8, "f64", "ozaki"), (8, "f64", "ozaki2"), (4, "f32", "ozaki")])
+                                          (8, "f64", "ozaki2"), (4, "f64", "ozaki2")])
 def test_concurrent_chunk_groups_bitwise(G, dt, variant, monkeypatch):
     """runtime.compute_groups with the later chunk groups on side streams, each
     task in its own libpdl scratch slot (PDL_TASK_SLOT) and reusing the B panel

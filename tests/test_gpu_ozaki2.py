@@ -23,7 +23,8 @@ from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
 
 @pytest.fixture(autouse=True)
 def _env(monkeypatch):
-    for k in ("PDL_DRY_RUN", "PDL_DGEMM_VARIANT", "PDL_OZAKI2_MODULI", "PDL_OZAKI2_BITS"):
+    for k in ("PDL_DRY_RUN", "PDL_DGEMM_VARIANT", "PDL_OZAKI2_MODULI", "PDL_OZAKI2_BITS", "PDL_OZAKI2_GUARD",
+              "PDL_OZAKI2_GUARD_TOL"):
         monkeypatch.delenv(k, raising=False)
     monkeypatch.setenv("PDL_ALLOW_OVERSUBSCRIBE", "1")
     pdl.unload()
@@ -75,8 +76,10 @@ def test_variant_selected_and_launch_count(monkeypatch):
     dC = torch.empty((300, 100), dtype=torch.float64, device="cuda")
     pdl.task_matmul(dA, dB, dC)
     pdl.run()
-    n = pdl.query_json("stats")["launches"] - 5
+    st = pdl.query_json("stats")
+    n = st["launches"] - 5 - 2    # - the certificate GEMM and K1's recompute launch
     assert 11 <= n <= 13, n       # fewer moduli suffice for K = 200
+    assert st["ozaki_guard"][0]["elements_recomputed"] == 0
     check(dC.cpu().numpy(), A, B)
 
 
@@ -194,8 +197,11 @@ def test_scaling_bits_above_50_residue_fallback():
 
 
 @pytest.mark.parametrize("moduli,tol", [(13, 1e-13), (14, 1e-14), (11, 1e-9)])
-def test_moduli_count_accuracy(moduli, tol):
-    """Fewer moduli force fewer scaling bits p (|X| <= K 2^(2p) < M/2)."""
+def test_moduli_count_accuracy(moduli, tol, monkeypatch):
+    """Fewer moduli force fewer scaling bits p (|X| <= K 2^(2p) < M/2): the
+    raw accuracy of the residue arithmetic, certificate off (with it on, 11
+    moduli send every element to K1)."""
+    monkeypatch.setenv("PDL_OZAKI2_GUARD", "off")
     A = W.uniform((256, 4096), np.float64, 41)
     B = W.signed((4096, 256), np.float64, 42)
     check(oz2_matmul(A, B, moduli=moduli), A, B, tol=tol)
@@ -242,3 +248,120 @@ def test_k0_and_tiny():
     check(oz2_matmul(A, B), A, B)           # 53-bit inputs, p-bit scaling: within the bar
     A, B = np.array([[3.0]]), np.array([[-0.625]])
     assert np.array_equal(oz2_matmul(A, B), A @ B)     # short mantissas: exact
+
+
+# ---- the certificate (R21) ----------------------------------------
+
+def oz2_run(A, B, guard=True, workers=1, tile=0, variant="ozaki2"):
+    """C and the certificate stats of one run (device-resident operands)."""
+    props = {"DGEMM_VARIANT": variant}
+    if variant == "ozaki2" and not guard:
+        props["OZAKI2_GUARD"] = "off"
+    pdl.load(pdl.descriptor_xml(workers, props=props))
+    try:
+        dA, dB = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+        dC = torch.full((A.shape[0], B.shape[1]), float("nan"), dtype=torch.float64, device="cuda")
+        pdl.task_matmul(dA, dB, dC, tile=tile)
+        pdl.run()
+        st = pdl.query_json("stats")
+        return dC.cpu().numpy(), st.get("ozaki_guard", [])
+    finally:
+        pdl.unload()
+
+
+def recomputed(g):
+    return sum(w["elements_recomputed"] for w in g)
+
+
+def adversarial(kind, seed):
+    rng = np.random.default_rng(seed)
+    if kind == "huge_times_zero":
+        # [2^60, 1] x [0, 1]^T: the 1 is below Ozaki II's 2^-43 row resolution
+        A = W.uniform((300, 200), np.float64, seed)
+        B = W.uniform((200, 260), np.float64, seed + 1)
+        A[7, :2] = [2.0 ** 60, 1.0]
+        A[7, 2:] = 0.0
+        B[:2, 11] = [0.0, 1.0]
+        A[150, 3] = 2.0 ** 60          # one huge element meeting zeros of B
+        B[3, :] = 0.0
+        return A, B
+    if kind == "in_row_spread":
+        # every element scaled by 2^u, u uniform in [-60, 60]: rows and columns
+        # spanning 120 binades
+        A = W.signed((256, 384), np.float64, seed) * np.exp2(rng.integers(-60, 61, (256, 384)))
+        B = W.signed((384, 200), np.float64, seed + 1) * np.exp2(rng.integers(-60, 61, (384, 200)))
+        return A, B
+    if kind.startswith("cancel_k"):
+        # small K with signed entries and exact cancellation partners: D_ij stays
+        # ~|a||b| while C_ij is tiny, and D_ij can be far below K max|a_i| max|b_j|
+        K = int(kind[8:])
+        A = W.signed((512, K), np.float64, seed) * np.exp2(rng.integers(-20, 21, (512, K)))
+        B = W.signed((K, 384), np.float64, seed + 1) * np.exp2(rng.integers(-20, 21, (K, 384)))
+        if K >= 2:
+            A[:, 1] = -A[:, 0] * (1 + 2.0 ** -30)
+            B[1, :] = B[0, :]
+        return A, B
+    raise ValueError(kind)
+
+
+KINDS = ["huge_times_zero", "in_row_spread"] + [f"cancel_k{k}" for k in (2, 3, 4, 8, 16)]
+
+
+@pytest.mark.parametrize("kind", KINDS)
+def test_certificate_holds_on_adversarial_inputs(kind):
+    """Seeded adversarial inputs at the plain 1e-12 componentwise bar through
+    DGEMM_VARIANT=ozaki2: the elements whose certified bound exceeds tau D_ij
+    are recomputed by K1; the others are certified."""
+    A, B = adversarial(kind, 7)
+    C, g = oz2_run(A, B)
+    check(C, A, B)
+    if kind in ("huge_times_zero", "in_row_spread"):
+        assert recomputed(g) > 0, "these inputs need the K1 recompute"
+    if kind == "huge_times_zero":
+        assert C[7, 11] == 1.0
+
+
+@pytest.mark.parametrize("kind", ["huge_times_zero", "in_row_spread"])
+def test_without_the_certificate_the_bar_fails(kind):
+    """Negative control: the same inputs with OZAKI2_GUARD=off break the 1e-12
+    bar, so the certificate is what holds it."""
+    A, B = adversarial(kind, 7)
+    C, _ = oz2_run(A, B, guard=False)
+    Cref, D = oracle.matmul(A, B)
+    assert oracle.scaled_error(C, Cref, D).max() > 1e-12
+
+
+def test_recomputed_elements_are_k1_bits_and_the_rest_ozaki_bits():
+    """Each element is either certified (bitwise the unguarded Ozaki-II value)
+    or recomputed (bitwise the K1 value) -- decided from its own row / column
+    sums and certificate product only."""
+    A, B = adversarial("in_row_spread", 11)
+    C, g = oz2_run(A, B)
+    C_off, _ = oz2_run(A, B, guard=False)
+    C_k1, _ = oz2_run(A, B, variant="dmma")
+    same_oz = C == C_off
+    same_k1 = C == C_k1
+    assert np.all(same_oz | same_k1)
+    assert recomputed(g) >= np.count_nonzero(~same_oz)
+
+
+def test_certificate_invariant_under_workers_and_tiles():
+    """The recompute set is per element, so Worker count and task tile change
+    no bit of the guarded result either (R14)."""
+    A, B = adversarial("cancel_k4", 13)
+    ref, _ = oz2_run(A, B)
+    for workers, tile in ((2, 64), (4, 32), (8, 0)):
+        C, _ = oz2_run(A, B, workers=workers, tile=tile)
+        assert np.array_equal(C, ref), (workers, tile)
+
+
+@pytest.mark.parametrize("name", ["C2", "C3"])
+def test_certificate_passes_benign_workloads(name):
+    """U[0,1) and U[-1,1) workloads of the configs are certified everywhere:
+    no element goes to K1 (the guard costs one INT8 GEMM, no recompute)."""
+    A, B = W.config_inputs(name, np.float64)
+    C, g = oz2_run(A, B)
+    assert recomputed(g) == 0
+    assert sum(w["tiles_checked"] for w in g) == -(-A.shape[0] // 128) * -(-B.shape[1] // 128)
+    Cs, gs = oz2_run(2 * A - 1, 2 * B - 1)
+    assert recomputed(gs) == 0

@@ -24,24 +24,16 @@ import workloads as W  # noqa: E402
 from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
 
 ROWS = [("C1", "f64", 1, None), ("C1", "f32", 1, None), ("C2", "f64", 1, None), ("C2", "f32", 1, None),
-        ("C2", "f64", 1, "ozaki"), ("C2", "f64", 1, "ozaki2"), ("C2", "f32", 1, "ozaki"), ("C3", "f64", 2, None),
-        ("C3", "f64", 4, None), ("C3", "f32", 4, None), ("C3", "f64", 4, "ozaki"), ("C3", "f64", 4, "ozaki2"),
-        ("C3", "f32", 4, "ozaki"), ("C0", "f64", 1, None), ("C0", "f64", 2, None), ("C0", "f64", 2, "ozaki"),
-        ("C0", "f64", 2, "ozaki2"),
-        ("C4", "f64", 1, None), ("C4", "f32", 1, None), ("C4", "f64", 1, "ozaki"), ("C4", "f64", 1, "ozaki2"),
-        ("C4", "f32", 1, "ozaki"),
-        ("C5", "f64", 8, None), ("C5", "f32", 8, None), ("C5", "f64", 8, "ozaki"), ("C5", "f64", 8, "ozaki2"),
-        ("C5", "f32", 8, "ozaki")]
+        ("C2", "f64", 1, "ozaki2"), ("C3", "f64", 2, None), ("C3", "f64", 4, None), ("C3", "f32", 4, None),
+        ("C3", "f64", 4, "ozaki2"), ("C0", "f64", 1, None), ("C0", "f64", 2, None), ("C0", "f64", 2, "ozaki2"),
+        ("C4", "f64", 1, None), ("C4", "f32", 1, None), ("C4", "f64", 1, "ozaki2"),
+        ("C5", "f64", 8, None), ("C5", "f32", 8, None), ("C5", "f64", 8, "ozaki2")]
 
 
 def descriptor(G, dt, variant):
     if variant == "ozaki2":
         return pdl.descriptor_xml(G, props={"DGEMM_VARIANT": "ozaki2"})
-    if variant != "ozaki":
-        return pdl.descriptor_xml(G)
-    if dt == "f64":
-        return pdl.descriptor_xml(G, "ozaki")
-    return pdl.descriptor_xml(G, props={"SGEMM_VARIANT": "ozaki"})
+    return pdl.descriptor_xml(G)
 
 
 def timed(fn, steps, stream):
