@@ -85,6 +85,19 @@ extern "C" {
                                 of this Worker: reuse its prepared form (FP32 split / Ozaki
                                 slices) instead of recomputing it; ignored when no matching
                                 prepared B exists */
+#define PDL_TASK_PREP_A 64u  /* with PDL_TASK_LOCAL: only prepare A -- write the task variant's
+                                prepared form of A's M rows (K wide) to C as packed rows of
+                                pdl_query("prepared_a/<dtype>/<K>") bytes (FP32 3xTF32:
+                                [TF32 hi: Kp floats][TF32 lo: Kp floats], Kp = K rounded up to
+                                32); B and N are ignored.  C: 16-byte aligned memory of the
+                                Worker's device.  PDL_EUNSUPPORTED for variants that exchange
+                                raw rows (query answers 0: FP64 dmma, ozaki2) */
+#define PDL_TASK_PREPARED_A 128u
+                             /* with PDL_TASK_LOCAL: A holds M prepared rows (PDL_TASK_PREP_A
+                                on a Worker with the same variant and K) in this Worker's
+                                memory region; lda is ignored; the task skips A's preparation.
+                                The multi-rank runtime exchanges prepared A chunks so each
+                                Worker prepares only its own chunk */
 #define PDL_TASK_SLOT(s) (((unsigned)(s) & 3u) << 4)
                              /* scratch slot s in 0..2 of the Worker: a task's own buffers (A
                                 split / slices / residues and exponents, residue planes,

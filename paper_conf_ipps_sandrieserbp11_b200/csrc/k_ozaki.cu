@@ -237,6 +237,7 @@ struct Oz2Moduli {
     // holding an element with (sa_i + sb_j + min(sa_i, sb_j)) > thr X^c_ij
     int check = -1;
     const unsigned long long *sa = nullptr, *sb = nullptr;
+    long long sa_ld = 1;
     uint32_t *flags = nullptr;
     long long ldf = 0;
     uint32_t *emask = nullptr;
@@ -373,7 +374,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
             const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
             const int cbase = tn * BN + cg * EPI_COLS;
             uint8_t *prow = R + (int64_t)t * plane + (int64_t)row * ldr + cbase;
-            const unsigned long long sai = cert && row < M ? mods.sa[row] : 0ull;
+            const unsigned long long sai = cert && row < M ? mods.sa[(int64_t)row * mods.sa_ld] : 0ull;
             mbar_wait(bar_tfull, ti & 1u);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #pragma unroll 1
@@ -620,8 +621,9 @@ static void oz2_persistent_launch(const CUtensorMap &ta, const CUtensorMap &tb, 
 
 cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
                                uint8_t *R, int64_t ldr, int64_t plane, int64_t rows, int64_t cols, cudaStream_t stream,
-                               int *launches, const Oz2Guard *guard) {
+                               int *launches, const Oz2Guard *guard, int64_t lda8) {
     using namespace koz;
+    if (lda8 <= 0) lda8 = P.ld8;
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 15u) || (ldr & 15) || (plane & 15)) return cudaErrorInvalidValue;
     if (P.check && (!guard || !guard->sa || !guard->sb || !guard->flags || !guard->emask || !guard->fallback))
@@ -655,6 +657,7 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
     }
     if (P.check) {
         all.sa = guard->sa;
+        all.sa_ld = guard->sa_ld;
         all.sb = guard->sb;
         all.flags = guard->flags;
         all.ldf = guard->ldf;
@@ -687,7 +690,7 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
                 const int t0 = l * np / nl, t1 = (l + 1) * np / nl, gl = t1 - t0;
                 const int64_t off = ((int64_t)c * np + t0) * P.Kc;
                 CUtensorMap ta, tb;
-                if (!map_i8(enc, &ta, A8 + off, (uint64_t)(gl * P.Kc), (uint64_t)rows, (uint64_t)P.ld8, BM) ||
+                if (!map_i8(enc, &ta, A8 + off, (uint64_t)(gl * P.Kc), (uint64_t)rows, (uint64_t)lda8, BM) ||
                     !map_i8(enc, &tb, Bt8 + off, (uint64_t)(gl * P.Kc), (uint64_t)cols, (uint64_t)P.ld8, BNH))
                     return cudaErrorInvalidValue;
                 oz2_persistent_launch<2>(ta, tb, R + ((int64_t)c * P.n + t0) * plane, ldr, plane, rows, cols, P.Kc,
@@ -701,7 +704,7 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
         for (int t = 0; t < np; ++t) {
             const int64_t off = ((int64_t)c * np + t) * P.Kc;
             CUtensorMap ta, tb;
-            if (!map_i8(enc, &ta, A8 + off, (uint64_t)P.Kc, (uint64_t)rows, (uint64_t)P.ld8, BM) ||
+            if (!map_i8(enc, &ta, A8 + off, (uint64_t)P.Kc, (uint64_t)rows, (uint64_t)lda8, BM) ||
                 !map_i8(enc, &tb, Bt8 + off, (uint64_t)P.Kc, (uint64_t)cols, (uint64_t)P.ld8, BNH))
                 return cudaErrorInvalidValue;
             if (t == P.n) {   // the certificate item: a persistent launch of one item group

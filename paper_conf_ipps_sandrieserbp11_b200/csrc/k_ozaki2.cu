@@ -202,7 +202,7 @@ __device__ __forceinline__ uint64_t pack8(const int (&r)[8]) {
 // One CTA per row (grid-stride): A (rows x K) -> A8 rows [c][t][kk].
 __global__ void oz2_split_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M, int64_t K, int n,
                                       int p, int64_t Kc, int nch, int8_t *__restrict__ A8, int64_t ld8,
-                                      int *__restrict__ ea) {
+                                      int *__restrict__ ea, int64_t ea_ld) {
     __shared__ double red[32];
     const int64_t Kpad = (int64_t)nch * Kc;
     for (int64_t i = blockIdx.x; i < M; i += gridDim.x) {
@@ -219,7 +219,7 @@ __global__ void oz2_split_rows_kernel(const double *__restrict__ A, int64_t lda,
         }
         __syncthreads();
         const int e = exp_of_max2(red[0]);
-        if (threadIdx.x == 0) ea[i] = e;
+        if (threadIdx.x == 0) ea[i * ea_ld] = e;
         int8_t *out = A8 + i * ld8;
         for (int64_t k8 = (int64_t)threadIdx.x * 8; k8 < Kpad; k8 += (int64_t)blockDim.x * 8) {
             double v[8];
@@ -243,7 +243,7 @@ __global__ void oz2_split_rows_kernel(const double *__restrict__ A, int64_t lda,
 // items -- every thread busy and 8 independent loads in flight, instead of one CTA
 // walking a row twice (oz2_split_rows_kernel, kept as PDL_OZ2_SPLIT=rows).
 __global__ void __launch_bounds__(256) oz2_rowmax_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
-                                                         int64_t K, int *__restrict__ ea) {
+                                                         int64_t K, int *__restrict__ ea, int64_t ea_ld) {
     const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
     if (row >= M) return;
     const int lane = threadIdx.x & 31;
@@ -251,14 +251,14 @@ __global__ void __launch_bounds__(256) oz2_rowmax_kernel(const double *__restric
     double mx = 0.0;
     for (int64_t k = lane; k < K; k += 32) mx = fmax(mx, fabs(r[k]));
     for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-    if (lane == 0) ea[row] = exp_of_max2(mx);
+    if (lane == 0) ea[row * ea_ld] = exp_of_max2(mx);
 }
 
 __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
                                                                int64_t K, int n, int np, int p, int64_t Kc, int nch,
                                                                int8_t *__restrict__ A8, int64_t ld8,
-                                                               const int *__restrict__ ea, int vec,
-                                                               unsigned long long *__restrict__ sa) {
+                                                               const int *__restrict__ ea, int64_t ea_ld, int vec,
+                                                               unsigned long long *__restrict__ sa, int64_t sa_ld) {
     const int64_t groups = (int64_t)nch * Kc / 8;   // Kc % 128 == 0
     const bool fast = p <= 50;                      // |A'| < 2^51: res8_fast (uniform)
     const bool check = np > n;                      // certificate plane n (one K chunk)
@@ -269,7 +269,7 @@ __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__r
          g8 += (int64_t)gridDim.x * blockDim.x) {
         const int64_t k8 = g8 * 8;
         const double *r = A + row * lda;
-        const int sh = p - ea[row];
+        const int sh = p - ea[row * ea_ld];
         double v[8];
         if (vec && k8 + 8 <= K) {   // 16-byte aligned row and a full group: 4 x LDG.128
 #pragma unroll
@@ -323,7 +323,7 @@ __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__r
     }
     if (check) {   // the warp's 32 lanes share the row (blockDim.x = 256 along k)
         rsum = warp_sum_u64(rsum, 32);
-        if ((threadIdx.x & 31) == 0 && rsum) atomicAdd(sa + row, rsum);
+        if ((threadIdx.x & 31) == 0 && rsum) atomicAdd(sa + row * sa_ld, rsum);
     }
     }
 }
@@ -438,7 +438,7 @@ __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__r
                                                               int64_t plane, const int *__restrict__ ea,
                                                               const int *__restrict__ fb, const Oz2Crt crt,
                                                               double *__restrict__ C, int64_t ldc, int64_t rows,
-                                                              int64_t cols) {
+                                                              int64_t cols, int64_t ea_ld) {
     const __int128 M = (__int128)(((u128)crt.Mw[1] << 64) | crt.Mw[0]);
     const __int128 H = (__int128)(((u128)crt.Hw[1] << 64) | crt.Hw[0]);
     // grid-stride over (row, 4-column group); the launch covers every item once
@@ -483,7 +483,7 @@ __global__ void __launch_bounds__(256) oz2_reconstruct_kernel(const uint8_t *__r
             acc[j] += (double)(long long)(X >> 64) * 18446744073709551616.0 + (double)(uint64_t)X;
         }
     }
-    const int er = ea[row] - 2 * crt.p;
+    const int er = ea[row * ea_ld] - 2 * crt.p;
     double *crow = C + row * ldc + c4;
 #pragma unroll
     for (int j = 0; j < 4; ++j)
@@ -524,7 +524,7 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
                                                               int64_t plane, const int *__restrict__ ea,
                                                               const int *__restrict__ fb, const Oz2CrtF crt,
                                                               double *__restrict__ C, int64_t ldc, int64_t rows,
-                                                              int64_t cols, int vec) {
+                                                              int64_t cols, int vec, int64_t ea_ld) {
     const double two52 = 4503599627370496.0, two39 = 549755813888.0, two78 = 302231454903657293676544.0;
     for (int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y; row < rows;
          row += (int64_t)gridDim.y * blockDim.y)
@@ -535,7 +535,7 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
 #pragma unroll
     for (int t = 0; t < NM; ++t)   // all planes' loads in flight together (ldr, plane % 16 == 0)
         u16[t] = __ldcs(reinterpret_cast<const uint2 *>(pr + (int64_t)t * plane));
-    const int er = ea[row] - 2 * crt.p;
+    const int er = ea[row * ea_ld] - 2 * crt.p;
     double *crow = C + row * ldc + c16;
 #pragma unroll
     for (int g = 0; g < 2; ++g) {
@@ -617,27 +617,31 @@ static cudaError_t upload_moduli(const Ozaki2Plan &P) {
 }
 
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
-                                  int8_t *A8, int *ea, cudaStream_t s, int *launches, unsigned long long *sa) {
+                                  int8_t *A8, int *ea, cudaStream_t s, int *launches, unsigned long long *sa,
+                                  int64_t lda8, int64_t ea_ld, int64_t sa_ld) {
     if (rows <= 0) return cudaSuccess;
+    if (lda8 <= 0) lda8 = P.ld8;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
     if (P.check) {
         if (!sa) return cudaErrorInvalidValue;
-        if ((e = cudaMemsetAsync(sa, 0, (size_t)rows * sizeof(unsigned long long), s)) != cudaSuccess) return e;
+        e = sa_ld == 1 ? cudaMemsetAsync(sa, 0, (size_t)rows * sizeof(unsigned long long), s)
+                       : cudaMemset2DAsync(sa, (size_t)(sa_ld * 8), 0, sizeof(unsigned long long), (size_t)rows, s);
+        if (e != cudaSuccess) return e;
     }
     const char *mode = getenv("PDL_OZ2_SPLIT");
     if (mode && !strcmp(mode, "rows") && !P.check) {
         const int blocks = (int)(rows < split_ctas() ? rows : split_ctas());
-        oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, P.ld8, ea);
+        oz2_split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, rows, K, P.n, P.p, P.Kc, P.nch, A8, lda8, ea, ea_ld);
         if (launches) *launches += 1;
         return cudaGetLastError();
     }
-    oz2_rowmax_kernel<<<(unsigned)((rows + 7) / 8), 256, 0, s>>>(A, lda, rows, K, ea);
+    oz2_rowmax_kernel<<<(unsigned)((rows + 7) / 8), 256, 0, s>>>(A, lda, rows, K, ea, ea_ld);
     const int64_t groups = (int64_t)P.nch * P.Kc / 8;
     dim3 grid((unsigned)std::min<int64_t>((groups + 255) / 256, 64), (unsigned)std::min<int64_t>(rows, 65535));
     const int vec = ((reinterpret_cast<uintptr_t>(A) & 15u) == 0 && (lda & 1) == 0) ? 1 : 0;
-    oz2_residue_rows_kernel<<<grid, 256, 0, s>>>(A, lda, rows, K, P.n, P.np, P.p, P.Kc, P.nch, A8, P.ld8, ea, vec,
-                                                 sa);
+    oz2_residue_rows_kernel<<<grid, 256, 0, s>>>(A, lda, rows, K, P.n, P.np, P.p, P.Kc, P.nch, A8, lda8, ea, ea_ld,
+                                                 vec, sa, sa_ld);
     if (launches) *launches += 2;
     return cudaGetLastError();
 }
@@ -679,7 +683,7 @@ bool oz2_crt_fast_ok(const Ozaki2Plan &P) {
 
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                                      cudaStream_t s) {
+                                      cudaStream_t s, int64_t ea_ld) {
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 3u) || (ldr & 3) || (plane & 3)) return cudaErrorInvalidValue;
     const char *crt_mode = getenv("PDL_OZ2_CRT");
@@ -701,7 +705,7 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
         dim3 grid((unsigned)((cols + 255) / 256), (unsigned)std::min<int64_t>((rows + 7) / 8, 65535));
         switch (P.n) {
 #define OZ2_CASE(k) \
-    case k: oz2_crt_fp64_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec); break;
+    case k: oz2_crt_fp64_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec, ea_ld); break;
             OZ2_CASE(2) OZ2_CASE(3) OZ2_CASE(4) OZ2_CASE(5) OZ2_CASE(6) OZ2_CASE(7) OZ2_CASE(8) OZ2_CASE(9)
             OZ2_CASE(10) OZ2_CASE(11) OZ2_CASE(12) OZ2_CASE(13) OZ2_CASE(14)
 #undef OZ2_CASE
@@ -725,7 +729,7 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
     dim3 grid((unsigned)((cols + 127) / 128), (unsigned)((rows + 7) / 8));
     switch (P.n) {
 #define OZ2_CASE(k) \
-    case k: oz2_reconstruct_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, crt, C, ldc, rows, cols); break;
+    case k: oz2_reconstruct_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, crt, C, ldc, rows, cols, ea_ld); break;
         OZ2_CASE(2) OZ2_CASE(3) OZ2_CASE(4) OZ2_CASE(5) OZ2_CASE(6) OZ2_CASE(7) OZ2_CASE(8) OZ2_CASE(9) OZ2_CASE(10)
         OZ2_CASE(11) OZ2_CASE(12) OZ2_CASE(13) OZ2_CASE(14)
 #undef OZ2_CASE

@@ -37,7 +37,7 @@ __device__ __forceinline__ float tf32_rna(float x) {
 }
 
 __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int64_t M, int64_t K,
-                                  float *__restrict__ hi, float *__restrict__ lo, int64_t Kp, int vec) {
+                                  float *__restrict__ hi, float *__restrict__ lo, int64_t Kp, int64_t ldo, int vec) {
     // one thread per 4 consecutive k of one row (Kp % 4 == 0)
     const int64_t q = Kp >> 2;
     const int64_t total = M * q;
@@ -57,8 +57,8 @@ __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int6
             h[u] = tf32_rna(v[u]);
             l[u] = tf32_rna(v[u] - h[u]);
         }
-        *reinterpret_cast<float4 *>(hi + i * Kp + k0) = make_float4(h[0], h[1], h[2], h[3]);
-        *reinterpret_cast<float4 *>(lo + i * Kp + k0) = make_float4(l[0], l[1], l[2], l[3]);
+        *reinterpret_cast<float4 *>(hi + i * ldo + k0) = make_float4(h[0], h[1], h[2], h[3]);
+        *reinterpret_cast<float4 *>(lo + i * ldo + k0) = make_float4(l[0], l[1], l[2], l[3]);
     }
 }
 
@@ -107,13 +107,14 @@ __global__ void __launch_bounds__(256) split_cols_t_kernel(const float *__restri
 }
 
 cudaError_t launch_split_rows(const float *A, int64_t lda, int64_t M, int64_t K, float *hi, float *lo, int64_t Kp,
-                              cudaStream_t s) {
+                              cudaStream_t s, int64_t ldo) {
+    if (ldo <= 0) ldo = Kp;
     if (M <= 0 || Kp <= 0) return cudaSuccess;
     const int64_t total = M * (Kp >> 2);
     int blocks = (int)((total + 255) / 256);
     if (blocks > 148 * 16) blocks = 148 * 16;
     const int vec = ((reinterpret_cast<uintptr_t>(A) & 15u) == 0 && (lda & 3) == 0) ? 1 : 0;
-    split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, M, K, hi, lo, Kp, vec);
+    split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, M, K, hi, lo, Kp, ldo, vec);
     return cudaGetLastError();
 }
 
@@ -298,9 +299,10 @@ __global__ void __launch_bounds__(k2::THREADS, 1)
     }
 }
 
-static bool map_f32(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_t Kp, uint64_t rows, uint32_t box_rows) {
+static bool map_f32(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_t Kp, uint64_t rows, uint32_t box_rows,
+                    uint64_t ld = 0) {
     cuuint64_t dims[2] = {Kp, rows};
-    cuuint64_t strides[1] = {Kp * 4};
+    cuuint64_t strides[1] = {(ld ? ld : Kp) * 4};
     cuuint32_t box[2] = {(cuuint32_t)k2::BK, box_rows};
     cuuint32_t es[2] = {1, 1};
     return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
@@ -310,11 +312,11 @@ static bool map_f32(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_
 
 cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                               cudaStream_t stream) {
+                               cudaStream_t stream, int64_t lda_s) {
     using namespace k2;
     if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
     CUtensorMap tah, tal, tbh, tbl;
-    if (!map_f32(enc, &tah, Ahi, Kp, M, BM) || !map_f32(enc, &tal, Alo, Kp, M, BM) ||
+    if (!map_f32(enc, &tah, Ahi, Kp, M, BM, lda_s) || !map_f32(enc, &tal, Alo, Kp, M, BM, lda_s) ||
         !map_f32(enc, &tbh, Bhi, Kp, N, BN) || !map_f32(enc, &tbl, Blo, Kp, N, BN))
         return cudaErrorInvalidValue;
     int dev = 0;

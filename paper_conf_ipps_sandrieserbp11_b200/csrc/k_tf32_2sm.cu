@@ -202,9 +202,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
 }
 
 static bool map_f32_2sm(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_t Kp, uint64_t rows,
-                        uint32_t box_rows) {
+                        uint32_t box_rows, uint64_t ld = 0) {
     cuuint64_t dims[2] = {Kp, rows};
-    cuuint64_t strides[1] = {Kp * 4};
+    cuuint64_t strides[1] = {(ld ? ld : Kp) * 4};
     cuuint32_t box[2] = {(cuuint32_t)k2x::BK, box_rows};
     cuuint32_t es[2] = {1, 1};
     return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
@@ -214,11 +214,11 @@ static bool map_f32_2sm(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uin
 
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                    const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                                   cudaStream_t stream, int *dyn_next, int *dyn_mine) {
+                                   cudaStream_t stream, int *dyn_next, int *dyn_mine, int64_t lda_s) {
     using namespace k2x;
     if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
     CUtensorMap tah, tal, tbh, tbl;
-    if (!map_f32_2sm(enc, &tah, Ahi, Kp, M, BM) || !map_f32_2sm(enc, &tal, Alo, Kp, M, BM) ||
+    if (!map_f32_2sm(enc, &tah, Ahi, Kp, M, BM, lda_s) || !map_f32_2sm(enc, &tal, Alo, Kp, M, BM, lda_s) ||
         !map_f32_2sm(enc, &tbh, Bhi, Kp, N, BNH) || !map_f32_2sm(enc, &tbl, Blo, Kp, N, BNH))
         return cudaErrorInvalidValue;
     int dev = 0;

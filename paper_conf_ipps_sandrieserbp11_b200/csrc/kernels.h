@@ -36,19 +36,21 @@ cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, con
 // set).  A stored element is bitwise the plain K1 result.
 
 // K3 -- TF32 hi/lo split pre-pass.  Kp = K rounded up to K2's BK (32).
-//  split_rows:   A (M x K, lda, fp32)  -> Ahi, Alo  (M x Kp, K-major, zero padded)
+//  split_rows:   A (M x K, lda, fp32)  -> Ahi, Alo  (M x Kp, K-major, zero padded; row stride
+//                ldo floats, default Kp -- the packed prepared-A rows [hi | lo] use 2 Kp)
 //  split_cols_t: B (K x N, ldb, fp32)  -> Bhi, Blo  (N x Kp, K-major = B^T, zero padded)
 constexpr int K2_BK = 32;
 cudaError_t launch_split_rows(const float *A, int64_t lda, int64_t M, int64_t K, float *hi, float *lo, int64_t Kp,
-                              cudaStream_t s);
+                              cudaStream_t s, int64_t ldo = 0);
 cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t N, float *hi, float *lo, int64_t Kp,
                                 cudaStream_t s);
 
 // K2 -- 3xTF32 tcgen05 GEMM on the split operands:
-//  C (M x N, ldc, fp32) = Ahi*Bhi^T + Ahi*Blo^T + Alo*Bhi^T   (hi/lo: M x Kp / N x Kp)
+//  C (M x N, ldc, fp32) = Ahi*Bhi^T + Ahi*Blo^T + Alo*Bhi^T   (hi/lo: M x Kp / N x Kp;
+//  lda_s = row stride of Ahi / Alo in floats, 0 = Kp)
 cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                               cudaStream_t stream);
+                               cudaStream_t stream, int64_t lda_s = 0);
 // K6/K7 -- FP64 DGEMM variant "ozaki2" (Ozaki scheme II: integer scaling and the
 // Chinese remainder theorem over INT8 GEMMs, k_ozaki2.cu).  A' = rint(A 2^(p-e_i))
 // row-wise, B' = rint(B 2^(p-f_j)) column-wise (|A'|, |B'| <= 2^p); for each of n
@@ -88,7 +90,8 @@ bool oz2_guard_ok(const Ozaki2Plan &P, int64_t K);
 // recomputed by K1 (IEEE FP64); K1 stores only the flagged elements, so every
 // element's value depends on its own certificate alone (bitwise invariance, R14).
 struct Oz2Guard {
-    unsigned long long *sa = nullptr;     // rows of the launch's rectangle
+    unsigned long long *sa = nullptr;     // rows of the launch's rectangle (stride sa_ld)
+    int64_t sa_ld = 1;
     unsigned long long *sb = nullptr;     // its columns
     uint32_t *flags = nullptr;            // tile (row / 128, col / 128) at flags[(row / 128) * ldf + col / 128]
     int64_t ldf = 0;
@@ -101,9 +104,16 @@ struct Oz2Guard {
 // `clusters` co-resident CTA pairs (k_ozaki.cu).
 int oz2_launches_per_chunk(int n, int64_t rows, int64_t cols, int clusters);
 // sa / sb (P.check): the certificate's row / column sums, zeroed and accumulated here.
+// lda8: row stride of A8 in bytes (0 = P.ld8); ea_ld / sa_ld: strides of ea / sa in
+// elements -- the packed prepared-A rows below use lda8 = P.ld8 + 16, ea_ld = lda8 / 4,
+// sa_ld = lda8 / 8.
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
                                   int8_t *A8, int *ea, cudaStream_t s, int *launches = nullptr,
-                                  unsigned long long *sa = nullptr);
+                                  unsigned long long *sa = nullptr, int64_t lda8 = 0, int64_t ea_ld = 1,
+                                  int64_t sa_ld = 1);
+// Prepared A rows of the ozaki2 variant (what PDL_TASK_PREP_A writes and
+// PDL_TASK_PREPARED_A reads): [residues: P.ld8 bytes][e_i: int32][4 bytes][sa_i: u64].
+inline int64_t oz2_prep_row_bytes(const Ozaki2Plan &P) { return P.ld8 + 16; }
 cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
                                   int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s,
                                   unsigned long long *sb = nullptr);
@@ -111,18 +121,19 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
 // launches and flags tiles into guard->flags (zeroed by the caller).
 cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
                                uint8_t *R, int64_t ldr, int64_t plane, int64_t rows, int64_t cols, cudaStream_t s,
-                               int *launches, const Oz2Guard *guard = nullptr);
+                               int *launches, const Oz2Guard *guard = nullptr, int64_t lda8 = 0);
 // The plan admits the FP64-pipe CRT pass (M < 2^117, M >= 2^(2p + lk + 1) (1 + 1/64));
 // otherwise launch_ozaki2_reconstruct uses the 128-bit integer pass.  PDL_OZ2_CRT=int
 // forces the integer pass.
 bool oz2_crt_fast_ok(const Ozaki2Plan &P);
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                                      cudaStream_t s);
+                                      cudaStream_t s, int64_t ea_ld = 1);
 
 // K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                    const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                                   cudaStream_t stream, int *dyn_next = nullptr, int *dyn_mine = nullptr);
+                                   cudaStream_t stream, int *dyn_next = nullptr, int *dyn_mine = nullptr,
+                                   int64_t lda_s = 0);
 
 }  // namespace pdlk

@@ -102,28 +102,17 @@ bool worker_sgemm_ozaki2(const WorkerCtx &w) {
     return lower(trim(v)) == "ozaki2";
 }
 
-// Ozaki-II per-row / per-column arrays of a task: the B side [bmax: cols u64][sb:
-// cols u64][fb: cols int] in the shared BUF_OZE of slot 0 (it does not move with
-// `rows`, so a prepared B survives row-chunk tasks, REUSE_B), the A side [ea: rows
-// int][sa: rows u64] after it for slot 0, in the slot's own BUF_OZE otherwise.
-// sa / sb: the certificate's row / column sums (R21).
-static int oz_exponents(WorkerCtx &w, int slot, int64_t rows, int64_t cols, unsigned long long **bmax, int **fb,
-                        int **ea, unsigned long long **sb, unsigned long long **sa) {
-    void *p = nullptr, *q = nullptr;
-    const size_t bside = (size_t)cols * 16 + (size_t)round_up(cols, 2) * 4;
-    const size_t aside = (size_t)round_up(rows, 2) * 4 + (size_t)rows * 8;
-    int rc = ensure_buf(w, BUF_OZE, bside + (slot == 0 ? aside : 0), &p);
+// Ozaki-II per-column arrays of a task: [bmax: cols u64][sb: cols u64][fb: cols int]
+// in the shared BUF_OZE (it does not move with `rows`, so a prepared B survives
+// row-chunk tasks, REUSE_B).  The A side (residues, e_i, sa_i) lives in the packed
+// prepared-A rows (pdlk::oz2_prep_row_bytes).  sb: the certificate's column sums.
+static int oz_b_arrays(WorkerCtx &w, int64_t cols, unsigned long long **bmax, int **fb, unsigned long long **sb) {
+    void *p = nullptr;
+    int rc = ensure_buf(w, BUF_OZE, (size_t)cols * 16 + (size_t)round_up(cols, 2) * 4, &p);
     if (rc) return rc;
     *bmax = (unsigned long long *)p;
     *sb = *bmax + cols;
     *fb = (int *)(*sb + cols);
-    if (slot == 0) {
-        *ea = *fb + round_up(cols, 2);
-    } else {
-        if ((rc = ensure_buf(w, slot_buf(BUF_OZE, slot), aside, &q))) return rc;
-        *ea = (int *)q;
-    }
-    *sa = (unsigned long long *)(*ea + round_up(rows, 2));
     return PDL_OK;
 }
 
@@ -167,7 +156,13 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     const int64_t pe = 16 / es;   // elements per 16 bytes
 
     // Where the operands live and whether they must be staged into this Worker's MR.
-    const bool a_st = K > 0 && (locate(A) != w.device || (f64 && (((uintptr_t)A % 16) || (t.lda * es) % 16)));
+    // PDL_TASK_PREPARED_A: A is a panel of prepared rows (PDL_TASK_PREP_A) in this
+    // Worker's memory region, read in place
+    const bool prepared = (t.flags & PDL_TASK_PREPARED_A) != 0;
+    if (prepared && K > 0 && (locate(A) != w.device || ((uintptr_t)A % 16)))
+        return set_err(PDL_EINVAL, "PDL_TASK_PREPARED_A: A must be 16-byte aligned memory of the Worker's device");
+    const bool a_st = K > 0 && !prepared &&
+                      (locate(A) != w.device || (f64 && (((uintptr_t)A % 16) || (t.lda * es) % 16)));
     const bool b_st = K > 0 && (locate(B) != w.device || (f64 && (((uintptr_t)B % 16) || (t.ldb * es) % 16)));
     const bool c_st = locate(C) != w.device;
 
@@ -287,11 +282,15 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     // FP32 split buffers (K-major hi/lo of A rows and of B^T rows)
     const int64_t Kp = round_up(std::max<int64_t>(K, 1), pdlk::K2_BK);
     float *ahi = nullptr, *alo = nullptr, *bhi = nullptr, *blo = nullptr;
+    const int64_t lda_s = 2 * Kp;   // prepared A rows [hi: Kp][lo: Kp] (PDL_TASK_PREP_A layout)
     if (!f64 && K > 0) {
-        if ((rc = ensure(BUF_AHI, (size_t)(rows * Kp * 4), &p))) return rc;
+        if (prepared) {
+            p = const_cast<void *>(A);
+        } else if ((rc = ensure(BUF_AHI, (size_t)(rows * lda_s * 4), &p))) {
+            return rc;
+        }
         ahi = (float *)p;
-        if ((rc = ensure(BUF_ALO, (size_t)(rows * Kp * 4), &p))) return rc;
-        alo = (float *)p;
+        alo = ahi + Kp;
         if ((rc = ensure_buf(w, BUF_BHI, (size_t)(cols * Kp * 4), &p))) return rc;
         bhi = (float *)p;
         if ((rc = ensure_buf(w, BUF_BLO, (size_t)(cols * Kp * 4), &p))) return rc;
@@ -310,12 +309,26 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     uint8_t *oz2_R = nullptr;
     int64_t oz2_ldr = 0, oz2_plane = 0;
     pdlk::Oz2Guard G2;
+    int64_t oz_pr = 0, oz_ea_ld = 1, oz_sa_ld = 1;
+    if (ozaki2 && prepared)
+        return set_err(PDL_EUNSUPPORTED, "PDL_TASK_PREPARED_A with DGEMM_VARIANT=ozaki2: the certificate's K1 "
+                                         "recompute needs the raw A rows (exchange raw A chunks for this variant)");
     if (ozaki2) {
-        if ((rc = ensure(BUF_OZA, P2.a8_bytes, &p))) return rc;
+        // packed prepared-A rows: [residues: ld8][e_i: int][pad][sa_i: u64]
+        oz_pr = pdlk::oz2_prep_row_bytes(P2);
+        if (prepared) {
+            p = const_cast<void *>(A);
+        } else if ((rc = ensure(BUF_OZA, (size_t)(rows * oz_pr), &p))) {
+            return rc;
+        }
         a8 = (int8_t *)p;
+        oz_ea = (int *)(a8 + P2.ld8);
+        oz_sa = (unsigned long long *)(a8 + P2.ld8 + 8);
+        oz_ea_ld = oz_pr / 4;
+        oz_sa_ld = oz_pr / 8;
         if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
         b8 = (int8_t *)p;
-        if ((rc = oz_exponents(w, slot, rows, cols, &oz_bmax, &oz_fb, &oz_ea, &oz_sb, &oz_sa))) return rc;
+        if ((rc = oz_b_arrays(w, cols, &oz_bmax, &oz_fb, &oz_sb))) return rc;
         oz2_ldr = round_up(cols, 16);
         oz2_plane = oz2_ldr * rows;
         if ((rc = ensure(BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
@@ -409,10 +422,13 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 e = cudaMemset2DAsync(Cs, (size_t)(ldcd * es), 0, (size_t)(nc * es), (size_t)nr, cs);
             } else if (ozaki2) {
                 // K7 scaling + residues of this band / panel once, shared by both compute streams
-                if (!a_prep[i]) {
+                if (!a_prep[i] && prepared) {
+                    a_prep[i] = 1;
+                } else if (!a_prep[i]) {
                     a_prep[i] = 1;
                     e = pdlk::launch_ozaki2_split_a((const double *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K, P2,
-                                                    a8 + r0 * P2.ld8, oz_ea + r0, cs, &w.launches, oz_sa + r0);
+                                                    a8 + r0 * oz_pr, oz_ea + r0 * oz_ea_ld, cs, &w.launches,
+                                                    oz_sa + r0 * oz_sa_ld, oz_pr, oz_ea_ld, oz_sa_ld);
                     if (piped) {
                         ev_sa[i] = ev_get(w, evn);
                         CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
@@ -440,7 +456,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 // the certificate of this band / panel (r0, c0: multiples of 128)
                 pdlk::Oz2Guard gs = G2;
                 if (P2.check) {
-                    gs.sa = oz_sa + r0;
+                    gs.sa = oz_sa + r0 * oz_sa_ld;
+                    gs.sa_ld = oz_sa_ld;
                     gs.sb = oz_sb + c0;
                     gs.flags = G2.flags + (r0 / 128) * G2.ldf + c0 / 128;
                     gs.emask = G2.emask + r0 * G2.ldw + c0 / 32;
@@ -451,11 +468,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                                               (size_t)nr, cs);
                 }
                 if (e == cudaSuccess)
-                    e = pdlk::launch_ozaki2_gemm(enc, a8 + r0 * P2.ld8, b8 + c0 * P2.ld8, P2, Rs, oz2_ldr, oz2_plane,
-                                                 nr, nc, cs, &nl, P2.check ? &gs : nullptr);
+                    e = pdlk::launch_ozaki2_gemm(enc, a8 + r0 * oz_pr, b8 + c0 * P2.ld8, P2, Rs, oz2_ldr, oz2_plane,
+                                                 nr, nc, cs, &nl, P2.check ? &gs : nullptr, oz_pr);
                 if (e == cudaSuccess)
-                    e = pdlk::launch_ozaki2_reconstruct(Rs, oz2_ldr, oz2_plane, oz_ea + r0, oz_fb + c0, P2,
-                                                        (double *)Cs, ldcd, nr, nc, cs);
+                    e = pdlk::launch_ozaki2_reconstruct(Rs, oz2_ldr, oz2_plane, oz_ea + r0 * oz_ea_ld, oz_fb + c0, P2,
+                                                        (double *)Cs, ldcd, nr, nc, cs, oz_ea_ld);
                 // flagged tiles: recomputed by K1 over the same operands (IEEE FP64)
                 if (e == cudaSuccess && P2.check) {
                     e = pdlk::launch_dgemm_k1(enc, (const double *)(Ad + (size_t)(r0 * lda) * es), lda,
@@ -474,10 +491,12 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 w.launches += 1;
             } else {
                 // K3 split of this band / panel once, shared by both compute streams
-                if (!a_prep[i]) {
+                if (!a_prep[i] && prepared) {
+                    a_prep[i] = 1;
+                } else if (!a_prep[i]) {
                     a_prep[i] = 1;
                     e = pdlk::launch_split_rows((const float *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K,
-                                                ahi + r0 * Kp, alo + r0 * Kp, Kp, cs);
+                                                ahi + r0 * lda_s, alo + r0 * lda_s, Kp, cs, lda_s);
                     w.launches += 1;
                     if (piped) {
                         ev_sa[i] = ev_get(w, evn);
@@ -502,11 +521,12 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
                 if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
                 if (k2v ? !strcmp(k2v, "1sm") : k2_pick_1sm(nr, nc, sms))
-                    e = pdlk::launch_gemm_3xtf32(enc, ahi + r0 * Kp, alo + r0 * Kp, bhi + c0 * Kp, blo + c0 * Kp, Kp,
-                                                 (float *)Cs, ldcd, nr, nc, cs);
+                    e = pdlk::launch_gemm_3xtf32(enc, ahi + r0 * lda_s, alo + r0 * lda_s, bhi + c0 * Kp, blo + c0 * Kp,
+                                                 Kp, (float *)Cs, ldcd, nr, nc, cs, lda_s);
                 else
-                    e = pdlk::launch_gemm_3xtf32_2sm(enc, ahi + r0 * Kp, alo + r0 * Kp, bhi + c0 * Kp, blo + c0 * Kp,
-                                                     Kp, (float *)Cs, ldcd, nr, nc, cs);
+                    e = pdlk::launch_gemm_3xtf32_2sm(enc, ahi + r0 * lda_s, alo + r0 * lda_s, bhi + c0 * Kp,
+                                                     blo + c0 * Kp, Kp, (float *)Cs, ldcd, nr, nc, cs, nullptr, nullptr,
+                                                     lda_s);
                 if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
                 w.launches += 1;
             }
@@ -553,6 +573,50 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         if (!w.ev_blast) CUDA_TRY(cudaEventCreateWithFlags(&w.ev_blast, cudaEventDisableTiming));
         CUDA_TRY(cudaEventRecord(w.ev_blast, w.stream));
     }
+    return PDL_OK;
+}
+
+// Bytes per prepared A row (PDL_TASK_PREP_A) of the task variant of PU `pu` for
+// inner dimension K, 0 when the variant exchanges raw rows: FP32 3xTF32 -> [hi:
+// Kp floats][lo: Kp floats]; FP64 (dmma; ozaki2, whose certificate recomputes from
+// the raw rows) -> 0.
+int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K) {
+    if (dtype != PDL_F32 || K <= 0) return 0;
+    WorkerCtx w;
+    w.pu = pu;
+    int sl, rn;
+    if (worker_ozaki(w, false, &sl, &rn) || worker_sgemm_ozaki2(w)) return 0;
+    return 2 * round_up(K, pdlk::K2_BK) * 4;
+}
+
+// PDL_TASK_PREP_A: the A preparation of the Worker's task variant for the task's M
+// rows, written as packed prepared rows to C (this Worker's memory region, 16-byte
+// aligned) -- the unit the multi-rank runtime exchanges instead of raw A chunks.
+int run_prep_a(WorkerCtx &w, const Task &t) {
+    CUDA_TRY(cudaSetDevice(w.device));
+    const int64_t pr = prepared_a_row_bytes(w.pu, t.dtype, t.K);
+    if (pr == 0)
+        return set_err(PDL_EUNSUPPORTED, "PDL_TASK_PREP_A: this Worker's %s task variant has no A preparation",
+                       t.dtype == PDL_F64 ? "FP64" : "FP32");
+    if (locate(t.C) != w.device || ((uintptr_t)t.C % 16))
+        return set_err(PDL_EINVAL, "PDL_TASK_PREP_A: the output must be 16-byte aligned memory of the Worker's device");
+    const int64_t Kp = round_up(t.K, pdlk::K2_BK);
+    const float *A = (const float *)t.A;
+    int64_t lda = t.lda;
+    if (locate(t.A) != w.device) {   // stage the raw rows into the Worker's memory region
+        void *p = nullptr;
+        lda = round_up(t.K, 4);
+        int rc = ensure_buf(w, BUF_A, (size_t)(t.M * lda * 4), &p);
+        if (rc) return rc;
+        CUDA_TRY(cudaMemcpy2DAsync(p, (size_t)(lda * 4), t.A, (size_t)(t.lda * 4), (size_t)(t.K * 4), (size_t)t.M,
+                                   cudaMemcpyDefault, w.stream));
+        g->xfer.count(locate(t.A), w.device, t.M * t.K * 4);
+        A = (const float *)p;
+    }
+    float *hi = (float *)t.C;
+    cudaError_t e = pdlk::launch_split_rows(A, lda, t.M, t.K, hi, hi + Kp, Kp, w.stream, 2 * Kp);
+    if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
+    w.launches += 1;
     return PDL_OK;
 }
 
@@ -866,7 +930,8 @@ int execute(bool sync) {
             pj << "{\"local\":true,\"M\":" << t.M << ",\"N\":" << t.N << ",\"K\":" << t.K << "}";
             if (g->dry_run) continue;
             if (g->workers.empty()) return set_err(PDL_ENOWORKER, "no Worker bound to this process");
-            rc = run_rect_g(g->workers[0], t, t.A, t.B, t.C, t.M, t.N);
+            rc = (t.flags & PDL_TASK_PREP_A) ? run_prep_a(g->workers[0], t)
+                                              : run_rect_g(g->workers[0], t, t.A, t.B, t.C, t.M, t.N);
             if (rc) return rc;
             continue;
         }

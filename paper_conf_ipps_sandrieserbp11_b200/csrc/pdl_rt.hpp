@@ -228,6 +228,8 @@ int run_dynamic(const Task &t, const std::vector<int> &gw);
 int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols);
 int execute(bool sync);
 int enable_peer(int from, int to);
+int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K);
+int run_prep_a(WorkerCtx &w, const Task &t);
 // pdl_xchg.cu
 bool exchange_applies(const Task &t, const Plan &plan, const std::vector<int> &gw);
 int run_exchange(const Task &t, const Plan &plan, const std::vector<int> &gw);

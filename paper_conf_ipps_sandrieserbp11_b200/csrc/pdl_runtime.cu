@@ -115,8 +115,24 @@ int enqueue(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb, v
     if (M < 0 || N < 0 || K < 0) return set_err(PDL_EINVAL, "negative size M=%lld N=%lld K=%lld", (long long)M,
                                                 (long long)N, (long long)K);
     if (tile < 0) return set_err(PDL_EINVAL, "negative tile %lld", (long long)tile);
-    if (flags & ~(PDL_TASK_PANELS | PDL_TASK_LOCAL | PDL_TASK_REUSE_B | PDL_TASK_GRAPH | PDL_TASK_SLOT(3)))
+    if (flags & ~(PDL_TASK_PANELS | PDL_TASK_LOCAL | PDL_TASK_REUSE_B | PDL_TASK_GRAPH | PDL_TASK_SLOT(3) |
+                  PDL_TASK_PREP_A | PDL_TASK_PREPARED_A))
         return set_err(PDL_EINVAL, "unknown flags 0x%x", flags);
+    if ((flags & (PDL_TASK_PREP_A | PDL_TASK_PREPARED_A)) && !(flags & PDL_TASK_LOCAL))
+        return set_err(PDL_EINVAL, "PDL_TASK_PREP_A / PDL_TASK_PREPARED_A need PDL_TASK_LOCAL");
+    if ((flags & PDL_TASK_PREP_A) && (flags & PDL_TASK_PREPARED_A))
+        return set_err(PDL_EINVAL, "PDL_TASK_PREP_A and PDL_TASK_PREPARED_A are exclusive");
+    if (flags & PDL_TASK_PREP_A) {
+        // A (M x K) -> prepared rows written to C; no product, no B
+        if (M < 0 || K < 0) return set_err(PDL_EINVAL, "negative size");
+        if (M == 0 || K == 0) return PDL_OK;
+        if (!A || !C) return set_err(PDL_EINVAL, "A or the output C is NULL");
+        const int64_t lda_ = lda ? lda : K;
+        if (lda_ < K) return set_err(PDL_EINVAL, "leading dimension smaller than the row width");
+        Task t{dtype, A, lda_, nullptr, 0, C, 0, M, 0, K, tile, group != nullptr, group ? group : "", flags, DistSpec()};
+        g->queue.push_back(t);
+        return PDL_OK;
+    }
     if (((flags >> 4) & 3u) >= 3u) return set_err(PDL_EINVAL, "scratch slot %u out of range (0..2)", (flags >> 4) & 3u);
     if ((flags & PDL_TASK_PANELS) && (flags & PDL_TASK_LOCAL))
         return set_err(PDL_EINVAL, "PDL_TASK_PANELS and PDL_TASK_LOCAL are exclusive");
@@ -419,6 +435,19 @@ int pdl_query(const char *key, char *out, size_t len) {
             bool any_green = false;
             for (auto &w : g->workers) any_green |= w.gctx != nullptr;
             res = g->workers.empty() || any_green ? "no" : "yes";
+        }
+        else if (k.rfind("prepared_a/", 0) == 0) {
+            // "prepared_a/<f64|f32>/<K>": bytes per prepared A row (PDL_TASK_PREP_A) of
+            // local Worker 0's task variant, 0 when it exchanges raw rows
+            char dts[8] = {0};
+            long long K = -1;
+            if (sscanf(k.c_str() + 11, "%3[^/]/%lld", dts, &K) != 2 || K < 0 ||
+                (strcmp(dts, "f64") && strcmp(dts, "f32")))
+                return set_err(PDL_EINVAL, "bad key '%s' (prepared_a/<f64|f32>/<K>)", key);
+            std::vector<int> gw = m.group_workers(nullptr);
+            if (gw.empty()) return set_err(PDL_ENOWORKER, "no gpu Worker");
+            const int pu = g->workers.empty() ? gw[0] : g->workers[0].pu;
+            res = std::to_string(prepared_a_row_bytes(pu, strcmp(dts, "f64") ? PDL_F32 : PDL_F64, K));
         }
         else if (k == "plan") res = g->plan_json;
         else if (k == "groups") {

@@ -138,14 +138,33 @@ def chunk_from_full(A, B, wp: WorkerPlan):
 
 
 class PanelBuffers:
-    def __init__(self, wp: WorkerPlan, dtype, device):
-        self.A = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dtype, device=device)
+    """The Worker's panels: B column-panel (Gr chunks of qb K-rows) and A
+    row-panel (Gc chunks of qa rows).  prep_bytes > 0 (the task variant prepares
+    A, pdl.prepared_a_row_bytes): the A panel holds PREPARED rows (bytes), so each
+    Worker prepares only its own chunk and the exchange moves prepared chunks
+    (FP32 3xTF32: TF32 hi/lo, 2x the raw bytes, instead of every Worker of a grid
+    row splitting the whole panel again)."""
+
+    def __init__(self, wp: WorkerPlan, dtype, device, prep_bytes: int = 0):
+        self.prepared = prep_bytes > 0
+        if self.prepared:
+            self.A = torch.empty((wp.Gc * wp.qa, prep_bytes), dtype=torch.uint8, device=device)
+        else:
+            self.A = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dtype, device=device)
         self.B = torch.empty((wp.Gr * wp.qb, wp.cols), dtype=dtype, device=device)
         if _test_delay_cycles():
             # fault injection (tests): panels start as NaN, so a compute that does
             # not wait for its chunk's landing produces NaN rows of C
-            self.A.fill_(float("nan"))
+            self.A.fill_(255 if self.prepared else float("nan"))
             self.B.fill_(float("nan"))
+
+
+def prepared_bytes(dtype, K, device) -> int:
+    """Prepared-A row bytes of this Worker's task variant for device panels
+    (0: exchange raw rows)."""
+    if device is None or torch.device(device).type != "cuda":
+        return 0
+    return pdl.prepared_a_row_bytes(dtype, K)
 
 
 def exchange(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers):
@@ -354,7 +373,12 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
         bufs.B.copy_(Bch)
     Bp = bufs.B[: wp.K]
     qa, c = wp.qa, wp.c
-    bufs.A[c * qa:(c + 1) * qa].copy_(Ach)
+    if bufs.prepared:
+        # the own chunk's prepared rows (TF32 hi/lo ...), straight into the panel
+        pdl.prepare_a(Ach, bufs.A[c * qa:(c + 1) * qa])
+        pdl.run_async()
+    else:
+        bufs.A[c * qa:(c + 1) * qa].copy_(Ach)
     works = {}
     if wp.Gc > 1:
         for j in range(wp.Gc):   # same order on every rank of the row
@@ -389,7 +413,7 @@ def tasks_may_overlap(*panels) -> bool:
     slot (PDL_TASK_SLOT; query "concurrent_tasks/<dtype>"), and stages nothing
     when every operand is on the Worker's device, 16-byte aligned, with 16-byte
     row pitches."""
-    dt = panels[0].dtype
+    dt = panels[-1].dtype   # the B panel: raw operand dtype (A may be prepared bytes)
     key = "concurrent_tasks/" + ("f64" if dt == torch.float64 else "f32")
     if not all(t.is_cuda for t in panels):
         return False
@@ -462,9 +486,10 @@ def chunk_task(Cblock, wp: WorkerPlan, tile=0):
     launch group its own)."""
     def compute(j, lo, hi, Arows, Bp, first, slot=0):
         Cv = Cblock[lo:hi]
+        prepared = Arows.dtype == torch.uint8   # prepared A rows (PanelBuffers prep_bytes)
         pdl.task_matmul(Arows, Bp, Cv, M=hi - lo, N=wp.cols, K=wp.K, tile=tile,
-                        lda=Arows.stride(0), ldb=Bp.stride(0), ldc=Cv.stride(0), local=True, reuse_b=not first,
-                        slot=slot)
+                        lda=0 if prepared else Arows.stride(0), ldb=Bp.stride(0), ldc=Cv.stride(0), local=True,
+                        reuse_b=not first, slot=slot, prepared_a=prepared)
         pdl.run_async()
     return compute
 
@@ -499,7 +524,7 @@ def distributed_matmul(A_full, B_full, C_full, tile=0, group=None, overlap=True)
     dev = torch.device("cuda", torch.cuda.current_device())
     Ach, Bch = chunk_from_full(A_full, B_full, wp)
     Ach, Bch = Ach.to(dev, non_blocking=True), Bch.to(dev, non_blocking=True)
-    bufs = PanelBuffers(wp, A_full.dtype, dev)
+    bufs = PanelBuffers(wp, A_full.dtype, dev, prepared_bytes(A_full.dtype, K, dev) if overlap else 0)
     Cb = torch.empty((wp.rows, wp.cols), dtype=C_full.dtype, device=dev)
     pdl.set_stream(torch.cuda.current_stream())
     if overlap:

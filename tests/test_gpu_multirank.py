@@ -140,3 +140,83 @@ def test_a_missing_wait_corrupts_c():
     r = _run_rc(4, "f64", 1000, 700, 300, 64,
                 env_extra={"PDL_TEST_EXCHANGE_DELAY_US": "3000", "PDL_OVERLAP_A": "1", "PDL_TEST_DROP_WAITS": "1"})
     assert r.returncode != 0 or "ok=False" in r.stdout, r.stdout[-2000:]
+
+
+@pytest.mark.parametrize("G", [2, 8])
+def test_prepared_a_chunks_bitwise(G, monkeypatch):
+    """FP32 3xTF32 exchanges PREPARED A chunks (PDL_TASK_PREP_A: TF32 hi/lo rows),
+    so each Worker splits only its own chunk: the chunk launches on the prepared
+    panel (PDL_TASK_PREPARED_A) give bitwise the raw-panel C, serial or on side
+    streams, for every Worker position."""
+    import numpy as np
+
+    sys.path.insert(0, ROOT)
+    from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime
+
+    M, N, K, tile = 1500, 1100, 260, 128
+    monkeypatch.setenv("PDL_ALLOW_OVERSUBSCRIBE", "1")
+    monkeypatch.setenv("PDL_DRY_RUN", "1")
+    pdl.load(pdl.descriptor_path(G))
+    try:
+        wps = [runtime.worker_plan(M, N, K, tile, r) for r in range(G)]
+    finally:
+        pdl.unload()
+        monkeypatch.delenv("PDL_DRY_RUN")
+    torch = pytest.importorskip("torch")
+    rng = np.random.default_rng(9)
+    A = torch.from_numpy(rng.uniform(-1, 1, (M, K)).astype(np.float32))
+    B = torch.from_numpy(rng.uniform(-1, 1, (K, N)).astype(np.float32))
+    dev = torch.device("cuda", 0)
+    pdl.load(pdl.descriptor_path(1))
+    try:
+        pb = runtime.prepared_bytes(torch.float32, K, dev)
+        assert pb == 2 * ((K + 31) // 32 * 32) * 4
+        assert runtime.prepared_bytes(torch.float64, K, dev) == 0     # dmma exchanges raw rows
+        for wp in wps:
+            raw = runtime.PanelBuffers(wp, torch.float32, dev)
+            prep = runtime.PanelBuffers(wp, torch.float32, dev, pb)
+            raw.A.zero_()
+            raw.A[: wp.rows].copy_(A[wp.row0: wp.row1])
+            for b in (raw, prep):
+                b.B[: wp.K].copy_(B[:, wp.col0: wp.col1])
+            pdl.set_stream(torch.cuda.current_stream())
+            for j in range(wp.Gc):   # every chunk prepared (here on one Worker)
+                pdl.prepare_a(raw.A[j * wp.qa:(j + 1) * wp.qa], prep.A[j * wp.qa:(j + 1) * wp.qa])
+            pdl.run()
+            out = []
+            for bufs, conc in ((raw, False), (prep, False), (prep, True)):
+                C = torch.full((wp.rows, wp.cols), float("nan"), device=dev)
+                runtime.compute_groups(wp, bufs, bufs.B[: wp.K], runtime.chunk_task(C, wp, tile), {}, conc)
+                pdl.sync()
+                torch.cuda.synchronize()
+                out.append(C.cpu())
+            assert torch.equal(out[0], out[1]) and torch.equal(out[0], out[2]), (wp.r, wp.c)
+    finally:
+        pdl.unload()
+
+
+def test_prep_a_errors():
+    sys.path.insert(0, ROOT)
+    torch = pytest.importorskip("torch")
+    from paper_conf_ipps_sandrieserbp11_b200 import pdl
+    pdl.load(pdl.descriptor_path(1))
+    try:
+        A = torch.rand((64, 96), dtype=torch.float64, device="cuda")
+        out = torch.empty((64, 2048), dtype=torch.uint8, device="cuda")
+        pdl.prepare_a(A, out)
+        with pytest.raises(pdl.PDLError) as e:
+            pdl.run()
+        assert e.value.code == pdl.PDL_EUNSUPPORTED      # FP64 dmma exchanges raw rows
+    finally:
+        pdl.unload()
+    pdl.load(pdl.descriptor_xml(1, props={"DGEMM_VARIANT": "ozaki2"}))
+    try:
+        Ap = torch.zeros((64, 4096), dtype=torch.uint8, device="cuda")
+        Bd = torch.rand((96, 32), dtype=torch.float64, device="cuda")
+        C = torch.empty((64, 32), dtype=torch.float64, device="cuda")
+        pdl.task_matmul(Ap, Bd, C, M=64, N=32, K=96, local=True, prepared_a=True)
+        with pytest.raises(pdl.PDLError) as e:
+            pdl.run()
+        assert e.value.code == pdl.PDL_EUNSUPPORTED      # the certificate recomputes from raw rows
+    finally:
+        pdl.unload()

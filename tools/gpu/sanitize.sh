@@ -9,7 +9,7 @@ for tool in racecheck synccheck memcheck; do
     name=$(echo $spec | tr ' ' '_')
     extra=""
     [ $tool = racecheck ] && extra="--racecheck-report all"
-    timeout 900 $CS --tool $tool $extra --kernel-name regex:pdlk --print-limit 50 python tools/sanitize_run.py $spec > $out/${tool}_${name}.txt 2>&1
+    timeout 900 $CS --tool $tool $extra --kernel-name kns=pdlk --print-limit 50 python tools/sanitize_run.py $spec > $out/${tool}_${name}.txt 2>&1
     echo "$tool $name rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_${name}.txt | tail -2 | tr '\n' ' ')"
   done
 done

@@ -36,26 +36,42 @@ def plans(M, N, K, tile, G):
         os.environ.pop("PDL_DRY_RUN", None)
 
 
-def time_worker(wp, dt, tile, concurrent, reps):
+def time_worker(wp, dt, tile, concurrent, reps, raw=False):
+    """The Worker's step after the exchange: (prepared-A variants) the preparation
+    of its own A chunk -- the other chunks arrive prepared -- then the chunk launches
+    of runtime.compute_groups."""
     dev = torch.device("cuda", torch.cuda.current_device())
     g = torch.Generator(device="cuda").manual_seed(11)
-    bufs = runtime.PanelBuffers(wp, dt, dev)
-    bufs.A.uniform_(generator=g)
+    prep = 0 if raw else runtime.prepared_bytes(dt, wp.K, dev)
+    bufs = runtime.PanelBuffers(wp, dt, dev, prep)
+    Araw = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dt, device=dev).uniform_(generator=g)
     bufs.B.uniform_(generator=g)
+    if prep:
+        pdl.prepare_a(Araw, bufs.A)   # the chunks the other Workers prepared (untimed)
+        pdl.run()
+    else:
+        bufs.A.copy_(Araw)
+    qa, c = wp.qa, wp.c
     Bp = bufs.B[: wp.K]
     C = torch.full((wp.rows, wp.cols), float("nan"), dtype=dt, device=dev)
     compute = runtime.chunk_task(C, wp, tile=tile)
     main = torch.cuda.current_stream()
     pdl.set_stream(main)
-    for _ in range(2):
+
+    def step():
+        if prep:
+            pdl.prepare_a(Araw[c * qa:(c + 1) * qa], bufs.A[c * qa:(c + 1) * qa])
+            pdl.run_async()
         runtime.compute_groups(wp, bufs, Bp, compute, {}, concurrent)
+    for _ in range(2):
+        step()
     pdl.sync()
     torch.cuda.synchronize()
     ms = []
     for _ in range(reps):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(main)
-        runtime.compute_groups(wp, bufs, Bp, compute, {}, concurrent)
+        step()
         e1.record(main)
         pdl.sync()
         torch.cuda.synchronize()
@@ -104,6 +120,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--gs", default="1,2,4,8")
     ap.add_argument("--variant", default=None, help="task variant (PDL_DGEMM_VARIANT / PDL_SGEMM_VARIANT)")
+    ap.add_argument("--raw", action="store_true", help="exchange raw A chunks (every Worker prepares its panel)")
     args = ap.parse_args()
     if args.variant:
         os.environ["PDL_DGEMM_VARIANT" if args.dtype == "f64" else "PDL_SGEMM_VARIANT"] = args.variant
@@ -114,6 +131,7 @@ def main():
         wps = plans(c.M, c.N, c.K, c.tile, G)
         pdl.load(pdl.descriptor_path(1))
         try:
+            a_ex = "raw" if args.raw or not runtime.prepared_bytes(dt, c.K, "cuda") else "prepared"
             seen = set()
             rows = []
             for wp in wps:
@@ -121,9 +139,9 @@ def main():
                 if key in seen:
                     continue
                 seen.add(key)
-                t_ser, C_ser = time_worker(wp, dt, c.tile, False, args.reps)
+                t_ser, C_ser = time_worker(wp, dt, c.tile, False, args.reps, args.raw)
                 C_ser = C_ser.clone()
-                t_con, C_con = time_worker(wp, dt, c.tile, None, args.reps)   # libpdl decides
+                t_con, C_con = time_worker(wp, dt, c.tile, None, args.reps, args.raw)   # libpdl decides
                 t_one = time_single(wp, dt, c.tile, args.reps)
                 flops = 2.0 * wp.rows * wp.cols * wp.K
                 rows.append({"c": wp.c, "rect": [wp.rows, wp.cols], "qa": wp.qa, "serial_ms": round(t_ser, 3),
@@ -134,7 +152,9 @@ def main():
                 torch.cuda.empty_cache()
         finally:
             pdl.unload()
-        r = {"config": args.config, "dtype": args.dtype, "variant": args.variant or "default", "G": G, "grid": [wps[0].Gr, wps[0].Gc],
+        r = {"config": args.config, "dtype": args.dtype, "variant": args.variant or "default", "G": G,
+             "a_exchange": a_ex,
+             "grid": [wps[0].Gr, wps[0].Gc],
              "max_serial_ms": max(x["serial_ms"] for x in rows),
              "max_concurrent_ms": max(x["concurrent_ms"] for x in rows),
              "max_single_launch_ms": max(x["single_launch_ms"] for x in rows), "workers": rows}
