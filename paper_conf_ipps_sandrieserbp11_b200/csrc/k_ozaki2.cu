@@ -181,11 +181,18 @@ __device__ __forceinline__ double scaled_magic(double x, int sh) {
 // max(0, |v| - 1) 2^(7-p) rounded down, in [0, 127] and at most |x| 2^(7-e)
 // (|v| - 1 < |x| 2^(p-e)); and the row / column sum term 2|v| + 1 for x != 0
 // (|x| 2^(p-e) <= |v| + 1/2).  DESIGN.md R21.
+// Both on the FP64 pipe, no conversion-unit op: x = max(|v| - 1, 0) 2^(7-p) < 2^7 is
+// exact, and x + 2^52 rounded down carries floor(x) in its low word; 2|v| + 1 <
+// 2^52 (p <= 50) is an exact integer whose sum with 2^52 holds it in the mantissa.
 __device__ __forceinline__ int cert8(double v, int p) {
-    return (int)floor(fmax(fabs(v) - 1.0, 0.0) * pow2d(7 - p));
+    const double x = fmax(fabs(v) - 1.0, 0.0) * pow2d(7 - p);
+    return __double2loint(__dadd_rd(x, 4503599627370496.0));
 }
-__device__ __forceinline__ unsigned long long cert_sum(double v, bool nz) {
-    return nz ? (unsigned long long)(2.0 * fabs(v) + 1.0) : 0ull;   // < 2^53: exact
+__device__ __forceinline__ unsigned long long cert_sum(double v, bool nz, int p) {
+    if (!nz) return 0ull;
+    const double d = fma(2.0, fabs(v), 1.0);
+    if (p <= 50) return (unsigned long long)(__double_as_longlong(d + 4503599627370496.0) - 0x4330000000000000ll);
+    return (unsigned long long)d;   // < 2^53: exact
 }
 __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x, int width) {
     for (int o = 1; o < width; o <<= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
@@ -316,7 +323,7 @@ __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__r
 #pragma unroll
             for (int j = 0; j < 8; ++j) {
                 cc[j] = cert8(v[j], p);
-                rsum += cert_sum(v[j], nz[j]);
+                rsum += cert_sum(v[j], nz[j], p);
             }
             *reinterpret_cast<uint64_t *>(o + (int64_t)n * Kc) = pack8(cc);
         }
@@ -341,78 +348,85 @@ __global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int
 // B (K x N) -> Bt8 (N rows of [c][t][kk]) through a shared tile stored transposed
 // (32 n rows x 64 k, row pitch 66 doubles): coalesced loads along n, then each
 // thread reads its column's 8 consecutive k as four 16-byte shared loads (every
-// quarter-warp on distinct banks) and writes one 8-byte word per modulus.
+// quarter-warp on distinct banks) and writes one 8-byte word per modulus.  A CTA
+// walks the k tiles blockIdx.y, blockIdx.y + gridDim.y, ... of its 32 columns, so
+// the certificate's column sums take one atomic per column and CTA (16 k tiles per
+// CTA at C4 instead of 256 single-tile CTAs contending on each column's sum).
 __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
     const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int n, int np, int p, int64_t Kc, int nch,
     const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
     unsigned long long *__restrict__ sb) {
     constexpr int PITCH = 66;
     __shared__ __align__(16) double tl[32 * PITCH];
-    const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 32;
+    const int64_t n0 = (int64_t)blockIdx.x * 32;
     const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
-#pragma unroll
-    for (int r = ty; r < 64; r += 8) {
-        const int64_t k = k0 + r, nn = n0 + tx;
-        tl[tx * PITCH + r] = (k < K && nn < N) ? __ldcs(B + k * ldb + nn) : 0.0;
-    }
-    __syncthreads();
-    const int64_t Kpad = (int64_t)nch * Kc;
+    const int64_t Kpad = (int64_t)nch * Kc, nkt = (Kpad + 63) / 64;
     const int nl = threadIdx.x >> 3, g = threadIdx.x & 7;
-    const int64_t col = n0 + nl, k8 = k0 + 8 * g;
+    const int64_t col = n0 + nl;
     const bool check = np > n;
+    const int f = col < N ? exp_of_max2(__longlong_as_double((long long)bmax[col])) : 0;
+    if (blockIdx.y == 0 && g == 0 && col < N) fb[col] = f;
     unsigned long long csum = 0;
-    if (col < N && k8 < Kpad) {   // (predicated, not returned: the certificate sum reduces over g)
-    const int f = exp_of_max2(__longlong_as_double((long long)bmax[col]));
-    if (blockIdx.y == 0 && g == 0) fb[col] = f;
-    double v[8];
+    for (int64_t kt = blockIdx.y; kt < nkt; kt += gridDim.y) {
+        const int64_t k0 = kt * 64;
+        __syncthreads();   // the previous tile's shared reads are done
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const double2 x = *reinterpret_cast<const double2 *>(&tl[nl * PITCH + 8 * g + 2 * j]);
-        v[2 * j] = x.x;
-        v[2 * j + 1] = x.y;
-    }
-    bool nz[8];
-#pragma unroll
-    for (int j = 0; j < 8; ++j) nz[j] = v[j] != 0.0;
-    const int64_t c = k8 / Kc, kk = k8 - c * Kc;
-    int8_t *o = Bt8 + col * ld8 + (c * np) * Kc + kk;
-    if (p <= 50) {
-        int lo[8];
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const double vm = scaled_magic(v[j], p - f);
-            lo[j] = __double2loint(vm);
-            v[j] = vm - 6755399441055744.0;
+        for (int r = ty; r < 64; r += 8) {
+            const int64_t k = k0 + r, nn = n0 + tx;
+            tl[tx * PITCH + r] = (k < K && nn < N) ? __ldcs(B + k * ldb + nn) : 0.0;
         }
-        for (int t = 0; t < n; ++t) {
-            int rr[8];
+        __syncthreads();
+        const int64_t k8 = k0 + 8 * g;
+        if (col >= N || k8 >= Kpad) continue;
+        double v[8];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) rr[j] = res8_fast(v[j], lo[j], t);
-            *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+        for (int j = 0; j < 4; ++j) {
+            const double2 x = *reinterpret_cast<const double2 *>(&tl[nl * PITCH + 8 * g + 2 * j]);
+            v[2 * j] = x.x;
+            v[2 * j + 1] = x.y;
         }
-    } else {
+        bool nz[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) v[j] = rint(scale2(v[j], p - f));
-        for (int t = 0; t < n; ++t) {
-            int rr[8];
+        for (int j = 0; j < 8; ++j) nz[j] = v[j] != 0.0;
+        const int64_t c = k8 / Kc, kk = k8 - c * Kc;
+        int8_t *o = Bt8 + col * ld8 + (c * np) * Kc + kk;
+        if (p <= 50) {
+            int lo[8];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
-            *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+            for (int j = 0; j < 8; ++j) {
+                const double vm = scaled_magic(v[j], p - f);
+                lo[j] = __double2loint(vm);
+                v[j] = vm - 6755399441055744.0;
+            }
+            for (int t = 0; t < n; ++t) {
+                int rr[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) rr[j] = res8_fast(v[j], lo[j], t);
+                *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[j] = rint(scale2(v[j], p - f));
+            for (int t = 0; t < n; ++t) {
+                int rr[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) rr[j] = res8(v[j], t);
+                *reinterpret_cast<uint64_t *>(o + (int64_t)t * Kc) = pack8(rr);
+            }
         }
-    }
-    if (check) {
-        int cc[8];
+        if (check) {
+            int cc[8];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            cc[j] = cert8(v[j], p);
-            csum += cert_sum(v[j], nz[j]);
+            for (int j = 0; j < 8; ++j) {
+                cc[j] = cert8(v[j], p);
+                csum += cert_sum(v[j], nz[j], p);
+            }
+            *reinterpret_cast<uint64_t *>(o + (int64_t)n * Kc) = pack8(cc);
         }
-        *reinterpret_cast<uint64_t *>(o + (int64_t)n * Kc) = pack8(cc);
-    }
     }
     if (check) {   // the 8 lanes of a column are consecutive: reduce, one atomic per column and CTA
         csum = warp_sum_u64(csum, 8);
-        if (g == 0 && csum) atomicAdd(sb + col, csum);
+        if (g == 0 && csum && col < N) atomicAdd(sb + col, csum);
     }
 }
 
@@ -663,7 +677,11 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
         oz2_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
     }
     const int64_t Kpad = (int64_t)P.nch * P.Kc;
-    dim3 g2((unsigned)((cols + 31) / 32), (unsigned)((Kpad + 63) / 64));
+    // k tiles per CTA: enough CTAs for the SMs (>= 8 waves' worth), at most 16 tiles each
+    const int64_t nkt = (Kpad + 63) / 64, ncb = (cols + 31) / 32;
+    int64_t gy = std::max<int64_t>(nkt / 16, (148 * 16 + ncb - 1) / ncb);
+    gy = std::max<int64_t>(1, std::min<int64_t>(gy, std::min<int64_t>(nkt, 65535)));
+    dim3 g2((unsigned)ncb, (unsigned)gy);
     oz2_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, P.n, P.np, P.p, P.Kc, P.nch, bmax, Bt8, P.ld8, fb,
                                                sb);
     return cudaGetLastError();
