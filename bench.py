@@ -472,7 +472,7 @@ def main():
         grid = runtime.Grid(wp.Gr, wp.Gc, rank, via_host=runtime.exchange_path() == "host")
         Ach, Bch = runtime.chunk_from_full(torch.from_numpy(A), torch.from_numpy(B), wp)
         Ach, Bch = Ach.to(dev), Bch.to(dev)
-        bufs = runtime.PanelBuffers(wp, tdt, dev, runtime.prepared_bytes(tdt, K, dev))
+        bufs = runtime.panel_buffers(wp, tdt, dev)
         dC = torch.empty((wp.rows, wp.cols), dtype=tdt, device=dev)
 
         compute = runtime.chunk_task(dC, wp, tile=c.tile)

@@ -89,15 +89,17 @@ extern "C" {
                                 prepared form of A's M rows (K wide) to C as packed rows of
                                 pdl_query("prepared_a/<dtype>/<K>") bytes (FP32 3xTF32:
                                 [TF32 hi: Kp floats][TF32 lo: Kp floats], Kp = K rounded up to
-                                32); B and N are ignored.  C: 16-byte aligned memory of the
-                                Worker's device.  PDL_EUNSUPPORTED for variants that exchange
-                                raw rows (query answers 0: FP64 dmma, ozaki2) */
+                                32; FP64 ozaki2: [residues: ld8 bytes][e_i: int32][4 bytes]
+                                [certificate row sum: u64]); B and N are ignored.  C: 16-byte
+                                aligned memory of the Worker's device.  PDL_EUNSUPPORTED for
+                                variants that exchange raw rows (query answers 0: FP64 dmma) */
 #define PDL_TASK_PREPARED_A 128u
                              /* with PDL_TASK_LOCAL: A holds M prepared rows (PDL_TASK_PREP_A
                                 on a Worker with the same variant and K) in this Worker's
                                 memory region; lda is ignored; the task skips A's preparation.
                                 The multi-rank runtime exchanges prepared A chunks so each
-                                Worker prepares only its own chunk */
+                                Worker prepares only its own chunk.  Variants that also read
+                                the raw rows (ozaki2) need task_matmul_prepared */
 #define PDL_TASK_SLOT(s) (((unsigned)(s) & 3u) << 4)
                              /* scratch slot s in 0..2 of the Worker: a task's own buffers (A
                                 split / slices / residues and exponents, residue planes,
@@ -204,6 +206,24 @@ int task_matmul_f32(const float *A, const float *B, float *C,
 int task_matmul_ex(int dtype, const void *A, int64_t lda, const void *B, int64_t ldb,
                    void *C, int64_t ldc, int64_t M, int64_t N, int64_t K, int64_t tile,
                    const char *group, const char *dist, unsigned flags);
+
+/*
+ * task_matmul_prepared -- a one-Worker task (PDL_TASK_LOCAL semantics) whose A
+ * is given as M prepared rows (PDL_TASK_PREP_A on a Worker with the same task
+ * variant and K; Aprep in this Worker's memory region, 16-byte aligned).
+ * Araw, lda_raw: the raw A rows (M x K, this Worker's device) for variants whose
+ * prepared tasks still read them -- ozaki2: the certificate's K1 recompute of
+ * uncertified elements, after the residue GEMMs (pdl_query("prepared_a/f64/<K>")
+ * ends in "+raw") -- else NULL.  raw_ready: a cudaEvent_t (as void *) the Worker
+ * stream waits on just before reading Araw, or NULL; so the raw rows may still be
+ * in flight while the residue GEMMs run.  B (K x N, ldb), C (M x N, ldc) as in
+ * task_matmul_ex.  flags: PDL_TASK_REUSE_B | PDL_TASK_GRAPH | PDL_TASK_SLOT(s).
+ * Errors: PDL_EINVAL (arguments; at pdl_run: Aprep or Araw not on the Worker's
+ * device), PDL_EUNSUPPORTED at pdl_run for variants without an A preparation.
+ */
+int task_matmul_prepared(int dtype, const void *Aprep, const void *Araw, int64_t lda_raw, void *raw_ready,
+                         const void *B, int64_t ldb, void *C, int64_t ldc, int64_t M, int64_t N, int64_t K,
+                         unsigned flags);
 
 /*
  * pdl_run -- map and execute all queued tasks in program order (access-mode

@@ -310,9 +310,9 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     int64_t oz2_ldr = 0, oz2_plane = 0;
     pdlk::Oz2Guard G2;
     int64_t oz_pr = 0, oz_ea_ld = 1, oz_sa_ld = 1;
-    if (ozaki2 && prepared)
-        return set_err(PDL_EUNSUPPORTED, "PDL_TASK_PREPARED_A with DGEMM_VARIANT=ozaki2: the certificate's K1 "
-                                         "recompute needs the raw A rows (exchange raw A chunks for this variant)");
+    if (ozaki2 && prepared && P2.check && !(t.Araw && locate(t.Araw) == w.device))
+        return set_err(PDL_EINVAL, "prepared A with DGEMM_VARIANT=ozaki2: the certificate's K1 recompute reads "
+                                   "the raw A rows -- pass them (task_matmul_prepared Araw, this Worker's device)");
     if (ozaki2) {
         // packed prepared-A rows: [residues: ld8][e_i: int][pad][sa_i: u64]
         oz_pr = pdlk::oz2_prep_row_bytes(P2);
@@ -473,9 +473,14 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (e == cudaSuccess)
                     e = pdlk::launch_ozaki2_reconstruct(Rs, oz2_ldr, oz2_plane, oz_ea + r0 * oz_ea_ld, oz_fb + c0, P2,
                                                         (double *)Cs, ldcd, nr, nc, cs, oz_ea_ld);
-                // flagged tiles: recomputed by K1 over the same operands (IEEE FP64)
+                // flagged tiles: recomputed by K1 over the same operands (IEEE FP64); a
+                // prepared task reads the raw rows it was given, once they are ready
+                const char *Ar = prepared ? (const char *)t.Araw : Ad;
+                const int64_t ldr_raw = prepared ? t.lda_raw : lda;
+                if (e == cudaSuccess && P2.check && prepared && t.raw_ready)
+                    e = cudaStreamWaitEvent(cs, (cudaEvent_t)t.raw_ready, 0);
                 if (e == cudaSuccess && P2.check) {
-                    e = pdlk::launch_dgemm_k1(enc, (const double *)(Ad + (size_t)(r0 * lda) * es), lda,
+                    e = pdlk::launch_dgemm_k1(enc, (const double *)(Ar + (size_t)(r0 * ldr_raw) * es), ldr_raw,
                                               (const double *)(Bd + (size_t)c0 * es), ldb, (double *)Cs, ldcd, nr, nc,
                                               K, cs, nullptr, nullptr, gs.flags, G2.ldf, gs.emask, G2.ldw);
                     ++nl;
@@ -578,15 +583,25 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
 
 // Bytes per prepared A row (PDL_TASK_PREP_A) of the task variant of PU `pu` for
 // inner dimension K, 0 when the variant exchanges raw rows: FP32 3xTF32 -> [hi:
-// Kp floats][lo: Kp floats]; FP64 (dmma; ozaki2, whose certificate recomputes from
-// the raw rows) -> 0.
-int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K) {
-    if (dtype != PDL_F32 || K <= 0) return 0;
+// Kp floats][lo: Kp floats]; FP64 ozaki2 -> [residues: ld8 bytes][e_i][pad][sa_i]
+// (pdlk::oz2_prep_row_bytes), and its prepared tasks still read the raw rows
+// (needs_raw: the certificate's K1 recompute); FP64 dmma -> 0.
+int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K, bool *needs_raw) {
+    if (needs_raw) *needs_raw = false;
+    if (K <= 0) return 0;
     WorkerCtx w;
     w.pu = pu;
     int sl, rn;
-    if (worker_ozaki(w, false, &sl, &rn) || worker_sgemm_ozaki2(w)) return 0;
-    return 2 * round_up(K, pdlk::K2_BK) * 4;
+    if (worker_ozaki(w, dtype == PDL_F64, &sl, &rn)) return 0;
+    if (dtype == PDL_F32) return worker_sgemm_ozaki2(w) ? 0 : 2 * round_up(K, pdlk::K2_BK) * 4;
+    int nmod = 0, bits = 0;
+    if (!worker_ozaki2(w, &nmod, &bits)) return 0;
+    double tau = 0.0;
+    const bool guard = worker_oz2_guard(w, &tau);
+    const pdlk::Ozaki2Plan P = pdlk::ozaki2_plan(1, 1, K, nmod, bits, guard);
+    if (guard && !P.check) return 0;   // runs K1: raw rows
+    if (needs_raw) *needs_raw = P.check != 0;
+    return pdlk::oz2_prep_row_bytes(P);
 }
 
 // PDL_TASK_PREP_A: the A preparation of the Worker's task variant for the task's M
@@ -600,23 +615,36 @@ int run_prep_a(WorkerCtx &w, const Task &t) {
                        t.dtype == PDL_F64 ? "FP64" : "FP32");
     if (locate(t.C) != w.device || ((uintptr_t)t.C % 16))
         return set_err(PDL_EINVAL, "PDL_TASK_PREP_A: the output must be 16-byte aligned memory of the Worker's device");
-    const int64_t Kp = round_up(t.K, pdlk::K2_BK);
-    const float *A = (const float *)t.A;
+    const int es = t.dtype == PDL_F64 ? 8 : 4;
+    const char *A = (const char *)t.A;
     int64_t lda = t.lda;
-    if (locate(t.A) != w.device) {   // stage the raw rows into the Worker's memory region
+    if (locate(t.A) != w.device || ((uintptr_t)A % 16) || (lda * es) % 16) {   // stage into the Worker's MR
         void *p = nullptr;
-        lda = round_up(t.K, 4);
-        int rc = ensure_buf(w, BUF_A, (size_t)(t.M * lda * 4), &p);
+        lda = round_up(t.K, 16 / es);
+        int rc = ensure_buf(w, BUF_A, (size_t)(t.M * lda * es), &p);
         if (rc) return rc;
-        CUDA_TRY(cudaMemcpy2DAsync(p, (size_t)(lda * 4), t.A, (size_t)(t.lda * 4), (size_t)(t.K * 4), (size_t)t.M,
+        CUDA_TRY(cudaMemcpy2DAsync(p, (size_t)(lda * es), t.A, (size_t)(t.lda * es), (size_t)(t.K * es), (size_t)t.M,
                                    cudaMemcpyDefault, w.stream));
-        g->xfer.count(locate(t.A), w.device, t.M * t.K * 4);
-        A = (const float *)p;
+        g->xfer.count(locate(t.A), w.device, t.M * t.K * es);
+        A = (const char *)p;
     }
-    float *hi = (float *)t.C;
-    cudaError_t e = pdlk::launch_split_rows(A, lda, t.M, t.K, hi, hi + Kp, Kp, w.stream, 2 * Kp);
-    if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
-    w.launches += 1;
+    pdlk::set_worker_sms(w.sm_limit);
+    cudaError_t e;
+    if (t.dtype == PDL_F32) {
+        const int64_t Kp = round_up(t.K, pdlk::K2_BK);
+        float *hi = (float *)t.C;
+        e = pdlk::launch_split_rows((const float *)A, lda, t.M, t.K, hi, hi + Kp, Kp, w.stream, 2 * Kp);
+        w.launches += 1;
+    } else {
+        int nmod = 0, bits = 0;
+        double tau = 0.0;
+        worker_ozaki2(w, &nmod, &bits);
+        const pdlk::Ozaki2Plan P = pdlk::ozaki2_plan(t.M, 1, t.K, nmod, bits, worker_oz2_guard(w, &tau));
+        int8_t *a8 = (int8_t *)t.C;
+        e = pdlk::launch_ozaki2_split_a((const double *)A, lda, t.M, t.K, P, a8, (int *)(a8 + P.ld8), w.stream,
+                                        &w.launches, (unsigned long long *)(a8 + P.ld8 + 8), pr, pr / 4, pr / 8);
+    }
+    if (e != cudaSuccess) return set_err(PDL_ECUDA, "A preparation launch failed: %s", cudaGetErrorString(e));
     return PDL_OK;
 }
 
@@ -808,7 +836,7 @@ std::string graph_key(const WorkerCtx &w, const Task &t, const void *A, const vo
 
 int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
     const bool want = (t.flags & PDL_TASK_GRAPH) || env_on("PDL_GRAPH");
-    if (!want || (t.flags & PDL_TASK_REUSE_B) || g->dry_run || rows <= 0 || cols <= 0)
+    if (!want || (t.flags & PDL_TASK_REUSE_B) || t.raw_ready || g->dry_run || rows <= 0 || cols <= 0)
         return run_rect(w, t, A, B, C, rows, cols);
     CUDA_TRY(cudaSetDevice(w.device));
     const std::string key = graph_key(w, t, A, B, C, rows, cols);

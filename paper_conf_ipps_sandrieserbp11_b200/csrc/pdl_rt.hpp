@@ -141,6 +141,11 @@ struct Task {
     std::string group;
     unsigned flags;
     DistSpec dist;
+    // task_matmul_prepared: the raw A rows a prepared task still reads (the
+    // Ozaki-II certificate's K1 recompute) and the event that makes them ready
+    const void *Araw = nullptr;
+    int64_t lda_raw = 0;
+    void *raw_ready = nullptr;
 };
 
 // Bytes moved along the descriptor's interconnects in the last run (pdl_query
@@ -228,7 +233,7 @@ int run_dynamic(const Task &t, const std::vector<int> &gw);
 int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols);
 int execute(bool sync);
 int enable_peer(int from, int to);
-int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K);
+int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K, bool *needs_raw = nullptr);
 int run_prep_a(WorkerCtx &w, const Task &t);
 // pdl_xchg.cu
 bool exchange_applies(const Task &t, const Plan &plan, const std::vector<int> &gw);

@@ -251,6 +251,30 @@ int task_matmul_ex(int dtype, const void *A, int64_t lda, const void *B, int64_t
     return enqueue(dtype, A, lda, B, ldb, C, ldc, M, N, K, tile, group, dist, flags);
 }
 
+int task_matmul_prepared(int dtype, const void *Aprep, const void *Araw, int64_t lda_raw, void *raw_ready,
+                         const void *B, int64_t ldb, void *C, int64_t ldc, int64_t M, int64_t N, int64_t K,
+                         unsigned flags) {
+    int rc = check_loaded();
+    if (rc) return rc;
+    if (dtype != PDL_F64 && dtype != PDL_F32) return set_err(PDL_EINVAL, "unknown dtype %d", dtype);
+    if (M < 0 || N < 0 || K < 0 || lda_raw < 0 || ldb < 0 || ldc < 0) return set_err(PDL_EINVAL, "negative size");
+    if (flags & ~(PDL_TASK_REUSE_B | PDL_TASK_GRAPH | PDL_TASK_SLOT(3)))
+        return set_err(PDL_EINVAL, "task_matmul_prepared: flags may be PDL_TASK_REUSE_B | PDL_TASK_GRAPH | "
+                                   "PDL_TASK_SLOT(s) (got 0x%x)", flags);
+    if (((flags >> 4) & 3u) >= 3u) return set_err(PDL_EINVAL, "scratch slot %u out of range (0..2)", (flags >> 4) & 3u);
+    if (M == 0 || N == 0) return PDL_OK;
+    if (!C || (K > 0 && (!Aprep || !B))) return set_err(PDL_EINVAL, "Aprep, B or C is NULL with nonzero sizes");
+    const int64_t ldb_ = ldb ? ldb : N, ldc_ = ldc ? ldc : N, ldr = lda_raw ? lda_raw : K;
+    if (ldb_ < N || ldc_ < N || (Araw && ldr < K)) return set_err(PDL_EINVAL, "leading dimension smaller than the row width");
+    Task t{dtype, Aprep, 0, B, ldb_, C, ldc_, M, N, K, 0, false, "", flags | PDL_TASK_LOCAL | PDL_TASK_PREPARED_A,
+           DistSpec()};
+    t.Araw = Araw;
+    t.lda_raw = ldr;
+    t.raw_ready = raw_ready;
+    g->queue.push_back(t);
+    return PDL_OK;
+}
+
 int pdl_run(void) { return execute(true); }
 
 int pdl_run_async(void) { return execute(false); }
@@ -447,7 +471,10 @@ int pdl_query(const char *key, char *out, size_t len) {
             std::vector<int> gw = m.group_workers(nullptr);
             if (gw.empty()) return set_err(PDL_ENOWORKER, "no gpu Worker");
             const int pu = g->workers.empty() ? gw[0] : g->workers[0].pu;
-            res = std::to_string(prepared_a_row_bytes(pu, strcmp(dts, "f64") ? PDL_F32 : PDL_F64, K));
+            bool raw = false;
+            const int64_t pr = prepared_a_row_bytes(pu, strcmp(dts, "f64") ? PDL_F32 : PDL_F64, K, &raw);
+            // "<bytes>" or "<bytes>+raw" (the prepared task also reads the raw rows)
+            res = std::to_string(pr) + (raw ? "+raw" : "");
         }
         else if (k == "plan") res = g->plan_json;
         else if (k == "groups") {

@@ -145,10 +145,16 @@ class PanelBuffers:
     (FP32 3xTF32: TF32 hi/lo, 2x the raw bytes, instead of every Worker of a grid
     row splitting the whole panel again)."""
 
-    def __init__(self, wp: WorkerPlan, dtype, device, prep_bytes: int = 0):
+    def __init__(self, wp: WorkerPlan, dtype, device, prep_bytes: int = 0, keep_raw: bool = False):
         self.prepared = prep_bytes > 0
+        # raw A rows beside the prepared ones: variants whose prepared tasks still
+        # read them (ozaki2: the certificate's K1 recompute); they travel after the
+        # prepared chunks and are needed only at the end of each chunk task
+        self.Araw = None
         if self.prepared:
             self.A = torch.empty((wp.Gc * wp.qa, prep_bytes), dtype=torch.uint8, device=device)
+            if keep_raw:
+                self.Araw = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dtype, device=device)
         else:
             self.A = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dtype, device=device)
         self.B = torch.empty((wp.Gr * wp.qb, wp.cols), dtype=dtype, device=device)
@@ -157,14 +163,26 @@ class PanelBuffers:
             # not wait for its chunk's landing produces NaN rows of C
             self.A.fill_(255 if self.prepared else float("nan"))
             self.B.fill_(float("nan"))
+            if self.Araw is not None:
+                self.Araw.fill_(float("nan"))
+
+
+def prepared_info(dtype, K, device):
+    """(prepared-A row bytes, prepared tasks read raw rows too) of this Worker's
+    task variant for device panels; (0, False): exchange raw rows."""
+    if device is None or torch.device(device).type != "cuda":
+        return 0, False
+    return pdl.prepared_a_info(dtype, K)
 
 
 def prepared_bytes(dtype, K, device) -> int:
-    """Prepared-A row bytes of this Worker's task variant for device panels
-    (0: exchange raw rows)."""
-    if device is None or torch.device(device).type != "cuda":
-        return 0
-    return pdl.prepared_a_row_bytes(dtype, K)
+    return prepared_info(dtype, K, device)[0]
+
+
+def panel_buffers(wp: WorkerPlan, dtype, device, prepared: bool = True) -> PanelBuffers:
+    """PanelBuffers in the exchange format of this Worker's task variant."""
+    pb, raw = prepared_info(dtype, wp.K, device) if prepared else (0, False)
+    return PanelBuffers(wp, dtype, device, pb, raw)
 
 
 def exchange(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers):
@@ -374,25 +392,33 @@ def exchange_overlapped(Ach, Bch, wp: WorkerPlan, grid: Grid, bufs: PanelBuffers
     Bp = bufs.B[: wp.K]
     qa, c = wp.qa, wp.c
     if bufs.prepared:
-        # the own chunk's prepared rows (TF32 hi/lo ...), straight into the panel
+        # the own chunk's prepared rows (TF32 hi/lo, Ozaki-II residues ...), straight
+        # into the panel: each Worker prepares only its own chunk
         pdl.prepare_a(Ach, bufs.A[c * qa:(c + 1) * qa])
         pdl.run_async()
+        if bufs.Araw is not None:
+            bufs.Araw[c * qa:(c + 1) * qa].copy_(Ach)
     else:
         bufs.A[c * qa:(c + 1) * qa].copy_(Ach)
-    works = {}
+    works, raw_works = {}, {}
     if wp.Gc > 1:
         for j in range(wp.Gc):   # same order on every rank of the row
             works[j] = _broadcast(bufs.A[j * qa:(j + 1) * qa], grid.row_ranks[j], grid.row_group)
+        if bufs.Araw is not None:   # after every prepared chunk: needed only by the recompute
+            for j in range(wp.Gc):
+                raw_works[j] = _broadcast(bufs.Araw[j * qa:(j + 1) * qa], grid.row_ranks[j], grid.row_group)
     if overlap_a is None:
-        overlap_a = wp.Gc == 1 or not bufs.A.is_cuda or overlap_pays(wp, bufs.A.element_size())
+        overlap_a = wp.Gc == 1 or not bufs.A.is_cuda or \
+            overlap_pays(wp, bufs.A.shape[1] * bufs.A.element_size() / max(1, wp.K))
     if overlap_a:
-        compute_groups(wp, bufs, Bp, compute, works, concurrent)
+        compute_groups(wp, bufs, Bp, compute, works, concurrent, raw_works)
     else:
-        for w in works.values():
+        for w in list(works.values()) + list(raw_works.values()):
             w.wait()
         if wp.rows > 0 and wp.cols > 0:
-            compute(wp.c, 0, wp.rows, bufs.A[: wp.rows], Bp, True)
-    for w in works.values():
+            kw = {} if bufs.Araw is None else {"raw": (bufs.Araw[: wp.rows], None)}
+            compute(wp.c, 0, wp.rows, bufs.A[: wp.rows], Bp, True, **kw)
+    for w in list(works.values()) + list(raw_works.values()):
         w.wait()
     return bufs.A[: wp.rows], Bp
 
@@ -425,7 +451,28 @@ def tasks_may_overlap(*panels) -> bool:
     return pdl.query(key) == "yes"
 
 
-def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concurrent=None):
+_raw_streams = {}
+
+
+def _raw_ready(grp, raw_works):
+    """An event after the landing of the raw chunks of `grp` (None: all local),
+    recorded on a helper stream so no compute stream waits for them early."""
+    pending = [raw_works[j] for j in grp if j in raw_works]
+    if not pending:
+        return None
+    dev = torch.cuda.current_device()
+    if dev not in _raw_streams:
+        _raw_streams[dev] = torch.cuda.Stream(device=dev)
+    s = _raw_streams[dev]
+    ev = torch.cuda.Event()
+    with torch.cuda.stream(s):
+        for w in pending:
+            w.wait()
+        ev.record(s)
+    return ev
+
+
+def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concurrent=None, raw_works=None):
     """The chunk computations of exchange_overlapped, in at most three launches
     so each stays wave-efficient: the own chunk at once, then the chunks before
     it (broadcast first, so they land first), then the chunks after it.
@@ -454,11 +501,14 @@ def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concu
         lo, hi = chunk_rows(wp, grp[0])[0], chunk_rows(wp, grp[-1])[1]
         if hi <= lo or wp.cols <= 0:
             continue
+        kw = {}   # raw A rows only for variants that read them (compute callbacks may not take them)
+        if bufs.Araw is not None:
+            kw["raw"] = (bufs.Araw[lo:hi], _raw_ready(grp, raw_works or {}))
         if first or not concurrent:
             for j in grp:
                 if j != c and j in works:
                     works[j].wait()
-            compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first)
+            compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first, **kw)
         else:
             side = _side_stream(len(joins))
             side.wait_event(ready)
@@ -468,7 +518,7 @@ def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concu
                         works[j].wait()
                 pdl.set_stream(side)
                 try:
-                    compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first, slot=len(joins) + 1)
+                    compute(grp[0], lo, hi, bufs.A[lo:hi], Bp, first, slot=len(joins) + 1, **kw)
                 finally:
                     pdl.set_stream(main)
                 done = torch.cuda.Event()
@@ -484,12 +534,16 @@ def chunk_task(Cblock, wp: WorkerPlan, tile=0):
     on this process's Worker; the prepared B panel is reused after the first;
     `slot` is the task's scratch slot (compute_groups gives each concurrent
     launch group its own)."""
-    def compute(j, lo, hi, Arows, Bp, first, slot=0):
+    def compute(j, lo, hi, Arows, Bp, first, slot=0, raw=None):
         Cv = Cblock[lo:hi]
-        prepared = Arows.dtype == torch.uint8   # prepared A rows (PanelBuffers prep_bytes)
-        pdl.task_matmul(Arows, Bp, Cv, M=hi - lo, N=wp.cols, K=wp.K, tile=tile,
-                        lda=0 if prepared else Arows.stride(0), ldb=Bp.stride(0), ldc=Cv.stride(0), local=True,
-                        reuse_b=not first, slot=slot, prepared_a=prepared)
+        if Arows.dtype == torch.uint8:   # prepared A rows (PanelBuffers prep_bytes)
+            Araw, ev = raw if raw is not None else (None, None)
+            pdl.task_matmul_prepared(Arows, Bp, Cv, M=hi - lo, N=wp.cols, K=wp.K, Araw=Araw,
+                                     lda_raw=0 if Araw is None else Araw.stride(0), raw_ready=ev,
+                                     ldb=Bp.stride(0), ldc=Cv.stride(0), reuse_b=not first, slot=slot)
+        else:
+            pdl.task_matmul(Arows, Bp, Cv, M=hi - lo, N=wp.cols, K=wp.K, tile=tile, lda=Arows.stride(0),
+                            ldb=Bp.stride(0), ldc=Cv.stride(0), local=True, reuse_b=not first, slot=slot)
         pdl.run_async()
     return compute
 
@@ -524,7 +578,7 @@ def distributed_matmul(A_full, B_full, C_full, tile=0, group=None, overlap=True)
     dev = torch.device("cuda", torch.cuda.current_device())
     Ach, Bch = chunk_from_full(A_full, B_full, wp)
     Ach, Bch = Ach.to(dev, non_blocking=True), Bch.to(dev, non_blocking=True)
-    bufs = PanelBuffers(wp, A_full.dtype, dev, prepared_bytes(A_full.dtype, K, dev) if overlap else 0)
+    bufs = panel_buffers(wp, A_full.dtype, dev, prepared=overlap)
     Cb = torch.empty((wp.rows, wp.cols), dtype=C_full.dtype, device=dev)
     pdl.set_stream(torch.cuda.current_stream())
     if overlap:

@@ -32,6 +32,13 @@ def main():
     pdl.load(pdl.descriptor_xml(world, variant), rank=rank, nranks=world)
     A = W.signed((M, K), dt, 501)
     B = W.signed((K, N), dt, 502)
+    if os.environ.get("DIST_CHECK_ADVERSARIAL") == "1" and K >= 2:
+        # elements the Ozaki-II certificate cannot certify (a 2^60 entry meeting a
+        # zero of B): they go through the K1 recompute, which reads raw A rows
+        for i in (3, M // 2, M - 2):
+            A[i, :] = 0.0
+            A[i, :2] = [2.0 ** 60, 1.0]
+        B[:2, 5] = [0.0, 1.0]
     C = np.full((M, N), np.nan, dtype=dt)
     wp = runtime.distributed_matmul(torch.from_numpy(A), torch.from_numpy(B), torch.from_numpy(C), tile=tile)
     rows = np.arange(wp.row0, wp.row1)
@@ -43,6 +50,10 @@ def main():
                                 D[:, wp.col0:wp.col1])
         err = float(e.max())
         ok = err <= (1e-12 if dt == np.float64 else 1e-5)
+        if not ok:
+            bad = np.argwhere(~(e <= (1e-12 if dt == np.float64 else 1e-5)))
+            print(f"dist_check rank {rank} rect {wp.row0}:{wp.row1} x {wp.col0}:{wp.col1}: {len(bad)} bad, "
+                  f"first {bad[:5].tolist()} err {err:.3e}", file=sys.stderr, flush=True)
     t = torch.tensor([0.0 if ok else 1.0, err])
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     if rank == 0:

@@ -33,7 +33,8 @@ def _run(world, *args, env_extra=None):
     env = dict(os.environ, PDL_ALLOW_OVERSUBSCRIBE="1", **(env_extra or {}))
     env.pop("PDL_DRY_RUN", None)
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
-    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    errs = [ln for ln in r.stderr.splitlines() if "Error" in ln or "error" in ln or "dist_check" in ln]
+    assert r.returncode == 0, r.stdout[-3000:] + "\n".join(errs[:40]) + r.stderr[-1500:]
     assert "ok=True" in r.stdout
 
 
@@ -133,6 +134,16 @@ def test_late_chunks_are_waited_for(world, dt):
          env_extra={"PDL_TEST_EXCHANGE_DELAY_US": "3000", "PDL_OVERLAP_A": "1"})
 
 
+@pytest.mark.parametrize("world", [4, 8])
+def test_ozaki2_prepared_exchange_with_late_raw_rows(world):
+    """Ozaki-II exchanges prepared chunks (residues + row scales + certificate
+    sums) and, after them, the raw chunks its certificate's K1 recompute reads;
+    with every landing 3 ms late and adversarial rows that force the recompute,
+    C is still right: the recompute waits for its raw rows (raw_ready event)."""
+    _run(world, "f64", 1000, 700, 300, 64, "ozaki2",
+         env_extra={"PDL_TEST_EXCHANGE_DELAY_US": "3000", "PDL_OVERLAP_A": "1", "DIST_CHECK_ADVERSARIAL": "1"})
+
+
 def test_a_missing_wait_corrupts_c():
     """Negative control for the test above: with the A-chunk waits dropped
     (PDL_TEST_DROP_WAITS=1) the same run computes on chunks that have not landed
@@ -142,12 +153,14 @@ def test_a_missing_wait_corrupts_c():
     assert r.returncode != 0 or "ok=False" in r.stdout, r.stdout[-2000:]
 
 
-@pytest.mark.parametrize("G", [2, 8])
-def test_prepared_a_chunks_bitwise(G, monkeypatch):
-    """FP32 3xTF32 exchanges PREPARED A chunks (PDL_TASK_PREP_A: TF32 hi/lo rows),
-    so each Worker splits only its own chunk: the chunk launches on the prepared
-    panel (PDL_TASK_PREPARED_A) give bitwise the raw-panel C, serial or on side
-    streams, for every Worker position."""
+@pytest.mark.parametrize("G,variant", [(2, None), (8, None), (4, "ozaki2"), (8, "ozaki2")])
+def test_prepared_a_chunks_bitwise(G, variant, monkeypatch):
+    """Variants with an A preparation exchange PREPARED A chunks (PDL_TASK_PREP_A:
+    FP32 TF32 hi/lo rows; Ozaki-II residues, scales and certificate sums), so each
+    Worker prepares only its own chunk: the chunk launches on the prepared panel
+    (task_matmul_prepared) give bitwise the raw-panel C, serial or on side
+    streams, for every Worker position -- Ozaki-II with adversarial rows whose
+    elements its certificate sends to the K1 recompute over the raw rows."""
     import numpy as np
 
     sys.path.insert(0, ROOT)
@@ -164,28 +177,39 @@ def test_prepared_a_chunks_bitwise(G, monkeypatch):
         monkeypatch.delenv("PDL_DRY_RUN")
     torch = pytest.importorskip("torch")
     rng = np.random.default_rng(9)
-    A = torch.from_numpy(rng.uniform(-1, 1, (M, K)).astype(np.float32))
-    B = torch.from_numpy(rng.uniform(-1, 1, (K, N)).astype(np.float32))
+    npdt, tdt = (np.float64, torch.float64) if variant else (np.float32, torch.float32)
+    A = torch.from_numpy(rng.uniform(-1, 1, (M, K)).astype(npdt))
+    B = torch.from_numpy(rng.uniform(-1, 1, (K, N)).astype(npdt))
+    if variant:
+        for i in (7, 700, 1400):
+            A[i, :] = 0.0
+            A[i, :2] = torch.tensor([2.0 ** 60, 1.0], dtype=tdt)
+        B[:2, 11] = torch.tensor([0.0, 1.0], dtype=tdt)
     dev = torch.device("cuda", 0)
-    pdl.load(pdl.descriptor_path(1))
+    pdl.load(pdl.descriptor_xml(1, props={"DGEMM_VARIANT": variant}) if variant else pdl.descriptor_path(1))
     try:
-        pb = runtime.prepared_bytes(torch.float32, K, dev)
-        assert pb == 2 * ((K + 31) // 32 * 32) * 4
-        assert runtime.prepared_bytes(torch.float64, K, dev) == 0     # dmma exchanges raw rows
+        pb, needs_raw = runtime.prepared_info(tdt, K, dev)
+        if variant:
+            assert pb > 0 and needs_raw
+        else:
+            assert pb == 2 * ((K + 31) // 32 * 32) * 4 and not needs_raw
+            assert runtime.prepared_bytes(torch.float64, K, dev) == 0     # dmma exchanges raw rows
         for wp in wps:
-            raw = runtime.PanelBuffers(wp, torch.float32, dev)
-            prep = runtime.PanelBuffers(wp, torch.float32, dev, pb)
+            raw = runtime.PanelBuffers(wp, tdt, dev)
+            prep = runtime.panel_buffers(wp, tdt, dev)
             raw.A.zero_()
             raw.A[: wp.rows].copy_(A[wp.row0: wp.row1])
             for b in (raw, prep):
                 b.B[: wp.K].copy_(B[:, wp.col0: wp.col1])
+            if prep.Araw is not None:
+                prep.Araw.copy_(raw.A)
             pdl.set_stream(torch.cuda.current_stream())
             for j in range(wp.Gc):   # every chunk prepared (here on one Worker)
                 pdl.prepare_a(raw.A[j * wp.qa:(j + 1) * wp.qa], prep.A[j * wp.qa:(j + 1) * wp.qa])
             pdl.run()
             out = []
             for bufs, conc in ((raw, False), (prep, False), (prep, True)):
-                C = torch.full((wp.rows, wp.cols), float("nan"), device=dev)
+                C = torch.full((wp.rows, wp.cols), float("nan"), dtype=tdt, device=dev)
                 runtime.compute_groups(wp, bufs, bufs.B[: wp.K], runtime.chunk_task(C, wp, tile), {}, conc)
                 pdl.sync()
                 torch.cuda.synchronize()
@@ -217,6 +241,6 @@ def test_prep_a_errors():
         pdl.task_matmul(Ap, Bd, C, M=64, N=32, K=96, local=True, prepared_a=True)
         with pytest.raises(pdl.PDLError) as e:
             pdl.run()
-        assert e.value.code == pdl.PDL_EUNSUPPORTED      # the certificate recomputes from raw rows
+        assert e.value.code == pdl.PDL_EINVAL            # the certificate recomputes from raw rows: none given
     finally:
         pdl.unload()

@@ -42,13 +42,15 @@ def time_worker(wp, dt, tile, concurrent, reps, raw=False):
     of runtime.compute_groups."""
     dev = torch.device("cuda", torch.cuda.current_device())
     g = torch.Generator(device="cuda").manual_seed(11)
-    prep = 0 if raw else runtime.prepared_bytes(dt, wp.K, dev)
-    bufs = runtime.PanelBuffers(wp, dt, dev, prep)
+    bufs = runtime.panel_buffers(wp, dt, dev, prepared=not raw)
+    prep = bufs.prepared
     Araw = torch.empty((wp.Gc * wp.qa, wp.K), dtype=dt, device=dev).uniform_(generator=g)
     bufs.B.uniform_(generator=g)
     if prep:
         pdl.prepare_a(Araw, bufs.A)   # the chunks the other Workers prepared (untimed)
         pdl.run()
+        if bufs.Araw is not None:     # raw rows for the certificate's recompute (landed)
+            bufs.Araw.copy_(Araw)
     else:
         bufs.A.copy_(Araw)
     qa, c = wp.qa, wp.c
