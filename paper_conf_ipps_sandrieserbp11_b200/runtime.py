@@ -451,6 +451,21 @@ def tasks_may_overlap(*panels) -> bool:
     return pdl.query(key) == "yes"
 
 
+def chunk_groups(wp: WorkerPlan):
+    """The Worker's chunk launches, in order: its own chunk (computes at once), then
+    two groups of contiguous chunks.  The broadcasts arrive in chunk order, so the
+    second group is the chunk that lands first when the own chunk sits at an end of
+    the row (c = 0: [1], then [2..]; c = Gc-1: [0], then [1..Gc-2]) -- it computes
+    while the rest lands -- and otherwise the chunks before / after the own one
+    (whose earlier chunks already landed while the own chunk computed)."""
+    c, G = wp.c, wp.Gc
+    if G >= 3 and c == 0:
+        return [[0], [1], list(range(2, G))]
+    if G >= 3 and c == G - 1:
+        return [[c], [0], list(range(1, c))]
+    return [[c], list(range(0, c)), list(range(c + 1, G))]
+
+
 _raw_streams = {}
 
 
@@ -489,7 +504,7 @@ def compute_groups(wp: WorkerPlan, bufs: PanelBuffers, Bp, compute, works, concu
     if concurrent is None:
         concurrent = tasks_may_overlap(bufs.A, Bp)
     main = torch.cuda.current_stream() if concurrent else None
-    groups = [[c], list(range(0, c)), list(range(c + 1, wp.Gc))]
+    groups = chunk_groups(wp)
     first = True
     joins = []
     if concurrent:

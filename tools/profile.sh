@@ -6,7 +6,7 @@
 #    roofline "traffic" of a step: tools/ncu_traffic_sum.py)
 set -x
 OUT=${OUT:-gpurun_out}
-WHAT=${WHAT:-"k1 k2 k3 oz oz2 oz32"}
+WHAT=${WHAT:-"k1 k2 k3 oz2"}
 mkdir -p $OUT
 B="python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-cublas --no-alt --e2e-steps 1"
 P="python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-cublas --no-e2e --no-alt"
@@ -18,16 +18,13 @@ for w in $WHAT; do
     k2) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_f32.csv $B --dtype f32 > $OUT/launches_f32.log 2>&1
         ncu --set full --clock-control none --import-source on -k regex:gemm_3xtf32 -s 1 -c 1 -o $OUT/prof_k2 -f $P --dtype f32 > $OUT/prof_k2.log 2>&1 ;;
     k3) ncu --set full --clock-control none --import-source on -k regex:split -s 2 -c 2 -o $OUT/prof_k3 -f $P --dtype f32 > $OUT/prof_k3.log 2>&1 ;;
-    oz) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_oz.csv $B --variant ozaki > $OUT/launches_oz.log 2>&1
-        ncu --set full --clock-control none --import-source on -k regex:oz_gemm -s 7 -c 1 -o $OUT/prof_oz -f $P --variant ozaki > $OUT/prof_oz.log 2>&1
-        ncu --set full --clock-control none --import-source on -k regex:oz_split -s 2 -c 2 -o $OUT/prof_ozsplit -f $P --variant ozaki > $OUT/prof_ozsplit.log 2>&1
-        ncu $DR -k regex:oz_gemm -s 6 -c 6 --log-file $OUT/traffic_ozaki.csv $P --variant ozaki > $OUT/traffic_oz.log 2>&1 ;;
     oz2) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_oz2.csv $B --variant ozaki2 > $OUT/launches_oz2.log 2>&1
+        # 14 GEMM launches per step at C4 (13 moduli + the certificate, R21); step 2 of the
+        # warm-up + timed run: skip the first step's 14, capture a residue GEMM and the certificate
         ncu --set full --clock-control none --import-source on -k 'regex:oz2?_gemm' -s 14 -c 1 -o $OUT/prof_oz2 -f $P --variant ozaki2 > $OUT/prof_oz2.log 2>&1
-        ncu --set full --clock-control none --import-source on -k 'regex:oz2_(rowmax|residue|colmax|split|crt|reconstruct)' -s 5 -c 5 -o $OUT/prof_oz2aux -f $P --variant ozaki2 > $OUT/prof_oz2aux.log 2>&1
-        ncu $DR -k 'regex:oz2?_gemm' -s 13 -c 13 --log-file $OUT/traffic_ozaki2.csv $P --variant ozaki2 > $OUT/traffic_oz2.log 2>&1 ;;
-    oz32) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_oz32.csv $B --dtype f32 --variant ozaki > $OUT/launches_oz32.log 2>&1
-        ncu $DR -k regex:oz_gemm -s 3 -c 3 --log-file $OUT/traffic_ozaki32.csv $P --dtype f32 --variant ozaki > $OUT/traffic_oz32.log 2>&1 ;;
+        ncu --set full --clock-control none --import-source on -k 'regex:oz2?_gemm' -s 27 -c 1 -o $OUT/prof_oz2cert -f $P --variant ozaki2 > $OUT/prof_oz2cert.log 2>&1
+        ncu --set full --clock-control none --import-source on -k 'regex:oz2_(rowmax|residue|colmax|split|crt|reconstruct)|dgemm_k1' -s 6 -c 6 -o $OUT/prof_oz2aux -f $P --variant ozaki2 > $OUT/prof_oz2aux.log 2>&1
+        ncu $DR -k 'regex:oz2?_gemm' -s 14 -c 14 --log-file $OUT/traffic_ozaki2.csv $P --variant ozaki2 > $OUT/traffic_oz2.log 2>&1 ;;
   esac
 done
 ls -la $OUT

@@ -26,6 +26,7 @@ from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
 NVLINK = 770e9
 # the task variants of this build (Ozaki scheme I is retired)
 CURRENT = {("f64", "dmma"), ("f32", "3xtf32"), ("f64", "ozaki2")}
+CLOCK = {}   # (dtype, variant, G) -> median SM MHz during the worst Worker's timing (if recorded)
 
 
 def rates():
@@ -44,7 +45,8 @@ def emulated():
     certificate, override round 1's)."""
     out = {}
     for fn in sorted(os.listdir(os.path.join(ROOT, "profiles")), key=lambda f: (not f.startswith("r01"), f)):
-        if (fn.startswith("r01_worker_emulate_") or fn.startswith("r02_worker_emulate_")) and fn.endswith(".jsonl"):
+        if (fn.startswith("r01_worker_emulate_") or fn.startswith("r02_worker_emulate_")) and fn.endswith(".jsonl") \
+                and "_raw" not in fn:   # r02 "_raw": the raw-exchange comparison runs
             with open(os.path.join(ROOT, "profiles", fn)) as f:
                 for line in f:
                     d = json.loads(line)
@@ -52,32 +54,56 @@ def emulated():
                         var = {"default": "dmma" if d["dtype"] == "f64" else "3xtf32"}.get(
                             d.get("variant", "default"), d.get("variant"))
                         out[(d["dtype"], var, d["G"])] = d["max_concurrent_ms"] / 1e3
+                        CLOCK[(d["dtype"], var, d["G"])] = d.get("sm_mhz_worst")
     return out
 
 
 def a_bytes_per_elem(dt, var, K):
-    """Bytes per A element on NVLink: FP32 3xTF32 exchanges prepared TF32 hi/lo rows
-    (runtime.PanelBuffers prep_bytes: 2 Kp floats per row), the others raw rows."""
+    """Latency-critical bytes per A element on NVLink: the prepared rows of the
+    variants that exchange them (runtime.panel_buffers; pdl prepared_a): FP32
+    3xTF32 TF32 hi/lo (2 Kp floats per row); FP64 Ozaki-II residues of 13 moduli +
+    the certificate plane + 16 bytes of row scale / certificate sum.  Ozaki-II's
+    raw rows travel after them and are read only by each chunk task's final K1
+    recompute (hidden behind the residue GEMMs; not counted here).  K1: raw rows."""
     if dt == "f32" and var == "3xtf32":
         return 2 * (-(-K // 32) * 32) * 4 / K
+    if dt == "f64" and var == "ozaki2":
+        import json
+        n = json.loads(pdl.query(f"ozaki2_plan/{K}"))["n"]
+        kc = -(-K // 128) * 128
+        return ((n + 1) * kc + 16) / K
     return 8 if dt == "f64" else 4
 
 
 def model(M, N, K, tile, G, rate, es, t_meas=None, a_es=None):
+    """Worst Worker's step: B column-panel all-gather (exposed), then its chunk
+    launches in runtime.chunk_groups order, each starting when the previous one
+    ends and its chunks have landed (broadcasts in chunk order, one chunk's bytes
+    at a time at NVLINK), compute split over the chunks by rows."""
+    from paper_conf_ipps_sandrieserbp11_b200 import runtime
     pdl.unload()
     pdl.load(pdl.descriptor_path(G))
     worst = 0.0
     for w in range(G):
         p = pdl.plan(M, N, K, tile, worker=w)
-        rows, cols = p["row1"] - p["row0"], p["col1"] - p["col0"]
+        wp = runtime.WorkerPlan(p["G"], p["Gr"], p["Gc"], p["r"], p["c"], p["row0"], p["row1"], p["col0"],
+                                p["col1"], p["qa"], p["qb"], M, N, K)
+        rows, cols = wp.rows, wp.cols
         t_comp = t_meas if t_meas is not None else 2.0 * rows * cols * K / rate
-        b_bytes = K * cols * es * (1 - 1 / p["Gr"])            # received B chunks
-        a_chunk = p["qa"] * K * (a_es or es)                    # one A chunk (raw or prepared)
-        t_b = b_bytes / NVLINK
-        # the own chunk (1/Gc of the work) computes while the other Gc-1 chunks arrive
-        t_own = t_comp / p["Gc"]
-        t_a_exposed = max(0.0, (p["Gc"] - 1) * a_chunk / NVLINK - t_own)
-        worst = max(worst, t_b + t_a_exposed + t_comp)
+        t_b = K * cols * es * (1 - 1 / wp.Gr) / NVLINK                 # received B chunks
+        chunk_t = wp.qa * K * (a_es or es) / NVLINK                     # one A chunk (raw or prepared)
+        arrive, t = {}, 0.0
+        for j in range(wp.Gc):                                          # broadcasts in chunk order
+            if j != wp.c:
+                t += chunk_t
+            arrive[j] = 0.0 if j == wp.c else t
+        now = 0.0
+        for grp in runtime.chunk_groups(wp):
+            if not grp:
+                continue
+            lo, hi = runtime.chunk_rows(wp, grp[0])[0], runtime.chunk_rows(wp, grp[-1])[1]
+            now = max(now, max(arrive[j] for j in grp)) + t_comp * (hi - lo) / max(1, rows)
+        worst = max(worst, t_b + now)
     pdl.unload()
     return worst
 
@@ -86,14 +112,22 @@ def main():
     r = rates()
     em = emulated()
     M = N = K = 16384
-    rows = ["| variant | G=1 ms | G=2 | G=4 | G=8 | predicted S_8 |", "|---|---|---|---|---|---|"]
+    rows = ["| variant | G=1 ms | G=2 | G=4 | G=8 | predicted S_8 | S_8 at the G=1 clock |",
+            "|---|---|---|---|---|---|---|"]
     for (dt, var), rate in sorted(r.items()):
         es = 8 if dt == "f64" else 4
         ts = [model(M, N, K, 1024, G, rate, es, em.get((dt, var, G)), a_bytes_per_elem(dt, var, K))
               for G in (1, 2, 4, 8)]
         src = "measured" if all((dt, var, G) in em for G in (1, 2, 4, 8)) else "rate"
+        # power-capped variants run a short G = 8 step at a higher clock than the long
+        # G = 1 step; scaling the G = 8 compute to the G = 1 clock removes that gain
+        f1, f8 = CLOCK.get((dt, var, 1)), CLOCK.get((dt, var, 8))
+        norm = "-"
+        if f1 and f8 and (dt, var, 8) in em:
+            t8c = em[(dt, var, 8)] * f8 / f1
+            norm = f"{ts[0] / (ts[3] - em[(dt, var, 8)] + t8c):.2f} ({f1:.0f} / {f8:.0f} MHz)"
         rows.append(f"| {dt} {var} ({src}) | {ts[0] * 1e3:.1f} | {ts[1] * 1e3:.1f} | {ts[2] * 1e3:.1f} | "
-                    f"{ts[3] * 1e3:.1f} | {ts[0] / ts[3]:.2f} |")
+                    f"{ts[3] * 1e3:.1f} | {ts[0] / ts[3]:.2f} | {norm} |")
     print("\n".join(rows))
 
 

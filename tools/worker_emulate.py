@@ -23,6 +23,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 import workloads as W  # noqa: E402
 from paper_conf_ipps_sandrieserbp11_b200 import pdl, runtime  # noqa: E402
+from bench import ClockSampler  # noqa: E402
 
 
 def plans(M, N, K, tile, G):
@@ -143,11 +144,14 @@ def main():
                 seen.add(key)
                 t_ser, C_ser = time_worker(wp, dt, c.tile, False, args.reps, args.raw)
                 C_ser = C_ser.clone()
-                t_con, C_con = time_worker(wp, dt, c.tile, None, args.reps, args.raw)   # libpdl decides
+                with ClockSampler(torch.cuda.current_device()) as clk:
+                    t_con, C_con = time_worker(wp, dt, c.tile, None, args.reps, args.raw)   # libpdl decides
+                ck = clk.summary() or {}
                 t_one = time_single(wp, dt, c.tile, args.reps)
                 flops = 2.0 * wp.rows * wp.cols * wp.K
                 rows.append({"c": wp.c, "rect": [wp.rows, wp.cols], "qa": wp.qa, "serial_ms": round(t_ser, 3),
                              "concurrent_ms": round(t_con, 3), "single_launch_ms": round(t_one, 3),
+                             "sm_mhz": ck.get("sm_mhz"), "clock_reasons": ck.get("reasons"),
                              "bitwise": bool(torch.equal(C_ser, C_con)),
                              "concurrent_tflops": round(flops / t_con / 1e9, 1)})
                 del C_ser, C_con
@@ -159,7 +163,9 @@ def main():
              "grid": [wps[0].Gr, wps[0].Gc],
              "max_serial_ms": max(x["serial_ms"] for x in rows),
              "max_concurrent_ms": max(x["concurrent_ms"] for x in rows),
-             "max_single_launch_ms": max(x["single_launch_ms"] for x in rows), "workers": rows}
+             "max_single_launch_ms": max(x["single_launch_ms"] for x in rows),
+             "sm_mhz_worst": next(x["sm_mhz"] for x in rows if x["concurrent_ms"] == max(y["concurrent_ms"] for y in rows)),
+             "workers": rows}
         print(json.dumps(r), flush=True)
         out.append(r)
     t1 = out[0]["max_concurrent_ms"] if out[0]["G"] == 1 else None
