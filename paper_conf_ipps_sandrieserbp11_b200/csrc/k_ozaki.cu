@@ -233,18 +233,35 @@ struct Oz2Moduli {
     int m[OZ2_MAX_MODULI + 1];
     unsigned magic[OZ2_MAX_MODULI + 1];   // ceil(2^39 / m): exact division-by-constant multiplier
     // certificate item (R21): item modulus index `check` of this launch is
-    // the GEMM of the certificate operands; its epilogue flags the 128 x 128 tiles
-    // holding an element with (sa_i + sb_j + min(sa_i, sb_j)) > thr X^c_ij
+    // the GEMM of the certificate operands; its epilogue flags the elements with
+    // X^c_ij < kappa (sa_i + sb_j + min(sa_i, sb_j)), kappa = 2^(14-2p-2) / (tau - 2^-51):
+    // the row term kappa sa_i and the column term kappa sb_j (sbd, from
+    // oz2_cert_cols_kernel) are doubles rounded up, the sum too, so the test is
+    // conservative and costs four FP64-pipe operations per element
     int check = -1;
-    const unsigned long long *sa = nullptr, *sb = nullptr;
+    const unsigned long long *sa = nullptr;
+    const double *sbd = nullptr;
     long long sa_ld = 1;
     uint32_t *flags = nullptr;
     long long ldf = 0;
     uint32_t *emask = nullptr;
     long long ldw = 0;
     unsigned *fallback = nullptr;
-    double thr = 0.0;   // tau' 2^(2p + 2 - 14)
+    double kappa = 0.0;
 };
+
+// kappa sb_j rounded up, once per launch (the epilogue's per-column term)
+__global__ void oz2_cert_cols_kernel(const unsigned long long *__restrict__ sb, int64_t cols, double kappa,
+                                     double *__restrict__ sbd) {
+    const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < cols) sbd[j] = __dmul_ru(__ull2double_ru(sb[j]), kappa);
+}
+
+// int32 -> double on the FP64 pipe (no conversion-unit op): the bits
+// 0x43380000:(x ^ 2^31) are 1.5 * 2^52 + 2^31 + x exactly
+__device__ __forceinline__ double i2d_fp64pipe(int32_t x) {
+    return __hiloint2double(0x43380000, x ^ (int)0x80000000) - 6755401588539392.0;
+}
 
 template <int NSUB>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::THREADS, 1)
@@ -374,7 +391,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
             const int row = tm * (2 * BM) + (int)rank * BM + q * 32 + lane;
             const int cbase = tn * BN + cg * EPI_COLS;
             uint8_t *prow = R + (int64_t)t * plane + (int64_t)row * ldr + cbase;
-            const unsigned long long sai = cert && row < M ? mods.sa[(int64_t)row * mods.sa_ld] : 0ull;
+            const double sad = cert && row < M ? __dmul_ru(__ull2double_ru(mods.sa[(int64_t)row * mods.sa_ld]),
+                                                          mods.kappa)
+                                               : 0.0;
             mbar_wait(bar_tfull, ti & 1u);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #pragma unroll 1
@@ -391,16 +410,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
                     // the componentwise bound against the lower bound 2^(e+f-14) X^c of D
                     // (both scaled by 2^-(e_i+f_j)); a zero row or column has no error
                     uint32_t bad = 0;
-                    if (sai) {
+                    if (sad != 0.0) {
 #pragma unroll
                         for (int jj = 0; jj < 16; ++jj) {
                             const int col = cbase + c0 + jj;
                             if (col >= N) break;
-                            const unsigned long long sbj = mods.sb[col];
-                            if (!sbj) continue;
-                            const double lhs =
-                                ((double)sai + (double)sbj + (double)(sai < sbj ? sai : sbj)) * (1.0 + 0x1p-50);
-                            if (lhs > mods.thr * (double)(int)r[jj]) bad |= 1u << jj;
+                            const double sbj = mods.sbd[col];
+                            const double t = __dadd_ru(__dadd_ru(sad, sbj), fmin(sad, sbj));
+                            if (sbj != 0.0 && i2d_fp64pipe((int32_t)r[jj]) < t) bad |= 1u << jj;
                         }
                     }
                     if (bad) {   // 16 columns aligned to 16: one word of the element mask
@@ -626,7 +643,8 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
     if (lda8 <= 0) lda8 = P.ld8;
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 15u) || (ldr & 15) || (plane & 15)) return cudaErrorInvalidValue;
-    if (P.check && (!guard || !guard->sa || !guard->sb || !guard->flags || !guard->emask || !guard->fallback))
+    if (P.check && (!guard || !guard->sa || !guard->sb || !guard->sbd || !guard->flags || !guard->emask ||
+                    !guard->fallback))
         return cudaErrorInvalidValue;
     cudaError_t e0 = oz_set_attrs<uint8_t>();
     if (e0 != cudaSuccess) return e0;
@@ -658,15 +676,20 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
     if (P.check) {
         all.sa = guard->sa;
         all.sa_ld = guard->sa_ld;
-        all.sb = guard->sb;
+        all.sbd = guard->sbd;
         all.flags = guard->flags;
         all.ldf = guard->ldf;
         all.emask = guard->emask;
         all.ldw = guard->ldw;
         all.fallback = guard->fallback;
-        // flag iff (sa + sb + min) 2^(-2p-2) > tau' 2^-14 X^c; tau' leaves 2^-51 for the
-        // rounding of X to double (|X 2^..| <= 4 D)
-        all.thr = (guard->tau - 0x1p-51) * std::ldexp(1.0, 2 * P.p + 2 - 14);
+        // certified iff (sa + sb + min) 2^(-2p-2) <= tau' 2^-14 X^c; tau' = tau - 2^-51 leaves
+        // 2^-51 for the rounding of X to double (|X 2^..| <= 4 D); kappa rounded up
+        all.kappa = std::ldexp(1.0, 14 - 2 * P.p - 2) / (guard->tau - 0x1p-51) * (1.0 + 0x1p-50);
+        oz2_cert_cols_kernel<<<(unsigned)((cols + 255) / 256), 256, 0, stream>>>(guard->sb, cols, all.kappa,
+                                                                                 guard->sbd);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        if (launches) ++*launches;
     }
     auto group_mods = [&](int t0, int gl) {
         Oz2Moduli g = all;

@@ -93,6 +93,7 @@ struct Oz2Guard {
     unsigned long long *sa = nullptr;     // rows of the launch's rectangle (stride sa_ld)
     int64_t sa_ld = 1;
     unsigned long long *sb = nullptr;     // its columns
+    double *sbd = nullptr;                // cols doubles of scratch (the epilogue's column term)
     uint32_t *flags = nullptr;            // tile (row / 128, col / 128) at flags[(row / 128) * ldf + col / 128]
     int64_t ldf = 0;
     uint32_t *emask = nullptr;            // element (row, col): bit col % 32 of emask[row * ldw + col / 32]

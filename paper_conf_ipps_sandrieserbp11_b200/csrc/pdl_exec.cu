@@ -106,13 +106,15 @@ bool worker_sgemm_ozaki2(const WorkerCtx &w) {
 // in the shared BUF_OZE (it does not move with `rows`, so a prepared B survives
 // row-chunk tasks, REUSE_B).  The A side (residues, e_i, sa_i) lives in the packed
 // prepared-A rows (pdlk::oz2_prep_row_bytes).  sb: the certificate's column sums.
-static int oz_b_arrays(WorkerCtx &w, int64_t cols, unsigned long long **bmax, int **fb, unsigned long long **sb) {
+static int oz_b_arrays(WorkerCtx &w, int64_t cols, unsigned long long **bmax, int **fb, unsigned long long **sb,
+                       double **sbd) {
     void *p = nullptr;
-    int rc = ensure_buf(w, BUF_OZE, (size_t)cols * 16 + (size_t)round_up(cols, 2) * 4, &p);
+    int rc = ensure_buf(w, BUF_OZE, (size_t)cols * 24 + (size_t)round_up(cols, 2) * 4, &p);
     if (rc) return rc;
     *bmax = (unsigned long long *)p;
     *sb = *bmax + cols;
-    *fb = (int *)(*sb + cols);
+    *sbd = (double *)(*sb + cols);
+    *fb = (int *)(*sbd + cols);
     return PDL_OK;
 }
 
@@ -306,6 +308,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     int8_t *a8 = nullptr, *b8 = nullptr;
     int *oz_ea = nullptr, *oz_fb = nullptr;
     unsigned long long *oz_bmax = nullptr, *oz_sa = nullptr, *oz_sb = nullptr;
+    double *oz_sbd = nullptr;
     uint8_t *oz2_R = nullptr;
     int64_t oz2_ldr = 0, oz2_plane = 0;
     pdlk::Oz2Guard G2;
@@ -328,7 +331,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         oz_sa_ld = oz_pr / 8;
         if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
         b8 = (int8_t *)p;
-        if ((rc = oz_b_arrays(w, cols, &oz_bmax, &oz_fb, &oz_sb))) return rc;
+        if ((rc = oz_b_arrays(w, cols, &oz_bmax, &oz_fb, &oz_sb, &oz_sbd))) return rc;
         oz2_ldr = round_up(cols, 16);
         oz2_plane = oz2_ldr * rows;
         if ((rc = ensure(BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
@@ -459,6 +462,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                     gs.sa = oz_sa + r0 * oz_sa_ld;
                     gs.sa_ld = oz_sa_ld;
                     gs.sb = oz_sb + c0;
+                    gs.sbd = oz_sbd + c0;
                     gs.flags = G2.flags + (r0 / 128) * G2.ldf + c0 / 128;
                     gs.emask = G2.emask + r0 * G2.ldw + c0 / 32;
                     e = cudaMemset2DAsync(gs.flags, (size_t)(G2.ldf * 4), 0, (size_t)((nc + 127) / 128) * 4,

@@ -343,8 +343,9 @@ def chunk_rows(wp: WorkerPlan, j):
     return lo, min(lo + wp.qa, wp.rows)
 
 
-# NVLink 5 peer bandwidth per direction (the measured peer-copy figure quoted in
-# /opt/skills/guides/B200_PROFILING.md) and the A exchange below which one launch
+# NVLink 5 peer bandwidth per direction -- an ESTIMATE: the B200 peer-copy figure
+# quoted in /opt/skills/guides/B200_PROFILING.md, not re-measured on this pool (one GPU
+# per gpurun call) -- and the A exchange below which one launch
 # over the whole Worker rectangle beats the chunked overlap: tools/worker_emulate.py
 # (profiles/r01_worker_emulate_single_*.jsonl) measured the chunk launches 0.41-0.46
 # ms slower than one launch for C3 at G = 4 / 8 (host issue of three short tasks

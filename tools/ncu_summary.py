@@ -85,10 +85,10 @@ def main():
         for d in s:
             rd = to_bytes(d.get("dram__bytes_read.sum", 0), d.get("dram__bytes_read.sum [unit]", "byte"))
             wr = to_bytes(d.get("dram__bytes_write.sum", 0), d.get("dram__bytes_write.sum [unit]", "byte"))
-            key = None
-            if "dgemm_k1" in d["kernel"]:
+            key = None   # only the bench's dominant-kernel captures (not e.g. the Ozaki-II recompute K1)
+            if "dgemm_k1" in d["kernel"] and name.startswith("prof_k1"):
                 key = "f64/C4"
-            elif "gemm_3xtf32" in d["kernel"]:
+            elif "gemm_3xtf32" in d["kernel"] and name.startswith("prof_k2"):
                 key = "f32/C4"
             if key:
                 traffic[key] = int(rd + wr)
