@@ -414,6 +414,17 @@ def k_roofline(ktimes, steps, pipe_flops, peak_dtype, kname, traffic_key, cfg, a
     return r
 
 
+def clock_context(roof, clocks):
+    """The peaks are issue rates at the maximum SM clock; a power-capped kernel runs
+    at a lower one.  Report the fraction of the peak scaled to the median SM clock
+    measured during the timed region beside the headline fraction (context only:
+    `frac` stays against the fixed measured peak)."""
+    if roof and roof.get("achieved") and clocks and clocks.get("sm_mhz") and clocks.get("sm_max_mhz"):
+        f = clocks["sm_mhz"] / clocks["sm_max_mhz"]
+        roof["frac_at_measured_clock"] = round(roof["achieved"] / (roof["peak"] * f), 4)
+        roof["measured_clock_mhz"] = clocks["sm_mhz"]
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -510,6 +521,8 @@ def main():
     if ozaki:
         roofline["note"] = ("achieved counts int8 tensor ops (one residue GEMM per modulus + the certificate "
                             "GEMM, 2 ops per MAC); useful FP64 FLOP = 2MNK")
+
+    clock_context(roofline, clocks)
 
     # ---- e2e: host pinned operands through the public API, --steps steps ----
     e2e = None
@@ -608,6 +621,7 @@ def main():
                                   "kernel_ms": round(float(np.mean(akt)), 3) if akt else None,
                                   "peak_source": apsrc},
                      "clocks": aclk})
+        clock_context(alts[-1]["roofline"], aclk)
 
     # ---- FP32 (north star (2)): the tcgen05/TMEM 3xTF32 path K3+K2 on the same config ----
     f32 = None
@@ -687,6 +701,7 @@ def fp32_leg(args, torch, dist, pdl, stream, dev, local, c):
            "parity": "max rel err <= 1e-5 vs oracle (tests/test_gpu_parity.py)",
            "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} (f32)",
            "roofline": roof, "clocks": clk}
+    clock_context(roof, clk)
     if not args.no_e2e:
         hA = torch.from_numpy(A).pin_memory()
         hB = torch.from_numpy(B).pin_memory()

@@ -394,6 +394,50 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
             const double sad = cert && row < M ? __dmul_ru(__ull2double_ru(mods.sa[(int64_t)row * mods.sa_ld]),
                                                           mods.kappa)
                                                : 0.0;
+            if (cert) {
+                // The certificate: the componentwise bound against the lower bound
+                // 2^(e+f-14) X^c of D (both scaled by 2^-(e_i+f_j)); a zero row or column
+                // has no error.  The warp's EPI_COLS column terms are fetched into
+                // registers (lane l: columns l, l + 32, ...) before the accumulator is
+                // ready and handed out by shuffles, so nothing but FP64-pipe arithmetic
+                // runs while the item's TMEM is held (it gates the next item's MMAs).
+                constexpr int NR = EPI_COLS / 32;
+                double sbr[NR];
+#pragma unroll
+                for (int k = 0; k < NR; ++k) {
+                    const int col = cbase + 32 * k + lane;
+                    sbr[k] = col < N ? mods.sbd[col] : 0.0;
+                }
+                mbar_wait(bar_tfull, ti & 1u);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll
+                for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
+                    uint32_t r[16];
+                    tmem_ld16(tl + c0, r);
+                    if (c0 + 16 == EPI_COLS) {   // this warp's last TMEM read is complete
+                        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive_cluster(tempty_leader);
+                    }
+                    uint32_t bad = 0;
+#pragma unroll
+                    for (int jj = 0; jj < 16; ++jj) {
+                        const int idx = c0 + jj;   // compile-time: register and lane of the column term
+                        const double sbj = __shfl_sync(0xffffffffu, sbr[idx >> 5], idx & 31);
+                        const double t = __dadd_ru(__dadd_ru(sad, sbj), fmin(sad, sbj));
+                        if (sbj != 0.0 && i2d_fp64pipe((int32_t)r[jj]) < t) bad |= 1u << jj;
+                    }
+                    if (row >= M || sad == 0.0) continue;   // (columns >= N carry sbj = 0)
+                    if (bad) {   // 16 columns aligned to 16: one word of the element mask
+                        const int c16 = cbase + c0;
+                        atomicOr(mods.emask + (int64_t)row * mods.ldw + (c16 >> 5), bad << (c16 & 31));
+                        uint32_t *f = mods.flags + (int64_t)(row >> 7) * mods.ldf + (c16 >> 7);
+                        if (atomicExch(f, 1u) == 0u) atomicAdd(mods.fallback, 1u);
+                        atomicAdd(mods.fallback + 1, (unsigned)__popc(bad));
+                    }
+                }
+                continue;
+            }
             mbar_wait(bar_tfull, ti & 1u);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 #pragma unroll 1
@@ -406,29 +450,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
                     if (lane == 0) mbar_arrive_cluster(tempty_leader);
                 }
                 if (row >= M) continue;
-                if (cert) {
-                    // the componentwise bound against the lower bound 2^(e+f-14) X^c of D
-                    // (both scaled by 2^-(e_i+f_j)); a zero row or column has no error
-                    uint32_t bad = 0;
-                    if (sad != 0.0) {
-#pragma unroll
-                        for (int jj = 0; jj < 16; ++jj) {
-                            const int col = cbase + c0 + jj;
-                            if (col >= N) break;
-                            const double sbj = mods.sbd[col];
-                            const double t = __dadd_ru(__dadd_ru(sad, sbj), fmin(sad, sbj));
-                            if (sbj != 0.0 && i2d_fp64pipe((int32_t)r[jj]) < t) bad |= 1u << jj;
-                        }
-                    }
-                    if (bad) {   // 16 columns aligned to 16: one word of the element mask
-                        const int c16 = cbase + c0;
-                        atomicOr(mods.emask + (int64_t)row * mods.ldw + (c16 >> 5), bad << (c16 & 31));
-                        uint32_t *f = mods.flags + (int64_t)(row >> 7) * mods.ldf + (c16 >> 7);
-                        if (atomicExch(f, 1u) == 0u) atomicAdd(mods.fallback, 1u);
-                        atomicAdd(mods.fallback + 1, (unsigned)__popc(bad));
-                    }
-                    continue;
-                }
                 uint32_t pk[4];
 #pragma unroll
                 for (int w4 = 0; w4 < 4; ++w4) {

@@ -349,9 +349,9 @@ __global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int
 // (32 n rows x 64 k, row pitch 66 doubles): coalesced loads along n, then each
 // thread reads its column's 8 consecutive k as four 16-byte shared loads (every
 // quarter-warp on distinct banks) and writes one 8-byte word per modulus.  A CTA
-// walks the k tiles blockIdx.y, blockIdx.y + gridDim.y, ... of its 32 columns, so
-// the certificate's column sums take one atomic per column and CTA (4 k tiles per
-// CTA at C4: 64 atomics per column instead of 256).
+// walks the k tiles blockIdx.y, blockIdx.y + gridDim.y, ... of its 32 columns (one
+// tile per CTA below 65536 tiles) and adds its certificate column sums with one
+// atomic per column.
 __global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
     const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int n, int np, int p, int64_t Kc, int nch,
     const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
@@ -677,11 +677,10 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
         oz2_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
     }
     const int64_t Kpad = (int64_t)P.nch * P.Kc;
-    // k tiles per CTA: 4 (many CTAs in flight keep the loads overlapped; 16 per CTA
-    // measured slower), at least 16 CTAs per SM's worth
+    // one k tile per CTA (C4: 1.70 ms; 4 or 16 tiles per CTA with fewer column-sum
+    // atomics measured 1.87 / 1.88 ms -- many CTAs in flight keep the loads overlapped)
     const int64_t nkt = (Kpad + 63) / 64, ncb = (cols + 31) / 32;
-    int64_t gy = std::max<int64_t>(nkt / 4, (148 * 16 + ncb - 1) / ncb);
-    gy = std::max<int64_t>(1, std::min<int64_t>(gy, std::min<int64_t>(nkt, 65535)));
+    const int64_t gy = std::max<int64_t>(1, std::min<int64_t>(nkt, 65535));
     dim3 g2((unsigned)ncb, (unsigned)gy);
     oz2_split_cols_t_kernel<<<g2, 256, 0, s>>>(B, ldb, K, cols, P.n, P.np, P.p, P.Kc, P.nch, bmax, Bt8, P.ld8, fb,
                                                sb);

@@ -70,6 +70,8 @@ def time_worker(wp, dt, tile, concurrent, reps, raw=False):
         step()
     pdl.sync()
     torch.cuda.synchronize()
+    if SUSTAIN_S > 0:
+        return sustained_ms(step, main), C
     ms = []
     for _ in range(reps):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -81,6 +83,33 @@ def time_worker(wp, dt, tile, concurrent, reps, raw=False):
         ms.append(e0.elapsed_time(e1))
     ms.sort()
     return ms[len(ms) // 2], C
+
+
+# --sustain S: time each Worker step back to back for >= S seconds (after as long a
+# warm-up), the way every GPU of a strong-scaling run repeats its step, so a short
+# G = 8 step meets the same power cap as the long G = 1 step (the INT8 / TF32 paths
+# run under sw_power_cap; a few isolated short steps run at boost clocks).
+SUSTAIN_S = 0.0
+
+
+def sustained_ms(step, stream):
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    step()
+    e1.record(stream)
+    pdl.sync()
+    torch.cuda.synchronize()
+    est = max(e0.elapsed_time(e1), 1e-3)
+    n = max(3, int(SUSTAIN_S * 1e3 / est))
+    for _ in range(n):   # warm-up at the sustained clock
+        step()
+    e0.record(stream)
+    for _ in range(n):
+        step()
+    e1.record(stream)
+    pdl.sync()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / n
 
 
 def time_single(wp, dt, tile, reps):
@@ -124,7 +153,11 @@ def main():
     ap.add_argument("--gs", default="1,2,4,8")
     ap.add_argument("--variant", default=None, help="task variant (PDL_DGEMM_VARIANT / PDL_SGEMM_VARIANT)")
     ap.add_argument("--raw", action="store_true", help="exchange raw A chunks (every Worker prepares its panel)")
+    ap.add_argument("--sustain", type=float, default=0.0,
+                    help="seconds of back-to-back steps per timing (sustained power-capped clock)")
     args = ap.parse_args()
+    global SUSTAIN_S
+    SUSTAIN_S = args.sustain
     if args.variant:
         os.environ["PDL_DGEMM_VARIANT" if args.dtype == "f64" else "PDL_SGEMM_VARIANT"] = args.variant
     c = W.CONFIGS[args.config]
@@ -159,6 +192,7 @@ def main():
         finally:
             pdl.unload()
         r = {"config": args.config, "dtype": args.dtype, "variant": args.variant or "default", "G": G,
+             "sustain_s": args.sustain,
              "a_exchange": a_ex,
              "grid": [wps[0].Gr, wps[0].Gc],
              "max_serial_ms": max(x["serial_ms"] for x in rows),
