@@ -65,10 +65,11 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cublas", action="store_true")
-    p.add_argument("--variant", choices=("default", "ozaki2"), default="default",
+    p.add_argument("--variant", choices=("default", "ozaki2", "tf32bf16", "3xtf32"), default="default",
                    help="task variant pinned in the PDL descriptor: default (FP64 K1 DMMA / FP32 K3+K2 3xTF32) "
                         "or ozaki2 (FP64 only: K6/K7 Ozaki scheme II, INT8 residue GEMMs + CRT, with its "
-                        "certificate and K1 recompute, DESIGN.md R21)")
+                        "certificate and K1 recompute, DESIGN.md R21); FP32: tf32bf16 (the default: TF32 main "
+                        "product + two BF16 correction products, DESIGN.md R22) or 3xtf32")
     p.add_argument("--no-alt", action="store_true", help="skip timing the other task variants")
     p.add_argument("--dist-backend", choices=("auto", "nccl", "gloo"), default="auto",
                    help="auto: NCCL when every rank has its own GPU, else gloo (ranks share GPUs: "
@@ -191,6 +192,8 @@ def variant_descriptor(pdl, world, dtype, variant):
     """PDL descriptor XML with the task variant pinned as a Worker property."""
     if variant == "default":
         return pdl.descriptor_xml(world)
+    if variant in ("tf32bf16", "3xtf32"):
+        return pdl.descriptor_xml(world, props={"SGEMM_VARIANT": variant})
     return pdl.descriptor_xml(world, props={"DGEMM_VARIANT": "ozaki2"})
 
 
@@ -452,6 +455,8 @@ def main():
 
     if args.variant == "ozaki2" and args.dtype != "f64":
         sys.exit("--variant ozaki2 is an FP64 task variant")
+    if args.variant in ("tf32bf16", "3xtf32") and args.dtype != "f32":
+        sys.exit(f"--variant {args.variant} is an FP32 task variant")
     ozaki = args.variant == "ozaki2"
     # the task variant is pre-selected through the Worker's PDL properties (L1316-1326)
     desc = variant_descriptor(pdl, world, args.dtype, args.variant)
@@ -510,14 +515,17 @@ def main():
     if ozaki:
         pipe_flops, kname = variant_ops(args.variant, wp.rows, wp.cols, K)
     else:
-        pipe_flops = flops_worker * (3 if args.dtype == "f32" else 1)
-        kname = "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else "K2 gemm_3xtf32_2sm_kernel (tcgen05)"
-    traffic_key = args.variant if ozaki else args.dtype
+        f32name = "3xtf32" if args.variant == "3xtf32" else "tf32bf16"
+        f32v = F32_VARIANTS[f32name]
+        pipe_flops = flops_worker * (f32v[0] if args.dtype == "f32" else 1)
+        kname = "K1 dgemm_k1_kernel (DMMA)" if args.dtype == "f64" else f32v[1]
+    traffic_key = args.variant if ozaki else (
+        "f32_tf32bf16" if args.dtype == "f32" and args.variant != "3xtf32" else args.dtype)
     roofline = k_roofline(ktimes, args.steps, pipe_flops, peak_dtype, kname, traffic_key, args.config,
                           (wp.rows * K + K * wp.cols + wp.rows * wp.cols) * es, wp.rows, wp.cols, args.dtype, ozaki)
     peak_tf = roofline["peak"]
     if args.dtype == "f32":
-        roofline["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
+        roofline["note"] = f32v[2]
     if ozaki:
         roofline["note"] = ("achieved counts int8 tensor ops (one residue GEMM per modulus + the certificate "
                             "GEMM, 2 ops per MAC); useful FP64 FLOP = 2MNK")
@@ -624,9 +632,10 @@ def main():
         clock_context(alts[-1]["roofline"], aclk)
 
     # ---- FP32 (north star (2)): the tcgen05/TMEM 3xTF32 path K3+K2 on the same config ----
-    f32 = None
+    f32 = f32_mix = None
     if world == 1 and args.dtype == "f64" and not args.no_f32:
         f32 = fp32_leg(args, torch, dist, pdl, stream, dev, local, c)
+        f32_mix = fp32_leg(args, torch, dist, pdl, stream, dev, local, c, variant="tf32bf16")
 
     # ---- the oracle on the host cores, after the GPU timings (rank 0, every N) ----
     cpu = None
@@ -645,7 +654,8 @@ def main():
             "config": {"workload": workload,
                        "M": M, "N": N, "K": K, "tile": c.tile, "parallelism": f"block2d {wp.Gr}x{wp.Gc}",
                        "task_variant": (variant_label(args.variant, args.dtype, K)[1] if ozaki else
-                                        ("dmma (K1)" if args.dtype == "f64" else "3xtf32 (K3+K2)")),
+                                        ("dmma (K1)" if args.dtype == "f64" else
+                                         ("3xtf32" if args.variant == "3xtf32" else "tf32bf16") + " (K3+K2)")),
                        "l2": "inputs larger than L2 (operands >> 126 MB), no flush needed"},
             "pct_of_tensor_peak": round(100 * (pipe_flops / flops_worker) * value / world / (peak_tf * 1e3), 2),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
@@ -663,20 +673,34 @@ def main():
             line["alt_variants"] = alts
         if f32 is not None:
             line["f32_3xtf32"] = f32
+        if f32_mix is not None:
+            line["f32_tf32bf16"] = f32_mix
         print(json.dumps(line), flush=True)
     pdl.unload()
     if world > 1:
         dist.destroy_process_group()
 
 
-def fp32_leg(args, torch, dist, pdl, stream, dev, local, c):
-    """FP32 inputs through the default SGEMM variant (K3 TF32 split + K2 3xTF32
-    tcgen05 CTA-pair kernel), device-resident and end to end, on the same
-    config: the tcgen05/TMEM kernel of north star (2) with a driver-run number."""
+F32_VARIANTS = {
+    # SGEMM_VARIANT -> (tensor passes per K block in TF32-equivalents, kernel label, note)
+    "3xtf32": (3, "K2 gemm_3xtf32_2sm_kernel<false> (tcgen05 cta_group::2 kind::tf32 x3)",
+               "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"),
+    "tf32bf16": (2, "K2 gemm_3xtf32_2sm_kernel<true> (tcgen05 cta_group::2 kind::tf32 + 2x kind::f16)",
+                 "achieved counts TF32-equivalent tensor work: a_hi*b_hi (TF32) + two BF16 correction "
+                 "products at twice the TF32 rate = 2 TF32 passes; useful FLOP = 1/2 (DESIGN.md R22)"),
+}
+
+
+def fp32_leg(args, torch, dist, pdl, stream, dev, local, c, variant="3xtf32"):
+    """FP32 inputs through an SGEMM task variant (K3 split + K2 tcgen05 CTA-pair
+    kernel; `variant` pinned through the Worker's SGEMM_VARIANT PDL property),
+    device-resident and end to end, on the same config: the tcgen05/TMEM kernel
+    of north star (2) with a driver-run number."""
     M, N, K = c.M, c.N, c.K
     A, B = host_inputs(args.config, np.float32)
+    passes, kname, note = F32_VARIANTS[variant]
     pdl.unload()
-    pdl.load(pdl.descriptor_xml(1))
+    pdl.load(pdl.descriptor_xml(1, props={"SGEMM_VARIANT": variant}))
     pdl.set_stream(stream)
     dA = torch.from_numpy(A).to(dev)
     dB = torch.from_numpy(B).to(dev)
@@ -693,12 +717,14 @@ def fp32_leg(args, torch, dist, pdl, stream, dev, local, c):
     ms, clk = device_timed(torch, dist, step, args.steps, stream, 1, dev, local, pdl.sync)
     kt = pdl.kernel_times()
     flops = 2.0 * M * N * K
-    roof = k_roofline(kt, args.steps, 3 * flops, "f32", "K2 gemm_3xtf32_2sm_kernel (tcgen05 cta_group::2 kind::tf32)",
-                      "f32", args.config, (M * K + K * N + M * N) * 4, M, N, "f32", False)
-    roof["note"] = "achieved counts the 3 TF32 tensor products; useful FLOP = 1/3"
+    roof = k_roofline(kt, args.steps, passes * flops, "f32", kname,
+                      "f32" if variant == "3xtf32" else "f32_" + variant, args.config,
+                      (M * K + K * N + M * N) * 4, M, N, "f32", False)
+    roof["note"] = note
     out = {"value": round(flops * args.steps / (ms / 1e3) / 1e9, 1), "unit": "GFLOP/s", "dtype": "f32",
-           "ms_per_step": round(ms / args.steps, 3), "task_variant": "3xtf32 (K3+K2)",
-           "parity": "max rel err <= 1e-5 vs oracle (tests/test_gpu_parity.py)",
+           "ms_per_step": round(ms / args.steps, 3), "task_variant": f"{variant} (K3+K2)",
+           "parity": ("max rel err <= 1e-5 vs oracle (tests/test_gpu_parity.py)" if variant == "3xtf32" else
+                      "max rel err <= 1e-5 vs oracle (tests/test_gpu_tf32bf16.py; split bound R22)"),
            "data": f"synthetic: numpy PCG64 U[0,1) seeds {W.seeds(c.cid)} (f32)",
            "roofline": roof, "clocks": clk}
     clock_context(roof, clk)

@@ -36,15 +36,52 @@ __device__ __forceinline__ float tf32_rna(float x) {
     return __uint_as_float(r);
 }
 
+// bf16 bits of x, round to nearest even
+__device__ __forceinline__ uint32_t bf16_rn_bits(float x) {
+    uint16_t r;
+    asm("cvt.rn.bf16.f32 %0, %1;" : "=h"(r) : "f"(x));
+    return r;
+}
+
+// Split of 4 consecutive k (k0 % 4 == 0) of one row into its K-major outputs.
+//  3xTF32 (mix = 0): hi[k] = rna_tf32(x), lo[k] = rna_tf32(x - hi)      (fp32 planes)
+//  TF32+BF16 (mix = 1, R22): hi[k] = rna_tf32(x) as before; the second
+//  plane holds bf16 pairs per 16-wide K block b: halves [32 b, 32 b + 16) =
+//  rn_bf16(hi), [32 b + 16, 32 b + 32) = rn_bf16(x - hi)  (64 bytes per block: one
+//  kind::f16 K = 16 step reads 32 of them; the K2 TMA boxes take 1 or 2 blocks)
+__device__ __forceinline__ void split_store4(const float (&v)[4], float *hi, float *lo, int64_t k0, int mix) {
+    float h[4], l[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+        h[u] = tf32_rna(v[u]);
+        l[u] = v[u] - h[u];   // exact in fp32
+    }
+    *reinterpret_cast<float4 *>(hi + k0) = make_float4(h[0], h[1], h[2], h[3]);
+    if (!mix) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) l[u] = tf32_rna(l[u]);
+        *reinterpret_cast<float4 *>(lo + k0) = make_float4(l[0], l[1], l[2], l[3]);
+    } else {
+        uint16_t *pl = reinterpret_cast<uint16_t *>(lo) + (k0 >> 4) * 32 + (k0 & 15);
+        const uint2 hb = make_uint2(bf16_rn_bits(h[0]) | (bf16_rn_bits(h[1]) << 16),
+                                    bf16_rn_bits(h[2]) | (bf16_rn_bits(h[3]) << 16));
+        const uint2 lb = make_uint2(bf16_rn_bits(l[0]) | (bf16_rn_bits(l[1]) << 16),
+                                    bf16_rn_bits(l[2]) | (bf16_rn_bits(l[3]) << 16));
+        *reinterpret_cast<uint2 *>(pl) = hb;
+        *reinterpret_cast<uint2 *>(pl + 16) = lb;
+    }
+}
+
 __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int64_t M, int64_t K,
-                                  float *__restrict__ hi, float *__restrict__ lo, int64_t Kp, int64_t ldo, int vec) {
+                                  float *__restrict__ hi, float *__restrict__ lo, int64_t Kp, int64_t ldo, int vec,
+                                  int mix) {
     // one thread per 4 consecutive k of one row (Kp % 4 == 0)
     const int64_t q = Kp >> 2;
     const int64_t total = M * q;
     for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
         const int64_t i = t / q, k0 = (t - i * q) << 2;
         const float *src = A + i * lda;
-        float v[4], h[4], l[4];
+        float v[4];
         if (vec && k0 + 3 < K) {   // 16-byte aligned rows: one LDG.128
             const float4 x = __ldcs(reinterpret_cast<const float4 *>(src + k0));
             v[0] = x.x, v[1] = x.y, v[2] = x.z, v[3] = x.w;
@@ -52,13 +89,7 @@ __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int6
 #pragma unroll
             for (int u = 0; u < 4; ++u) v[u] = (k0 + u < K) ? __ldg(src + k0 + u) : 0.0f;
         }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            h[u] = tf32_rna(v[u]);
-            l[u] = tf32_rna(v[u] - h[u]);
-        }
-        *reinterpret_cast<float4 *>(hi + i * ldo + k0) = make_float4(h[0], h[1], h[2], h[3]);
-        *reinterpret_cast<float4 *>(lo + i * ldo + k0) = make_float4(l[0], l[1], l[2], l[3]);
+        split_store4(v, hi + i * ldo, lo + i * ldo, k0, mix);
     }
 }
 
@@ -68,7 +99,7 @@ __global__ void split_rows_kernel(const float *__restrict__ A, int64_t lda, int6
 // (profiles/r01_ncu_prof_k3.json).
 __global__ void __launch_bounds__(256) split_cols_t_kernel(const float *__restrict__ B, int64_t ldb, int64_t K,
                                                            int64_t N, float *__restrict__ hi, float *__restrict__ lo,
-                                                           int64_t Kp, int vec) {
+                                                           int64_t Kp, int vec, int mix) {
     __shared__ float t[64][65];
     const int64_t k0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 64;
     const int cq = threadIdx.x & 15, r0 = threadIdx.x >> 4;
@@ -93,37 +124,32 @@ __global__ void __launch_bounds__(256) split_cols_t_kernel(const float *__restri
         const int nr = r0 + 16 * i;
         const int64_t n = n0 + nr, k = k0 + 4 * cq;
         if (n < N && k < Kp) {   // Kp % 32 == 0: a group of 4 k is all inside or all outside
-            float h[4], l[4];
+            float v[4];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const float v = t[4 * cq + j][nr];
-                h[j] = tf32_rna(v);
-                l[j] = tf32_rna(v - h[j]);
-            }
-            *reinterpret_cast<float4 *>(hi + n * Kp + k) = make_float4(h[0], h[1], h[2], h[3]);
-            *reinterpret_cast<float4 *>(lo + n * Kp + k) = make_float4(l[0], l[1], l[2], l[3]);
+            for (int j = 0; j < 4; ++j) v[j] = t[4 * cq + j][nr];
+            split_store4(v, hi + n * Kp, lo + n * Kp, k, mix);
         }
     }
 }
 
 cudaError_t launch_split_rows(const float *A, int64_t lda, int64_t M, int64_t K, float *hi, float *lo, int64_t Kp,
-                              cudaStream_t s, int64_t ldo) {
+                              cudaStream_t s, int64_t ldo, int mix) {
     if (ldo <= 0) ldo = Kp;
     if (M <= 0 || Kp <= 0) return cudaSuccess;
     const int64_t total = M * (Kp >> 2);
     int blocks = (int)((total + 255) / 256);
     if (blocks > 148 * 16) blocks = 148 * 16;
     const int vec = ((reinterpret_cast<uintptr_t>(A) & 15u) == 0 && (lda & 3) == 0) ? 1 : 0;
-    split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, M, K, hi, lo, Kp, ldo, vec);
+    split_rows_kernel<<<blocks, 256, 0, s>>>(A, lda, M, K, hi, lo, Kp, ldo, vec, mix);
     return cudaGetLastError();
 }
 
 cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t N, float *hi, float *lo, int64_t Kp,
-                                cudaStream_t s) {
+                                cudaStream_t s, int mix) {
     if (N <= 0 || Kp <= 0) return cudaSuccess;
     dim3 grid((unsigned)((N + 63) / 64), (unsigned)((Kp + 63) / 64));
     const int vec = ((reinterpret_cast<uintptr_t>(B) & 15u) == 0 && (ldb & 3) == 0) ? 1 : 0;
-    split_cols_t_kernel<<<grid, 256, 0, s>>>(B, ldb, K, N, hi, lo, Kp, vec);
+    split_cols_t_kernel<<<grid, 256, 0, s>>>(B, ldb, K, N, hi, lo, Kp, vec, mix);
     return cudaGetLastError();
 }
 
@@ -149,6 +175,7 @@ constexpr int KCB = 4;
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
 }  // namespace k2
 
+template <bool MIX>
 __global__ void __launch_bounds__(k2::THREADS, 1)
     gemm_3xtf32_kernel(const __grid_constant__ CUtensorMap tAh, const __grid_constant__ CUtensorMap tAl,
                        const __grid_constant__ CUtensorMap tBh, const __grid_constant__ CUtensorMap tBl,
@@ -216,9 +243,10 @@ __global__ void __launch_bounds__(k2::THREADS, 1)
                 mbar_arrive_expect_tx(fb, STAGE_BYTES);
                 const uint32_t st = base + s * STAGE_BYTES;
                 tma_load_2d(st, &tAh, fb, kb * BK, m0);
-                tma_load_2d(st + A_BYTES, &tAl, fb, kb * BK, m0);
+                const int kl = kb * (MIX ? 2 * BK : BK);   // bf16 [hi' | lo'] rows: 64 halves per block
+                tma_load_2d(st + A_BYTES, &tAl, fb, kl, m0);
                 tma_load_2d(st + 2 * A_BYTES, &tBh, fb, kb * BK, n0);
-                tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBl, fb, kb * BK, n0);
+                tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBl, fb, kl, n0);
             }
         }
     } else if (warp == 1) {
@@ -240,14 +268,30 @@ __global__ void __launch_bounds__(k2::THREADS, 1)
                 asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
                 const uint32_t st = base + s * STAGE_BYTES;
                 const uint32_t ah = st, al = st + A_BYTES, bh = st + 2 * A_BYTES, bl = bh + B_BYTES;
+                if constexpr (MIX) {
+                    // TF32+BF16 (R22), per 16-wide K step (the order of K2 v3): the two
+                    // correction products as kind::f16 on the bf16 [hi'(16) | lo'(16)]
+                    // blocks (K = 16 = 32 B per instruction), then hi*hi in TF32 for k, k + 8
+                    constexpr uint32_t idesc16 = idesc_bf16(BM, BN);
 #pragma unroll
-                for (int kk = 0; kk < BK / UMMA_K; ++kk) {
-                    const uint32_t off = kk * UMMA_K * 4;   // 32 B per K step inside the swizzle atom
-                    const uint32_t acc0 = (kin == 0 && kk == 0) ? 0u : 1u;
-                    // small terms first: lo*hi, hi*lo, then hi*hi
-                    umma_tf32(dtm, umma_desc_k_sw128(al + off), umma_desc_k_sw128(bh + off), idesc, acc0);
-                    umma_tf32(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bl + off), idesc, 1u);
-                    umma_tf32(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bh + off), idesc, 1u);
+                    for (int k16 = 0; k16 < BK / 16; ++k16) {
+                        const uint32_t o = k16 * 64;
+                        const uint32_t acc0 = (kin == 0 && k16 == 0) ? 0u : 1u;
+                        umma_bf16(dtm, umma_desc_k_sw128(al + o + 32), umma_desc_k_sw128(bl + o), idesc16, acc0);
+                        umma_bf16(dtm, umma_desc_k_sw128(al + o), umma_desc_k_sw128(bl + o + 32), idesc16, 1u);
+                        umma_tf32(dtm, umma_desc_k_sw128(ah + o), umma_desc_k_sw128(bh + o), idesc, 1u);
+                        umma_tf32(dtm, umma_desc_k_sw128(ah + o + 32), umma_desc_k_sw128(bh + o + 32), idesc, 1u);
+                    }
+                } else {
+#pragma unroll
+                    for (int kk = 0; kk < BK / UMMA_K; ++kk) {
+                        const uint32_t off = kk * UMMA_K * 4;   // 32 B per K step inside the swizzle atom
+                        const uint32_t acc0 = (kin == 0 && kk == 0) ? 0u : 1u;
+                        // small terms first: lo*hi, hi*lo, then hi*hi
+                        umma_tf32(dtm, umma_desc_k_sw128(al + off), umma_desc_k_sw128(bh + off), idesc, acc0);
+                        umma_tf32(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bl + off), idesc, 1u);
+                        umma_tf32(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bh + off), idesc, 1u);
+                    }
                 }
                 umma_commit(bar_empty + 8 * s);                 // smem stage free when these MMAs finish
                 if (kin == KCB - 1 || kb == nk - 1) umma_commit(bar_tfull + 8 * buf);   // chunk sum ready
@@ -299,38 +343,42 @@ __global__ void __launch_bounds__(k2::THREADS, 1)
     }
 }
 
+// bf16 = 1: the plane holds the bf16 [hi' | lo'] rows of the TF32+BF16 split (2 Kp
+// halves per row, boxes of 64 halves = the same 128 bytes per K block)
 static bool map_f32(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_t Kp, uint64_t rows, uint32_t box_rows,
-                    uint64_t ld = 0) {
-    cuuint64_t dims[2] = {Kp, rows};
+                    uint64_t ld = 0, int bf16 = 0) {
+    cuuint64_t dims[2] = {bf16 ? 2 * Kp : Kp, rows};
     cuuint64_t strides[1] = {(ld ? ld : Kp) * 4};
-    cuuint32_t box[2] = {(cuuint32_t)k2::BK, box_rows};
+    cuuint32_t box[2] = {(cuuint32_t)(bf16 ? 2 * k2::BK : k2::BK), box_rows};
     cuuint32_t es[2] = {1, 1};
-    return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
+    return enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr),
+               dims, strides, box, es,
                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                               cudaStream_t stream, int64_t lda_s) {
+                               cudaStream_t stream, int64_t lda_s, int mix) {
     using namespace k2;
     if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
     CUtensorMap tah, tal, tbh, tbl;
-    if (!map_f32(enc, &tah, Ahi, Kp, M, BM, lda_s) || !map_f32(enc, &tal, Alo, Kp, M, BM, lda_s) ||
-        !map_f32(enc, &tbh, Bhi, Kp, N, BN) || !map_f32(enc, &tbl, Blo, Kp, N, BN))
+    if (!map_f32(enc, &tah, Ahi, Kp, M, BM, lda_s) || !map_f32(enc, &tal, Alo, Kp, M, BM, lda_s, mix) ||
+        !map_f32(enc, &tbh, Bhi, Kp, N, BN) || !map_f32(enc, &tbl, Blo, Kp, N, BN, 0, mix))
         return cudaErrorInvalidValue;
     int dev = 0;
     cudaGetDevice(&dev);
-    static bool attr_done[64] = {false};
-    if (dev < 64 && !attr_done[dev]) {
-        cudaError_t e = cudaFuncSetAttribute(gemm_3xtf32_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    static bool attr_done[2][64] = {};
+    if (dev < 64 && !attr_done[mix ? 1 : 0][dev]) {
+        cudaError_t e = cudaFuncSetAttribute(mix ? gemm_3xtf32_kernel<true> : gemm_3xtf32_kernel<false>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
         if (e != cudaSuccess) return e;
-        attr_done[dev] = true;
+        attr_done[mix ? 1 : 0][dev] = true;
     }
     const int tiles_m = (int)((M + BM - 1) / BM), tiles_n = (int)((N + BN - 1) / BN);
     const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 3) == 0) ? 1 : 0;
-    gemm_3xtf32_kernel<<<tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(tah, tal, tbh, tbl, C, ldc, (int)M, (int)N,
-                                                                          (int)Kp, tiles_m, tiles_n, vec_ok);
+    (mix ? gemm_3xtf32_kernel<true> : gemm_3xtf32_kernel<false>)<<<tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(
+        tah, tal, tbh, tbl, C, ldc, (int)M, (int)N, (int)Kp, tiles_m, tiles_n, vec_ok);
     return cudaGetLastError();
 }
 

@@ -33,26 +33,53 @@ namespace k2x {
 constexpr int BM = 128;                 // A rows per CTA (UMMA M = 256 over the pair)
 constexpr int BN = 256;                 // UMMA N (cluster tile columns)
 constexpr int BNH = BN / 2;             // B^T rows per CTA
-constexpr int BK = K2_BK, STAGES = 3, UMMA_K = 8;
-constexpr int A_BYTES = BM * BK * 4;    // 16 KiB
-constexpr int B_BYTES = BNH * BK * 4;   // 16 KiB
-constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;   // 64 KiB per CTA
+constexpr int UMMA_K = 8;
 constexpr int EPI_WARPS = 16;
 constexpr int EPI_COLS = BN / (EPI_WARPS / 4);           // 64 columns per epilogue warp
 constexpr int FIRST_EPI_WARP = 2;   // warps 2..17: each TMEM lane quarter (warp % 4) gets 4 warps
 constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
 constexpr int TMEM_COLS = 512;
-constexpr int KCB = 4;                  // K chunk = KCB * BK = 128 (R16)
-constexpr int GROUP_M = 4;              // cluster-tile rows per raster group (sweep: 4 best)
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+constexpr int KCHUNK = 128;             // K chunk promoted from TMEM (R16)
+constexpr int GROUP_M = 8;              // cluster-tile rows per raster group (r2 sweep at C4: 8 best, DRAM/power)
+// K-block width BKF (floats per stage row): 32 = one 128-byte swizzle row (SWIZZLE_128B),
+// 3-stage ring of 64 KiB; 16 = 64-byte rows (SWIZZLE_64B), 7-stage ring of 32 KiB -- the same
+// 224 KiB of shared memory holds 6 stages ahead of the MMAs instead of 2 (deeper TMA
+// prefetch: the 2 x 1024-cycle lead of the 64 KiB ring does not cover the L2 / DRAM
+// latency plus the stage's own transfer at tf32bf16's feed rate, 64 B/clk per SM).
+template <int BKF>
+struct Cfg {
+    static constexpr int BK = BKF;
+    static constexpr int A_BYTES = BM * BKF * 4;
+    static constexpr int B_BYTES = BNH * BKF * 4;
+    static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+    static constexpr int STAGES = BKF == 32 ? 3 : 7;
+    static constexpr int KCB = KCHUNK / BKF;
+    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+    static constexpr CUtensorMapSwizzle SWZ = BKF == 32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
+};
 }  // namespace k2x
 
+// UMMA descriptor of a K-major operand tile with BKF-float rows (SW128 or SW64)
+template <int BKF>
+__device__ __forceinline__ uint64_t k2_desc(uint32_t saddr) {
+    if constexpr (BKF == 32) return umma_desc_k_sw128(saddr);
+    else return umma_desc_k_sw64(saddr);
+}
+
+// MIX = tf32bf16 (R22), BKF = K-block width of the TMA ring (see k2x::Cfg).  The MMA
+// order is fixed per 16-wide K step -- MIX: a_lo'*b_hi', a_hi'*b_lo' (kind::f16), then
+// a_hi*b_hi for k and k+8 (kind::tf32); 3xTF32: per 8-wide step lo*hi, hi*lo, hi*hi --
+// so every BKF (and K2 v1) accumulates in the same order: bitwise the same C.
+template <bool MIX, int BKF>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
     gemm_3xtf32_2sm_kernel(const __grid_constant__ CUtensorMap tAh, const __grid_constant__ CUtensorMap tAl,
                            const __grid_constant__ CUtensorMap tBh, const __grid_constant__ CUtensorMap tBl,
                            float *__restrict__ C, int64_t ldc, int M, int N, int Kp, int tiles_m, int tiles_n,
-                           int group_m, int vec_ok, int *dyn_next, int *dyn_mine) {
+                           int group_m, int vec_ok, int *dyn_next, int *dyn_mine, int dbg) {
     using namespace k2x;
+    using G = Cfg<BKF>;
+    constexpr int BK = G::BK, STAGES = G::STAGES, A_BYTES = G::A_BYTES, B_BYTES = G::B_BYTES;
+    constexpr int STAGE_BYTES = G::STAGE_BYTES, KCB = G::KCB;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t base = (smem_u32(smem_raw) + 1023u) & ~1023u;
     const uint32_t bar_full = base + STAGES * STAGE_BYTES;   // STAGES x 8 (used in the leader)
@@ -114,18 +141,24 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
                 const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
                 mbar_wait(bar_empty + 8 * s, ph ^ 1u);
                 const uint32_t fb_leader = mapa_shared(bar_full + 8 * s, 0);
+                if (dbg == 2 || dbg == 3) {   // measurement only: no operand traffic (PDL_K2_DEBUG=2, 3)
+                    if (rank == 0) mbar_arrive(bar_full + 8 * s);
+                    continue;
+                }
                 if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * STAGE_BYTES);
                 const uint32_t st = base + s * STAGE_BYTES;
+                const int kl = kb * (MIX ? 2 * BK : BK);   // bf16 [hi' | lo'] rows: 2 BK halves per block
                 tma_load_2d_2sm(st, &tAh, fb_leader, kb * BK, m0);
-                tma_load_2d_2sm(st + A_BYTES, &tAl, fb_leader, kb * BK, m0);
+                tma_load_2d_2sm(st + A_BYTES, &tAl, fb_leader, kl, m0);
                 tma_load_2d_2sm(st + 2 * A_BYTES, &tBh, fb_leader, kb * BK, nb0);
-                tma_load_2d_2sm(st + 2 * A_BYTES + B_BYTES, &tBl, fb_leader, kb * BK, nb0);
+                tma_load_2d_2sm(st + 2 * A_BYTES + B_BYTES, &tBl, fb_leader, kl, nb0);
             }
         }
     } else if (warp == 1) {
         // ---------------- MMA issuer (leader CTA, one thread) ----------------
         if (rank == 0 && lane == 0) {
             constexpr uint32_t idesc = idesc_tf32(2 * BM, BN);
+            constexpr uint32_t idesc16 = idesc_bf16(2 * BM, BN);
             for (int kb = 0; kb < nk; ++kb) {
                 const int chunk = kb / KCB, kin = kb - chunk * KCB;
                 const uint32_t buf = (uint32_t)chunk & 1u;
@@ -140,13 +173,27 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
                 asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
                 const uint32_t st = base + s * STAGE_BYTES;
                 const uint32_t ah = st, al = st + A_BYTES, bh = st + 2 * A_BYTES, bl = bh + B_BYTES;
+                if (dbg == 1) {   // measurement only: no MMAs, the TMA ring alone (PDL_K2_DEBUG=1)
+                } else if constexpr (MIX) {
+                    // per 16-wide K step: the BF16 plane holds [hi'(16) | lo'(16)] = 64 bytes
 #pragma unroll
-                for (int kk = 0; kk < BK / UMMA_K; ++kk) {
-                    const uint32_t off = kk * UMMA_K * 4;
-                    const uint32_t acc0 = (kin == 0 && kk == 0) ? 0u : 1u;
-                    umma_tf32_2sm(dtm, umma_desc_k_sw128(al + off), umma_desc_k_sw128(bh + off), idesc, acc0);
-                    umma_tf32_2sm(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bl + off), idesc, 1u);
-                    umma_tf32_2sm(dtm, umma_desc_k_sw128(ah + off), umma_desc_k_sw128(bh + off), idesc, 1u);
+                    for (int k16 = 0; k16 < BK / 16; ++k16) {
+                        const uint32_t o16 = k16 * 64, o32 = k16 * 64;
+                        const uint32_t acc0 = (kin == 0 && k16 == 0) ? 0u : 1u;
+                        umma_bf16_2sm(dtm, k2_desc<BKF>(al + o16 + 32), k2_desc<BKF>(bl + o16), idesc16, acc0);
+                        umma_bf16_2sm(dtm, k2_desc<BKF>(al + o16), k2_desc<BKF>(bl + o16 + 32), idesc16, 1u);
+                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + o32), k2_desc<BKF>(bh + o32), idesc, 1u);
+                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + o32 + 32), k2_desc<BKF>(bh + o32 + 32), idesc, 1u);
+                    }
+                } else {
+#pragma unroll
+                    for (int kk = 0; kk < BK / UMMA_K; ++kk) {
+                        const uint32_t off = kk * UMMA_K * 4;
+                        const uint32_t acc0 = (kin == 0 && kk == 0) ? 0u : 1u;
+                        umma_tf32_2sm(dtm, k2_desc<BKF>(al + off), k2_desc<BKF>(bh + off), idesc, acc0);
+                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + off), k2_desc<BKF>(bl + off), idesc, 1u);
+                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + off), k2_desc<BKF>(bh + off), idesc, 1u);
+                    }
                 }
                 umma_commit_2sm(bar_empty + 8 * s);
                 if (kin == KCB - 1 || kb == nk - 1) umma_commit_2sm(bar_tfull + 8 * buf);
@@ -167,12 +214,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
             const uint32_t buf = (uint32_t)chunk & 1u;
             mbar_wait(bar_tfull + 8 * buf, (uint32_t)(chunk >> 1) & 1u);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            if (dbg < 3) {   // PDL_K2_DEBUG=3 (measurement only): chunks are not promoted
 #pragma unroll
-            for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
-                uint32_t r[16];
-                tmem_ld16(tl + buf * BN + c0, r);
+                for (int c0 = 0; c0 < EPI_COLS; c0 += 16) {
+                    uint32_t r[16];
+                    tmem_ld16(tl + buf * BN + c0, r);
 #pragma unroll
-                for (int j = 0; j < 16; ++j) acc[c0 + j] += __uint_as_float(r[j]);
+                    for (int j = 0; j < 16; ++j) acc[c0 + j] += __uint_as_float(r[j]);
+                }
             }
             asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
             __syncwarp();
@@ -201,41 +250,70 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
     }
 }
 
+// bf16 = 1: the bf16 [hi' | lo'] plane of the TF32+BF16 split (2 Kp halves per row).
+// Box rows of BKF floats = BKF * 4 bytes either way.
 static bool map_f32_2sm(EncodeTiledFn enc, CUtensorMap *m, const float *ptr, uint64_t Kp, uint64_t rows,
-                        uint32_t box_rows, uint64_t ld = 0) {
-    cuuint64_t dims[2] = {Kp, rows};
+                        uint32_t box_rows, uint64_t ld, int bf16, int bkf) {
+    cuuint64_t dims[2] = {bf16 ? 2 * Kp : Kp, rows};
     cuuint64_t strides[1] = {(ld ? ld : Kp) * 4};
-    cuuint32_t box[2] = {(cuuint32_t)k2x::BK, box_rows};
+    cuuint32_t box[2] = {(cuuint32_t)(bf16 ? 2 * bkf : bkf), box_rows};
     cuuint32_t es[2] = {1, 1};
-    return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float *>(ptr), dims, strides, box, es,
-               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+    return enc(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+               const_cast<float *>(ptr), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+               bkf == 32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
-                                   const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                                   cudaStream_t stream, int *dyn_next, int *dyn_mine, int64_t lda_s) {
+// K-block width of the CTA-pair kernel: PDL_K2_BK = 16 | 32 (measurement knob),
+// default 32: the 7-stage SW64 ring measured slower at C4 (tf32bf16 29.8 vs 23.9 ms,
+// 3xtf32 33.1 vs 32.1 ms; r2s19), so a deeper prefetch is not what the kernel lacks.
+// Both give bitwise the same C.
+static int k2_bkf() {
+    const char *e = getenv("PDL_K2_BK");
+    return (e && atoi(e) == 16) ? 16 : 32;
+}
+
+template <bool MIX, int BKF>
+static cudaError_t launch_k2x(const CUtensorMap &tah, const CUtensorMap &tal, const CUtensorMap &tbh,
+                              const CUtensorMap &tbl, float *C, int64_t ldc, int64_t M, int64_t N, int64_t Kp,
+                              cudaStream_t stream, int *dyn_next, int *dyn_mine) {
     using namespace k2x;
-    if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
-    CUtensorMap tah, tal, tbh, tbl;
-    if (!map_f32_2sm(enc, &tah, Ahi, Kp, M, BM, lda_s) || !map_f32_2sm(enc, &tal, Alo, Kp, M, BM, lda_s) ||
-        !map_f32_2sm(enc, &tbh, Bhi, Kp, N, BNH) || !map_f32_2sm(enc, &tbl, Blo, Kp, N, BNH))
-        return cudaErrorInvalidValue;
+    auto kern = gemm_3xtf32_2sm_kernel<MIX, BKF>;
+    // measurement knob (C is garbage): 1 = TMA ring only, 2 = MMAs only, 3 = MMAs only, no chunk promotion
+    const char *de = getenv("PDL_K2_DEBUG");
+    const int dbg = de ? atoi(de) : 0;
+    constexpr int SMEM = Cfg<BKF>::SMEM_BYTES;
     int dev = 0;
     cudaGetDevice(&dev);
-    static bool attr_done[64] = {false};
+    static bool attr_done[64] = {};
     if (dev < 64 && !attr_done[dev]) {
-        cudaError_t e =
-            cudaFuncSetAttribute(gemm_3xtf32_2sm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
         if (e != cudaSuccess) return e;
         attr_done[dev] = true;
     }
     const int tiles_m = (int)((M + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((N + BN - 1) / BN);
     const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 3) == 0) ? 1 : 0;
-    gemm_3xtf32_2sm_kernel<<<2 * tiles_m * tiles_n, THREADS, SMEM_BYTES, stream>>>(
-        tah, tal, tbh, tbl, C, ldc, (int)M, (int)N, (int)Kp, tiles_m, tiles_n, raster_group_m(GROUP_M), vec_ok, dyn_next,
-        dyn_mine);
+    kern<<<2 * tiles_m * tiles_n, THREADS, SMEM, stream>>>(tah, tal, tbh, tbl, C, ldc, (int)M, (int)N, (int)Kp,
+                                                          tiles_m, tiles_n, raster_group_m(GROUP_M), vec_ok,
+                                                          dyn_next, dyn_mine, dbg);
     return cudaGetLastError();
+}
+
+cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
+                                   const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
+                                   cudaStream_t stream, int *dyn_next, int *dyn_mine, int64_t lda_s, int mix) {
+    using namespace k2x;
+    if (M <= 0 || N <= 0 || Kp <= 0) return cudaSuccess;
+    const int bkf = k2_bkf();
+    CUtensorMap tah, tal, tbh, tbl;
+    if (!map_f32_2sm(enc, &tah, Ahi, Kp, M, BM, lda_s, 0, bkf) || !map_f32_2sm(enc, &tal, Alo, Kp, M, BM, lda_s, mix, bkf) ||
+        !map_f32_2sm(enc, &tbh, Bhi, Kp, N, BNH, 0, 0, bkf) || !map_f32_2sm(enc, &tbl, Blo, Kp, N, BNH, 0, mix, bkf))
+        return cudaErrorInvalidValue;
+    if (bkf == 32)
+        return mix ? launch_k2x<true, 32>(tah, tal, tbh, tbl, C, ldc, M, N, Kp, stream, dyn_next, dyn_mine)
+                   : launch_k2x<false, 32>(tah, tal, tbh, tbl, C, ldc, M, N, Kp, stream, dyn_next, dyn_mine);
+    return mix ? launch_k2x<true, 16>(tah, tal, tbh, tbl, C, ldc, M, N, Kp, stream, dyn_next, dyn_mine)
+               : launch_k2x<false, 16>(tah, tal, tbh, tbl, C, ldc, M, N, Kp, stream, dyn_next, dyn_mine);
 }
 
 }  // namespace pdlk

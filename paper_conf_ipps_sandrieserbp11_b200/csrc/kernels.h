@@ -40,17 +40,23 @@ cudaError_t launch_dgemm_k1(EncodeTiledFn enc, const double *A, int64_t lda, con
 //                ldo floats, default Kp -- the packed prepared-A rows [hi | lo] use 2 Kp)
 //  split_cols_t: B (K x N, ldb, fp32)  -> Bhi, Blo  (N x Kp, K-major = B^T, zero padded)
 constexpr int K2_BK = 32;
+// mix = 1 (FP32 task variant "tf32bf16", R22): hi as above; the `lo` plane
+//                holds bf16 pairs per 32-wide K block b -- halves [64 b, 64 b + 32) =
+//                rn_bf16(hi), [64 b + 32, 64 b + 64) = rn_bf16(x - hi) (same bytes per row).
 cudaError_t launch_split_rows(const float *A, int64_t lda, int64_t M, int64_t K, float *hi, float *lo, int64_t Kp,
-                              cudaStream_t s, int64_t ldo = 0);
+                              cudaStream_t s, int64_t ldo = 0, int mix = 0);
 cudaError_t launch_split_cols_t(const float *B, int64_t ldb, int64_t K, int64_t N, float *hi, float *lo, int64_t Kp,
-                                cudaStream_t s);
+                                cudaStream_t s, int mix = 0);
 
 // K2 -- 3xTF32 tcgen05 GEMM on the split operands:
 //  C (M x N, ldc, fp32) = Ahi*Bhi^T + Ahi*Blo^T + Alo*Bhi^T   (hi/lo: M x Kp / N x Kp;
 //  lda_s = row stride of Ahi / Alo in floats, 0 = Kp)
+// mix = 1 (R22): the lo planes are the bf16 [hi' | lo'] planes of the mixed split and
+//  C = Ahi*Bhi^T (kind::tf32) + Ahi'*Blo'^T + Alo'*Bhi'^T (kind::f16, BF16 operands):
+//  two TF32-equivalent tensor passes per K block instead of three.
 cudaError_t launch_gemm_3xtf32(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
-                               cudaStream_t stream, int64_t lda_s = 0);
+                               cudaStream_t stream, int64_t lda_s = 0, int mix = 0);
 // K6/K7 -- FP64 DGEMM variant "ozaki2" (Ozaki scheme II: integer scaling and the
 // Chinese remainder theorem over INT8 GEMMs, k_ozaki2.cu).  A' = rint(A 2^(p-e_i))
 // row-wise, B' = rint(B 2^(p-f_j)) column-wise (|A'|, |B'| <= 2^p); for each of n
@@ -135,6 +141,6 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,
                                    const float *Blo, int64_t Kp, float *C, int64_t ldc, int64_t M, int64_t N,
                                    cudaStream_t stream, int *dyn_next = nullptr, int *dyn_mine = nullptr,
-                                   int64_t lda_s = 0);
+                                   int64_t lda_s = 0, int mix = 0);
 
 }  // namespace pdlk

@@ -102,6 +102,22 @@ bool worker_sgemm_ozaki2(const WorkerCtx &w) {
     return lower(trim(v)) == "ozaki2";
 }
 
+// FP32 task variant of the Worker (PDL property SGEMM_VARIANT, env PDL_SGEMM_VARIANT):
+// "tf32bf16" (default; R22: a_hi*b_hi in TF32 plus the two correction
+// products in BF16 -- two TF32-equivalent tensor passes per K block) or "3xtf32"
+// (three TF32 products, the round-1 default; split error ~2^-21 instead of <= 2^-17
+// of |A||B|).  Returns 1 for tf32bf16, 0 for 3xtf32, -1 for a name this build does
+// not know ("ozaki" / "ozaki2" are reported by their own checks).
+int worker_sgemm_mix(const WorkerCtx &w) {
+    std::string v;
+    if (const char *e = getenv("PDL_SGEMM_VARIANT")) v = e;
+    else if (const Property *p = g->model.prop(w.pu, "SGEMM_VARIANT")) v = p->value;
+    v = lower(trim(v));
+    if (v.empty() || v == "tf32bf16" || v == "default") return 1;
+    if (v == "3xtf32" || v == "ozaki" || v == "ozaki2") return 0;
+    return -1;
+}
+
 // Ozaki-II per-column arrays of a task: [bmax: cols u64][sb: cols u64][fb: cols int]
 // in the shared BUF_OZE (it does not move with `rows`, so a prepared B survives
 // row-chunk tasks, REUSE_B).  The A side (residues, e_i, sa_i) lives in the packed
@@ -208,7 +224,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     const bool piped = RB * CP > 1;
     // Task variant of this Worker, pre-selected from its PDL properties (task
     // repository + static pre-selection, L1307-1326): FP64 K1 (DMMA) or K6/K7
-    // (Ozaki scheme II with its certificate), FP32 K3+K2 (3xTF32).
+    // (Ozaki scheme II with its certificate), FP32 K3+K2 (TF32+BF16 or 3xTF32).
     int oz2_nmod = 0, oz2_bits = 0;
     if (K > 0 && (f64 ? false : worker_sgemm_ozaki2(w)))
         return set_err(PDL_EUNSUPPORTED, "SGEMM_VARIANT ozaki2: Ozaki scheme II is an FP64 variant");
@@ -219,8 +235,10 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                            "%s_VARIANT ozaki (Ozaki scheme I) is retired: its dropped slice products bound the "
                            "error only by %s of K max|a| max|b|, which cannot certify the componentwise bar; use %s",
                            f64 ? "DGEMM" : "SGEMM", f64 ? "~2^-42" : "~2^-21",
-                           f64 ? "DGEMM_VARIANT=ozaki2 (certified, DESIGN.md R21) or dmma" : "the default 3xtf32");
+                           f64 ? "DGEMM_VARIANT=ozaki2 (certified, DESIGN.md R21) or dmma" : "tf32bf16 (default) or 3xtf32");
     }
+    const int mix = (K > 0 && !f64) ? worker_sgemm_mix(w) : 0;
+    if (mix < 0) return set_err(PDL_EINVAL, "SGEMM_VARIANT: unknown FP32 task variant (3xtf32 | tf32bf16)");
     bool ozaki2 = K > 0 && f64 && worker_ozaki2(w, &oz2_nmod, &oz2_bits);
     double oz2_tau = 0.0;
     const bool oz2_guard = ozaki2 && worker_oz2_guard(w, &oz2_tau);
@@ -240,7 +258,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     want.dtype = t.dtype;
     want.oz = ozaki2 ? 2 + P2.check : 0;
     want.S = ozaki2 ? P2.n : 0;
-    want.rn = ozaki2 ? P2.p : 0;
+    want.rn = ozaki2 ? P2.p : mix;
     const bool prep_b = K > 0 && (ozaki2 || !f64);
     // A task that re-prepares B while another task of this Worker may still read
     // the shared B-side buffers on another stream (a side-stream chunk task, slot
@@ -505,7 +523,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 } else if (!a_prep[i]) {
                     a_prep[i] = 1;
                     e = pdlk::launch_split_rows((const float *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K,
-                                                ahi + r0 * lda_s, alo + r0 * lda_s, Kp, cs, lda_s);
+                                                ahi + r0 * lda_s, alo + r0 * lda_s, Kp, cs, lda_s, mix);
                     w.launches += 1;
                     if (piped) {
                         ev_sa[i] = ev_get(w, evn);
@@ -517,7 +535,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (e == cudaSuccess && !b_prep[j] && !b_ready) {
                     b_prep[j] = 1;
                     e = pdlk::launch_split_cols_t((const float *)(Bd + (size_t)c0 * es), ldb, K, nc, bhi + c0 * Kp,
-                                                  blo + c0 * Kp, Kp, cs);
+                                                  blo + c0 * Kp, Kp, cs, mix);
                     w.launches += 1;
                     if (e == cudaSuccess && mark_bprep(cs)) return set_err(PDL_ECUDA, "event record failed");
                     if (piped) {
@@ -531,11 +549,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (kt_mark(w, true, cs)) return set_err(PDL_ECUDA, "event record failed");
                 if (k2v ? !strcmp(k2v, "1sm") : k2_pick_1sm(nr, nc, sms))
                     e = pdlk::launch_gemm_3xtf32(enc, ahi + r0 * lda_s, alo + r0 * lda_s, bhi + c0 * Kp, blo + c0 * Kp,
-                                                 Kp, (float *)Cs, ldcd, nr, nc, cs, lda_s);
+                                                 Kp, (float *)Cs, ldcd, nr, nc, cs, lda_s, mix);
                 else
                     e = pdlk::launch_gemm_3xtf32_2sm(enc, ahi + r0 * lda_s, alo + r0 * lda_s, bhi + c0 * Kp,
                                                      blo + c0 * Kp, Kp, (float *)Cs, ldcd, nr, nc, cs, nullptr, nullptr,
-                                                     lda_s);
+                                                     lda_s, mix);
                 if (e == cudaSuccess && kt_mark(w, false, cs)) return set_err(PDL_ECUDA, "event record failed");
                 w.launches += 1;
             }
@@ -612,6 +630,7 @@ int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K, bool *needs_raw) {
 // rows, written as packed prepared rows to C (this Worker's memory region, 16-byte
 // aligned) -- the unit the multi-rank runtime exchanges instead of raw A chunks.
 int run_prep_a(WorkerCtx &w, const Task &t) {
+    NvtxRange nv("prepare A");
     CUDA_TRY(cudaSetDevice(w.device));
     const int64_t pr = prepared_a_row_bytes(w.pu, t.dtype, t.K);
     if (pr == 0)
@@ -637,7 +656,9 @@ int run_prep_a(WorkerCtx &w, const Task &t) {
     if (t.dtype == PDL_F32) {
         const int64_t Kp = round_up(t.K, pdlk::K2_BK);
         float *hi = (float *)t.C;
-        e = pdlk::launch_split_rows((const float *)A, lda, t.M, t.K, hi, hi + Kp, Kp, w.stream, 2 * Kp);
+        const int mix = worker_sgemm_mix(w);
+        if (mix < 0) return set_err(PDL_EINVAL, "SGEMM_VARIANT: unknown FP32 task variant (3xtf32 | tf32bf16)");
+        e = pdlk::launch_split_rows((const float *)A, lda, t.M, t.K, hi, hi + Kp, Kp, w.stream, 2 * Kp, mix);
         w.launches += 1;
     } else {
         int nmod = 0, bits = 0;
@@ -680,6 +701,7 @@ int enable_peer(int from, int to) {
 }
 
 int run_dynamic(const Task &t, const std::vector<int> &gw) {
+    NvtxRange nv("DYNAMIC");
     std::vector<WorkerCtx *> ws;
     for (int pu : gw)
         for (auto &w : g->workers)
@@ -782,13 +804,15 @@ int run_dynamic(const Task &t, const std::vector<int> &gw) {
                     buf4[b] = (float *)p;
                 }
                 w.bsig.valid = false;
-                e = pdlk::launch_split_rows((const float *)Ad, lda, M, K, buf4[0], buf4[1], Kp, w.stream);
+                const int mix = worker_sgemm_mix(w);
+                if (mix < 0) return set_err(PDL_EINVAL, "SGEMM_VARIANT: unknown FP32 task variant (3xtf32 | tf32bf16)");
+                e = pdlk::launch_split_rows((const float *)Ad, lda, M, K, buf4[0], buf4[1], Kp, w.stream, 0, mix);
                 if (e == cudaSuccess)
-                    e = pdlk::launch_split_cols_t((const float *)Bd, ldb, K, N, buf4[2], buf4[3], Kp, w.stream);
+                    e = pdlk::launch_split_cols_t((const float *)Bd, ldb, K, N, buf4[2], buf4[3], Kp, w.stream, mix);
                 if (e != cudaSuccess) return set_err(PDL_ECUDA, "K3 split launch failed: %s", cudaGetErrorString(e));
                 if (kt_mark(w, true, w.stream)) return set_err(PDL_ECUDA, "event record failed");
                 e = pdlk::launch_gemm_3xtf32_2sm(enc, buf4[0], buf4[1], buf4[2], buf4[3], Kp, (float *)Cd, ldc, M, N,
-                                                 w.stream, g->dyn, mine);
+                                                 w.stream, g->dyn, mine, 0, mix);
                 w.launches += 3;
             }
             if (e != cudaSuccess) return set_err(PDL_ECUDA, "tile kernel launch failed: %s", cudaGetErrorString(e));
@@ -839,6 +863,7 @@ std::string graph_key(const WorkerCtx &w, const Task &t, const void *A, const vo
 }
 
 int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols) {
+    NvtxRange nv("worker rect %lldx%lld (pu %lld)", (long long)rows, (long long)cols, (long long)w.pu);
     const bool want = (t.flags & PDL_TASK_GRAPH) || env_on("PDL_GRAPH");
     if (!want || (t.flags & PDL_TASK_REUSE_B) || t.raw_ready || g->dry_run || rows <= 0 || cols <= 0)
         return run_rect(w, t, A, B, C, rows, cols);
@@ -929,6 +954,7 @@ int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *
 }
 
 int execute(bool sync) {
+    NvtxRange nv_run(sync ? "pdl_run" : "pdl_run_async");
     int rc = check_loaded();
     if (rc) return rc;
     std::vector<Task> q;
@@ -956,6 +982,7 @@ int execute(bool sync) {
             }
     for (size_t ti = 0; ti < q.size(); ++ti) {
         const Task &t = q[ti];
+        NvtxRange nv_task("task %lldx%lldx%lld", (long long)t.M, (long long)t.N, (long long)t.K);
         if (t.flags & PDL_TASK_LOCAL) {
             // one tile task of this process's (first) Worker, no mapping
             if (ti) pj << ",";

@@ -22,6 +22,8 @@
 #include <dlfcn.h>
 #include <unistd.h>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/libpdl.h"
 #include "kernels.h"
 #include "pdl_model.hpp"
@@ -30,6 +32,21 @@
 namespace pdlrt {
 
 using namespace pdl;
+
+// NVTX range for profilers (nsys / ncu --nvtx): header-only NVTX v3, a no-op unless a
+// tool injects itself (SURVEY.md SS5 tracing).  Ranges: pdl_run, each task, each
+// Worker rectangle, the Worker<->Worker exchange, DYNAMIC, A preparation.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    NvtxRange(const char *fmt, long long a, long long b, long long c) {
+        char buf[96];
+        snprintf(buf, sizeof buf, fmt, a, b, c);
+        nvtxRangePushA(buf);
+    }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
 
 extern thread_local std::string g_err;
 int set_err(int code, const char *fmt, ...);
@@ -228,6 +245,7 @@ int ensure_aux(WorkerCtx &w);
 bool worker_ozaki(const WorkerCtx &w, bool f64, int *slices, int *rn);
 bool worker_ozaki2(const WorkerCtx &w, int *nmod, int *bits);
 bool worker_sgemm_ozaki2(const WorkerCtx &w);
+int worker_sgemm_mix(const WorkerCtx &w);
 int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols);
 int run_dynamic(const Task &t, const std::vector<int> &gw);
 int run_rect_g(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C, int64_t rows, int64_t cols);

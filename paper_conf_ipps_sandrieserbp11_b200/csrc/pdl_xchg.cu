@@ -70,6 +70,7 @@ struct XW {
 }  // namespace
 
 int run_exchange(const Task &t, const Plan &plan, const std::vector<int> &gw) {
+    NvtxRange nv("worker<->worker exchange");
     const int G = (int)gw.size();
     const int es = t.dtype == PDL_F64 ? 8 : 4, pe = 16 / es;
     const int64_t K = t.K;

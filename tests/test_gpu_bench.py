@@ -49,6 +49,17 @@ def test_bench_two_ranks_plain_invocation():
 def test_bench_one_gpu_carries_the_fp32_leg():
     line = _bench("--gpus", 1, "--config", "C2", "--steps", 3, "--warmup", 3, "--cpu-seconds", 2, "--no-alt")
     _common(line, 1)
-    f32 = line["f32_3xtf32"]
-    assert f32["value"] > 0 and f32["roofline"]["frac"] > 0 and f32["e2e"]["value"] > 0
-    assert "K2" in f32["roofline"]["kernel"]
+    for key, variant in (("f32_3xtf32", "3xtf32"), ("f32_tf32bf16", "tf32bf16")):
+        f32 = line[key]
+        assert f32["value"] > 0 and f32["roofline"]["frac"] > 0 and f32["e2e"]["value"] > 0
+        assert "K2" in f32["roofline"]["kernel"] and f32["task_variant"].startswith(variant)
+
+
+def test_bench_fp32_variants_main_line():
+    for variant in ("default", "3xtf32"):
+        line = _bench("--dtype", "f32", "--variant", variant, "--config", "C2", "--steps", 3, "--warmup", 3,
+                      "--cpu-seconds", 1)
+        _common(line, 1)
+        want = "3xtf32" if variant == "3xtf32" else "tf32bf16"
+        assert line["config"]["task_variant"].startswith(want)
+        assert ("kind::f16" in line["roofline"]["kernel"]) == (want == "tf32bf16")

@@ -90,6 +90,8 @@ def main():
                 key = "f64/C4"
             elif "gemm_3xtf32" in d["kernel"] and name.startswith("prof_k2"):
                 key = "f32/C4"
+            elif "gemm_3xtf32" in d["kernel"] and name.startswith("prof_mix"):
+                key = "f32_tf32bf16/C4"
             if key:
                 traffic[key] = int(rd + wr)
             print(name, d["kernel"][:40], "dram bytes", int(rd + wr), d.get("stall_share"))

@@ -25,7 +25,7 @@ from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
 
 NVLINK = 770e9
 # the task variants of this build (Ozaki scheme I is retired)
-CURRENT = {("f64", "dmma"), ("f32", "3xtf32"), ("f64", "ozaki2")}
+CURRENT = {("f64", "dmma"), ("f32", "3xtf32"), ("f32", "tf32bf16"), ("f64", "ozaki2")}
 CLOCK = {}   # (dtype, variant, G) -> median SM MHz during the worst Worker's timing (if recorded)
 
 
@@ -65,7 +65,7 @@ def a_bytes_per_elem(dt, var, K):
     the certificate plane + 16 bytes of row scale / certificate sum.  Ozaki-II's
     raw rows travel after them and are read only by each chunk task's final K1
     recompute (hidden behind the residue GEMMs; not counted here).  K1: raw rows."""
-    if dt == "f32" and var == "3xtf32":
+    if dt == "f32" and var in ("3xtf32", "tf32bf16"):   # hi + lo / hi + bf16 [hi'|lo']: 8 bytes
         return 2 * (-(-K // 32) * 32) * 4 / K
     if dt == "f64" and var == "ozaki2":
         import json
@@ -114,6 +114,9 @@ def main():
     M = N = K = 16384
     rows = ["| variant | G=1 ms | G=2 | G=4 | G=8 | predicted S_8 | S_8 at the G=1 clock |",
             "|---|---|---|---|---|---|---|"]
+    for key in CURRENT:   # variants measured only by the emulations: rate from their G = 1 step
+        if key not in r and (*key, 1) in em:
+            r[key] = 2.0 * M * N * K / em[(*key, 1)]
     for (dt, var), rate in sorted(r.items()):
         es = 8 if dt == "f64" else 4
         ts = [model(M, N, K, 1024, G, rate, es, em.get((dt, var, G)), a_bytes_per_elem(dt, var, K))

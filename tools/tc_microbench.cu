@@ -4,6 +4,10 @@
 // TMEM (no global traffic), CUDA-event timed.
 //   kind::tf32  M=128 N=256 K=8   (cta_group::1) and M=256 N=256 (cta_group::2)
 //   kind::i8    M=128 N=256 K=32  (cta_group::1) and M=256 N=256 (cta_group::2)
+//   kind::f16   M=256 N=256 K=16  BF16 operands (cta_group::2), and the tf32bf16 K2 mix
+//               (per 4 instructions: 2 kind::f16 K=16 + 2 kind::tf32 K=8, cta_group::2),
+//               reported as TF32-equivalent TFLOP/s (one f16 K=16 instruction = one
+//               tf32 K=8 instruction's worth of time if BF16 runs at twice the TF32 rate)
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tools/tc_microbench tools/tc_microbench.cu
 #include <cuda_runtime.h>
 
@@ -17,10 +21,11 @@ __device__ __forceinline__ uint64_t desc_k_sw128(uint32_t saddr) {
            ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
 }
 
-// kind: 0 = tf32 (a/b fmt 2, c F32), 1 = i8 (a/b fmt 1 signed, c S32)
+// kind: 0 = tf32 (a/b fmt 2, c F32), 1 = i8 (a/b fmt 1 signed, c S32), 2 = f16 with BF16 (a/b fmt 1, c F32)
 __host__ __device__ constexpr uint32_t idesc(int kind, int M, int N) {
     return kind == 0 ? ((1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24))
-                     : ((2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24));
+           : kind == 1 ? ((2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24))
+                       : ((1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24));
 }
 
 template <int KIND, int CG>
@@ -56,14 +61,21 @@ __global__ void __launch_bounds__(128, 1) tc_peak(int iters, int *flag) {
     const uint32_t tmem = tslot;
     const uint32_t sa = su32(smem), sb = sa + 16384;
     constexpr int M = CG == 1 ? 128 : 256;
-    constexpr uint32_t id = idesc(KIND, M, 256);
+    constexpr uint32_t id = idesc(KIND == 3 ? 0 : KIND, M, 256);
+    constexpr uint32_t id16 = idesc(2, M, 256);
     if (threadIdx.x == 0 && rank == 0) {
         for (int it = 0; it < iters; ++it) {
 #pragma unroll
             for (int kk = 0; kk < 4; ++kk) {
                 const uint64_t da = desc_k_sw128(sa + kk * 32), db = desc_k_sw128(sb + kk * 32);
                 const uint32_t acc = (it | kk) ? 1u : 0u;
-                if (KIND == 0 && CG == 1)
+                if (KIND == 2 || (KIND == 3 && kk < 2))
+                    asm volatile("{.reg .pred p; setp.ne.b32 p, %4, 0; tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;}"
+                                 ::"r"(tmem), "l"(da), "l"(db), "r"(id16), "r"(acc));
+                else if (KIND == 3)
+                    asm volatile("{.reg .pred p; setp.ne.b32 p, %4, 0; tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;}"
+                                 ::"r"(tmem), "l"(da), "l"(db), "r"(id), "r"(acc));
+                else if (KIND == 0 && CG == 1)
                     asm volatile("{.reg .pred p; setp.ne.b32 p, %4, 0; tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;}"
                                  ::"r"(tmem), "l"(da), "l"(db), "r"(id), "r"(acc));
                 else if (KIND == 0)
@@ -132,7 +144,7 @@ double run(int sms, int iters) {
     cudaEventSynchronize(e1);
     float ms;
     cudaEventElapsedTime(&ms, e0, e1);
-    const double K = KIND == 0 ? 8 : 32;
+    const double K = (KIND == 0 || KIND == 3) ? 8 : KIND == 2 ? 16 : 32;   // KIND 3: TF32-equivalent
     const double per_instr = 2.0 * (CG == 1 ? 128 : 256) * 256 * K;
     const double issuers = CG == 1 ? sms : sms / 2;
     cudaFree(flag);
@@ -148,8 +160,11 @@ int main() {
     double tf2 = run<0, 2>(sms, iters);
     double i1 = run<1, 1>(sms, iters);
     double i2 = run<1, 2>(sms, iters);
+    double b2 = run<2, 2>(sms, iters);
+    double m2 = run<3, 2>(sms, iters);
     printf("{\"device\":\"%s\",\"sms\":%d,\"tf32_tflops_1sm_m128n256\":%.1f,\"tf32_tflops_2sm_m256n256\":%.1f,"
-           "\"i8_tops_1sm_m128n256\":%.1f,\"i8_tops_2sm_m256n256\":%.1f,\"err\":\"%s\"}\n",
-           p.name, sms, tf1, tf2, i1, i2, cudaGetErrorString(cudaGetLastError()));
+           "\"i8_tops_1sm_m128n256\":%.1f,\"i8_tops_2sm_m256n256\":%.1f,\"bf16_tflops_2sm_m256n256\":%.1f,"
+           "\"tf32bf16_mix_tf32eq_tflops_2sm\":%.1f,\"err\":\"%s\"}\n",
+           p.name, sms, tf1, tf2, i1, i2, b2, m2, cudaGetErrorString(cudaGetLastError()));
     return 0;
 }
