@@ -136,7 +136,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
             tma_prefetch_desc(&tAl);
             tma_prefetch_desc(&tBh);
             tma_prefetch_desc(&tBl);
-            for (int kb = 0; kb < nk; ++kb) {
+            for (int kb = 0; kb < (dbg == 4 ? 0 : nk); ++kb) {
                 const int s = kb % STAGES;
                 const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
                 mbar_wait(bar_empty + 8 * s, ph ^ 1u);
@@ -145,13 +145,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
                     if (rank == 0) mbar_arrive(bar_full + 8 * s);
                     continue;
                 }
-                if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * STAGE_BYTES);
+                // PDL_K2_DEBUG=5 (measurement only): the B lo plane is not loaded (a 25 % smaller feed)
+                if (rank == 0) mbar_arrive_expect_tx(bar_full + 8 * s, 2 * (STAGE_BYTES - (dbg == 5 ? B_BYTES : 0)));
                 const uint32_t st = base + s * STAGE_BYTES;
                 const int kl = kb * (MIX ? 2 * BK : BK);   // bf16 [hi' | lo'] rows: 2 BK halves per block
                 tma_load_2d_2sm(st, &tAh, fb_leader, kb * BK, m0);
                 tma_load_2d_2sm(st + A_BYTES, &tAl, fb_leader, kl, m0);
                 tma_load_2d_2sm(st + 2 * A_BYTES, &tBh, fb_leader, kb * BK, nb0);
-                tma_load_2d_2sm(st + 2 * A_BYTES + B_BYTES, &tBl, fb_leader, kl, nb0);
+                if (dbg != 5) tma_load_2d_2sm(st + 2 * A_BYTES + B_BYTES, &tBl, fb_leader, kl, nb0);
             }
         }
     } else if (warp == 1) {
@@ -169,7 +170,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
                 }
                 const int s = kb % STAGES;
                 const uint32_t ph = (uint32_t)(kb / STAGES) & 1u;
-                mbar_wait(bar_full + 8 * s, ph);
+                if (dbg != 4) mbar_wait(bar_full + 8 * s, ph);
                 asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
                 const uint32_t st = base + s * STAGE_BYTES;
                 const uint32_t ah = st, al = st + A_BYTES, bh = st + 2 * A_BYTES, bl = bh + B_BYTES;
@@ -195,7 +196,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
                         umma_tf32_2sm(dtm, k2_desc<BKF>(ah + off), k2_desc<BKF>(bh + off), idesc, 1u);
                     }
                 }
-                umma_commit_2sm(bar_empty + 8 * s);
+                if (dbg != 4) umma_commit_2sm(bar_empty + 8 * s);   // 4: MMAs only, no stage barriers
                 if (kin == KCB - 1 || kb == nk - 1) umma_commit_2sm(bar_tfull + 8 * buf);
             }
         }
@@ -279,7 +280,8 @@ static cudaError_t launch_k2x(const CUtensorMap &tah, const CUtensorMap &tal, co
                               cudaStream_t stream, int *dyn_next, int *dyn_mine) {
     using namespace k2x;
     auto kern = gemm_3xtf32_2sm_kernel<MIX, BKF>;
-    // measurement knob (C is garbage): 1 = TMA ring only, 2 = MMAs only, 3 = MMAs only, no chunk promotion
+    // measurement knob (C is garbage): 1 = TMA ring only, 2 = MMAs only, 3 = MMAs only, no chunk promotion,
+    // 4 = MMAs only without the per-stage full / empty barriers
     const char *de = getenv("PDL_K2_DEBUG");
     const int dbg = de ? atoi(de) : 0;
     constexpr int SMEM = Cfg<BKF>::SMEM_BYTES;

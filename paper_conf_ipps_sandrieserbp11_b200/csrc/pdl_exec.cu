@@ -210,17 +210,20 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     for (int j = 0; j <= CP; ++j) cp[j] = std::min<int64_t>(cols, round_up((int64_t)j * cols / CP, 128));
     rb[RB] = rows;
     cp[CP] = cols;
-    // PDL_PIPE_FIRST=f: the first row band is 1/f of the others (the first kernel waits
-    // for less staging; the rest of the rows spread over the remaining bands)
-    if (RB > 1) {
-        if (const char *e = getenv("PDL_PIPE_FIRST")) {
-            const int f = std::max(1, atoi(e));
-            const int64_t first = std::max<int64_t>(128, round_up(rows / RB / f, 128));
-            rb[1] = std::min<int64_t>(rows, first);
-            for (int i = 2; i < RB; ++i)
-                rb[i] = std::min<int64_t>(rows, round_up(first + (int64_t)(i - 1) * (rows - first) / (RB - 1), 128));
-        }
-    }
+    // PDL_PIPE_FIRST=f / PDL_PIPE_FIRST_COL=f: the first row band / column panel is 1/f of
+    // the others (the first kernel waits for less staging; the rest spreads over the
+    // remaining bands / panels)
+    auto shrink_first = [](std::vector<int64_t> &cut, int n, int64_t len, const char *name) {
+        const char *e = getenv(name);
+        if (n <= 1 || !e) return;
+        const int f = std::max(1, atoi(e));
+        const int64_t first = std::max<int64_t>(128, round_up(len / n / f, 128));
+        cut[1] = std::min<int64_t>(len, first);
+        for (int i = 2; i < n; ++i)
+            cut[i] = std::min<int64_t>(len, round_up(first + (int64_t)(i - 1) * (len - first) / (n - 1), 128));
+    };
+    shrink_first(rb, RB, rows, "PDL_PIPE_FIRST");
+    shrink_first(cp, CP, cols, "PDL_PIPE_FIRST_COL");
     const bool piped = RB * CP > 1;
     // Task variant of this Worker, pre-selected from its PDL properties (task
     // repository + static pre-selection, L1307-1326): FP64 K1 (DMMA) or K6/K7
