@@ -1,6 +1,6 @@
 """One task through libpdl for compute-sanitizer (memcheck / racecheck /
 synccheck) runs: `python tools/sanitize_run.py <variant> <M> <N> <K> [workers]`
-with variant in dmma | 3xtf32 | ozaki2 | ozaki2-flagged (adversarial inputs that
+with variant in dmma | tf32bf16 | 3xtf32 | ozaki2 | ozaki2-flagged (adversarial inputs that
 send elements through the certificate's K1 recompute) | exchange (host operands,
 8 Workers, the Worker<->Worker peer-copy path).  Checks the result against the
 oracle on a few rows so a silent corruption under the tool also fails."""
@@ -23,13 +23,14 @@ def main():
     workers = int(sys.argv[5]) if len(sys.argv) > 5 else 1
     os.environ.pop("PDL_DRY_RUN", None)
     os.environ["PDL_ALLOW_OVERSUBSCRIBE"] = "1"
-    dt = np.float32 if variant == "3xtf32" else np.float64
+    dt = np.float32 if variant in ("3xtf32", "tf32bf16") else np.float64
     A = W.signed((M, K), dt, 1)
     B = W.signed((K, N), dt, 2)
     if variant == "ozaki2-flagged":
         A[3, :2] = [2.0 ** 60, 1.0]
         B[:2, 5] = [0.0, 1.0]
-    props = {"DGEMM_VARIANT": "ozaki2"} if variant.startswith("ozaki2") else None
+    props = ({"DGEMM_VARIANT": "ozaki2"} if variant.startswith("ozaki2") else
+             {"SGEMM_VARIANT": variant} if dt == np.float32 else None)
     pdl.load(pdl.descriptor_xml(workers, props=props) if props else pdl.descriptor_path(workers))
     if variant == "exchange":
         C = np.full((M, N), np.nan, dtype=dt)
