@@ -52,6 +52,18 @@ TF32_TCGEN05_PEAK_TFLOPS = 1107.0
 INT8_TCGEN05_PEAK_TOPS = 4571.0
 
 
+# The paper's own result and hardware, quoted as context: it
+# reports speedups only (Fig. 5), whose values PAPER.md does not retain.
+PAPER_CONTEXT = {
+    "workload": "FP64 DGEMM of two 8192x8192 matrices (PAPER.md L1402-1406)",
+    "hardware": "2x Xeon X5550 (8 cores) + GTX 480 + GTX 285, CUBLAS DGEMM / GotoBLAS2 under StarPU "
+                "(L1396-1431)",
+    "published": "speedup over a single-threaded program only (Fig. 5); the values are not recoverable "
+                 "from PAPER.md",
+    "box_fp64_peak_gflops_derived": 340,
+}
+
+
 def parse():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
@@ -661,6 +673,7 @@ def main():
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": int(timed_launches),
             "clocks": clocks,
+            "paper_context": PAPER_CONTEXT,
         }
         if world > 1:
             line["config"]["dist_backend"] = backend
