@@ -6,7 +6,7 @@ scaled error against the oracle on sampled rows, and the oracle's own rate.
 Multi-Worker configs run their Worker count oversubscribed on the one GPU (the
 mapping and per-Worker launches are real; NVLink scaling is not measured).
 
-    python tools/bench_table.py [--out profiles/r01_bench_table.md]
+    python tools/bench_table.py [--out profiles/r02_bench_table.md]
 """
 import argparse
 import json
@@ -23,16 +23,20 @@ import oracle  # noqa: E402
 import workloads as W  # noqa: E402
 from paper_conf_ipps_sandrieserbp11_b200 import pdl  # noqa: E402
 
-ROWS = [("C1", "f64", 1, None), ("C1", "f32", 1, None), ("C2", "f64", 1, None), ("C2", "f32", 1, None),
-        ("C2", "f64", 1, "ozaki2"), ("C3", "f64", 2, None), ("C3", "f64", 4, None), ("C3", "f32", 4, None),
+# (config, dtype, Workers, variant): None = the dtype's default (FP64 dmma, FP32 tf32bf16)
+ROWS = [("C1", "f64", 1, None), ("C1", "f32", 1, None), ("C1", "f32", 1, "3xtf32"),
+        ("C2", "f64", 1, None), ("C2", "f32", 1, None), ("C2", "f32", 1, "3xtf32"), ("C2", "f64", 1, "ozaki2"),
+        ("C3", "f64", 2, None), ("C3", "f64", 4, None), ("C3", "f32", 4, None), ("C3", "f32", 4, "3xtf32"),
         ("C3", "f64", 4, "ozaki2"), ("C0", "f64", 1, None), ("C0", "f64", 2, None), ("C0", "f64", 2, "ozaki2"),
-        ("C4", "f64", 1, None), ("C4", "f32", 1, None), ("C4", "f64", 1, "ozaki2"),
-        ("C5", "f64", 8, None), ("C5", "f32", 8, None), ("C5", "f64", 8, "ozaki2")]
+        ("C4", "f64", 1, None), ("C4", "f32", 1, None), ("C4", "f32", 1, "3xtf32"), ("C4", "f64", 1, "ozaki2"),
+        ("C5", "f64", 8, None), ("C5", "f32", 8, None), ("C5", "f32", 8, "3xtf32"), ("C5", "f64", 8, "ozaki2")]
 
 
 def descriptor(G, dt, variant):
     if variant == "ozaki2":
         return pdl.descriptor_xml(G, props={"DGEMM_VARIANT": "ozaki2"})
+    if variant in ("3xtf32", "tf32bf16"):
+        return pdl.descriptor_xml(G, props={"SGEMM_VARIANT": variant})
     return pdl.descriptor_xml(G)
 
 
@@ -85,7 +89,7 @@ def run_row(cfg, dt, G, variant, steps):
     ot = time.perf_counter() - t0
     err = float(oracle.scaled_error(C[rows], Cref, D).max())
     return {"config": cfg, "M": c.M, "N": c.N, "K": c.K, "tile": c.tile, "dtype": dt, "workers": G,
-            "variant": variant or ("dmma" if dt == "f64" else "3xtf32"), "ms": round(ms, 3),
+            "variant": variant or ("dmma" if dt == "f64" else "tf32bf16"), "ms": round(ms, 3),
             "gflops": round(flops / ms / 1e6, 1), "e2e_gflops": round(flops / ems / 1e6, 1),
             "max_scaled_err": err, "oracle_rows": int(len(rows)),
             "oracle_gflops": round(2.0 * len(rows) * c.N * c.K / ot / 1e9, 2)}
