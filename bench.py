@@ -375,7 +375,17 @@ def setup_dist(args, torch, dist):
     dev = torch.device("cuda", local)
     if world > 1:
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
+            try:
+                dist.init_process_group("nccl", device_id=dev)
+            except Exception as e:   # noqa: BLE001 -- reported in the line, not hidden
+                # every rank sees the same failure (NCCL's init is collective): fall back to
+                # gloo with host-staged exchange so the run still yields a (labelled) line
+                print(f"bench.py rank {rank}: NCCL init failed ({type(e).__name__}: {e}); using gloo",
+                      file=sys.stderr, flush=True)
+                if dist.is_initialized():
+                    dist.destroy_process_group()
+                dist.init_process_group("gloo")
+                backend = "gloo (NCCL init failed)"
         else:
             dist.init_process_group("gloo")
     return world, rank, local, dev, backend, shared
