@@ -6,7 +6,8 @@ the launch configuration bench.py times.
   B = x y^T with integer factors in [-4, 4]; C = (v.x) u y^T exactly (|C| <= 2^22,
   exact in FP32 and TF32 too).  Compared bitwise on EVERY element against the
   closed form computed in int64 on the host -- no oracle run, no GPU arithmetic
-  in the expected value -- for K1 (FP64 DMMA), K2 (FP32 3xTF32) and Ozaki II.
+  in the expected value -- for K1 (FP64 DMMA), K2 (FP32: the default tf32bf16 and
+  3xTF32) and Ozaki II.
 * P5 integer matrices in {-8..8} at C4: every partial sum is an integer below
   2^20, so C equals the oracle bitwise on 256 sampled rows (all columns).
 * P7 at C4 on the 8-Worker descriptor (oversubscribed on this GPU): C is
@@ -37,7 +38,9 @@ def _env(monkeypatch):
 
 def run(A, B, dt, tile, workers=1, variant=None):
     """One task on device-resident operands through the C ABI; C back on the host."""
-    props = {"DGEMM_VARIANT": variant} if variant else None
+    props = None
+    if variant:
+        props = {("SGEMM_VARIANT" if dt == np.float32 else "DGEMM_VARIANT"): variant}
     pdl.load(pdl.descriptor_xml(workers, props=props) if props else pdl.descriptor_path(workers))
     try:
         dA = torch.from_numpy(A).cuda()
@@ -63,7 +66,8 @@ def rank1(name, dt):
 
 
 @pytest.mark.parametrize("name", ["C4", "C5"])
-@pytest.mark.parametrize("dt,variant", [(np.float64, None), (np.float32, None), (np.float64, "ozaki2")])
+@pytest.mark.parametrize("dt,variant", [(np.float64, None), (np.float32, None), (np.float32, "3xtf32"),
+                                        (np.float64, "ozaki2")])
 def test_rank1_closed_form_every_element(name, dt, variant):
     c = W.CONFIGS[name]
     A, B, expect = rank1(name, dt)
@@ -73,7 +77,8 @@ def test_rank1_closed_form_every_element(name, dt, variant):
     assert bad == 0, f"{bad} of {C.size} elements differ from the closed form"
 
 
-@pytest.mark.parametrize("dt,variant", [(np.float64, None), (np.float32, None), (np.float64, "ozaki2")])
+@pytest.mark.parametrize("dt,variant", [(np.float64, None), (np.float32, None), (np.float32, "3xtf32"),
+                                        (np.float64, "ozaki2")])
 def test_integer_matrices_c4_bitwise_sampled(dt, variant):
     c = W.CONFIGS["C4"]
     A, B = W.config_inputs("C4", dt, dist="integers")
