@@ -1,6 +1,6 @@
 """Pinned host <-> device copy bandwidth on this box (the e2e legs' PCIe floor):
-contiguous 1 GiB H2D / D2H, both directions at once, and the 2-D copy shape of the
-pipelined B column panels (K rows of 16 KiB).  CUDA events; JSON line on stdout."""
+contiguous 1 GiB H2D / D2H and both directions at once.  CUDA events; JSON line on
+stdout."""
 import json
 
 import torch
@@ -38,13 +38,6 @@ def main():
         torch.cuda.current_stream().wait_stream(s2)
     t = timed(both)
     out["duplex_total_gbs"] = 2 * n * 4 / t / 1e9
-    # B column panel of the pipelined staging: 16384 rows x 4096 fp32 out of 16384
-    K, N, w = 16384, 16384, 4096
-    hb = h[: K * N // 4 * 4].view(-1)[: K * (N // 4)]   # reuse the pinned buffer
-    hB = h.view(-1)[: K * N // 4].view(K // 4, N)       # 4096 x 16384 view
-    dB = d.view(-1)[: (K // 4) * w].view(K // 4, w)
-    out["h2d_2d_panel_gbs"] = (K // 4) * w * 4 / timed(lambda: dB.copy_(hB[:, :w], non_blocking=True)) / 1e9
-    del hb
     print(json.dumps({k: round(v, 2) for k, v in out.items()}))
 
 
