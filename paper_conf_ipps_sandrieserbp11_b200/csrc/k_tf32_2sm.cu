@@ -40,7 +40,9 @@ constexpr int FIRST_EPI_WARP = 2;   // warps 2..17: each TMEM lane quarter (warp
 constexpr int THREADS = (FIRST_EPI_WARP + EPI_WARPS) * 32;
 constexpr int TMEM_COLS = 512;
 constexpr int KCHUNK = 128;             // K chunk promoted from TMEM (R16)
-constexpr int GROUP_M = 8;              // cluster-tile rows per raster group (r2 sweep at C4: 8 best, DRAM/power)
+// cluster-tile rows per raster group (r2 sweeps at C4): tf32bf16 8 (DRAM 49.7 -> 36.6 GB per
+// launch, higher power-capped clock), 3xtf32 4 (ncu DRAM 54 GB at 4 vs 67 GB at 8)
+constexpr int GROUP_M_MIX = 8, GROUP_M_3X = 4;
 // K-block width BKF (floats per stage row): 32 = one 128-byte swizzle row (SWIZZLE_128B),
 // 3-stage ring of 64 KiB; 16 = 64-byte rows (SWIZZLE_64B), 7-stage ring of 32 KiB -- the same
 // 224 KiB of shared memory holds 6 stages ahead of the MMAs instead of 2 (deeper TMA
@@ -296,7 +298,7 @@ static cudaError_t launch_k2x(const CUtensorMap &tah, const CUtensorMap &tal, co
     const int tiles_m = (int)((M + 2 * BM - 1) / (2 * BM)), tiles_n = (int)((N + BN - 1) / BN);
     const int vec_ok = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 3) == 0) ? 1 : 0;
     kern<<<2 * tiles_m * tiles_n, THREADS, SMEM, stream>>>(tah, tal, tbh, tbl, C, ldc, (int)M, (int)N, (int)Kp,
-                                                          tiles_m, tiles_n, raster_group_m(GROUP_M), vec_ok,
+                                                          tiles_m, tiles_n, raster_group_m(MIX ? GROUP_M_MIX : GROUP_M_3X), vec_ok,
                                                           dyn_next, dyn_mine, dbg);
     return cudaGetLastError();
 }

@@ -88,10 +88,10 @@ def main():
             key = None   # only the bench's dominant-kernel captures (not e.g. the Ozaki-II recompute K1)
             if "dgemm_k1" in d["kernel"] and name.startswith("prof_k1"):
                 key = "f64/C4"
-            elif "gemm_3xtf32" in d["kernel"] and name.startswith("prof_k2"):
-                key = "f32/C4"
-            elif "gemm_3xtf32" in d["kernel"] and name.startswith("prof_mix"):
-                key = "f32_tf32bf16/C4"
+            elif "gemm_3xtf32" in d["kernel"] and name.startswith("prof_k2x3"):
+                key = "f32/C4"                      # 3xtf32 (bench's f32_3xtf32 leg)
+            elif "gemm_3xtf32" in d["kernel"] and (name.startswith("prof_k2") or name.startswith("prof_mix")):
+                key = "f32_tf32bf16/C4"             # the FP32 default
             if key:
                 traffic[key] = int(rd + wr)
             print(name, d["kernel"][:40], "dram bytes", int(rd + wr), d.get("stall_share"))

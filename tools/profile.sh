@@ -6,7 +6,7 @@
 #    roofline "traffic" of a step: tools/ncu_traffic_sum.py)
 set -x
 OUT=${OUT:-gpurun_out}
-WHAT=${WHAT:-"k1 k2 k3 oz2"}
+WHAT=${WHAT:-"k1 k2 k2x3 k3 oz2"}   # k2: the FP32 default (tf32bf16), k2x3: 3xtf32
 mkdir -p $OUT
 B="python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-cublas --no-alt --e2e-steps 1"
 P="python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-cublas --no-e2e --no-alt"
@@ -17,6 +17,7 @@ for w in $WHAT; do
         ncu --set full --clock-control none --import-source on -k regex:dgemm_k1 -s 1 -c 1 -o $OUT/prof_k1 -f $P --dtype f64 > $OUT/prof_k1.log 2>&1 ;;
     k2) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_f32.csv $B --dtype f32 > $OUT/launches_f32.log 2>&1
         ncu --set full --clock-control none --import-source on -k regex:gemm_3xtf32 -s 1 -c 1 -o $OUT/prof_k2 -f $P --dtype f32 > $OUT/prof_k2.log 2>&1 ;;
+    k2x3) ncu --set full --clock-control none --import-source on -k regex:gemm_3xtf32 -s 1 -c 1 -o $OUT/prof_k2x3 -f $P --dtype f32 --variant 3xtf32 > $OUT/prof_k2x3.log 2>&1 ;;
     k3) ncu --set full --clock-control none --import-source on -k regex:split -s 2 -c 2 -o $OUT/prof_k3 -f $P --dtype f32 > $OUT/prof_k3.log 2>&1 ;;
     oz2) ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_oz2.csv $B --variant ozaki2 > $OUT/launches_oz2.log 2>&1
         # 14 GEMM launches per step at C4 (13 moduli + the certificate, R21); step 2 of the
