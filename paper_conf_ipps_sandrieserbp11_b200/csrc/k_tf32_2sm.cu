@@ -44,10 +44,10 @@ constexpr int KCHUNK = 128;             // K chunk promoted from TMEM (R16)
 // launch, higher power-capped clock), 3xtf32 4 (ncu DRAM 54 GB at 4 vs 67 GB at 8)
 constexpr int GROUP_M_MIX = 8, GROUP_M_3X = 4;
 // K-block width BKF (floats per stage row): 32 = one 128-byte swizzle row (SWIZZLE_128B),
-// 3-stage ring of 64 KiB; 16 = 64-byte rows (SWIZZLE_64B), 7-stage ring of 32 KiB -- the same
-// 224 KiB of shared memory holds 6 stages ahead of the MMAs instead of 2 (deeper TMA
-// prefetch: the 2 x 1024-cycle lead of the 64 KiB ring does not cover the L2 / DRAM
-// latency plus the stage's own transfer at tf32bf16's feed rate, 64 B/clk per SM).
+// 3-stage ring of 64 KiB (default); 16 = 64-byte rows (SWIZZLE_64B), 7-stage ring of 32 KiB,
+// which keeps 6 stages in flight ahead of the MMAs instead of 2.  The deeper ring measured
+// slower (profiles/r02_k2_measurements.md): the kernel is bound by the chip-wide L2 -> SM
+// feed, not by prefetch depth, and the smaller stages double the barrier round trips.
 template <int BKF>
 struct Cfg {
     static constexpr int BK = BKF;
@@ -57,7 +57,6 @@ struct Cfg {
     static constexpr int STAGES = BKF == 32 ? 3 : 7;
     static constexpr int KCB = KCHUNK / BKF;
     static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
-    static constexpr CUtensorMapSwizzle SWZ = BKF == 32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B;
 };
 }  // namespace k2x
 
@@ -181,12 +180,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(k2x::THREADS, 1)
                     // per 16-wide K step: the BF16 plane holds [hi'(16) | lo'(16)] = 64 bytes
 #pragma unroll
                     for (int k16 = 0; k16 < BK / 16; ++k16) {
-                        const uint32_t o16 = k16 * 64, o32 = k16 * 64;
+                        // 64 bytes per 16-wide step in both planes: bf16 [hi' | lo'], tf32 hi (k, k + 8)
+                        const uint32_t o = k16 * 64;
                         const uint32_t acc0 = (kin == 0 && k16 == 0) ? 0u : 1u;
-                        umma_bf16_2sm(dtm, k2_desc<BKF>(al + o16 + 32), k2_desc<BKF>(bl + o16), idesc16, acc0);
-                        umma_bf16_2sm(dtm, k2_desc<BKF>(al + o16), k2_desc<BKF>(bl + o16 + 32), idesc16, 1u);
-                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + o32), k2_desc<BKF>(bh + o32), idesc, 1u);
-                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + o32 + 32), k2_desc<BKF>(bh + o32 + 32), idesc, 1u);
+                        umma_bf16_2sm(dtm, k2_desc<BKF>(al + o + 32), k2_desc<BKF>(bl + o), idesc16, acc0);
+                        umma_bf16_2sm(dtm, k2_desc<BKF>(al + o), k2_desc<BKF>(bl + o + 32), idesc16, 1u);
+                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + o), k2_desc<BKF>(bh + o), idesc, 1u);
+                        umma_tf32_2sm(dtm, k2_desc<BKF>(ah + o + 32), k2_desc<BKF>(bh + o + 32), idesc, 1u);
                     }
                 } else {
 #pragma unroll
