@@ -64,7 +64,8 @@ extern "C" {
 
 /* Element types of task_matmul_ex. */
 #define PDL_F64 0            /* the paper's precision: DGEMM (L1402-1406); FP64 DMMA tensor cores */
-#define PDL_F32 1            /* FP32 in/out; 3xTF32 split on tcgen05 tensor cores (north star (2)) */
+#define PDL_F32 1            /* FP32 in/out; TF32 split on tcgen05 tensor cores (north star (2)):
+                                TF32 main product + BF16 corrections (default) or 3xTF32 */
 
 /* task_matmul_ex flags. */
 #define PDL_TASK_PANELS 1u   /* operands are this process's Worker panels (after the exchange):
@@ -87,9 +88,10 @@ extern "C" {
                                 prepared B exists */
 #define PDL_TASK_PREP_A 64u  /* with PDL_TASK_LOCAL: only prepare A -- write the task variant's
                                 prepared form of A's M rows (K wide) to C as packed rows of
-                                pdl_query("prepared_a/<dtype>/<K>") bytes (FP32 3xTF32:
-                                [TF32 hi: Kp floats][TF32 lo: Kp floats], Kp = K rounded up to
-                                32; FP64 ozaki2: [residues: ld8 bytes][e_i: int32][4 bytes]
+                                pdl_query("prepared_a/<dtype>/<K>") bytes (FP32: [TF32 hi: Kp
+                                floats][second plane: Kp floats -- tf32bf16: per 16-wide K block
+                                16 BF16 hi' then 16 BF16 lo'; 3xtf32: TF32 lo], Kp = K rounded up
+                                to 32; FP64 ozaki2: [residues: ld8 bytes][e_i: int32][4 bytes]
                                 [certificate row sum: u64]); B and N are ignored.  C: 16-byte
                                 aligned memory of the Worker's device.  PDL_EUNSUPPORTED for
                                 variants that exchange raw rows (query answers 0: FP64 dmma) */
@@ -139,8 +141,11 @@ extern "C" {
  *   bound of |A||B|, and K1 recomputes each element whose bound exceeds
  *   tau |A||B| -- so |C - AB| <= tau |A||B| holds element by element for any
  *   finite input (R20, R21); tasks with K > 65536 run K1.
- *   SGEMM_VARIANT = 3xtf32 (default: K3 + K2).  The round-1 variant "ozaki"
- *   (Ozaki scheme I) is retired: PDL_EUNSUPPORTED at pdl_run.
+ *   SGEMM_VARIANT = tf32bf16 (default: K3 + K2, a_hi*b_hi in TF32 plus the
+ *   two correction products in BF16, split error <= 7.9e-6 |A||B|, DESIGN.md
+ *   R22) | 3xtf32 (three TF32 products); another name is PDL_EINVAL at
+ *   pdl_run.  The round-1 variant "ozaki" (Ozaki scheme I) is retired:
+ *   PDL_EUNSUPPORTED at pdl_run.
  *   RELATIVE_SPEED weights the BLOCK mapping.  Env PDL_<PROPERTY> overrides a
  *   property for every Worker.
  * This process is the single Master driving every Worker of the descriptor.
@@ -172,7 +177,8 @@ int pdl_load_rank(const char *descriptor, int rank, int nranks);
 int task_matmul(const double *A, const double *B, double *C,
                 int64_t M, int64_t N, int64_t K, int64_t tile);
 
-/* task_matmul_f32 -- FP32 variant of the same task interface (3xTF32 tcgen05). */
+/* task_matmul_f32 -- FP32 variant of the same task interface (TF32-split tcgen05;
+ * SGEMM_VARIANT picks tf32bf16 or 3xtf32). */
 int task_matmul_f32(const float *A, const float *B, float *C,
                     int64_t M, int64_t N, int64_t K, int64_t tile);
 
