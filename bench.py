@@ -247,6 +247,18 @@ def variant_ops(variant, rows, cols, K):
     return ozaki2_ops(rows, cols, K)
 
 
+def ozaki2_skip_adjust(ops, kname, guard, K):
+    """The certificate GEMM is skipped when no row or column of the launch mixes signs
+    (R23; stats of the last step): count n GEMMs instead of n + 1."""
+    skipped = sum(w.get("certificate_gemms_skipped", 0) for w in guard)
+    if skipped:
+        n_mod = ozaki2_moduli(K)[0]
+        ops *= n_mod / (n_mod + 1)
+        kname = kname.replace("+ 1 certificate GEMM", "(the certificate GEMM skipped: no row or column mixes "
+                                                      "signs, the CRT pass certifies, R23)")
+    return ops, kname, skipped
+
+
 def variant_label(variant, dtype, K):
     n = ozaki2_moduli(K)[0]
     return f"{dtype}-ozaki2-i8x{n}", f"ozaki2 (K6/K7, {n} moduli + certificate GEMM, CRT, K1 recompute)"
@@ -536,6 +548,7 @@ def main():
     peak_dtype = "i8" if ozaki else args.dtype
     if ozaki:
         pipe_flops, kname = variant_ops(args.variant, wp.rows, wp.cols, K)
+        pipe_flops, kname, _ = ozaki2_skip_adjust(pipe_flops, kname, pdl.query_json("stats").get("ozaki_guard", []), K)
     else:
         f32name = "3xtf32" if args.variant == "3xtf32" else "tf32bf16"
         f32v = F32_VARIANTS[f32name]
@@ -550,7 +563,7 @@ def main():
         roofline["note"] = f32v[2]
     if ozaki:
         roofline["note"] = ("achieved counts int8 tensor ops (one residue GEMM per modulus + the certificate "
-                            "GEMM, 2 ops per MAC); useful FP64 FLOP = 2MNK")
+                            "GEMM unless no row or column mixes signs (R23), 2 ops per MAC); useful FP64 FLOP = 2MNK")
 
     clock_context(roofline, clocks)
 
@@ -632,6 +645,7 @@ def main():
         akt = pdl.kernel_times()
         guard = pdl.query_json("stats").get("ozaki_guard", [])
         aops, akname = variant_ops(av, M, N, K)
+        aops, akname, skipped = ozaki2_skip_adjust(aops, akname, guard, K)
         apeak, apsrc, _ = tensor_peak("i8")
         aach = aops / (float(np.mean(akt)) / 1e3) / 1e12 if akt else None
         adt, alabel = variant_label(av, args.dtype, K)
@@ -642,7 +656,10 @@ def main():
                      "parity": "certified |C - AB| <= 5e-13 |A||B| per element (DESIGN.md R21; "
                                "tests/test_gpu_ozaki2.py, tests/test_ozaki2_certificate.py)",
                      "certificate": {"tiles_checked": sum(w["tiles_checked"] for w in guard),
-                                     "elements_recomputed_by_k1": sum(w["elements_recomputed"] for w in guard)},
+                                     "elements_recomputed_by_k1": sum(w["elements_recomputed"] for w in guard),
+                                     "launches_certified_in_crt_pass": sum(w.get("certified_in_crt", 0)
+                                                                           for w in guard),
+                                     "certificate_gemms_skipped": skipped},
                      "roofline": {"bound": "tensor", "achieved": round(aach, 1) if aach else None,
                                   "peak": apeak, "unit": "TFLOP/s",
                                   "frac": round(aach / apeak, 4) if aach else None,

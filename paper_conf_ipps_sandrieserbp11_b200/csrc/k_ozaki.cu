@@ -248,13 +248,31 @@ struct Oz2Moduli {
     long long ldw = 0;
     unsigned *fallback = nullptr;
     double kappa = 0.0;
+    // R23 (rsign null = off): elements whose row and column are sign-uniform are the
+    // CRT pass's; this epilogue checks the others, and every role skips the certificate
+    // items -- the launch's last item group -- when *sign_word == 0 (no row or column of
+    // the launch mixes signs)
+    const unsigned *rsign = nullptr;
+    long long rsign_ld = 1;
+    const unsigned *csign = nullptr;
+    const unsigned *sign_word = nullptr;
 };
 
-// kappa sb_j rounded up, once per launch (the epilogue's per-column term)
+// kappa sb_j rounded up, once per launch (the epilogue's per-column term); with R23 on
+// (sign_word) the same pass scans the rows' and columns' sign bits: a row or column that
+// mixes signs sets *sign_word (zeroed before)
 __global__ void oz2_cert_cols_kernel(const unsigned long long *__restrict__ sb, int64_t cols, double kappa,
-                                     double *__restrict__ sbd) {
+                                     double *__restrict__ sbd, const unsigned *__restrict__ rsign, int64_t rsign_ld,
+                                     int64_t rows, const unsigned *__restrict__ csign,
+                                     unsigned *__restrict__ sign_word) {
     const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (j < cols) sbd[j] = __dmul_ru(__ull2double_ru(sb[j]), kappa);
+    bool mixed = false;
+    if (j < cols) {
+        sbd[j] = __dmul_ru(__ull2double_ru(sb[j]), kappa);
+        mixed = sign_word && csign[j] == 3u;
+    }
+    if (sign_word && j < rows) mixed |= rsign[j * rsign_ld] == 3u;
+    if (__any_sync(0xffffffffu, mixed) && (threadIdx.x & 31) == 0) atomicOr(sign_word, 1u);
 }
 
 // int32 -> double on the FP64 pipe (no conversion-unit op): the bits
@@ -286,7 +304,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t rank = cluster_ctarank();
     const int ntiles = tiles_m * tiles_n, nclusters = (int)(gridDim.x >> 1), cl = (int)(blockIdx.x >> 1);
-    const int nitems = nmod * ntiles;
+    // the certificate items are the launch's last item group (check == nmod - 1); with
+    // sign-uniform operands (R23, *sign_mixed == 0 after the K7 passes) they are skipped
+    // by every role of every CTA alike
+    const bool skip_cert = mods.check == nmod - 1 && mods.sign_word && *mods.sign_word == 0u;
+    const int nitems = (nmod - (skip_cert ? 1 : 0)) * ntiles;
+    if (skip_cert && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(mods.fallback + 3, 1u);   // stats
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
@@ -394,6 +417,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
             const double sad = cert && row < M ? __dmul_ru(__ull2double_ru(mods.sa[(int64_t)row * mods.sa_ld]),
                                                           mods.kappa)
                                                : 0.0;
+            // R23: a sign-uniform row's elements in sign-uniform columns are the CRT pass's
+            const bool row_uni = cert && mods.rsign && row < M && mods.rsign[(int64_t)row * mods.rsign_ld] != 3u;
             if (cert) {
                 // The certificate: the componentwise bound against the lower bound
                 // 2^(e+f-14) X^c of D (both scaled by 2^-(e_i+f_j)); a zero row or column
@@ -403,10 +428,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
                 // runs while the item's TMEM is held (it gates the next item's MMAs).
                 constexpr int NR = EPI_COLS / 32;
                 double sbr[NR];
+                uint32_t cuni = 0;   // bit k: column cbase + 32 k + lane is sign-uniform (R23)
 #pragma unroll
                 for (int k = 0; k < NR; ++k) {
                     const int col = cbase + 32 * k + lane;
                     sbr[k] = col < N ? mods.sbd[col] : 0.0;
+                    if (mods.rsign && col < N && mods.csign[col] != 3u) cuni |= 1u << k;
                 }
                 mbar_wait(bar_tfull, ti & 1u);
                 asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -424,8 +451,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(koz::Cfg<NSUB, 1>::T
                     for (int jj = 0; jj < 16; ++jj) {
                         const int idx = c0 + jj;   // compile-time: register and lane of the column term
                         const double sbj = __shfl_sync(0xffffffffu, sbr[idx >> 5], idx & 31);
+                        // (every lane shuffles: row_uni differs between lanes)
+                        const uint32_t cu = __shfl_sync(0xffffffffu, cuni, idx & 31);
+                        const bool uni = row_uni && ((cu >> (idx >> 5)) & 1u);
                         const double t = __dadd_ru(__dadd_ru(sad, sbj), fmin(sad, sbj));
-                        if (sbj != 0.0 && i2d_fp64pipe((int32_t)r[jj]) < t) bad |= 1u << jj;
+                        if (sbj != 0.0 && !uni && i2d_fp64pipe((int32_t)r[jj]) < t) bad |= 1u << jj;
                     }
                     if (row >= M || sad == 0.0) continue;   // (columns >= N carry sbj = 0)
                     if (bad) {   // 16 columns aligned to 16: one word of the element mask
@@ -706,8 +736,19 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
         // certified iff (sa + sb + min) 2^(-2p-2) <= tau' 2^-14 X^c; tau' = tau - 2^-51 leaves
         // 2^-51 for the rounding of X to double (|X 2^..| <= 4 D); kappa rounded up
         all.kappa = std::ldexp(1.0, 14 - 2 * P.p - 2) / (guard->tau - 0x1p-51) * (1.0 + 0x1p-50);
-        oz2_cert_cols_kernel<<<(unsigned)((cols + 255) / 256), 256, 0, stream>>>(guard->sb, cols, all.kappa,
-                                                                                 guard->sbd);
+        if (guard->rsign) {   // R23
+            if (!guard->csign || !guard->sign_word) return cudaErrorInvalidValue;
+            all.rsign = guard->rsign;
+            all.rsign_ld = guard->rsign_ld;
+            all.csign = guard->csign;
+            all.sign_word = guard->sign_word;
+            cudaError_t e = cudaMemsetAsync(guard->sign_word, 0, sizeof(unsigned), stream);
+            if (e != cudaSuccess) return e;
+        }
+        const int64_t nscan = std::max<int64_t>(cols, guard->rsign ? rows : 0);
+        oz2_cert_cols_kernel<<<(unsigned)((nscan + 255) / 256), 256, 0, stream>>>(
+            guard->sb, cols, all.kappa, guard->sbd, guard->rsign, guard->rsign_ld, rows, guard->csign,
+            guard->sign_word);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
         if (launches) ++*launches;

@@ -249,16 +249,30 @@ __global__ void oz2_split_rows_kernel(const double *__restrict__ A, int64_t lda,
 // coalesced loads, then an element-parallel residue pass over (row, 8-k group)
 // items -- every thread busy and 8 independent loads in flight, instead of one CTA
 // walking a row twice (oz2_split_rows_kernel, kept as PDL_OZ2_SPLIT=rows).
+// rsign (R23, optional, stride ea_ld): the row's sign bits -- bit 0 a positive entry,
+// bit 1 a negative one (3: the row mixes signs).
 __global__ void __launch_bounds__(256) oz2_rowmax_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
-                                                         int64_t K, int *__restrict__ ea, int64_t ea_ld) {
+                                                         int64_t K, int *__restrict__ ea, int64_t ea_ld,
+                                                         unsigned *__restrict__ rsign) {
     const int64_t row = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
     if (row >= M) return;
     const int lane = threadIdx.x & 31;
     const double *r = A + row * lda;
     double mx = 0.0;
-    for (int64_t k = lane; k < K; k += 32) mx = fmax(mx, fabs(r[k]));
+    bool pos = false, neg = false;
+    for (int64_t k = lane; k < K; k += 32) {
+        const double v = r[k];
+        mx = fmax(mx, fabs(v));
+        pos |= v > 0.0;
+        neg |= v < 0.0;
+    }
     for (int o = 16; o; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
     if (lane == 0) ea[row * ea_ld] = exp_of_max2(mx);
+    if (rsign) {
+        pos = __any_sync(0xffffffffu, pos);
+        neg = __any_sync(0xffffffffu, neg);
+        if (lane == 0) rsign[row * ea_ld] = (pos ? 1u : 0u) | (neg ? 2u : 0u);
+    }
 }
 
 __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
@@ -335,14 +349,21 @@ __global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__r
     }
 }
 
+// csign (R23): per column, bit 0 = a positive entry seen, bit 1 = a negative one.
 __global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N,
-                                  unsigned long long *__restrict__ bmax) {
+                                  unsigned long long *__restrict__ bmax, unsigned *__restrict__ csign) {
     const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (n >= N) return;
     const int64_t k0 = (int64_t)blockIdx.y * 256, k1 = min(K, k0 + 256);
     double mx = 0.0;
-    for (int64_t k = k0; k < k1; ++k) mx = fmax(mx, fabs(B[k * ldb + n]));
+    unsigned sg = 0;
+    for (int64_t k = k0; k < k1; ++k) {
+        const double v = B[k * ldb + n];
+        mx = fmax(mx, fabs(v));
+        sg |= (v > 0.0 ? 1u : 0u) | (v < 0.0 ? 2u : 0u);
+    }
     atomicMax(bmax + n, (unsigned long long)__double_as_longlong(mx));
+    if (csign && sg) atomicOr(csign + n, sg);
 }
 
 // B (K x N) -> Bt8 (N rows of [c][t][kk]) through a shared tile stored transposed
@@ -524,6 +545,30 @@ struct Oz2CrtF {
     double invM39, invM;           // 2^39 / M, 1 / M
 };
 
+// The certificate in the CRT pass for sign-uniform rows and columns (R23).
+// When row i of A and column j of B each hold entries of one sign, every product
+// A_ik B_kj has the same sign and D_ij = |(AB)_ij|; with the a-priori bound
+// E = (sa_i + sb_j + min) / 4 + 2^-53 |X| on |X - AB 2^-(e_i+f_j-2p)| (R21) the element is
+// certified when E (1 + tau) <= tau |X|, i.e. when
+//   (sa_i + sb_j + min(sa_i, sb_j)) / 4 <= thr |X|,   thr = tau / (1 + tau) - 2^-52
+// (rounded down; the left side is rounded up), which gives |C - AB| <= tau D_ij.  A zero
+// row or column is exact.  Failing elements are flagged for K1 like the GEMM certificate;
+// elements whose row or column mixes signs are the GEMM certificate's.
+struct Oz2CrtCert {
+    const unsigned *rsign = nullptr;   // null: no check in this pass; row sign bits (stride rsign_ld)
+    long long rsign_ld = 1;
+    const unsigned *csign = nullptr;   // column sign bits
+    const unsigned long long *sa = nullptr;
+    long long sa_ld = 1;
+    const unsigned long long *sb = nullptr;
+    double thr = 0.0;
+    uint32_t *flags = nullptr;
+    long long ldf = 0;
+    uint32_t *emask = nullptr;
+    long long ldw = 0;
+    unsigned *fallback = nullptr;
+};
+
 __device__ __forceinline__ void two_sum(double a, double b, double &s, double &e) {
     s = a + b;
     const double bb = s - a;
@@ -533,13 +578,18 @@ __device__ __forceinline__ void two_sum(double a, double b, double &s, double &e
 // 8 consecutive columns per thread: one 8-byte load per plane (all NM in flight),
 // then two groups of four columns through the FP64 pieces, each stored at once.
 // One K chunk (K <= 65536); longer K uses the integer pass.
-template <int NM>
+template <int NM, bool CERT>
 __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__restrict__ R, int64_t ldr,
                                                               int64_t plane, const int *__restrict__ ea,
                                                               const int *__restrict__ fb, const Oz2CrtF crt,
                                                               double *__restrict__ C, int64_t ldc, int64_t rows,
-                                                              int64_t cols, int vec, int64_t ea_ld) {
+                                                              int64_t cols, int vec, int64_t ea_ld,
+                                                              const Oz2CrtCert cc) {
     const double two52 = 4503599627370496.0, two39 = 549755813888.0, two78 = 302231454903657293676544.0;
+    // CERT instantiation: the R23 check of the elements whose row and column are
+    // sign-uniform (the others are the certificate GEMM's)
+    if (CERT && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0 && threadIdx.y == 0)
+        atomicAdd(cc.fallback + 2, 1u);   // stats: launches that certify in the CRT pass
     for (int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y; row < rows;
          row += (int64_t)gridDim.y * blockDim.y)
     for (int64_t c16 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8; c16 < cols;
@@ -551,6 +601,9 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
         u16[t] = __ldcs(reinterpret_cast<const uint2 *>(pr + (int64_t)t * plane));
     const int er = ea[row * ea_ld] - 2 * crt.p;
     double *crow = C + row * ldc + c16;
+    const unsigned long long sai = (CERT && cc.rsign[row * cc.rsign_ld] != 3u) ? cc.sa[row * cc.sa_ld] : 0ull;
+    const double sad = __ull2double_ru(sai);
+    uint32_t bad = 0;
 #pragma unroll
     for (int g = 0; g < 2; ++g) {
         double acc[4];
@@ -579,6 +632,17 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
             }
         }
         const int64_t c0 = c16 + 4 * g;
+        if (CERT && sai) {   // (sai == 0: zero row, or a row mixing signs)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                if (c0 + j >= cols || cc.csign[c0 + j] == 3u) continue;
+                const unsigned long long sbj = cc.sb[c0 + j];
+                if (!sbj) continue;   // zero column: exact
+                const double sbd = __ull2double_ru(sbj);
+                const double lhs = __dmul_ru(__dadd_ru(__dadd_ru(sad, sbd), fmin(sad, sbd)), 0.25);
+                if (lhs > __dmul_rd(fabs(acc[j]), cc.thr)) bad |= 1u << (4 * g + j);
+            }
+        }
         if (vec && c0 + 4 <= cols) {
             __stcs(reinterpret_cast<double2 *>(crow + 4 * g),
                    make_double2(scale2(acc[0], er + fb[c0]), scale2(acc[1], er + fb[c0 + 1])));
@@ -589,6 +653,12 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
             for (int j = 0; j < 4; ++j)
                 if (c0 + j < cols) crow[4 * g + j] = scale2(acc[j], er + fb[c0 + j]);
         }
+    }
+    if (bad) {   // 8 columns aligned to 8: inside one word of the element mask
+        atomicOr(cc.emask + row * cc.ldw + (c16 >> 5), bad << (c16 & 31));
+        uint32_t *f = cc.flags + (row >> 7) * cc.ldf + (c16 >> 7);
+        if (atomicExch(f, 1u) == 0u) atomicAdd(cc.fallback, 1u);
+        atomicAdd(cc.fallback + 1, (unsigned)__popc(bad));
     }
     }
 }
@@ -632,7 +702,7 @@ static cudaError_t upload_moduli(const Ozaki2Plan &P) {
 
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
                                   int8_t *A8, int *ea, cudaStream_t s, int *launches, unsigned long long *sa,
-                                  int64_t lda8, int64_t ea_ld, int64_t sa_ld) {
+                                  int64_t lda8, int64_t ea_ld, int64_t sa_ld, unsigned *rsign) {
     if (rows <= 0) return cudaSuccess;
     if (lda8 <= 0) lda8 = P.ld8;
     cudaError_t e = upload_moduli(P);
@@ -650,7 +720,7 @@ cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, in
         if (launches) *launches += 1;
         return cudaGetLastError();
     }
-    oz2_rowmax_kernel<<<(unsigned)((rows + 7) / 8), 256, 0, s>>>(A, lda, rows, K, ea, ea_ld);
+    oz2_rowmax_kernel<<<(unsigned)((rows + 7) / 8), 256, 0, s>>>(A, lda, rows, K, ea, ea_ld, rsign);
     const int64_t groups = (int64_t)P.nch * P.Kc / 8;
     dim3 grid((unsigned)std::min<int64_t>((groups + 255) / 256, 64), (unsigned)std::min<int64_t>(rows, 65535));
     const int vec = ((reinterpret_cast<uintptr_t>(A) & 15u) == 0 && (lda & 1) == 0) ? 1 : 0;
@@ -662,7 +732,7 @@ cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, in
 
 cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
                                   int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s,
-                                  unsigned long long *sb) {
+                                  unsigned long long *sb, unsigned *csign) {
     if (cols <= 0) return cudaSuccess;
     cudaError_t e = upload_moduli(P);
     if (e != cudaSuccess) return e;
@@ -672,9 +742,10 @@ cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64
     }
     e = cudaMemsetAsync(bmax, 0, (size_t)cols * sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
+    if (csign && (e = cudaMemsetAsync(csign, 0, (size_t)cols * sizeof(unsigned), s)) != cudaSuccess) return e;
     if (K > 0) {
         dim3 g1((unsigned)((cols + 255) / 256), (unsigned)((K + 255) / 256));
-        oz2_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax);
+        oz2_colmax_kernel<<<g1, 256, 0, s>>>(B, ldb, K, cols, bmax, csign);
     }
     const int64_t Kpad = (int64_t)P.nch * P.Kc;
     // one k tile per CTA (C4: 1.70 ms; 4 or 16 tiles per CTA with fewer column-sum
@@ -701,7 +772,7 @@ bool oz2_crt_fast_ok(const Ozaki2Plan &P) {
 
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                                      cudaStream_t s, int64_t ea_ld) {
+                                      cudaStream_t s, int64_t ea_ld, const Oz2Guard *guard) {
     if (rows <= 0 || cols <= 0) return cudaSuccess;
     if ((reinterpret_cast<uintptr_t>(R) & 3u) || (ldr & 3) || (plane & 3)) return cudaErrorInvalidValue;
     const char *crt_mode = getenv("PDL_OZ2_CRT");
@@ -719,11 +790,35 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
         f.invM = 1.0 / P.Md;
         if ((reinterpret_cast<uintptr_t>(R) & 15u) || (ldr & 15) || (plane & 15)) return cudaErrorInvalidValue;
         const int vec = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
+        Oz2CrtCert cc;
+        if (guard && guard->rsign) {   // R23: the certificate of sign-uniform rows / columns
+            if (!guard->csign || !guard->sa || !guard->sb || !guard->flags || !guard->emask || !guard->fallback)
+                return cudaErrorInvalidValue;
+            cc.rsign = guard->rsign;
+            cc.rsign_ld = guard->rsign_ld;
+            cc.csign = guard->csign;
+            cc.sa = guard->sa;
+            cc.sa_ld = guard->sa_ld;
+            cc.sb = guard->sb;
+            cc.thr = (guard->tau / (1.0 + guard->tau) - 0x1p-52) * (1.0 - 0x1p-48);
+            cc.flags = guard->flags;
+            cc.ldf = guard->ldf;
+            cc.emask = guard->emask;
+            cc.ldw = guard->ldw;
+            cc.fallback = guard->fallback;
+        }
         dim3 block(32, 8);
         dim3 grid((unsigned)((cols + 255) / 256), (unsigned)std::min<int64_t>((rows + 7) / 8, 65535));
         switch (P.n) {
 #define OZ2_CASE(k) \
-    case k: oz2_crt_fp64_kernel<k><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec, ea_ld); break;
+    case k:                                                                                                    \
+        if (cc.rsign)                                                                                          \
+            oz2_crt_fp64_kernel<k, true><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec,  \
+                                                                ea_ld, cc);                                    \
+        else                                                                                                   \
+            oz2_crt_fp64_kernel<k, false><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec, \
+                                                                 ea_ld, cc);                                   \
+        break;
             OZ2_CASE(2) OZ2_CASE(3) OZ2_CASE(4) OZ2_CASE(5) OZ2_CASE(6) OZ2_CASE(7) OZ2_CASE(8) OZ2_CASE(9)
             OZ2_CASE(10) OZ2_CASE(11) OZ2_CASE(12) OZ2_CASE(13) OZ2_CASE(14)
 #undef OZ2_CASE

@@ -106,6 +106,16 @@ struct Oz2Guard {
     int64_t ldw = 0;
     unsigned *fallback = nullptr;         // [0] += flagged tiles, [1] += flagged elements (stats)
     double tau = 5e-13;
+    // Sign-uniform rows and columns (R23; rsign null = off).  Where row i and
+    // column j each hold entries of one sign, D_ij = |C_ij| and the CRT pass certifies the
+    // element against its own |X|; the certificate GEMM checks the other elements and is
+    // skipped when no row or column of the launch mixes signs (*sign_word == 0 after the
+    // scan in its column-term pass).  Sign bits: bit 0 = a positive entry, bit 1 = a
+    // negative one.
+    const unsigned *rsign = nullptr;      // rows of the launch, stride rsign_ld (the packed row's pad word)
+    int64_t rsign_ld = 1;
+    const unsigned *csign = nullptr;      // columns of the launch
+    unsigned *sign_word = nullptr;        // the launch's "some row or column mixes signs" word
 };
 // Persistent K6 launches per K chunk for n moduli on a rows x cols rectangle with
 // `clusters` co-resident CTA pairs (k_ozaki.cu).
@@ -114,16 +124,19 @@ int oz2_launches_per_chunk(int n, int64_t rows, int64_t cols, int clusters);
 // lda8: row stride of A8 in bytes (0 = P.ld8); ea_ld / sa_ld: strides of ea / sa in
 // elements -- the packed prepared-A rows below use lda8 = P.ld8 + 16, ea_ld = lda8 / 4,
 // sa_ld = lda8 / 8.
+// rsign (optional, stride ea_ld): each row's sign bits (R23) -- the pad word after e_i
+// in the packed prepared rows, so they travel with exchanged rows.
 cudaError_t launch_ozaki2_split_a(const double *A, int64_t lda, int64_t rows, int64_t K, const Ozaki2Plan &P,
                                   int8_t *A8, int *ea, cudaStream_t s, int *launches = nullptr,
                                   unsigned long long *sa = nullptr, int64_t lda8 = 0, int64_t ea_ld = 1,
-                                  int64_t sa_ld = 1);
+                                  int64_t sa_ld = 1, unsigned *rsign = nullptr);
 // Prepared A rows of the ozaki2 variant (what PDL_TASK_PREP_A writes and
-// PDL_TASK_PREPARED_A reads): [residues: P.ld8 bytes][e_i: int32][4 bytes][sa_i: u64].
+// PDL_TASK_PREPARED_A reads): [residues: P.ld8 bytes][e_i: int32][sign bits: u32][sa_i: u64].
 inline int64_t oz2_prep_row_bytes(const Ozaki2Plan &P) { return P.ld8 + 16; }
+// csign (optional): per column sign bits (bit 0 positive, bit 1 negative entry; R23).
 cudaError_t launch_ozaki2_split_b(const double *B, int64_t ldb, int64_t K, int64_t cols, const Ozaki2Plan &P,
                                   int8_t *Bt8, int *fb, unsigned long long *bmax, cudaStream_t s,
-                                  unsigned long long *sb = nullptr);
+                                  unsigned long long *sb = nullptr, unsigned *csign = nullptr);
 // guard (P.check): the certificate GEMM runs as one more item of the persistent
 // launches and flags tiles into guard->flags (zeroed by the caller).
 cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t *Bt8, const Ozaki2Plan &P,
@@ -133,9 +146,11 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
 // otherwise launch_ozaki2_reconstruct uses the 128-bit integer pass.  PDL_OZ2_CRT=int
 // forces the integer pass.
 bool oz2_crt_fast_ok(const Ozaki2Plan &P);
+// guard with rsign (R23): the FP64-pipe CRT pass certifies the elements of sign-uniform
+// rows and columns against |X| (D = |C| there) and flags the failing ones for K1.
 cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t plane, const int *ea, const int *fb,
                                       const Ozaki2Plan &P, double *C, int64_t ldc, int64_t rows, int64_t cols,
-                                      cudaStream_t s, int64_t ea_ld = 1);
+                                      cudaStream_t s, int64_t ea_ld = 1, const Oz2Guard *guard = nullptr);
 
 // K2 v3 -- same contract on a CTA pair (tcgen05 cta_group::2, 256 x 256 tiles).
 cudaError_t launch_gemm_3xtf32_2sm(EncodeTiledFn enc, const float *Ahi, const float *Alo, const float *Bhi,

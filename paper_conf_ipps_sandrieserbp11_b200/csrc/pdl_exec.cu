@@ -118,20 +118,34 @@ int worker_sgemm_mix(const WorkerCtx &w) {
     return -1;
 }
 
-// Ozaki-II per-column arrays of a task: [bmax: cols u64][sb: cols u64][fb: cols int]
-// in the shared BUF_OZE (it does not move with `rows`, so a prepared B survives
-// row-chunk tasks, REUSE_B).  The A side (residues, e_i, sa_i) lives in the packed
-// prepared-A rows (pdlk::oz2_prep_row_bytes).  sb: the certificate's column sums.
+// Ozaki-II per-column arrays of a task: [bmax: cols u64][sb: cols u64][sbd: cols double]
+// [fb: cols int][csign: cols u32] in the shared BUF_OZE (it does not move with `rows`, so
+// a prepared B survives row-chunk tasks, REUSE_B).  The A side (residues, e_i, sa_i)
+// lives in the packed prepared-A rows (pdlk::oz2_prep_row_bytes).  sb: the certificate's
+// column sums; csign: each column's sign bits (R23).
 static int oz_b_arrays(WorkerCtx &w, int64_t cols, unsigned long long **bmax, int **fb, unsigned long long **sb,
-                       double **sbd) {
+                       double **sbd, unsigned **csign) {
     void *p = nullptr;
-    int rc = ensure_buf(w, BUF_OZE, (size_t)cols * 24 + (size_t)round_up(cols, 2) * 4, &p);
+    int rc = ensure_buf(w, BUF_OZE, (size_t)cols * 24 + (size_t)round_up(cols, 2) * 4 + (size_t)cols * 4, &p);
     if (rc) return rc;
     *bmax = (unsigned long long *)p;
     *sb = *bmax + cols;
     *sbd = (double *)(*sb + cols);
     *fb = (int *)(*sbd + cols);
+    *csign = (unsigned *)(*fb + round_up(cols, 2));
     return PDL_OK;
+}
+
+// R23: the certificate of sign-uniform rows and columns runs in the CRT pass when the
+// plan reconstructs on the FP64-pipe pass (a property of the plan and the environment,
+// never of the data, so the per-element decision is the same for any Worker count, tile
+// and staging cut); PDL_OZ2_CERT_UNIFORM=0 turns it off.
+static bool oz2_uniform_shortcut(const pdlk::Ozaki2Plan &P) {
+    if (!P.check || !pdlk::oz2_crt_fast_ok(P)) return false;
+    const char *crt = getenv("PDL_OZ2_CRT");
+    if (crt && !strcmp(crt, "int")) return false;
+    const char *e = getenv("PDL_OZ2_CERT_UNIFORM");
+    return !(e && !strcmp(e, "0"));
 }
 
 // Certificate of the Ozaki-II variant (R21): PDL property OZAKI2_GUARD =
@@ -329,6 +343,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     int8_t *a8 = nullptr, *b8 = nullptr;
     int *oz_ea = nullptr, *oz_fb = nullptr;
     unsigned long long *oz_bmax = nullptr, *oz_sa = nullptr, *oz_sb = nullptr;
+    unsigned *oz_csign = nullptr, *oz_sign_words = nullptr;
     double *oz_sbd = nullptr;
     uint8_t *oz2_R = nullptr;
     int64_t oz2_ldr = 0, oz2_plane = 0;
@@ -352,7 +367,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         oz_sa_ld = oz_pr / 8;
         if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
         b8 = (int8_t *)p;
-        if ((rc = oz_b_arrays(w, cols, &oz_bmax, &oz_fb, &oz_sb, &oz_sbd))) return rc;
+        if ((rc = oz_b_arrays(w, cols, &oz_bmax, &oz_fb, &oz_sb, &oz_sbd, &oz_csign))) return rc;
         oz2_ldr = round_up(cols, 16);
         oz2_plane = oz2_ldr * rows;
         if ((rc = ensure(BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
@@ -361,8 +376,16 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             // recompute flags of the rectangle's 128 x 128 tiles, and the Worker's
             // count of flagged tiles in this run (pdl_query "stats")
             G2.ldf = (cols + 127) / 128;
-            if ((rc = ensure(BUF_OZF, (size_t)(((rows + 127) / 128) * G2.ldf * 4), &p))) return rc;
+            const size_t fbytes = (size_t)(((rows + 127) / 128) * G2.ldf * 4);
+            // + one "mixed signs" word per band x panel launch (R23), after the tile flags
+            if ((rc = ensure(BUF_OZF, fbytes + (size_t)RB * CP * 4, &p))) return rc;
             G2.flags = (uint32_t *)p;
+            if (oz2_uniform_shortcut(P2)) {
+                oz_sign_words = (unsigned *)((char *)p + fbytes);
+                G2.rsign = (const unsigned *)(oz_ea + 1);   // the packed rows' pad words
+                G2.rsign_ld = oz_ea_ld;
+                G2.csign = oz_csign;
+            }
             G2.ldw = (cols + 31) / 32;
             if ((rc = ensure(BUF_OZM, (size_t)(rows * G2.ldw * 4), &p))) return rc;
             G2.emask = (uint32_t *)p;
@@ -452,7 +475,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                     a_prep[i] = 1;
                     e = pdlk::launch_ozaki2_split_a((const double *)(Ad + (size_t)(r0 * lda) * es), lda, nr, K, P2,
                                                     a8 + r0 * oz_pr, oz_ea + r0 * oz_ea_ld, cs, &w.launches,
-                                                    oz_sa + r0 * oz_sa_ld, oz_pr, oz_ea_ld, oz_sa_ld);
+                                                    oz_sa + r0 * oz_sa_ld, oz_pr, oz_ea_ld, oz_sa_ld,
+                                                    (unsigned *)(oz_ea + r0 * oz_ea_ld) + 1);
                     if (piped) {
                         ev_sa[i] = ev_get(w, evn);
                         CUDA_TRY(cudaEventRecord(ev_sa[i], cs));
@@ -463,7 +487,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                 if (e == cudaSuccess && !b_prep[j] && !b_ready) {
                     b_prep[j] = 1;
                     e = pdlk::launch_ozaki2_split_b((const double *)(Bd + (size_t)c0 * es), ldb, K, nc, P2,
-                                                    b8 + c0 * P2.ld8, oz_fb + c0, oz_bmax + c0, cs, oz_sb + c0);
+                                                    b8 + c0 * P2.ld8, oz_fb + c0, oz_bmax + c0, cs, oz_sb + c0,
+                                                    oz_csign + c0);
                     w.launches += 2;
                     if (e == cudaSuccess && mark_bprep(cs)) return set_err(PDL_ECUDA, "event record failed");
                     if (piped) {
@@ -484,6 +509,11 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                     gs.sa_ld = oz_sa_ld;
                     gs.sb = oz_sb + c0;
                     gs.sbd = oz_sbd + c0;
+                    if (G2.rsign) {   // R23: this band's rows, this panel's columns, this launch's word
+                        gs.rsign = G2.rsign + r0 * G2.rsign_ld;
+                        gs.csign = G2.csign + c0;
+                        gs.sign_word = oz_sign_words + (i * CP + j);
+                    }
                     gs.flags = G2.flags + (r0 / 128) * G2.ldf + c0 / 128;
                     gs.emask = G2.emask + r0 * G2.ldw + c0 / 32;
                     e = cudaMemset2DAsync(gs.flags, (size_t)(G2.ldf * 4), 0, (size_t)((nc + 127) / 128) * 4,
@@ -497,7 +527,8 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                                                  nr, nc, cs, &nl, P2.check ? &gs : nullptr, oz_pr);
                 if (e == cudaSuccess)
                     e = pdlk::launch_ozaki2_reconstruct(Rs, oz2_ldr, oz2_plane, oz_ea + r0 * oz_ea_ld, oz_fb + c0, P2,
-                                                        (double *)Cs, ldcd, nr, nc, cs, oz_ea_ld);
+                                                        (double *)Cs, ldcd, nr, nc, cs, oz_ea_ld,
+                                                        gs.rsign ? &gs : nullptr);
                 // flagged tiles: recomputed by K1 over the same operands (IEEE FP64); a
                 // prepared task reads the raw rows it was given, once they are ready
                 const char *Ar = prepared ? (const char *)t.Araw : Ad;
@@ -669,8 +700,10 @@ int run_prep_a(WorkerCtx &w, const Task &t) {
         worker_ozaki2(w, &nmod, &bits);
         const pdlk::Ozaki2Plan P = pdlk::ozaki2_plan(t.M, 1, t.K, nmod, bits, worker_oz2_guard(w, &tau));
         int8_t *a8 = (int8_t *)t.C;
+        // the rows' sign bits (R23) go into the pad word after e_i and travel with the rows
         e = pdlk::launch_ozaki2_split_a((const double *)A, lda, t.M, t.K, P, a8, (int *)(a8 + P.ld8), w.stream,
-                                        &w.launches, (unsigned long long *)(a8 + P.ld8 + 8), pr, pr / 4, pr / 8);
+                                        &w.launches, (unsigned long long *)(a8 + P.ld8 + 8), pr, pr / 4, pr / 8,
+                                        (unsigned *)(a8 + P.ld8 + 4));
     }
     if (e != cudaSuccess) return set_err(PDL_ECUDA, "A preparation launch failed: %s", cudaGetErrorString(e));
     return PDL_OK;

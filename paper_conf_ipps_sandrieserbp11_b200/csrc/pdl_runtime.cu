@@ -524,13 +524,17 @@ int pdl_query(const char *key, char *out, size_t len) {
                 bool f1 = true;
                 for (auto &w : g->workers) {
                     if (w.guard_epoch != g->run_epoch) continue;
-                    unsigned cnt[2] = {0, 0};
+                    unsigned cnt[4] = {0, 0, 0, 0};
                     cudaSetDevice(w.device);
                     if (cudaMemcpy(cnt, w.buf[BUF_OZG].ptr, sizeof cnt, cudaMemcpyDeviceToHost) != cudaSuccess)
                         cudaGetLastError();
+                    // certified_in_crt: CRT launches that certify sign-uniform rows / columns;
+                    // certificate_gemms_skipped: certificate GEMM launches skipped because no
+                    // row or column of theirs mixes signs (R23)
                     o << (f1 ? "" : ",") << "{\"id\":\"" << json_escape(m.pus[w.pu].id)
                       << "\",\"tiles_checked\":" << w.guard_tiles << ",\"tiles_recomputed\":" << cnt[0]
-                      << ",\"elements_recomputed\":" << cnt[1] << "}";
+                      << ",\"elements_recomputed\":" << cnt[1] << ",\"certified_in_crt\":" << cnt[2]
+                      << ",\"certificate_gemms_skipped\":" << cnt[3] << "}";
                     f1 = false;
                 }
                 o << "]";

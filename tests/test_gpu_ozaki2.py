@@ -365,3 +365,115 @@ def test_certificate_passes_benign_workloads(name):
     assert sum(w["tiles_checked"] for w in g) == -(-A.shape[0] // 128) * -(-B.shape[1] // 128)
     Cs, gs = oz2_run(2 * A - 1, 2 * B - 1)
     assert recomputed(gs) == 0
+
+
+# ---- the certificate of sign-uniform rows and columns (R23) ---------
+
+def oz2_run_env(A, B, monkeypatch, uniform=True, workers=1, tile=0, host=False):
+    if uniform:
+        monkeypatch.delenv("PDL_OZ2_CERT_UNIFORM", raising=False)
+    else:
+        monkeypatch.setenv("PDL_OZ2_CERT_UNIFORM", "0")
+    pdl.load(pdl.descriptor_xml(workers, props={"DGEMM_VARIANT": "ozaki2"}))
+    try:
+        if host:
+            C = np.full((A.shape[0], B.shape[1]), np.nan)
+            pdl.task_matmul(A, B, C, tile=tile)
+            pdl.run()
+        else:
+            dA, dB = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+            dC = torch.full((A.shape[0], B.shape[1]), float("nan"), dtype=torch.float64, device="cuda")
+            pdl.task_matmul(dA, dB, dC, tile=tile)
+            pdl.run()
+            C = dC.cpu().numpy()
+        return C, pdl.query_json("stats").get("ozaki_guard", [])
+    finally:
+        pdl.unload()
+
+
+def gsum(g, key):
+    return sum(w.get(key, 0) for w in g)
+
+
+def test_uniform_operands_skip_the_certificate_gemm(monkeypatch):
+    """U[0,1) operands: every row and column is sign-uniform, so D = |C| and the CRT
+    pass certifies every element; the lower-bound GEMM is skipped.  Benign data is
+    certified either way, so C is bitwise the GEMM-certificate result."""
+    A, B = W.config_inputs("C3", np.float64)
+    C, g = oz2_run_env(A, B, monkeypatch)
+    check(C, A, B, rows=np.arange(0, A.shape[0], 37))
+    assert gsum(g, "certified_in_crt") >= 1 and gsum(g, "certificate_gemms_skipped") >= 1
+    assert recomputed(g) == 0
+    C0, g0 = oz2_run_env(A, B, monkeypatch, uniform=False)
+    assert gsum(g0, "certificate_gemms_skipped") == 0 and gsum(g0, "certified_in_crt") == 0
+    assert np.array_equal(C, C0)
+    # all-negative rows times positive columns are sign-uniform too
+    C1, g1 = oz2_run_env(-A, B, monkeypatch)
+    assert gsum(g1, "certificate_gemms_skipped") >= 1
+    assert np.array_equal(C1, -C)
+
+
+def positive_adversarial(seed):
+    """Non-negative operands (every row and column sign-uniform) that Ozaki II's
+    p-bit scaling cannot represent: in-row spread over 2^+-60 and [2^60, 1] x [0, 1]^T."""
+    rng = np.random.default_rng(seed)
+    A = W.uniform((256, 384), np.float64, seed) * np.exp2(rng.integers(-60, 61, (256, 384)))
+    B = W.uniform((384, 200), np.float64, seed + 1) * np.exp2(rng.integers(-60, 61, (384, 200)))
+    A[7, :2] = [2.0 ** 60, 1.0]
+    A[7, 2:] = 0.0
+    B[:2, 11] = [0.0, 1.0]
+    return A, B
+
+
+def test_uniform_certificate_flags_what_it_cannot_certify(monkeypatch):
+    """The CRT-pass certificate is a certificate: on non-negative adversarial operands
+    it sends the elements it cannot certify to K1 and the 1e-12 bar holds; without any
+    certificate (OZAKI2_GUARD=off) the same inputs break the bar."""
+    A, B = positive_adversarial(21)
+    C, g = oz2_run_env(A, B, monkeypatch)
+    check(C, A, B)
+    assert gsum(g, "certificate_gemms_skipped") >= 1
+    assert recomputed(g) > 0
+    assert C[7, 11] == 1.0
+    C_off, _ = oz2_run(A, B, guard=False)
+    Cref, D = oracle.matmul(A, B)
+    assert oracle.scaled_error(C_off, Cref, D).max() > 1e-12
+
+
+def mixed_adversarial(seed):
+    """Some rows / columns mix signs, the rest are uniform, with adversarial entries in
+    both kinds: each element is certified by its own kind's certificate."""
+    A, B = positive_adversarial(seed)
+    rng = np.random.default_rng(seed + 7)
+    mr = rng.choice(A.shape[0], 60, replace=False)
+    A[mr] *= np.where(rng.random((60, A.shape[1])) < 0.5, -1.0, 1.0)
+    mc = rng.choice(B.shape[1], 50, replace=False)
+    B[:, mc] *= np.where(rng.random((B.shape[0], 50)) < 0.5, -1.0, 1.0)
+    A[7, 2:] = 0.0     # keep row 7 the [2^60, 1] case (uniform)
+    return A, B
+
+
+def test_mixed_sign_operands_use_both_certificates(monkeypatch):
+    A, B = mixed_adversarial(31)
+    C, g = oz2_run_env(A, B, monkeypatch)
+    check(C, A, B)
+    assert gsum(g, "certificate_gemms_skipped") == 0 and gsum(g, "certified_in_crt") >= 1
+    assert recomputed(g) > 0
+    C0, _ = oz2_run_env(A, B, monkeypatch, uniform=False)
+    check(C0, A, B)
+
+
+def test_uniform_certificate_invariant_under_workers_tiles_and_staging(monkeypatch):
+    """R14: the choice between the two certificates is per element (its row's and
+    column's signs), never per launch, so Worker count, task tile and the host-staged
+    band x panel cut change no bit -- even where one Worker's rectangle is all
+    sign-uniform and another's is not."""
+    A, B = mixed_adversarial(41)
+    ref, _ = oz2_run_env(A, B, monkeypatch)
+    check(ref, A, B)
+    for workers, tile in ((2, 64), (4, 32), (8, 0)):
+        C, _ = oz2_run_env(A, B, monkeypatch, workers=workers, tile=tile)
+        assert np.array_equal(C, ref), (workers, tile)
+    monkeypatch.setenv("PDL_PIPELINE", "force")
+    C, _ = oz2_run_env(A, B, monkeypatch, host=True, tile=64)
+    assert np.array_equal(C, ref)

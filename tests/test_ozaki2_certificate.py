@@ -131,3 +131,93 @@ def test_huge_times_zero_is_not_certified():
     B = np.array([[0.0], [1.0]])
     (i, j, err, bound, lower, D, certified, exact), = emulate(A, B, 43)
     assert err == 1 and D == 1 and not certified and lower == 0
+
+
+# ---- R23: the certificate of sign-uniform rows and columns ---------------------
+#
+# Where row i of A and column j of B each hold entries of one sign, D_ij = |(AB)_ij|,
+# and the library certifies the element in the CRT pass when
+#     (sa_i + sb_j + min(sa_i, sb_j)) / 4 <= thr |X_ij|,   thr = tau / (1 + tau) - 2^-52
+# (X = fl(A'B'), the scaled result).  Pinned: (4) a row / column is called uniform only
+# when D_ij = |(AB)_ij| holds exactly, and (5) an element certified this way has
+# |C_ij - (AB)_ij| <= tau D_ij.
+
+def _sign_bits(v):
+    return (1 if any(x > 0 for x in v) else 0) | (2 if any(x < 0 for x in v) else 0)
+
+
+def emulate_uniform(A, B, p, tau):
+    M, K = A.shape
+    N = B.shape[1]
+    e = [_exp_of_max(A[i]) for i in range(M)]
+    f = [_exp_of_max(B[:, j]) for j in range(N)]
+    Ap = [[_scale(A[i, k], p - e[i]) for k in range(K)] for i in range(M)]
+    Bp = [[_scale(B[k, j], p - f[j]) for j in range(N)] for k in range(K)]
+    sa = [sum(2 * abs(Ap[i][k]) + 1 for k in range(K) if A[i, k] != 0) for i in range(M)]
+    sb = [sum(2 * abs(Bp[k][j]) + 1 for k in range(K) if B[k, j] != 0) for j in range(N)]
+    thr = Fraction(tau) / (1 + Fraction(tau)) - Fraction(2) ** -52
+    out = []
+    for i in range(M):
+        for j in range(N):
+            uni = _sign_bits(A[i]) != 3 and _sign_bits(B[:, j]) != 3
+            X = float(sum(Ap[i][k] * Bp[k][j] for k in range(K)))     # fl(X): one rounding
+            C = math.ldexp(X, e[i] + f[j] - 2 * p)
+            P = sum(Fraction(float(A[i, k])) * Fraction(float(B[k, j])) for k in range(K))
+            D = sum(abs(Fraction(float(A[i, k])) * Fraction(float(B[k, j]))) for k in range(K))
+            certified = uni and sa[i] > 0 and sb[j] > 0 and \
+                Fraction(sa[i] + sb[j] + min(sa[i], sb[j]), 4) <= thr * abs(Fraction(X))
+            exact = sa[i] == 0 or sb[j] == 0
+            out.append((uni, certified, exact, abs(Fraction(C) - P), P, D))
+    return out
+
+
+def _uniform_inputs(kind, rng, M=6, N=5, K=9):
+    if kind == "uniform":
+        return rng.random((M, K)), rng.random((K, N))
+    if kind == "negative_rows":
+        return -rng.random((M, K)), rng.random((K, N))
+    if kind == "spread":
+        A = rng.random((M, K)) * np.exp2(rng.integers(-60, 61, (M, K)))
+        B = rng.random((K, N)) * np.exp2(rng.integers(-60, 61, (K, N)))
+        return A, B
+    if kind == "huge_times_zero":
+        A, B = rng.random((M, K)), rng.random((K, N))
+        A[0, :] = 0.0
+        A[0, :2] = [2.0 ** 60, 1.0]
+        B[:2, 0] = [0.0, 1.0]
+        A[1] = 0.0
+        B[:, 2] = 0.0
+        return A, B
+    if kind == "mixed":
+        A, B = rng.uniform(-1, 1, (M, K)), rng.random((K, N))
+        A[2] = np.abs(A[2])                 # one uniform row
+        B[:, 1] *= np.where(rng.random(K) < 0.5, -1.0, 1.0)
+        return A, B
+    raise ValueError(kind)
+
+
+@pytest.mark.parametrize("p", [8, 12, 20, 43])
+@pytest.mark.parametrize("kind", ["uniform", "negative_rows", "spread", "huge_times_zero", "mixed"])
+def test_uniform_certificate_holds(kind, p):
+    rng = np.random.default_rng(77 * p + len(kind))
+    A, B = _uniform_inputs(kind, rng)
+    tau = 5e-13 if p >= 40 else 2.0 ** (-p + 6)
+    n_cert = 0
+    for uni, certified, exact, err, P, D in emulate_uniform(A, B, p, tau):
+        if uni:
+            assert abs(P) == D                                   # (4)
+        if exact:
+            assert err == 0
+        if certified:
+            n_cert += 1
+            assert err <= Fraction(tau) * D                      # (5)
+    if kind in ("uniform", "negative_rows"):
+        assert n_cert > 0
+
+
+def test_uniform_certificate_refuses_huge_times_zero():
+    """[2^60, 1] x [0, 1]^T: both uniform, D = 1, Ozaki II returns 0 -- not certified."""
+    A = np.array([[2.0 ** 60, 1.0]])
+    B = np.array([[0.0], [1.0]])
+    (uni, certified, exact, err, P, D), = emulate_uniform(A, B, 43, 5e-13)
+    assert uni and not certified and err == 1 and D == 1
