@@ -1,6 +1,8 @@
 """One task through libpdl for compute-sanitizer (memcheck / racecheck /
 synccheck) runs: `python tools/sanitize_run.py <variant> <M> <N> <K> [workers]`
-with variant in dmma | tf32bf16 | 3xtf32 | ozaki2 | ozaki2-flagged (adversarial inputs that
+with variant in dmma | tf32bf16 | 3xtf32 | ozaki2 | ozaki2-uniform (non-negative operands: the
+certificate in the CRT pass, R23) | ozaki2-mixed (some rows / columns mix signs: both
+certificates, the GEMM epilogue's per-lane column bits) | ozaki2-flagged (adversarial inputs that
 send elements through the certificate's K1 recompute) | exchange (host operands,
 8 Workers, the Worker<->Worker peer-copy path).  Checks the result against the
 oracle on a few rows so a silent corruption under the tool also fails."""
@@ -29,6 +31,14 @@ def main():
     if variant == "ozaki2-flagged":
         A[3, :2] = [2.0 ** 60, 1.0]
         B[:2, 5] = [0.0, 1.0]
+    if variant in ("ozaki2-uniform", "ozaki2-mixed"):
+        A, B = np.abs(A), np.abs(B)
+        A[3, :2] = [2.0 ** 60, 1.0]
+        A[3, 2:] = 0.0
+        B[:2, 5] = [0.0, 1.0]
+        if variant == "ozaki2-mixed":
+            A[10:60] *= np.where(np.random.default_rng(3).random((50, K)) < 0.5, -1.0, 1.0)
+            B[:, 20:40] *= np.where(np.random.default_rng(4).random((K, 20)) < 0.5, -1.0, 1.0)
     props = ({"DGEMM_VARIANT": "ozaki2"} if variant.startswith("ozaki2") else
              {"SGEMM_VARIANT": variant} if dt == np.float32 else None)
     pdl.load(pdl.descriptor_xml(workers, props=props) if props else pdl.descriptor_path(workers))
