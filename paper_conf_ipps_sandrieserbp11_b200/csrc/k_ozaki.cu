@@ -264,15 +264,45 @@ struct Oz2Moduli {
 __global__ void oz2_cert_cols_kernel(const unsigned long long *__restrict__ sb, int64_t cols, double kappa,
                                      double *__restrict__ sbd, const unsigned *__restrict__ rsign, int64_t rsign_ld,
                                      int64_t rows, const unsigned *__restrict__ csign,
-                                     unsigned *__restrict__ sign_word) {
+                                     unsigned *__restrict__ sign_word, double *__restrict__ sbu,
+                                     unsigned long long *__restrict__ sbmax) {
     const int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     bool mixed = false;
+    unsigned long long um = 0;   // bits of a non-negative double: ordered like the value
     if (j < cols) {
-        sbd[j] = __dmul_ru(__ull2double_ru(sb[j]), kappa);
+        const double s = __ull2double_ru(sb[j]);
+        sbd[j] = __dmul_ru(s, kappa);
         mixed = sign_word && csign[j] == 3u;
+        if (sign_word) {
+            sbu[j] = mixed ? -1.0 : s;   // the CRT pass's column term (R23)
+            if (!mixed) um = (unsigned long long)__double_as_longlong(s);
+        }
     }
     if (sign_word && j < rows) mixed |= rsign[j * rsign_ld] == 3u;
     if (__any_sync(0xffffffffu, mixed) && (threadIdx.x & 31) == 0) atomicOr(sign_word, 1u);
+    if (sign_word) {   // the launch's largest uniform column term, for the CRT pass's row bound
+        for (int o = 16; o; o >>= 1) um = max(um, __shfl_xor_sync(0xffffffffu, um, o));
+        if ((threadIdx.x & 31) == 0 && um) atomicMax(sbmax, um);
+    }
+}
+
+// R23: the CRT pass's per-row bound T_i = (sa_i + sbmax + min(sa_i, sbmax)) / thr4, every
+// step rounded up (sbmax: the launch's largest uniform column term, from the column-term
+// pass): |X_ij| >= T_i certifies element (i, j) of a sign-uniform row and column by one
+// compare.  T_i = 0 for a row mixing signs (the GEMM's) or a zero row (exact).
+__global__ void oz2_row_bound_kernel(const unsigned *__restrict__ rsign, int64_t rsign_ld,
+                                     const unsigned long long *__restrict__ sa, int64_t sa_ld, int64_t rows,
+                                     const unsigned long long *__restrict__ sbmax, double thr4,
+                                     double *__restrict__ rowT) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= rows) return;
+    double T = 0.0;
+    const unsigned long long sai = sa[i * sa_ld];
+    if (rsign[i * rsign_ld] != 3u && sai) {
+        const double sad = __ull2double_ru(sai), sbm = __longlong_as_double((long long)*sbmax);
+        T = __ddiv_ru(__dadd_ru(__dadd_ru(sad, sbm), fmin(sad, sbm)), thr4);
+    }
+    rowT[i] = T;
 }
 
 // int32 -> double on the FP64 pipe (no conversion-unit op): the bits
@@ -737,21 +767,30 @@ cudaError_t launch_ozaki2_gemm(EncodeTiledFn enc, const int8_t *A8, const int8_t
         // 2^-51 for the rounding of X to double (|X 2^..| <= 4 D); kappa rounded up
         all.kappa = std::ldexp(1.0, 14 - 2 * P.p - 2) / (guard->tau - 0x1p-51) * (1.0 + 0x1p-50);
         if (guard->rsign) {   // R23
-            if (!guard->csign || !guard->sign_word) return cudaErrorInvalidValue;
+            if (!guard->csign || !guard->sign_word || !guard->sbu || !guard->sbmax) return cudaErrorInvalidValue;
             all.rsign = guard->rsign;
             all.rsign_ld = guard->rsign_ld;
             all.csign = guard->csign;
             all.sign_word = guard->sign_word;
             cudaError_t e = cudaMemsetAsync(guard->sign_word, 0, sizeof(unsigned), stream);
+            if (e == cudaSuccess) e = cudaMemsetAsync(guard->sbmax, 0, sizeof(unsigned long long), stream);
             if (e != cudaSuccess) return e;
         }
         const int64_t nscan = std::max<int64_t>(cols, guard->rsign ? rows : 0);
         oz2_cert_cols_kernel<<<(unsigned)((nscan + 255) / 256), 256, 0, stream>>>(
             guard->sb, cols, all.kappa, guard->sbd, guard->rsign, guard->rsign_ld, rows, guard->csign,
-            guard->sign_word);
+            guard->sign_word, guard->sbu, guard->sbmax);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
         if (launches) ++*launches;
+        if (guard->rsign) {   // R23: the CRT pass's row bounds
+            if (!guard->rowT) return cudaErrorInvalidValue;
+            oz2_row_bound_kernel<<<(unsigned)((rows + 255) / 256), 256, 0, stream>>>(
+                guard->rsign, guard->rsign_ld, guard->sa, guard->sa_ld, rows, guard->sbmax,
+                oz2_uniform_thr4(guard->tau), guard->rowT);
+            if ((e = cudaGetLastError()) != cudaSuccess) return e;
+            if (launches) ++*launches;
+        }
     }
     auto group_mods = [&](int t0, int gl) {
         Oz2Moduli g = all;

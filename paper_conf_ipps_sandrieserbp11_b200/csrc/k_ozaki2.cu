@@ -553,15 +553,19 @@ struct Oz2CrtF {
 //   (sa_i + sb_j + min(sa_i, sb_j)) / 4 <= thr |X|,   thr = tau / (1 + tau) - 2^-52
 // (rounded down; the left side is rounded up), which gives |C - AB| <= tau D_ij.  A zero
 // row or column is exact.  Failing elements are flagged for K1 like the GEMM certificate;
-// elements whose row or column mixes signs are the GEMM certificate's.
+// elements whose row or column mixes signs are the GEMM certificate's.  The column term
+// sb_j (rounded up to double; -1 marks a column mixing signs) comes from the column-term
+// pass.  Per row, T = (sa_i + sbmax + min) / (4 thr) rounded up (sbmax: the launch's
+// largest uniform column term) certifies every element with |X| >= T by one compare; only
+// the elements below it (none on benign data) read their own column term.
 struct Oz2CrtCert {
     const unsigned *rsign = nullptr;   // null: no check in this pass; row sign bits (stride rsign_ld)
     long long rsign_ld = 1;
-    const unsigned *csign = nullptr;   // column sign bits
+    const double *sbu = nullptr;       // column term: sb_j rounded up, -1 for a column mixing signs
+    const double *rowT = nullptr;      // per row: the bound T_i (oz2_row_bound_kernel)
     const unsigned long long *sa = nullptr;
     long long sa_ld = 1;
-    const unsigned long long *sb = nullptr;
-    double thr = 0.0;
+    double thr4 = 0.0;                 // 4 thr, rounded down
     uint32_t *flags = nullptr;
     long long ldf = 0;
     uint32_t *emask = nullptr;
@@ -586,10 +590,8 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
                                                               int64_t cols, int vec, int64_t ea_ld,
                                                               const Oz2CrtCert cc) {
     const double two52 = 4503599627370496.0, two39 = 549755813888.0, two78 = 302231454903657293676544.0;
-    // CERT instantiation: the R23 check of the elements whose row and column are
-    // sign-uniform (the others are the certificate GEMM's)
     if (CERT && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0 && threadIdx.y == 0)
-        atomicAdd(cc.fallback + 2, 1u);   // stats: launches that certify in the CRT pass
+        atomicAdd(cc.fallback + 2, 1u);   // stats: CRT launches certifying sign-uniform rows / columns
     for (int64_t row = (int64_t)blockIdx.y * blockDim.y + threadIdx.y; row < rows;
          row += (int64_t)gridDim.y * blockDim.y)
     for (int64_t c16 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8; c16 < cols;
@@ -601,8 +603,10 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
         u16[t] = __ldcs(reinterpret_cast<const uint2 *>(pr + (int64_t)t * plane));
     const int er = ea[row * ea_ld] - 2 * crt.p;
     double *crow = C + row * ldc + c16;
-    const unsigned long long sai = (CERT && cc.rsign[row * cc.rsign_ld] != 3u) ? cc.sa[row * cc.sa_ld] : 0ull;
-    const double sad = __ull2double_ru(sai);
+    // R23: |X| >= T_i certifies the element by one compare (T_i: the row's bound over the
+    // launch's largest uniform column term, 0 for a mixing or zero row); below it, the
+    // element's own column term decides
+    const double T = CERT ? cc.rowT[row] : 0.0;
     uint32_t bad = 0;
 #pragma unroll
     for (int g = 0; g < 2; ++g) {
@@ -632,15 +636,15 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
             }
         }
         const int64_t c0 = c16 + 4 * g;
-        if (CERT && sai) {   // (sai == 0: zero row, or a row mixing signs)
+        if (CERT) {
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
-                if (c0 + j >= cols || cc.csign[c0 + j] == 3u) continue;
-                const unsigned long long sbj = cc.sb[c0 + j];
-                if (!sbj) continue;   // zero column: exact
-                const double sbd = __ull2double_ru(sbj);
-                const double lhs = __dmul_ru(__dadd_ru(__dadd_ru(sad, sbd), fmin(sad, sbd)), 0.25);
-                if (lhs > __dmul_rd(fabs(acc[j]), cc.thr)) bad |= 1u << (4 * g + j);
+                if (fabs(acc[j]) >= T || c0 + j >= cols) continue;   // certified by the row bound
+                const double sbd = cc.sbu[c0 + j];   // -1: a column mixing signs (the GEMM's); 0: exact
+                if (sbd <= 0.0) continue;
+                const double sad = __ull2double_ru(cc.sa[row * cc.sa_ld]);   // (T > 0: a uniform nonzero row)
+                if (__dadd_ru(__dadd_ru(sad, sbd), fmin(sad, sbd)) > __dmul_rd(fabs(acc[j]), cc.thr4))
+                    bad |= 1u << (4 * g + j);
             }
         }
         if (vec && c0 + 4 <= cols) {
@@ -654,7 +658,7 @@ __global__ void __launch_bounds__(256, 3) oz2_crt_fp64_kernel(const uint8_t *__r
                 if (c0 + j < cols) crow[4 * g + j] = scale2(acc[j], er + fb[c0 + j]);
         }
     }
-    if (bad) {   // 8 columns aligned to 8: inside one word of the element mask
+    if (CERT && bad) {   // 8 columns aligned to 8: inside one word of the element mask
         atomicOr(cc.emask + row * cc.ldw + (c16 >> 5), bad << (c16 & 31));
         uint32_t *f = cc.flags + (row >> 7) * cc.ldf + (c16 >> 7);
         if (atomicExch(f, 1u) == 0u) atomicAdd(cc.fallback, 1u);
@@ -792,15 +796,15 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
         const int vec = ((reinterpret_cast<uintptr_t>(C) & 15u) == 0 && (ldc & 1) == 0) ? 1 : 0;
         Oz2CrtCert cc;
         if (guard && guard->rsign) {   // R23: the certificate of sign-uniform rows / columns
-            if (!guard->csign || !guard->sa || !guard->sb || !guard->flags || !guard->emask || !guard->fallback)
+            if (!guard->sbu || !guard->rowT || !guard->sa || !guard->flags || !guard->emask || !guard->fallback)
                 return cudaErrorInvalidValue;
+            cc.rowT = guard->rowT;
             cc.rsign = guard->rsign;
             cc.rsign_ld = guard->rsign_ld;
-            cc.csign = guard->csign;
+            cc.sbu = guard->sbu;
             cc.sa = guard->sa;
             cc.sa_ld = guard->sa_ld;
-            cc.sb = guard->sb;
-            cc.thr = (guard->tau / (1.0 + guard->tau) - 0x1p-52) * (1.0 - 0x1p-48);
+            cc.thr4 = oz2_uniform_thr4(guard->tau);
             cc.flags = guard->flags;
             cc.ldf = guard->ldf;
             cc.emask = guard->emask;
@@ -811,13 +815,13 @@ cudaError_t launch_ozaki2_reconstruct(const uint8_t *R, int64_t ldr, int64_t pla
         dim3 grid((unsigned)((cols + 255) / 256), (unsigned)std::min<int64_t>((rows + 7) / 8, 65535));
         switch (P.n) {
 #define OZ2_CASE(k) \
-    case k:                                                                                                    \
-        if (cc.rsign)                                                                                          \
-            oz2_crt_fp64_kernel<k, true><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec,  \
-                                                                ea_ld, cc);                                    \
-        else                                                                                                   \
-            oz2_crt_fp64_kernel<k, false><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, vec, \
-                                                                 ea_ld, cc);                                   \
+    case k:                                                                                              \
+        if (cc.rsign)                                                                                    \
+            oz2_crt_fp64_kernel<k, true><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows, cols, \
+                                                                vec, ea_ld, cc);                         \
+        else                                                                                             \
+            oz2_crt_fp64_kernel<k, false><<<grid, block, 0, s>>>(R, ldr, plane, ea, fb, f, C, ldc, rows,      \
+                                                                 cols, vec, ea_ld, cc);                  \
         break;
             OZ2_CASE(2) OZ2_CASE(3) OZ2_CASE(4) OZ2_CASE(5) OZ2_CASE(6) OZ2_CASE(7) OZ2_CASE(8) OZ2_CASE(9)
             OZ2_CASE(10) OZ2_CASE(11) OZ2_CASE(12) OZ2_CASE(13) OZ2_CASE(14)

@@ -116,7 +116,13 @@ struct Oz2Guard {
     int64_t rsign_ld = 1;
     const unsigned *csign = nullptr;      // columns of the launch
     unsigned *sign_word = nullptr;        // the launch's "some row or column mixes signs" word
+    double *sbu = nullptr;                // per column (written by the column-term pass): sb_j rounded
+                                          // up to double, -1 for a column that mixes signs
+    unsigned long long *sbmax = nullptr;  // the launch's largest uniform column term (double bits)
+    double *rowT = nullptr;               // per row of the launch: the CRT pass's bound T_i (0: none)
 };
+// thr4 = 4 (tau / (1 + tau) - 2^-52), rounded down: the R23 certificate's scale
+inline double oz2_uniform_thr4(double tau) { return 4.0 * (tau / (1.0 + tau) - 0x1p-52) * (1.0 - 0x1p-48); }
 // Persistent K6 launches per K chunk for n moduli on a rows x cols rectangle with
 // `clusters` co-resident CTA pairs (k_ozaki.cu).
 int oz2_launches_per_chunk(int n, int64_t rows, int64_t cols, int clusters);

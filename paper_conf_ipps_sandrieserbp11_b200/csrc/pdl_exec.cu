@@ -119,20 +119,21 @@ int worker_sgemm_mix(const WorkerCtx &w) {
 }
 
 // Ozaki-II per-column arrays of a task: [bmax: cols u64][sb: cols u64][sbd: cols double]
-// [fb: cols int][csign: cols u32] in the shared BUF_OZE (it does not move with `rows`, so
+// [fb: cols int][csign: cols u32][sbu: cols double] in the shared BUF_OZE (it does not move with `rows`, so
 // a prepared B survives row-chunk tasks, REUSE_B).  The A side (residues, e_i, sa_i)
 // lives in the packed prepared-A rows (pdlk::oz2_prep_row_bytes).  sb: the certificate's
-// column sums; csign: each column's sign bits (R23).
+// column sums; csign: each column's sign bits, sbu: the CRT certificate's column term (R23).
 static int oz_b_arrays(WorkerCtx &w, int64_t cols, unsigned long long **bmax, int **fb, unsigned long long **sb,
-                       double **sbd, unsigned **csign) {
+                       double **sbd, unsigned **csign, double **sbu) {
     void *p = nullptr;
-    int rc = ensure_buf(w, BUF_OZE, (size_t)cols * 24 + (size_t)round_up(cols, 2) * 4 + (size_t)cols * 4, &p);
+    int rc = ensure_buf(w, BUF_OZE, (size_t)cols * 32 + (size_t)round_up(cols, 2) * 8, &p);
     if (rc) return rc;
     *bmax = (unsigned long long *)p;
     *sb = *bmax + cols;
     *sbd = (double *)(*sb + cols);
     *fb = (int *)(*sbd + cols);
     *csign = (unsigned *)(*fb + round_up(cols, 2));
+    *sbu = (double *)(*csign + round_up(cols, 2));
     return PDL_OK;
 }
 
@@ -344,6 +345,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
     int *oz_ea = nullptr, *oz_fb = nullptr;
     unsigned long long *oz_bmax = nullptr, *oz_sa = nullptr, *oz_sb = nullptr;
     unsigned *oz_csign = nullptr, *oz_sign_words = nullptr;
+    double *oz_sbu = nullptr, *oz_rowT = nullptr;
     double *oz_sbd = nullptr;
     uint8_t *oz2_R = nullptr;
     int64_t oz2_ldr = 0, oz2_plane = 0;
@@ -367,7 +369,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         oz_sa_ld = oz_pr / 8;
         if ((rc = ensure_buf(w, BUF_OZB, P2.b8_bytes, &p))) return rc;
         b8 = (int8_t *)p;
-        if ((rc = oz_b_arrays(w, cols, &oz_bmax, &oz_fb, &oz_sb, &oz_sbd, &oz_csign))) return rc;
+        if ((rc = oz_b_arrays(w, cols, &oz_bmax, &oz_fb, &oz_sb, &oz_sbd, &oz_csign, &oz_sbu))) return rc;
         oz2_ldr = round_up(cols, 16);
         oz2_plane = oz2_ldr * rows;
         if ((rc = ensure(BUF_OZR, (size_t)(oz2_plane * P2.n * P2.nch), &p))) return rc;
@@ -376,12 +378,15 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
             // recompute flags of the rectangle's 128 x 128 tiles, and the Worker's
             // count of flagged tiles in this run (pdl_query "stats")
             G2.ldf = (cols + 127) / 128;
-            const size_t fbytes = (size_t)(((rows + 127) / 128) * G2.ldf * 4);
-            // + one "mixed signs" word per band x panel launch (R23), after the tile flags
-            if ((rc = ensure(BUF_OZF, fbytes + (size_t)RB * CP * 4, &p))) return rc;
+            const size_t fbytes = (size_t)round_up((int64_t)(((rows + 127) / 128) * G2.ldf * 4), 16);
+            // + 16 bytes per band x panel launch (R23), after the tile flags: the "mixed signs"
+            // word and the largest uniform column term
+            // and the rows' bounds T_i (8 bytes per row)
+            if ((rc = ensure(BUF_OZF, fbytes + (size_t)RB * CP * 16 + (size_t)rows * 8, &p))) return rc;
             G2.flags = (uint32_t *)p;
             if (oz2_uniform_shortcut(P2)) {
                 oz_sign_words = (unsigned *)((char *)p + fbytes);
+                oz_rowT = (double *)((char *)p + fbytes + (size_t)RB * CP * 16);
                 G2.rsign = (const unsigned *)(oz_ea + 1);   // the packed rows' pad words
                 G2.rsign_ld = oz_ea_ld;
                 G2.csign = oz_csign;
@@ -512,7 +517,10 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
                     if (G2.rsign) {   // R23: this band's rows, this panel's columns, this launch's word
                         gs.rsign = G2.rsign + r0 * G2.rsign_ld;
                         gs.csign = G2.csign + c0;
-                        gs.sign_word = oz_sign_words + (i * CP + j);
+                        gs.sign_word = oz_sign_words + 4 * (i * CP + j);
+                        gs.sbmax = (unsigned long long *)(gs.sign_word + 2);
+                        gs.rowT = oz_rowT + r0;
+                        gs.sbu = oz_sbu + c0;
                     }
                     gs.flags = G2.flags + (r0 / 128) * G2.ldf + c0 / 128;
                     gs.emask = G2.emask + r0 * G2.ldw + c0 / 32;
