@@ -275,7 +275,9 @@ __global__ void __launch_bounds__(256) oz2_rowmax_kernel(const double *__restric
     }
 }
 
-__global__ void __launch_bounds__(256) oz2_residue_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
+// (256, 3): 80 registers, three CTAs per SM -- more loads in flight than the 96-register
+// two-CTA build (C4: 1.57 -> 1.29 ms; a 64-register four-CTA build spills)
+__global__ void __launch_bounds__(256, 3) oz2_residue_rows_kernel(const double *__restrict__ A, int64_t lda, int64_t M,
                                                                int64_t K, int n, int np, int p, int64_t Kc, int nch,
                                                                int8_t *__restrict__ A8, int64_t ld8,
                                                                const int *__restrict__ ea, int64_t ea_ld, int vec,
@@ -373,7 +375,7 @@ __global__ void oz2_colmax_kernel(const double *__restrict__ B, int64_t ldb, int
 // walks the k tiles blockIdx.y, blockIdx.y + gridDim.y, ... of its 32 columns (one
 // tile per CTA below 65536 tiles) and adds its certificate column sums with one
 // atomic per column.
-__global__ void __launch_bounds__(256) oz2_split_cols_t_kernel(
+__global__ void __launch_bounds__(256, 3) oz2_split_cols_t_kernel(
     const double *__restrict__ B, int64_t ldb, int64_t K, int64_t N, int n, int np, int p, int64_t Kc, int nch,
     const unsigned long long *__restrict__ bmax, int8_t *__restrict__ Bt8, int64_t ld8, int *__restrict__ fb,
     unsigned long long *__restrict__ sb) {
