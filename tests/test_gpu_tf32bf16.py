@@ -282,3 +282,29 @@ def test_c4_full_size_sampled():
     C = mm(A, B, tile=c.tile)
     rows = W.sampled_rows(c.M, (), c.tile, n_random=64)
     check(C, A, B, rows=rows)
+
+
+def test_prepared_b_is_not_shared_between_variants(monkeypatch):
+    """The prepared-B cache (PDL_TASK_REUSE_B) keys on the task variant: a B split for
+    tf32bf16 (TF32 hi + BF16 pairs) is not read by a 3xtf32 task asking for reuse (TF32
+    hi/lo in the same buffers), and vice versa -- C equals a fresh run of each variant."""
+    M, N, K = 500, 390, 700
+    A = W.signed((M, K), np.float32, 91)
+    B = W.signed((K, N), np.float32, 92)
+    fresh = {v: mm(A, B, props={"SGEMM_VARIANT": v}) for v in ("tf32bf16", "3xtf32")}
+    assert not np.array_equal(fresh["tf32bf16"], fresh["3xtf32"])
+    pdl.load(pdl.descriptor_xml(1))
+    try:
+        dA, dB = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+        out = torch.empty((M, N), dtype=torch.float32, device="cuda")
+        for first, second in (("tf32bf16", "3xtf32"), ("3xtf32", "tf32bf16")):
+            monkeypatch.setenv("PDL_SGEMM_VARIANT", first)
+            pdl.task_matmul(dA, dB, out, local=True)
+            pdl.run()
+            assert np.array_equal(out.cpu().numpy(), fresh[first])
+            monkeypatch.setenv("PDL_SGEMM_VARIANT", second)
+            pdl.task_matmul(dA, dB, out, local=True, reuse_b=True)
+            pdl.run()
+            assert np.array_equal(out.cpu().numpy(), fresh[second])
+    finally:
+        pdl.unload()
