@@ -139,8 +139,10 @@ def test_huge_times_zero_is_not_certified():
 # and the library certifies the element in the CRT pass when
 #     (sa_i + sb_j + min(sa_i, sb_j)) / 4 <= thr |X_ij|,   thr = tau / (1 + tau) - 2^-52
 # (X = fl(A'B'), the scaled result).  Pinned: (4) a row / column is called uniform only
-# when D_ij = |(AB)_ij| holds exactly, and (5) an element certified this way has
-# |C_ij - (AB)_ij| <= tau D_ij.
+# when D_ij = |(AB)_ij| holds exactly, (5) an element certified this way has
+# |C_ij - (AB)_ij| <= tau D_ij, and (6) the same test is sound for any element, uniform or
+# not (D >= |AB| >= |C| - E always): the sign classification decides only where the test
+# is tight enough to make the lower-bound GEMM unnecessary, never correctness.
 
 def _sign_bits(v):
     return (1 if any(x > 0 for x in v) else 0) | (2 if any(x < 0 for x in v) else 0)
@@ -164,10 +166,11 @@ def emulate_uniform(A, B, p, tau):
             C = math.ldexp(X, e[i] + f[j] - 2 * p)
             P = sum(Fraction(float(A[i, k])) * Fraction(float(B[k, j])) for k in range(K))
             D = sum(abs(Fraction(float(A[i, k])) * Fraction(float(B[k, j]))) for k in range(K))
-            certified = uni and sa[i] > 0 and sb[j] > 0 and \
+            crt_ok = sa[i] > 0 and sb[j] > 0 and \
                 Fraction(sa[i] + sb[j] + min(sa[i], sb[j]), 4) <= thr * abs(Fraction(X))
+            certified = uni and crt_ok
             exact = sa[i] == 0 or sb[j] == 0
-            out.append((uni, certified, exact, abs(Fraction(C) - P), P, D))
+            out.append((uni, certified, exact, abs(Fraction(C) - P), P, D, crt_ok))
     return out
 
 
@@ -203,7 +206,7 @@ def test_uniform_certificate_holds(kind, p):
     A, B = _uniform_inputs(kind, rng)
     tau = 5e-13 if p >= 40 else 2.0 ** (-p + 6)
     n_cert = 0
-    for uni, certified, exact, err, P, D in emulate_uniform(A, B, p, tau):
+    for uni, certified, exact, err, P, D, crt_ok in emulate_uniform(A, B, p, tau):
         if uni:
             assert abs(P) == D                                   # (4)
         if exact:
@@ -211,6 +214,8 @@ def test_uniform_certificate_holds(kind, p):
         if certified:
             n_cert += 1
             assert err <= Fraction(tau) * D                      # (5)
+        if crt_ok:   # (6) the CRT-pass test is sound for ANY element: D >= |AB| >= |C| - E
+            assert err <= Fraction(tau) * D
     if kind in ("uniform", "negative_rows"):
         assert n_cert > 0
 
@@ -219,5 +224,5 @@ def test_uniform_certificate_refuses_huge_times_zero():
     """[2^60, 1] x [0, 1]^T: both uniform, D = 1, Ozaki II returns 0 -- not certified."""
     A = np.array([[2.0 ** 60, 1.0]])
     B = np.array([[0.0], [1.0]])
-    (uni, certified, exact, err, P, D), = emulate_uniform(A, B, 43, 5e-13)
+    (uni, certified, exact, err, P, D, _), = emulate_uniform(A, B, 43, 5e-13)
     assert uni and not certified and err == 1 and D == 1
