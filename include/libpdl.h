@@ -91,7 +91,7 @@ extern "C" {
                                 pdl_query("prepared_a/<dtype>/<K>") bytes (FP32: [TF32 hi: Kp
                                 floats][second plane: Kp floats -- tf32bf16: per 16-wide K block
                                 16 BF16 hi' then 16 BF16 lo'; 3xtf32: TF32 lo], Kp = K rounded up
-                                to 32; FP64 ozaki2: [residues: ld8 bytes][e_i: int32][4 bytes]
+                                to 32; FP64 ozaki2: [residues: ld8 bytes][e_i: int32][sign bits: u32]
                                 [certificate row sum: u64]); B and N are ignored.  C: 16-byte
                                 aligned memory of the Worker's device.  PDL_EUNSUPPORTED for
                                 variants that exchange raw rows (query answers 0: FP64 dmma) */

@@ -355,7 +355,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
         return set_err(PDL_EINVAL, "prepared A with DGEMM_VARIANT=ozaki2: the certificate's K1 recompute reads "
                                    "the raw A rows -- pass them (task_matmul_prepared Araw, this Worker's device)");
     if (ozaki2) {
-        // packed prepared-A rows: [residues: ld8][e_i: int][pad][sa_i: u64]
+        // packed prepared-A rows: [residues: ld8][e_i: int][sign bits: u32 (R23)][sa_i: u64]
         oz_pr = pdlk::oz2_prep_row_bytes(P2);
         if (prepared) {
             p = const_cast<void *>(A);
@@ -647,7 +647,7 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
 
 // Bytes per prepared A row (PDL_TASK_PREP_A) of the task variant of PU `pu` for
 // inner dimension K, 0 when the variant exchanges raw rows: FP32 3xTF32 -> [hi:
-// Kp floats][lo: Kp floats]; FP64 ozaki2 -> [residues: ld8 bytes][e_i][pad][sa_i]
+// Kp floats][lo: Kp floats]; FP64 ozaki2 -> [residues: ld8 bytes][e_i][sign bits][sa_i]
 // (pdlk::oz2_prep_row_bytes), and its prepared tasks still read the raw rows
 // (needs_raw: the certificate's K1 recompute); FP64 dmma -> 0.
 int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K, bool *needs_raw) {
