@@ -646,8 +646,9 @@ int run_rect(WorkerCtx &w, const Task &t, const void *A, const void *B, void *C,
 }
 
 // Bytes per prepared A row (PDL_TASK_PREP_A) of the task variant of PU `pu` for
-// inner dimension K, 0 when the variant exchanges raw rows: FP32 3xTF32 -> [hi:
-// Kp floats][lo: Kp floats]; FP64 ozaki2 -> [residues: ld8 bytes][e_i][sign bits][sa_i]
+// inner dimension K, 0 when the variant exchanges raw rows: FP32 -> [TF32 hi: Kp
+// floats][second plane: Kp floats (tf32bf16: BF16 [hi' | lo'] per 16-wide K block; 3xtf32:
+// TF32 lo)]; FP64 ozaki2 -> [residues: ld8 bytes][e_i][sign bits][sa_i]
 // (pdlk::oz2_prep_row_bytes), and its prepared tasks still read the raw rows
 // (needs_raw: the certificate's K1 recompute); FP64 dmma -> 0.
 int64_t prepared_a_row_bytes(int pu, int dtype, int64_t K, bool *needs_raw) {
