@@ -51,6 +51,8 @@ def emulated():
                 for line in f:
                     d = json.loads(line)
                     if "G" in d and d.get("config") == "C4":
+                        # "default" = the FP32 default when the file was written (3xtf32 before
+                        # round 2's tf32bf16; newer files name the variant)
                         var = {"default": "dmma" if d["dtype"] == "f64" else "3xtf32"}.get(
                             d.get("variant", "default"), d.get("variant"))
                         out[(d["dtype"], var, d["G"])] = d["max_concurrent_ms"] / 1e3

@@ -191,7 +191,10 @@ def main():
                 torch.cuda.empty_cache()
         finally:
             pdl.unload()
-        r = {"config": args.config, "dtype": args.dtype, "variant": args.variant or "default", "G": G,
+        # the variant by name (the FP32 default is tf32bf16 since round 2; older files say
+        # "default" for 3xtf32)
+        vname = args.variant or ("dmma" if args.dtype == "f64" else "tf32bf16")
+        r = {"config": args.config, "dtype": args.dtype, "variant": vname, "G": G,
              "sustain_s": args.sustain,
              "a_exchange": a_ex,
              "grid": [wps[0].Gr, wps[0].Gc],
