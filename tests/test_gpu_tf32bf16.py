@@ -308,3 +308,15 @@ def test_prepared_b_is_not_shared_between_variants(monkeypatch):
             assert np.array_equal(out.cpu().numpy(), fresh[second])
     finally:
         pdl.unload()
+
+
+@pytest.mark.parametrize("dist", ["uniform", "signed"])
+def test_long_k_2_pow_20(props, dist):
+    """Long-K edge for FP32: K = 2^20 + 3 (8192 promoted 128-wide chunks summed in FP32
+    registers with round-to-nearest, a ragged last K block) on a small ragged C; the
+    1e-5 bar holds for both variants."""
+    M, N, K = 70, 37, (1 << 20) + 3
+    gen = W.uniform if dist == "uniform" else W.signed
+    A = gen((M, K), np.float32, 83)
+    B = gen((K, N), np.float32, 84)
+    check(mm(A, B, props=props), A, B)
