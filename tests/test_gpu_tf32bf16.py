@@ -320,3 +320,48 @@ def test_long_k_2_pow_20(props, dist):
     A = gen((M, K), np.float32, 83)
     B = gen((K, N), np.float32, 84)
     check(mm(A, B, props=props), A, B)
+
+
+def _rz32(x):
+    """float64 -> float32 rounded toward zero (the TMEM accumulate, R16)."""
+    x = np.asarray(x, np.float64)
+    f = x.astype(np.float32)
+    over = np.abs(f.astype(np.float64)) > np.abs(x)
+    f[over] = np.nextafter(f[over], np.float32(0))
+    return f
+
+
+def _split_products(a, b, variant):
+    """The three exact products each K = 1 element of C is built from, in the kernel's
+    MMA order: the split of R22 / 3xTF32 (p1, p2: the corrections, p3 = hi*hi)."""
+    import test_tf32bf16_bound as tb
+    f = np.float64
+    ah, ahb, alb = (p.astype(f) for p in tb.split(a))
+    bh, bhb, blb = (p.astype(f) for p in tb.split(b))
+    A, Bt = np.meshgrid(np.arange(a.size), np.arange(b.size), indexing="ij")
+    if variant == "tf32bf16":   # per 16-wide K step: lo'*hi', hi'*lo', hi*hi
+        return alb[A] * bhb[Bt], ahb[A] * blb[Bt], ah[A] * bh[Bt]
+    al = tb.rna_tf32((a - tb.rna_tf32(a)).astype(np.float32)).astype(f)   # lo = rna_tf32(x - hi)
+    bl = tb.rna_tf32((b - tb.rna_tf32(b)).astype(np.float32)).astype(f)
+    return al[A] * bh[Bt], ah[A] * bl[Bt], ah[A] * bh[Bt]
+
+
+def test_k1_products_match_the_documented_arithmetic(props):
+    """Pin of the kernel's arithmetic independent of the oracle: for K = 1 every MMA adds
+    one exact product, so C follows from the split (R22 / 3xTF32), the MMA order and the
+    TMEM accumulate (R16), emulated on the CPU.  Where the corrections and hi*hi share a
+    sign, C is bitwise RZ(RZ(p1 + p2) + p3) (round-toward-zero adds); where they do not,
+    the accumulator truncates the aligned smaller addend toward zero first, so C is that
+    value or one FP32 ulp above it in magnitude (measured, R16).  A wrong operand
+    offset, plane or product would be far outside either."""
+    rng = np.random.default_rng(97)
+    a = ((rng.random(150) * 2 - 1) * np.exp2(rng.integers(-20, 21, 150))).astype(np.float32)
+    b = ((rng.random(130) * 2 - 1) * np.exp2(rng.integers(-20, 21, 130))).astype(np.float32)
+    C = mm(a[:, None].copy(), b[None, :].copy(), props=props)
+    p1, p2, p3 = _split_products(a, b, props["SGEMM_VARIANT"])
+    model = _rz32(_rz32(p1 + p2).astype(np.float64) + p3)
+    same = np.sign(p1 + p2) * np.sign(p3) >= 0
+    assert np.array_equal(C[same], model[same])
+    up = np.nextafter(model, np.copysign(np.float32(np.inf), model))   # one ulp away from zero
+    assert np.all((C == model) | (C == up))
+    assert same.mean() > 0.3 and (~same).mean() > 0.3
