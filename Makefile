@@ -24,7 +24,7 @@ all: $(LIB) $(ORACLE)
 examples: examples/dgemm_c_abi
 
 # measurement tools (peaks, tensor-core behaviour, green-context splits)
-TOOLS := tools/microbench tools/tc_microbench tools/tc_probe tools/fp64_mix_probe tools/green_probe tools/cluster_probe
+TOOLS := tools/microbench tools/tc_microbench tools/tc_probe tools/fp64_mix_probe tools/green_probe tools/cluster_probe tools/feed_probe
 tools: $(TOOLS)
 
 tools/%: tools/%.cu
