@@ -46,8 +46,8 @@ constexpr int GROUP_M_MIX = 8, GROUP_M_3X = 4;
 // K-block width BKF (floats per stage row): 32 = one 128-byte swizzle row (SWIZZLE_128B),
 // 3-stage ring of 64 KiB (default); 16 = 64-byte rows (SWIZZLE_64B), 7-stage ring of 32 KiB,
 // which keeps 6 stages in flight ahead of the MMAs instead of 2.  The deeper ring measured
-// slower (profiles/r02_k2_measurements.md): the kernel is bound by the chip-wide L2 -> SM
-// feed, not by prefetch depth, and the smaller stages double the barrier round trips.
+// slower (profiles/r02_k2_measurements.md): its smaller stages double the barrier round trips
+// and the MMAs lose more than the feed (16.3 TB/s, held back by L2 misses) gains.
 template <int BKF>
 struct Cfg {
     static constexpr int BK = BKF;
